@@ -105,6 +105,11 @@ mce_status mce_load_csr(int32_t device, int64_t n, const int64_t *row_ptr, const
 
 void mce_graph_free(mce_graph *g);
 
+/* Drop the cached preprocessing (core numbers, orientation) so that the next
+ * mce_enumerate / mce_find_one recomputes it -- used by benchmarks that time
+ * the whole pipeline from a resident CSR. */
+mce_status mce_graph_clear_cache(mce_graph *g);
+
 /* k-core decomposition + orientation (PAPER.md II-B-2 line 61, IV-C line
  * 131).  Run implicitly by mce_enumerate / mce_find_one; exposed for tests.
  * core_out (device or host per `where`, int32[n], may be NULL): core numbers.

@@ -1,0 +1,503 @@
+// Breadth-first maximum clique driver (PAPER.md IV-D Algorithm 2 MAXCLIQUES,
+// IV-E windowed search) over the device kernels of expand.cu.
+//
+//  run():   preprocess -> heuristic lower bound -> roots grouped by candidate
+//           set width W -> windows of roots -> level-synchronous expansion.
+//  process(k): one level: count pass (+ leaf capture) -> scan -> write pass
+//           of the next level -> recurse.  When the next level would exceed
+//           the frontier budget it is produced and explored in chunks
+//           (the paper's windowing applied at any depth, V-C-3 "Recursive
+//           Windowing"), so the frontier never exceeds the budget.
+#include <algorithm>
+#include <chrono>
+#include <cstdio>
+#include <cstring>
+#include <numeric>
+#include <vector>
+
+#include "engine.cuh"
+#include "expand.cuh"
+#include "heuristic.cuh"
+
+namespace mce {
+
+namespace {
+constexpr size_t kAlign = 256;
+
+struct Arena {
+    DevBuf<uint8_t> buf;
+    size_t top = 0;
+    void init(size_t bytes) {
+        buf.alloc(bytes);
+        top = 0;
+    }
+    size_t avail() const { return buf.n > top ? buf.n - top : 0; }
+    template <typename T>
+    T *alloc(int64_t count) {
+        size_t bytes = ((size_t)std::max<int64_t>(count, 1) * sizeof(T) + kAlign - 1) / kAlign * kAlign;
+        if (top + bytes > buf.n)
+            fail(MCE_ERR_BUDGET, "frontier budget exhausted (need " + std::to_string(bytes) + " more bytes, " +
+                                     std::to_string(avail()) + " available)");
+        T *p = reinterpret_cast<T *>(buf.p + top);
+        top += bytes;
+        return p;
+    }
+};
+
+struct Level {
+    int64_t count = 0;
+    uint64_t *P = nullptr;
+    int32_t *slot = nullptr;
+    int32_t *parent = nullptr;
+    int32_t *vloc = nullptr;
+};
+
+class Timer {
+   public:
+    explicit Timer(cudaStream_t s) : s_(s) {
+        MCE_CUDA(cudaEventCreate(&a_));
+        MCE_CUDA(cudaEventCreate(&b_));
+    }
+    ~Timer() {
+        cudaEventDestroy(a_);
+        cudaEventDestroy(b_);
+    }
+    void start() { MCE_CUDA(cudaEventRecord(a_, s_)); }
+    void stop() { MCE_CUDA(cudaEventRecord(b_, s_)); pending_ = true; }
+    // accumulate after the stream has been synchronised past stop()
+    double collect() {
+        if (!pending_) return 0.0;
+        float ms = 0;
+        MCE_CUDA(cudaEventElapsedTime(&ms, a_, b_));
+        pending_ = false;
+        return ms;
+    }
+
+   private:
+    cudaStream_t s_;
+    cudaEvent_t a_, b_;
+    bool pending_ = false;
+};
+
+class Engine {
+   public:
+    Engine(mce_graph *g, const mce_options &o, bool find_one) : g_(g), o_(o), find_one_(find_one), s_(g->stream) {}
+
+    mce_result *run();
+
+   private:
+    int32_t need() const { return find_one_ ? best_ + 1 : best_; }
+    void process(int32_t k, const Level &L);
+    void do_class(int32_t cls, const int32_t *list, int64_t count);
+    void handle_leaves(int32_t size, int64_t cnt, ExpandArgs &a);
+    void sync_bound(bool active);
+    void launch_timed(const ExpandArgs &a, bool write);
+
+    mce_graph *g_;
+    mce_options o_;
+    bool find_one_;
+    cudaStream_t s_;
+    Arena arena_;
+    int32_t best_ = 0;
+    int32_t W_ = 1;
+    int64_t stride_ = 1, offset_ = 0;
+
+    // leaves
+    DevBuf<unsigned long long> leaf_count_;
+    DevBuf<int32_t> stage_;
+    int64_t stage_rows_ = 0;
+    std::vector<int32_t> rows_;  // host copy of the stored cliques (width res_size_)
+    int32_t res_size_ = 0;
+    int64_t res_count_ = 0;
+    bool truncated_ = false;
+
+    // chain of levels for clique read-out
+    DevBuf<LevelLink> chain_dev_;
+    int32_t chain_cap_ = 0;
+
+    const RootInfo *roots_ = nullptr;
+    const uint64_t *adj_ = nullptr;
+
+    // stats
+    std::vector<int64_t> level_entries_;
+    double t_expand_ms_ = 0.0, t_count_ms_ = 0.0;
+    int64_t count_launches_ = 0, kernels_ = 0;
+    double count_bytes_ = 0.0;
+    DevBuf<unsigned long long> pbits_;  // sum of |P| over counted entries (algorithmic bytes)
+};
+
+void Engine::launch_timed(const ExpandArgs &a, bool write) {
+    Timer t(s_);
+    t.start();
+    launch_expand(a, write, s_);
+    t.stop();
+    MCE_CUDA(cudaStreamSynchronize(s_));
+    double ms = t.collect();
+    t_expand_ms_ += ms;
+    ++kernels_;
+    if (!write) {
+        t_count_ms_ += ms;
+        ++count_launches_;
+        const double n = (double)(a.end - a.begin);
+        count_bytes_ += n * (8.0 * a.W + 4 + 4 + 4 + sizeof(RootInfo));
+    }
+}
+
+void Engine::sync_bound(bool active) {
+    if (!o_.bound_sync) return;
+    int32_t gactive = 0;
+    int32_t gb = o_.bound_sync(best_, active ? 1 : 0, &gactive, o_.bound_sync_user);
+    if (gb > best_) best_ = gb;
+}
+
+void Engine::handle_leaves(int32_t size, int64_t cnt, ExpandArgs &a) {
+    if (cnt <= 0) return;
+    if (find_one_) {
+        // all leaves of this launch have size k+1 > best: keep the first
+        best_ = size;
+        res_size_ = size;
+        res_count_ = 1;
+        rows_.resize(size);
+        MCE_CUDA(cudaMemcpy(rows_.data(), stage_.get(), sizeof(int32_t) * size, cudaMemcpyDeviceToHost));
+        return;
+    }
+    if (size > res_size_) {
+        rows_.clear();
+        res_size_ = size;
+        res_count_ = 0;
+        truncated_ = false;
+    }
+    if (size > best_) best_ = size;
+    const int64_t stored = (int64_t)rows_.size() / std::max(res_size_, 1);
+    int64_t want = cnt;
+    if (o_.max_cliques > 0) want = std::min<int64_t>(want, std::max<int64_t>(o_.max_cliques - stored, 0));
+    if (want > a.leaf_cap) {  // staging too small: grow and replay the count pass (idempotent)
+        stage_rows_ = want;
+        stage_.alloc((size_t)want * std::max<int32_t>(g_->max_out + 2, 2));
+        a.leaf_rows = stage_.get();
+        a.leaf_cap = want;
+        MCE_CUDA(cudaMemsetAsync(leaf_count_.get(), 0, sizeof(unsigned long long), s_));
+        launch_expand(a, false, s_);
+        ++kernels_;
+        MCE_CUDA(cudaStreamSynchronize(s_));
+    }
+    const int64_t take = std::min<int64_t>(want, a.leaf_cap);
+    if (take > 0) {
+        size_t old = rows_.size();
+        rows_.resize(old + (size_t)take * size);
+        MCE_CUDA(cudaMemcpy(rows_.data() + old, stage_.get(), sizeof(int32_t) * take * size, cudaMemcpyDeviceToHost));
+    }
+    if (take < cnt) truncated_ = true;
+    res_count_ += cnt;
+}
+
+void Engine::process(int32_t k, const Level &L) {
+    if ((int64_t)level_entries_.size() <= k) level_entries_.resize(k + 1, 0);
+    level_entries_[k] += L.count;
+    if (k + 2 > chain_cap_) {
+        int32_t cap = std::max(256, 2 * (k + 2));
+        DevBuf<LevelLink> nc(cap);
+        if (chain_cap_) MCE_CUDA(cudaMemcpyAsync(nc.get(), chain_dev_.get(), sizeof(LevelLink) * chain_cap_,
+                                                 cudaMemcpyDeviceToDevice, s_));
+        chain_dev_ = std::move(nc);
+        chain_cap_ = cap;
+    }
+    LevelLink link{L.parent, L.vloc};
+    MCE_CUDA(cudaMemcpyAsync(chain_dev_.get() + k, &link, sizeof(link), cudaMemcpyHostToDevice, s_));
+
+    const size_t mark = arena_.top;
+    const int64_t N = L.count;
+    int32_t *counts = arena_.alloc<int32_t>(N);
+    int64_t *offs = arena_.alloc<int64_t>(N + 1);
+    int64_t *tmp = arena_.alloc<int64_t>(scan_tmp_items(N));
+    int64_t *chunk = arena_.alloc<int64_t>(4);
+
+    ExpandArgs a{};
+    a.P = L.P;
+    a.slot = L.slot;
+    a.parent = L.parent;
+    a.vloc = L.vloc;
+    a.begin = 0;
+    a.end = N;
+    a.k = k;
+    a.need = need();
+    a.bound = o_.bound;
+    a.W = W_;
+    a.roots = roots_;
+    a.adj = adj_;
+    a.ocol = g_->ocol.get();
+    a.order = g_->order.get();
+    a.counts = counts;
+    a.leaf_count = leaf_count_.get();
+    a.leaf_rows = stage_.get();
+    a.leaf_cap = stage_rows_;
+    a.chain = chain_dev_.get();
+
+    MCE_CUDA(cudaMemsetAsync(leaf_count_.get(), 0, sizeof(unsigned long long), s_));
+    launch_timed(a, false);
+    exclusive_scan_i32(counts, offs, N, tmp, s_);
+    kernels_ += 3;
+    int64_t total = 0;
+    unsigned long long leaves = 0;
+    MCE_CUDA(cudaMemcpyAsync(&total, offs + N, sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
+    MCE_CUDA(cudaMemcpyAsync(&leaves, leaf_count_.get(), sizeof(leaves), cudaMemcpyDeviceToHost, s_));
+    MCE_CUDA(cudaStreamSynchronize(s_));
+    if (o_.verbose > 0)
+        fprintf(stderr, "[mce] level k=%d entries=%lld children=%lld leaves=%llu need=%d\n", k, (long long)N,
+                (long long)total, leaves, a.need);
+    if (leaves) handle_leaves(k + 1, (int64_t)leaves, a);
+
+    const int64_t per_child = 8 * W_ + 12 + 12 + 16;
+    int64_t a0 = 0;
+    while (total > 0 && a0 < N) {
+        const int64_t cap = (int64_t)(arena_.avail() / 2) / per_child;
+        int64_t b, cnt, base;
+        if (a0 == 0 && total <= cap) {
+            b = N;
+            cnt = total;
+            base = 0;
+        } else {
+            launch_find_chunk_end(offs, a0, N, cap, chunk, s_);
+            ++kernels_;
+            int64_t h[3];
+            MCE_CUDA(cudaMemcpyAsync(h, chunk, sizeof(h), cudaMemcpyDeviceToHost, s_));
+            MCE_CUDA(cudaStreamSynchronize(s_));
+            b = h[0];
+            cnt = h[1];
+            base = h[2];
+            if (b == a0)
+                fail(MCE_ERR_BUDGET, "the children of one candidate at level " + std::to_string(k) +
+                                         " exceed the frontier budget");
+        }
+        const size_t cmark = arena_.top;
+        Level C;
+        C.count = cnt;
+        C.P = arena_.alloc<uint64_t>(cnt * W_);
+        C.slot = arena_.alloc<int32_t>(cnt);
+        C.parent = arena_.alloc<int32_t>(cnt);
+        C.vloc = arena_.alloc<int32_t>(cnt);
+        ExpandArgs w = a;
+        w.begin = a0;
+        w.end = b;
+        w.offsets = offs;
+        w.out_base = base;
+        w.cP = C.P;
+        w.cslot = C.slot;
+        w.cparent = C.parent;
+        w.cvloc = C.vloc;
+        launch_timed(w, true);
+        sync_bound(true);
+        if (cnt > 0) process(k + 1, C);
+        arena_.top = cmark;
+        a0 = b;
+    }
+    arena_.top = mark;
+}
+
+void Engine::do_class(int32_t cls, const int32_t *list, int64_t count) {
+    // this shard's view: positions offset_, offset_+stride_, ...
+    const int64_t mine = count > offset_ ? (count - offset_ + stride_ - 1) / stride_ : 0;
+    if (mine <= 0) return;
+    W_ = 1 << cls;
+    const int32_t *base = list + offset_;
+    // adjacency rows per root -> prefix (host copy, to cut windows)
+    std::vector<int64_t> prefix(mine + 1);
+    {
+        const size_t mark = arena_.top;
+        int32_t *len = arena_.alloc<int32_t>(mine);
+        int64_t *pre = arena_.alloc<int64_t>(mine + 1);
+        int64_t *tmp = arena_.alloc<int64_t>(scan_tmp_items(mine));
+        launch_root_lengths(base, mine, stride_, g_->orp.get(), len, s_);
+        exclusive_scan_i32(len, pre, mine, tmp, s_);
+        kernels_ += 4;
+        MCE_CUDA(cudaMemcpyAsync(prefix.data(), pre, sizeof(int64_t) * (mine + 1), cudaMemcpyDeviceToHost, s_));
+        MCE_CUDA(cudaStreamSynchronize(s_));
+        arena_.top = mark;
+    }
+    // windows from the highest ranks down (densest cores first)
+    int64_t hi = mine;
+    while (hi > 0) {
+        const size_t mark = arena_.top;
+        const int64_t room = (int64_t)(arena_.avail() / 4);
+        const int64_t per_root = sizeof(RootInfo) + 8 * W_ + 12 + 64;
+        int64_t lo = hi - 1;
+        int64_t maxw = o_.window > 0 ? o_.window : hi;
+        // grow the window while it fits a quarter of the free budget
+        {
+            int64_t l = std::max<int64_t>(0, hi - maxw), h = hi - 1;  // smallest lo that fits
+            while (l < h) {
+                int64_t mid = (l + h) / 2;
+                int64_t bytes = (prefix[hi] - prefix[mid]) * 8 * W_ + (hi - mid) * per_root;
+                if (bytes <= room)
+                    h = mid;
+                else
+                    l = mid + 1;
+            }
+            lo = l;
+        }
+        const int64_t nw = hi - lo;
+        const int64_t rows = prefix[hi] - prefix[lo];
+        RootInfo *roots = arena_.alloc<RootInfo>(nw);
+        int64_t *pre = arena_.alloc<int64_t>(nw + 1);
+        uint64_t *adj = arena_.alloc<uint64_t>(rows * W_);
+        // row prefix of this window, relative to lo
+        {
+            std::vector<int64_t> rel(nw + 1);
+            for (int64_t i = 0; i <= nw; ++i) rel[i] = prefix[lo + i] - prefix[lo];
+            MCE_CUDA(cudaMemcpyAsync(pre, rel.data(), sizeof(int64_t) * (nw + 1), cudaMemcpyHostToDevice, s_));
+            MCE_CUDA(cudaStreamSynchronize(s_));
+        }
+        launch_make_roots(base + lo * stride_, nw, stride_, W_, g_->orp.get(), pre, roots, s_);
+        launch_build_adj(roots, nw, W_, g_->orp.get(), g_->ocol.get(), adj, s_);
+        kernels_ += 2;
+        roots_ = roots;
+        adj_ = adj;
+        Level L1;
+        L1.count = nw;
+        L1.P = arena_.alloc<uint64_t>(nw * W_);
+        L1.slot = arena_.alloc<int32_t>(nw);
+        L1.parent = arena_.alloc<int32_t>(nw);
+        L1.vloc = arena_.alloc<int32_t>(nw);
+        launch_init_level1(roots, nw, W_, L1.P, L1.slot, L1.parent, L1.vloc, s_);
+        ++kernels_;
+        process(1, L1);
+        sync_bound(true);
+        arena_.top = mark;
+        hi = lo;
+    }
+}
+
+mce_result *Engine::run() {
+    auto *res = new mce_result();
+    const int64_t n = g_->n;
+    stride_ = o_.shard_count > 1 ? o_.shard_count : 1;
+    offset_ = o_.shard_count > 1 ? o_.shard_rank : 0;
+    if (n == 0) {  // the empty clique is the only clique of the null graph
+        res->omega = 0;
+        res->count = 1;
+        res->stored = 1;
+        sync_bound(false);
+        return res;
+    }
+    if (g_->nnz == 0) {  // edgeless: every vertex is a maximum clique
+        res->omega = 1;
+        for (int64_t v = offset_; v < n; v += stride_) {
+            if (find_one_ && !res->rows.empty()) break;
+            res->rows.push_back((int32_t)v);
+        }
+        res->stored = (int64_t)res->rows.size();
+        res->count = find_one_ ? 1 : res->stored;
+        if (o_.max_cliques > 0 && res->stored > o_.max_cliques) {
+            res->rows.resize(o_.max_cliques);
+            res->stored = o_.max_cliques;
+            res->truncated = 1;
+        }
+        sync_bound(false);
+        return res;
+    }
+    preprocess(g_, o_.orientation);
+    res->t_pre_ms = g_->t_pre_ms;
+    kernels_ += g_->kernels;
+
+    int heur = o_.heuristic;
+    if (find_one_ && heur == 0) heur = 1;  // find-one needs an incumbent clique
+    HeuristicResult hr = run_heuristic(g_, heur, o_.heuristic_runs, (int32_t)offset_, (int32_t)stride_, false);
+    res->t_heur_ms = hr.ms;
+    kernels_ += hr.kernels;
+    best_ = std::max<int32_t>(hr.omega_bar, 2);
+    if (find_one_) {
+        res_size_ = hr.omega_bar;
+        res_count_ = 1;
+        rows_ = hr.clique;
+        if (o_.bound_sync) sync_bound(true);
+    } else {
+        best_ = std::max(best_, o_.lower_bound);
+        sync_bound(true);
+    }
+
+    // frontier budget
+    size_t free_b = 0, total_b = 0;
+    MCE_CUDA(cudaMemGetInfo(&free_b, &total_b));
+    int64_t budget = o_.budget_bytes;
+    if (budget <= 0)
+        budget = std::min<int64_t>((int64_t)(free_b * 0.8), (int64_t)(1ll << 30) + 48ll * g_->nnz + 64ll * n);
+    budget = std::min<int64_t>(budget, (int64_t)(free_b * 0.95));
+    arena_.init((size_t)budget);
+    leaf_count_.alloc(1);
+    stage_rows_ = find_one_ ? 1 : 4096;
+    stage_.alloc((size_t)stage_rows_ * std::max<int32_t>(g_->max_out + 2, 2));
+    pbits_.alloc(1);
+
+    Timer tt(s_);
+    tt.start();
+    // roots worth expanding: 1 + |N+(r)| >= need
+    {
+        const size_t mark = arena_.top;
+        int32_t *cls = arena_.alloc<int32_t>(n);
+        int32_t *flag = arena_.alloc<int32_t>(n);
+        int64_t *pos = arena_.alloc<int64_t>(n + 1);
+        int64_t *tmp = arena_.alloc<int64_t>(scan_tmp_items(n));
+        launch_classify_roots(n, g_->orp.get(), std::max<int32_t>(need() - 1, 1), cls, s_);
+        ++kernels_;
+        std::vector<std::pair<int32_t, int64_t>> classes;
+        std::vector<int32_t *> lists;
+        for (int32_t c = kMaxClass - 1; c >= 0; --c) {
+            launch_flag_eq(n, cls, c, flag, s_);
+            exclusive_scan_i32(flag, pos, n, tmp, s_);
+            int64_t cnt = 0;
+            MCE_CUDA(cudaMemcpyAsync(&cnt, pos + n, sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
+            MCE_CUDA(cudaStreamSynchronize(s_));
+            kernels_ += 4;
+            if (cnt == 0) continue;
+            int32_t *list = arena_.alloc<int32_t>(cnt);
+            launch_compact(n, flag, pos, list, s_);
+            ++kernels_;
+            classes.push_back({c, cnt});
+            lists.push_back(list);
+        }
+        {  // any root too wide for the kernels?
+            launch_flag_eq(n, cls, 100, flag, s_);
+            exclusive_scan_i32(flag, pos, n, tmp, s_);
+            int64_t cnt = 0;
+            MCE_CUDA(cudaMemcpyAsync(&cnt, pos + n, sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
+            MCE_CUDA(cudaStreamSynchronize(s_));
+            if (cnt) fail(MCE_ERR_INVALID, "out-degree above 16384 after orientation is not supported");
+        }
+        // the class lists stay allocated below `mark` while the classes run
+        for (size_t i = 0; i < classes.size(); ++i) do_class(classes[i].first, lists[i], classes[i].second);
+        arena_.top = mark;
+    }
+    tt.stop();
+    MCE_CUDA(cudaStreamSynchronize(s_));
+    res->t_enum_ms = tt.collect();
+    // keep answering the other shards until everyone is done
+    if (o_.bound_sync) {
+        int32_t gactive = 1;
+        int guard = 0;
+        while (gactive && guard++ < (1 << 30)) {
+            int32_t gb = o_.bound_sync(best_, 0, &gactive, o_.bound_sync_user);
+            if (gb > best_) best_ = gb;
+        }
+    }
+    res->omega = res_size_;
+    res->count = res_count_;
+    res->rows = std::move(rows_);
+    res->stored = res_size_ > 0 ? (int64_t)res->rows.size() / res_size_ : 0;
+    res->truncated = truncated_ ? 1 : 0;
+    res->level_entries = level_entries_;
+    res->t_count_ms = t_count_ms_;
+    res->count_launches = count_launches_;
+    res->count_bytes = count_bytes_;
+    res->t_expand_ms = t_expand_ms_;
+    res->kernels = kernels_;
+    return res;
+}
+
+}  // namespace
+
+mce_result *run_engine(mce_graph *g, const mce_options &o, bool find_one) {
+    Engine e(g, o, find_one);
+    return e.run();
+}
+
+}  // namespace mce

@@ -1,0 +1,22 @@
+// Engine entry point and the result object behind the C ABI.
+#pragma once
+#include <vector>
+
+#include "graph.cuh"
+#include "mce.h"
+
+struct mce_result {
+    int32_t omega = 0;
+    int64_t count = 0;     // multiplicity (exact)
+    int64_t stored = 0;    // rows available
+    int32_t truncated = 0;
+    std::vector<int32_t> rows;  // stored * omega original vertex ids
+    bool canonical = false;     // rows sorted (each clique ascending, list lexicographic)
+    std::vector<int64_t> level_entries;
+    double t_pre_ms = 0, t_heur_ms = 0, t_enum_ms = 0, t_expand_ms = 0, t_count_ms = 0, count_bytes = 0;
+    int64_t count_launches = 0, kernels = 0;
+};
+
+namespace mce {
+mce_result *run_engine(mce_graph *g, const mce_options &o, bool find_one);
+}

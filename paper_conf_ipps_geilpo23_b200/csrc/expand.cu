@@ -1,0 +1,539 @@
+// Expansion kernels: every k-clique candidate (C, P) of a level is expanded
+// into its (k+1)-clique candidates (PAPER.md IV-D, Algorithm 2).
+//
+// Layout (B200 design, not the paper's clique list): the candidates of one
+// root r live in the root-local space V = N+(r) (the out-neighbours of r in
+// the degeneracy orientation, so |V| <= degeneracy); a candidate set P is a
+// W-word bitset over V and the root's induced adjacency is a bit matrix A
+// (|V| rows x W words) built once per root with warp-cooperative sorted-list
+// membership tests compacted by __ballot_sync (launch_build_adj).  Every
+// deeper intersection "P after v, restricted to N(v)" (Algorithm 2 lines 4-5)
+// is then one AND of W words instead of a binary search per pair.
+//
+// Pruning (PAPER.md II-B-3, line 63) against the running lower bound `need`:
+//   bound 0: |C| + |P|                 (Algorithm 2 line 8)
+//   bound 1: |C| + colours(P), greedy sequential colouring of G[P]
+//            ("a tighter upper bound using ... vertex coloring"), branching
+//            from the highest colour down (Tomita-Seki MCQ order), so a
+//            branch is cut as soon as |C| + colour(v) < need.
+// A child with an empty candidate set is a clique that cannot grow inside
+// its branch: when its size reaches `need` it is recorded (leaf).
+// Children go to the next level through the count pass -> scan -> write pass
+// (Algorithm 2 lines 29-35: COUNTCLIQUES, CUBSCAN, OUTPUTNEWCLIQUES).
+#include "expand.cuh"
+
+namespace mce {
+
+namespace {
+
+__device__ __forceinline__ bool adjacent_ranks(const int64_t *__restrict__ orp, const int32_t *__restrict__ ocol,
+                                               int32_t a, int32_t b) {
+    // edges point from lower to higher rank; rows sorted ascending
+    if (a > b) {
+        int32_t t = a;
+        a = b;
+        b = t;
+    }
+    return contains_sorted(ocol, __ldg(orp + a), __ldg(orp + a + 1), b);
+}
+
+// W == 1: one warp per root, lane i builds row i (and i+32) of the 64x64 matrix
+__global__ void build_adj_w1(const RootInfo *__restrict__ roots, int64_t nroots, const int64_t *__restrict__ orp,
+                             const int32_t *__restrict__ ocol, uint64_t *__restrict__ adj) {
+    const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    for (int64_t j = warp; j < nroots; j += nwarps) {
+        const RootInfo ri = roots[j];
+        const int32_t *V = ocol + ri.vbase;
+        for (int32_t i = lane; i < ri.L; i += 32) {
+            const int32_t a = __ldg(V + i);
+            uint64_t row = 0;
+            // j > i: V[j] in N+(a) -- one merge pass over two sorted lists
+            int64_t p = __ldg(orp + a), pe = __ldg(orp + a + 1);
+            for (int32_t c = i + 1; c < ri.L && p < pe; ++c) {
+                const int32_t b = __ldg(V + c);
+                while (p < pe && __ldg(ocol + p) < b) ++p;
+                if (p < pe && __ldg(ocol + p) == b) row |= 1ull << c;
+            }
+            // j < i: a in N+(V[j])
+            for (int32_t c = 0; c < i; ++c) {
+                const int32_t b = __ldg(V + c);
+                if (contains_sorted(ocol, __ldg(orp + b), __ldg(orp + b + 1), a)) row |= 1ull << c;
+            }
+            adj[ri.abase + i] = row;
+        }
+    }
+}
+
+// W >= 2: one block per root, one warp per row, 32 columns per __ballot_sync
+__global__ void build_adj_wide(const RootInfo *__restrict__ roots, int64_t nroots, int W,
+                               const int64_t *__restrict__ orp, const int32_t *__restrict__ ocol,
+                               uint64_t *__restrict__ adj) {
+    const int lane = threadIdx.x & 31;
+    const int wib = threadIdx.x >> 5, nwb = blockDim.x >> 5;
+    uint32_t *adj32 = reinterpret_cast<uint32_t *>(adj);
+    for (int64_t j = blockIdx.x; j < nroots; j += gridDim.x) {
+        const RootInfo ri = roots[j];
+        const int32_t *V = ocol + ri.vbase;
+        for (int32_t i = wib; i < ri.L; i += nwb) {
+            const int32_t a = __ldg(V + i);
+            uint32_t *row = adj32 + 2 * (ri.abase + (int64_t)i * W);
+            for (int32_t c0 = 0; c0 < 64 * W; c0 += 32) {
+                const int32_t c = c0 + lane;
+                bool e = false;
+                if (c < ri.L && c != i) e = adjacent_ranks(orp, ocol, a, __ldg(V + c));
+                const unsigned m = __ballot_sync(0xffffffffu, e);
+                if (lane == 0) row[c0 >> 5] = m;
+            }
+        }
+    }
+}
+
+__global__ void init_level1_kernel(const RootInfo *__restrict__ roots, int64_t nroots, int W, uint64_t *P,
+                                   int32_t *slot, int32_t *parent, int32_t *vloc) {
+    for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < nroots; j += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t L = roots[j].L;
+        for (int w = 0; w < W; ++w) {
+            int32_t lo = w * 64;
+            uint64_t m = L >= lo + 64 ? ~0ull : (L > lo ? ((1ull << (L - lo)) - 1) : 0ull);
+            P[j * W + w] = m;
+        }
+        slot[j] = (int32_t)j;
+        parent[j] = -1;
+        vloc[j] = -1;
+    }
+}
+
+__device__ void record_leaf(const ExpandArgs &a, int64_t e, int32_t v, const RootInfo &ri) {
+    const unsigned long long idx = atomicAdd(a.leaf_count, 1ull);
+    if ((int64_t)idx >= a.leaf_cap) return;
+    const int32_t size = a.k + 1;
+    int32_t *row = a.leaf_rows + (int64_t)idx * size;
+    const int32_t *V = a.ocol + ri.vbase;
+    row[a.k] = a.order[V[v]];
+    int64_t cur = e;
+    for (int32_t lev = a.k; lev >= 2; --lev) {
+        row[lev - 1] = a.order[V[a.chain[lev].vloc[cur]]];
+        cur = a.chain[lev].parent[cur];
+    }
+    row[0] = a.order[ri.r];
+}
+
+// ---------------------------------------------------------------------------
+// thread per candidate, W <= 2 words (|V| <= 128): the sparse-graph workhorse
+// ---------------------------------------------------------------------------
+template <int W, bool WRITE>
+__global__ void __launch_bounds__(256) expand_thread(const ExpandArgs a) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t e = a.begin + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < a.end; e += stride) {
+        int64_t out = 0;
+        if (WRITE) {
+            out = a.offsets[e];
+            if (a.offsets[e + 1] == out) continue;
+            out -= a.out_base;
+        }
+        uint64_t P[W];
+#pragma unroll
+        for (int w = 0; w < W; ++w) P[w] = a.P[e * W + w];
+        const RootInfo ri = a.roots[a.slot[e]];
+        const uint64_t *A = a.adj + ri.abase;
+        uint8_t ord[64 * W];
+        uint8_t colr[64 * W];
+        int np = 0;
+        int ncol = 0;
+        if (a.bound == 1) {
+            uint64_t U[W];
+#pragma unroll
+            for (int w = 0; w < W; ++w) U[w] = P[w];
+            while (true) {
+                bool any = false;
+#pragma unroll
+                for (int w = 0; w < W; ++w) any |= U[w] != 0;
+                if (!any) break;
+                ++ncol;
+                uint64_t Q[W];
+#pragma unroll
+                for (int w = 0; w < W; ++w) Q[w] = U[w];
+#pragma unroll
+                for (int w = 0; w < W; ++w) {
+                    while (Q[w]) {
+                        const int b = __ffsll((long long)Q[w]) - 1;
+                        const int v = w * 64 + b;
+                        const uint64_t *row = A + (int64_t)v * W;
+#pragma unroll
+                        for (int x = 0; x < W; ++x) Q[x] &= ~__ldg(row + x);
+                        Q[w] &= ~(1ull << b);
+                        U[w] &= ~(1ull << b);
+                        ord[np] = (uint8_t)v;
+                        colr[np] = (uint8_t)ncol;
+                        ++np;
+                    }
+                }
+            }
+        } else {
+#pragma unroll
+            for (int w = 0; w < W; ++w) {
+                uint64_t q = P[w];
+                while (q) {
+                    const int b = __ffsll((long long)q) - 1;
+                    q &= q - 1;
+                    ord[np] = (uint8_t)(w * 64 + b);
+                    colr[np] = (uint8_t)(np + 1);
+                    ++np;
+                }
+            }
+            ncol = np;
+        }
+        int32_t cnt = 0;
+        if (a.k + ncol >= a.need) {
+            uint64_t R[W];
+#pragma unroll
+            for (int w = 0; w < W; ++w) R[w] = P[w];
+            for (int i = np - 1; i >= 0; --i) {
+                if (a.k + colr[i] < a.need) break;
+                const int v = ord[i];
+                const uint64_t *row = A + (int64_t)v * W;
+                uint64_t C[W];
+                int pc = 0;
+#pragma unroll
+                for (int w = 0; w < W; ++w) {
+                    C[w] = R[w] & __ldg(row + w);
+                    pc += __popcll(C[w]);
+                }
+                R[v >> 6] &= ~(1ull << (v & 63));
+                if (pc == 0) {
+                    if (!WRITE && a.k + 1 >= a.need) record_leaf(a, e, v, ri);
+                } else if (a.k + 1 + pc >= a.need) {
+                    if (WRITE) {
+                        const int64_t c = out + cnt;
+#pragma unroll
+                        for (int w = 0; w < W; ++w) a.cP[c * W + w] = C[w];
+                        a.cslot[c] = a.slot[e];
+                        a.cparent[c] = (int32_t)e;
+                        a.cvloc[c] = v;
+                    }
+                    ++cnt;
+                }
+            }
+        }
+        if (!WRITE) a.counts[e] = cnt;
+    }
+}
+
+// ---------------------------------------------------------------------------
+// warp per candidate, W >= 4 words: lanes own words (WPL words per lane)
+// ---------------------------------------------------------------------------
+template <int WPL, bool WRITE>
+__global__ void expand_warp(const ExpandArgs a, int max_l) {
+    extern __shared__ uint16_t sm[];
+    const int lane = threadIdx.x & 31;
+    const int wib = threadIdx.x >> 5;
+    uint16_t *ord = sm + (int64_t)wib * 2 * max_l;
+    uint16_t *colr = ord + max_l;
+    const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int W = a.W;
+    for (int64_t e = a.begin + warp; e < a.end; e += nwarps) {
+        int64_t out = 0;
+        if (WRITE) {
+            out = a.offsets[e];
+            if (a.offsets[e + 1] == out) continue;
+            out -= a.out_base;
+        }
+        uint64_t P[WPL];
+#pragma unroll
+        for (int t = 0; t < WPL; ++t) {
+            const int j = lane + 32 * t;
+            P[t] = j < W ? a.P[e * W + j] : 0ull;
+        }
+        const RootInfo ri = a.roots[a.slot[e]];
+        const uint64_t *A = a.adj + ri.abase;
+        int np = 0, ncol = 0;
+        if (a.bound == 1) {
+            uint64_t U[WPL];
+#pragma unroll
+            for (int t = 0; t < WPL; ++t) U[t] = P[t];
+            while (true) {
+                bool any = false;
+#pragma unroll
+                for (int t = 0; t < WPL; ++t) any |= U[t] != 0;
+                if (!__any_sync(0xffffffffu, any)) break;
+                ++ncol;
+                uint64_t Q[WPL];
+#pragma unroll
+                for (int t = 0; t < WPL; ++t) Q[t] = U[t];
+                while (true) {
+                    int v = -1;
+#pragma unroll
+                    for (int t = 0; t < WPL; ++t) {
+                        if (v < 0) {
+                            const unsigned m = __ballot_sync(0xffffffffu, Q[t] != 0);
+                            if (m) {
+                                const int src = __ffs(m) - 1;
+                                const int bit = __shfl_sync(0xffffffffu, __ffsll((long long)Q[t]) - 1, src);
+                                v = (src + 32 * t) * 64 + bit;
+                            }
+                        }
+                    }
+                    if (v < 0) break;
+                    const uint64_t *row = A + (int64_t)v * W;
+#pragma unroll
+                    for (int t = 0; t < WPL; ++t) {
+                        const int j = lane + 32 * t;
+                        if (j < W) Q[t] &= ~__ldg(row + j);
+                    }
+                    const int jv = v >> 6;
+                    if ((jv & 31) == lane) {
+#pragma unroll
+                        for (int t = 0; t < WPL; ++t)
+                            if (t == (jv >> 5)) {
+                                Q[t] &= ~(1ull << (v & 63));
+                                U[t] &= ~(1ull << (v & 63));
+                            }
+                    }
+                    if (lane == 0) {
+                        ord[np] = (uint16_t)v;
+                        colr[np] = (uint16_t)ncol;
+                    }
+                    ++np;
+                }
+            }
+        } else {
+            // ascending bit order; colr[i] = i + 1
+            int base = 0;
+#pragma unroll
+            for (int t = 0; t < WPL; ++t) {
+                const int pc = __popcll(P[t]);
+                int incl = pc;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    int y = __shfl_up_sync(0xffffffffu, incl, o);
+                    if (lane >= o) incl += y;
+                }
+                int pos = base + incl - pc;
+                uint64_t q = P[t];
+                while (q) {
+                    const int b = __ffsll((long long)q) - 1;
+                    q &= q - 1;
+                    ord[pos] = (uint16_t)((lane + 32 * t) * 64 + b);
+                    colr[pos] = (uint16_t)(pos + 1);
+                    ++pos;
+                }
+                base += __shfl_sync(0xffffffffu, incl, 31);
+            }
+            np = base;
+            ncol = np;
+        }
+        __syncwarp();
+        int32_t cnt = 0;
+        if (a.k + ncol >= a.need) {
+            uint64_t R[WPL];
+#pragma unroll
+            for (int t = 0; t < WPL; ++t) R[t] = P[t];
+            for (int i = np - 1; i >= 0; --i) {
+                if (a.k + colr[i] < a.need) break;
+                const int v = ord[i];
+                const uint64_t *row = A + (int64_t)v * W;
+                uint64_t C[WPL];
+                int pc = 0;
+#pragma unroll
+                for (int t = 0; t < WPL; ++t) {
+                    const int j = lane + 32 * t;
+                    C[t] = j < W ? (R[t] & __ldg(row + j)) : 0ull;
+                    pc += __popcll(C[t]);
+                }
+                pc = __reduce_add_sync(0xffffffffu, pc);
+                const int jv = v >> 6;
+                if ((jv & 31) == lane) {
+#pragma unroll
+                    for (int t = 0; t < WPL; ++t)
+                        if (t == (jv >> 5)) R[t] &= ~(1ull << (v & 63));
+                }
+                if (pc == 0) {
+                    if (!WRITE && lane == 0 && a.k + 1 >= a.need) record_leaf(a, e, v, ri);
+                } else if (a.k + 1 + pc >= a.need) {
+                    if (WRITE) {
+                        const int64_t c = out + cnt;
+#pragma unroll
+                        for (int t = 0; t < WPL; ++t) {
+                            const int j = lane + 32 * t;
+                            if (j < W) a.cP[c * W + j] = C[t];
+                        }
+                        if (lane == 0) {
+                            a.cslot[c] = a.slot[e];
+                            a.cparent[c] = (int32_t)e;
+                            a.cvloc[c] = v;
+                        }
+                    }
+                    ++cnt;
+                }
+            }
+        }
+        if (!WRITE && lane == 0) a.counts[e] = cnt;
+        __syncwarp();
+    }
+}
+
+__global__ void classify_roots_kernel(int64_t n, const int64_t *__restrict__ orp, int32_t min_len, int32_t *cls) {
+    for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < n; r += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t L = orp[r + 1] - orp[r];
+        int32_t c = -1;
+        if (L >= min_len && L > 0) {
+            const int64_t words = (L + 63) / 64;
+            c = 0;
+            while ((1ll << c) < words) ++c;
+            if (c >= kMaxClass) c = 100;  // unsupported size: reported by the host
+        }
+        cls[r] = c;
+    }
+}
+
+__global__ void flag_eq_kernel(int64_t n, const int32_t *__restrict__ cls, int32_t c, int32_t *flag) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        flag[i] = cls[i] == c;
+}
+
+__global__ void compact_idx_kernel(int64_t n, const int32_t *__restrict__ flag, const int64_t *__restrict__ pos,
+                                   int32_t *out) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        if (flag[i]) out[pos[i]] = (int32_t)i;
+}
+
+__global__ void root_lengths_kernel(const int32_t *__restrict__ list, int64_t count, int64_t stride,
+                                    const int64_t *__restrict__ orp, int32_t *len) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < count; i += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t r = list[i * stride];
+        len[i] = (int32_t)(orp[r + 1] - orp[r]);
+    }
+}
+
+__global__ void make_roots_kernel(const int32_t *__restrict__ list, int64_t count, int64_t stride, int W,
+                                  const int64_t *__restrict__ orp, const int64_t *__restrict__ row_prefix,
+                                  RootInfo *roots) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < count; i += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t r = list[i * stride];
+        RootInfo ri;
+        ri.r = r;
+        ri.vbase = orp[r];
+        ri.L = (int32_t)(orp[r + 1] - ri.vbase);
+        ri.abase = row_prefix[i] * W;
+        roots[i] = ri;
+    }
+}
+
+// largest b in (a, n] with offsets[b] - offsets[a] <= cap (at least a+1 if possible)
+__global__ void find_chunk_end_kernel(const int64_t *__restrict__ offsets, int64_t a, int64_t n, int64_t cap,
+                                      int64_t *out) {
+    const int64_t base = offsets[a];
+    int64_t lo = a, hi = n;  // invariant: offsets[lo]-base <= cap
+    while (lo < hi) {
+        int64_t mid = (lo + hi + 1) >> 1;
+        if (offsets[mid] - base <= cap)
+            lo = mid;
+        else
+            hi = mid - 1;
+    }
+    out[0] = lo;
+    out[1] = offsets[lo] - base;
+    out[2] = base;
+}
+
+template <int WPL>
+void launch_warp(const ExpandArgs &a, bool write_pass, cudaStream_t s) {
+    const int max_l = 64 * a.W;
+    const int warps = WPL >= 4 ? 1 : (WPL == 2 ? 2 : 4);
+    const size_t smem = (size_t)warps * 2 * max_l * sizeof(uint16_t);
+    const int64_t items = a.end - a.begin;
+    const int grid = grid_for(items * 32, 32 * warps, 32);
+    if (write_pass) {
+        if (smem > 48 * 1024)
+            MCE_CUDA(cudaFuncSetAttribute(expand_warp<WPL, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        expand_warp<WPL, true><<<grid, 32 * warps, smem, s>>>(a, max_l);
+    } else {
+        if (smem > 48 * 1024)
+            MCE_CUDA(cudaFuncSetAttribute(expand_warp<WPL, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        expand_warp<WPL, false><<<grid, 32 * warps, smem, s>>>(a, max_l);
+    }
+    MCE_LAUNCH_CHECK();
+}
+
+}  // namespace
+
+void launch_build_adj(const RootInfo *roots, int64_t nroots, int W, const int64_t *orp, const int32_t *ocol,
+                      uint64_t *adj, cudaStream_t s) {
+    if (nroots <= 0) return;
+    if (W == 1) {
+        build_adj_w1<<<grid_for(nroots * 32, 256, 16), 256, 0, s>>>(roots, nroots, orp, ocol, adj);
+    } else {
+        build_adj_wide<<<grid_for(nroots, 1, 16), 256, 0, s>>>(roots, nroots, W, orp, ocol, adj);
+    }
+    MCE_LAUNCH_CHECK();
+}
+
+void launch_init_level1(const RootInfo *roots, int64_t nroots, int W, uint64_t *P, int32_t *slot, int32_t *parent,
+                        int32_t *vloc, cudaStream_t s) {
+    if (nroots <= 0) return;
+    init_level1_kernel<<<grid_for(nroots, 256), 256, 0, s>>>(roots, nroots, W, P, slot, parent, vloc);
+    MCE_LAUNCH_CHECK();
+}
+
+void launch_expand(const ExpandArgs &a, bool write_pass, cudaStream_t s) {
+    const int64_t items = a.end - a.begin;
+    if (items <= 0) return;
+    if (a.W == 1 || a.W == 2) {
+        const int grid = grid_for(items, 256, 8);
+        if (a.W == 1) {
+            if (write_pass)
+                expand_thread<1, true><<<grid, 256, 0, s>>>(a);
+            else
+                expand_thread<1, false><<<grid, 256, 0, s>>>(a);
+        } else {
+            if (write_pass)
+                expand_thread<2, true><<<grid, 256, 0, s>>>(a);
+            else
+                expand_thread<2, false><<<grid, 256, 0, s>>>(a);
+        }
+        MCE_LAUNCH_CHECK();
+    } else if (a.W <= 32) {
+        launch_warp<1>(a, write_pass, s);
+    } else if (a.W <= 64) {
+        launch_warp<2>(a, write_pass, s);
+    } else if (a.W <= 128) {
+        launch_warp<4>(a, write_pass, s);
+    } else {
+        launch_warp<8>(a, write_pass, s);
+    }
+}
+
+void launch_classify_roots(int64_t n, const int64_t *orp, int32_t min_len, int32_t *cls, cudaStream_t s) {
+    classify_roots_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, orp, min_len, cls);
+    MCE_LAUNCH_CHECK();
+}
+void launch_flag_eq(int64_t n, const int32_t *cls, int32_t c, int32_t *flag, cudaStream_t s) {
+    flag_eq_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, cls, c, flag);
+    MCE_LAUNCH_CHECK();
+}
+void launch_compact(int64_t n, const int32_t *flag, const int64_t *pos, int32_t *out, cudaStream_t s) {
+    compact_idx_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, flag, pos, out);
+    MCE_LAUNCH_CHECK();
+}
+void launch_make_roots(const int32_t *list, int64_t count, int64_t stride, int W, const int64_t *orp,
+                       const int64_t *row_prefix, RootInfo *roots, cudaStream_t s) {
+    if (count <= 0) return;
+    make_roots_kernel<<<grid_for(count, 256), 256, 0, s>>>(list, count, stride, W, orp, row_prefix, roots);
+    MCE_LAUNCH_CHECK();
+}
+void launch_root_lengths(const int32_t *list, int64_t count, int64_t stride, const int64_t *orp, int32_t *len,
+                         cudaStream_t s) {
+    if (count <= 0) return;
+    root_lengths_kernel<<<grid_for(count, 256), 256, 0, s>>>(list, count, stride, orp, len);
+    MCE_LAUNCH_CHECK();
+}
+void launch_find_chunk_end(const int64_t *offsets, int64_t a, int64_t n, int64_t cap, int64_t *out,
+                           cudaStream_t s) {
+    find_chunk_end_kernel<<<1, 1, 0, s>>>(offsets, a, n, cap, out);
+    MCE_LAUNCH_CHECK();
+}
+
+}  // namespace mce

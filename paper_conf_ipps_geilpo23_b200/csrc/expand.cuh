@@ -1,0 +1,74 @@
+// Frontier layout and expansion kernels (the hot path).
+#pragma once
+
+#include "common.cuh"
+
+namespace mce {
+
+// One root of the current window.  Its candidate space is V = the root's
+// out-neighbours (oriented CSR row, ranks ascending); local index i <-> V[i].
+struct RootInfo {
+    int32_t r;      // rank of the root
+    int32_t L;      // |V| = out-degree
+    int64_t vbase;  // orp[r]: V = ocol + vbase
+    int64_t abase;  // first word of the root's adjacency rows in the arena (L rows x W words)
+};
+
+// per-level arrays needed to read a clique back (PAPER.md IV-B: "sublistID ...
+// allows us ... at the end of the computation, to read out all of the vertices")
+struct LevelLink {
+    const int32_t *parent;  // index of the parent entry in the previous level (-1 at level 1)
+    const int32_t *vloc;    // local index of the vertex this entry added (-1 at level 1)
+};
+
+// A frontier level: |C| = k for every entry; P is the candidate set as a
+// bitset over the root's local space (W words per entry, structure of arrays).
+struct ExpandArgs {
+    const uint64_t *P;
+    const int32_t *slot;
+    const int32_t *parent;
+    const int32_t *vloc;
+    int64_t begin, end;  // entries [begin, end) of the input level
+    int32_t k;           // |C|
+    int32_t need;        // smallest clique size still of interest
+    int32_t bound;       // 0: |C|+|P|, 1: colouring
+    int32_t W;           // words per candidate set (runtime, warp kernels)
+    const RootInfo *roots;
+    const uint64_t *adj;
+    const int32_t *ocol;
+    const int32_t *order;  // rank -> original vertex id
+    // count pass
+    int32_t *counts;  // indexed by entry
+    // write pass
+    const int64_t *offsets;  // exclusive scan of counts (indexed by entry)
+    int64_t out_base;        // offsets[begin]
+    uint64_t *cP;
+    int32_t *cslot;
+    int32_t *cparent;
+    int32_t *cvloc;
+    // leaves of size k+1 (count pass only)
+    unsigned long long *leaf_count;
+    int32_t *leaf_rows;
+    int64_t leaf_cap;  // rows
+    const LevelLink *chain;  // chain[1..k]
+};
+
+// W classes: 0 -> 1 word, 1 -> 2, 2 -> 4, ... (W = 1 << class); L <= 64 W
+constexpr int kMaxClass = 9;  // W up to 256 words (L <= 16384)
+
+void launch_build_adj(const RootInfo *roots, int64_t nroots, int W, const int64_t *orp, const int32_t *ocol,
+                      uint64_t *adj, cudaStream_t s);
+void launch_init_level1(const RootInfo *roots, int64_t nroots, int W, uint64_t *P, int32_t *slot, int32_t *parent,
+                        int32_t *vloc, cudaStream_t s);
+void launch_expand(const ExpandArgs &a, bool write_pass, cudaStream_t s);
+void launch_classify_roots(int64_t n, const int64_t *orp, int32_t min_len, int32_t *cls, cudaStream_t s);
+void launch_flag_eq(int64_t n, const int32_t *cls, int32_t c, int32_t *flag, cudaStream_t s);
+void launch_compact(int64_t n, const int32_t *flag, const int64_t *pos, int32_t *out, cudaStream_t s);
+void launch_make_roots(const int32_t *list, int64_t count, int64_t stride, int W, const int64_t *orp,
+                       const int64_t *row_prefix, RootInfo *roots, cudaStream_t s);
+void launch_root_lengths(const int32_t *list, int64_t count, int64_t stride, const int64_t *orp, int32_t *len,
+                         cudaStream_t s);
+void launch_find_chunk_end(const int64_t *offsets, int64_t a, int64_t n, int64_t cap, int64_t *out,
+                           cudaStream_t s);
+
+}  // namespace mce

@@ -1,0 +1,37 @@
+// Device-resident graph handle and the preprocessing entry points.
+#pragma once
+
+#include "common.cuh"
+
+struct mce_graph {
+    int device = 0;
+    cudaStream_t stream = nullptr;
+    int64_t n = 0;
+    int64_t nnz = 0;  // 2|E|
+    int64_t max_deg = 0;
+    mce::DevBuf<int64_t> rowptr;  // [n+1] undirected CSR
+    mce::DevBuf<int32_t> col;     // [nnz], rows sorted ascending
+
+    // ---- preprocessing (PAPER.md II-B-2, IV-C), computed lazily ----
+    int orientation = -1;          // MCE_ORIENT_* the arrays below were built for
+    bool have_core = false;
+    mce::DevBuf<int32_t> core;     // [n] core numbers
+    mce::DevBuf<int32_t> peel;     // [n] k-core peel order (vertex removed i-th)
+    int32_t degeneracy = 0;
+    mce::DevBuf<int32_t> order;    // [n] rank -> vertex (orientation order)
+    mce::DevBuf<int32_t> rank;     // [n] vertex -> rank
+    mce::DevBuf<int64_t> orp;      // [n+1] oriented CSR over ranks
+    mce::DevBuf<int32_t> ocol;     // [nnz/2] out-neighbour ranks, rows ascending
+    int32_t max_out = 0;           // largest out-degree
+    double t_pre_ms = 0.0;         // device time of the last preprocessing
+    int64_t kernels = 0;           // kernels launched by the last preprocessing
+};
+
+namespace mce {
+// k-core numbers and peel order (cooperative persistent kernel)
+void kcore(mce_graph *g);
+// rank/order by the requested orientation + oriented CSR with sorted rows
+void orient(mce_graph *g, int orientation);
+// both, cached on the handle
+void preprocess(mce_graph *g, int orientation);
+}  // namespace mce

@@ -1,0 +1,271 @@
+// Greedy lower bound on omega (PAPER.md IV-A, lines 103-109, Algorithm 1).
+//
+// Multi-run: the h vertices with the highest threshold (degree or core
+// number) each seed one run; a run holds C = {seed}, P = N(seed) and
+// repeatedly adds the candidate with the highest threshold (ties: smaller id,
+// the first maximum of an id-sorted segment = Algorithm 1 line 34's segmented
+// max), then keeps only the candidates adjacent to it (lines 35-38).  The
+// single-run variants are the h = 1 case (the first pick from "all vertices"
+// is the top vertex).
+//
+// B200 mapping: one warp per run instead of Algorithm 1's segmented
+// CUB passes -- the argmax is a warp max-reduction over a 64-bit key
+// (threshold << 32 | ~id), the filter is a warp-cooperative membership test
+// (binary search in the sorted adjacency list of the added vertex) compacted
+// in place with __ballot_sync/__popc, so every run stays in one warp's
+// registers + one contiguous scratch segment and no host round trip is needed
+// per iteration.
+#include <algorithm>
+#include <vector>
+
+#include "graph.cuh"
+#include "heuristic.cuh"
+
+namespace mce {
+
+namespace {
+
+__device__ __forceinline__ unsigned long long warp_max_u64(unsigned long long x) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        unsigned long long y = __shfl_xor_sync(0xffffffffu, x, o);
+        x = y > x ? y : x;
+    }
+    return x;
+}
+
+__device__ __forceinline__ unsigned long long pick_key(const int32_t *__restrict__ thr, int32_t x) {
+    return ((unsigned long long)(uint32_t)__ldg(thr + x) << 32) | (unsigned long long)(0x7fffffffu - (uint32_t)x);
+}
+
+// One greedy run for seed s by the calling warp.  Writes the clique (in order
+// added) to `clique` when non-null.  Returns the clique size.
+__device__ int32_t greedy_run(int32_t s, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
+                              const int32_t *__restrict__ thr, int32_t *__restrict__ scratch, int32_t *clique) {
+    const int lane = threadIdx.x & 31;
+    const int64_t base = rowptr[s];
+    int64_t len = rowptr[s + 1] - base;
+    const int32_t *src = col + base;  // first round reads the CSR row directly
+    int32_t *buf = scratch + base;    // later rounds work in place in the seed's segment
+    int32_t csize = 1;
+    if (clique && lane == 0) clique[0] = s;
+    while (len > 0) {
+        unsigned long long key = 0;
+        for (int64_t i = lane; i < len; i += 32) {
+            unsigned long long k2 = pick_key(thr, src[i]);
+            key = k2 > key ? k2 : key;
+        }
+        key = warp_max_u64(key);
+        const int32_t w = (int32_t)(0x7fffffffu - (uint32_t)(key & 0xffffffffull));
+        if (clique && lane == 0) clique[csize] = w;
+        ++csize;
+        const int64_t wb = rowptr[w], we = rowptr[w + 1];
+        int64_t out = 0;
+        for (int64_t i0 = 0; i0 < len; i0 += 32) {
+            int64_t i = i0 + lane;
+            int32_t x = i < len ? src[i] : -1;
+            bool keep = i < len && x != w && contains_sorted(col, wb, we, x);
+            unsigned m = __ballot_sync(0xffffffffu, keep);
+            if (keep) buf[out + __popc(m & lanemask_lt())] = x;
+            out += __popc(m);
+        }
+        __syncwarp();
+        src = buf;
+        len = out;
+    }
+    return csize;
+}
+
+__global__ void greedy_kernel(int64_t nseeds, const int32_t *__restrict__ seeds, const int64_t *__restrict__ rowptr,
+                              const int32_t *__restrict__ col, const int32_t *__restrict__ thr,
+                              int32_t *__restrict__ scratch, int32_t *__restrict__ run_size, int32_t *best_size) {
+    const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    for (int64_t i = warp; i < nseeds; i += nwarps) {
+        int32_t s = seeds[i];
+        int32_t c = greedy_run(s, rowptr, col, thr, scratch, nullptr);
+        if (lane == 0) {
+            run_size[s] = c;
+            atomicMax(best_size, c);
+        }
+    }
+}
+
+// among seeds whose run reached best, the first in seed order (threshold desc, id asc)
+__global__ void best_seed_kernel(int64_t nseeds, const int32_t *__restrict__ seeds, const int32_t *__restrict__ thr,
+                                 const int32_t *__restrict__ run_size, const int32_t *best_size,
+                                 unsigned long long *best_key) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nseeds; i += (int64_t)gridDim.x * blockDim.x) {
+        int32_t s = seeds[i];
+        if (run_size[s] == *best_size) atomicMax(best_key, pick_key(thr, s));
+    }
+}
+
+__global__ void replay_kernel(const unsigned long long *best_key, const int64_t *__restrict__ rowptr,
+                              const int32_t *__restrict__ col, const int32_t *__restrict__ thr,
+                              int32_t *__restrict__ scratch, int32_t *clique) {
+    int32_t s = (int32_t)(0x7fffffffu - (uint32_t)(*best_key & 0xffffffffull));
+    greedy_run(s, rowptr, col, thr, scratch, clique);
+}
+
+__global__ void degree_thr_kernel(int64_t n, const int64_t *__restrict__ rowptr, int32_t *thr) {
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+        thr[v] = (int32_t)(rowptr[v + 1] - rowptr[v]);
+}
+
+__global__ void thr_hist_kernel(int64_t n, const int32_t *__restrict__ thr, int64_t *bins) {
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+        atomicAdd((unsigned long long *)(bins + thr[v]), 1ull);
+}
+
+__global__ void tie_flags_kernel(int64_t n, const int32_t *__restrict__ thr, int32_t tau, int32_t *flag) {
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+        flag[v] = thr[v] == tau;
+}
+
+// seed flag = thr > tau, or thr == tau and among the first `quota` ties by id
+__global__ void seed_flags_kernel(int64_t n, const int32_t *__restrict__ thr, int32_t tau,
+                                  const int64_t *__restrict__ tie_rank, int64_t quota, int32_t *flag) {
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+        flag[v] = thr[v] > tau || (thr[v] == tau && tie_rank[v] < quota);
+}
+
+__global__ void compact_kernel(int64_t n, const int32_t *__restrict__ flag, const int64_t *__restrict__ pos,
+                               int32_t *out) {
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+        if (flag[v]) out[pos[v]] = (int32_t)v;
+}
+
+__global__ void iota_kernel(int64_t n, int32_t *out) {
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+        out[v] = (int32_t)v;
+}
+
+}  // namespace
+
+HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_rank, int32_t shard_count,
+                              bool want_runs) {
+    HeuristicResult res;
+    const int64_t n = g->n;
+    cudaStream_t s = g->stream;
+    if (n == 0 || kind == 0) return res;
+    bool use_core = (kind == 2 || kind == 4);
+    bool single = (kind == 1 || kind == 2);
+    if (single) h = 1;
+    if (h <= 0 || h > n) h = n;
+    if (use_core) kcore(g);
+    cudaEvent_t e0, e1;
+    MCE_CUDA(cudaEventCreate(&e0));
+    MCE_CUDA(cudaEventCreate(&e1));
+    MCE_CUDA(cudaEventRecord(e0, s));
+    int64_t kernels = 0;
+
+    DevBuf<int32_t> thr_buf;
+    const int32_t *thr;
+    if (use_core) {
+        thr = g->core.get();
+    } else {
+        thr_buf.alloc(n);
+        degree_thr_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(), thr_buf.get());
+        MCE_LAUNCH_CHECK();
+        ++kernels;
+        thr = thr_buf.get();
+    }
+    // ---- seeds: the h vertices with the highest threshold (ties: smaller id)
+    DevBuf<int32_t> seeds(n);
+    int64_t nseeds = 0;
+    if (h == n) {
+        iota_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, seeds.get());
+        MCE_LAUNCH_CHECK();
+        ++kernels;
+        nseeds = n;
+    } else {
+        int64_t maxthr = use_core ? g->degeneracy : g->max_deg;
+        DevBuf<int64_t> bins(maxthr + 1);
+        MCE_CUDA(cudaMemsetAsync(bins.get(), 0, bins.bytes(), s));
+        thr_hist_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, thr, bins.get());
+        MCE_LAUNCH_CHECK();
+        std::vector<int64_t> hb(maxthr + 1);
+        MCE_CUDA(cudaMemcpyAsync(hb.data(), bins.get(), bins.bytes(), cudaMemcpyDeviceToHost, s));
+        MCE_CUDA(cudaStreamSynchronize(s));
+        int64_t above = 0;
+        int32_t tau = 0;
+        for (int64_t t = maxthr; t >= 0; --t) {
+            if (above + hb[t] >= h) {
+                tau = (int32_t)t;
+                break;
+            }
+            above += hb[t];
+        }
+        int64_t quota = h - above;
+        DevBuf<int32_t> flag(n);
+        DevBuf<int64_t> pos(n + 1), tmp(scan_tmp_items(n));
+        tie_flags_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, thr, tau, flag.get());
+        MCE_LAUNCH_CHECK();
+        exclusive_scan_i32(flag.get(), pos.get(), n, tmp.get(), s);
+        seed_flags_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, thr, tau, pos.get(), quota, flag.get());
+        MCE_LAUNCH_CHECK();
+        exclusive_scan_i32(flag.get(), pos.get(), n, tmp.get(), s);
+        compact_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, flag.get(), pos.get(), seeds.get());
+        MCE_LAUNCH_CHECK();
+        kernels += 10;
+        nseeds = h;
+    }
+    // ---- shard the runs across ranks (cyclic over the id-ordered seed list)
+    const int32_t *seed_ptr = seeds.get();
+    DevBuf<int32_t> shard_seeds;
+    if (shard_count > 1) {
+        std::vector<int32_t> hs(nseeds);
+        MCE_CUDA(cudaMemcpyAsync(hs.data(), seeds.get(), sizeof(int32_t) * nseeds, cudaMemcpyDeviceToHost, s));
+        MCE_CUDA(cudaStreamSynchronize(s));
+        std::vector<int32_t> mine;
+        for (int64_t i = shard_rank; i < nseeds; i += shard_count) mine.push_back(hs[i]);
+        shard_seeds.alloc(std::max<size_t>(mine.size(), 1));
+        if (!mine.empty())
+            MCE_CUDA(cudaMemcpyAsync(shard_seeds.get(), mine.data(), sizeof(int32_t) * mine.size(),
+                                     cudaMemcpyHostToDevice, s));
+        seed_ptr = shard_seeds.get();
+        nseeds = (int64_t)mine.size();
+    }
+    // ---- the runs
+    DevBuf<int32_t> scratch(std::max<int64_t>(g->nnz, 1)), run_size(n), best(1);
+    DevBuf<unsigned long long> best_key(1);
+    DevBuf<int32_t> clique(g->max_deg + 2);
+    MCE_CUDA(cudaMemsetAsync(run_size.get(), 0, run_size.bytes(), s));
+    MCE_CUDA(cudaMemsetAsync(best.get(), 0, best.bytes(), s));
+    MCE_CUDA(cudaMemsetAsync(best_key.get(), 0, best_key.bytes(), s));
+    if (nseeds > 0) {
+        greedy_kernel<<<grid_for(nseeds * 32, 256), 256, 0, s>>>(nseeds, seed_ptr, g->rowptr.get(), g->col.get(),
+                                                                  thr, scratch.get(), run_size.get(), best.get());
+        MCE_LAUNCH_CHECK();
+        best_seed_kernel<<<grid_for(nseeds, 256), 256, 0, s>>>(nseeds, seed_ptr, thr, run_size.get(), best.get(),
+                                                               best_key.get());
+        MCE_LAUNCH_CHECK();
+        replay_kernel<<<1, 32, 0, s>>>(best_key.get(), g->rowptr.get(), g->col.get(), thr, scratch.get(),
+                                       clique.get());
+        MCE_LAUNCH_CHECK();
+        kernels += 3;
+    }
+    MCE_CUDA(cudaEventRecord(e1, s));
+    MCE_CUDA(cudaMemcpyAsync(&res.omega_bar, best.get(), sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+    MCE_CUDA(cudaStreamSynchronize(s));
+    float ms = 0;
+    MCE_CUDA(cudaEventElapsedTime(&ms, e0, e1));
+    res.ms = ms;
+    res.kernels = kernels;
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    if (res.omega_bar > 0) {
+        res.clique.resize(res.omega_bar);
+        MCE_CUDA(cudaMemcpy(res.clique.data(), clique.get(), sizeof(int32_t) * res.omega_bar,
+                            cudaMemcpyDeviceToHost));
+    }
+    if (want_runs) {
+        res.run_size.resize(n);
+        MCE_CUDA(cudaMemcpy(res.run_size.data(), run_size.get(), sizeof(int32_t) * n, cudaMemcpyDeviceToHost));
+    }
+    return res;
+}
+
+}  // namespace mce

@@ -1,0 +1,227 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Bit-exact for everything (omega, multiplicity, the sorted list of sorted
+cliques, core numbers, greedy run sizes); find_one returns a clique whose
+size equals the oracle's omega (several answers are correct there, so the
+rest is checked for validity).
+"""
+
+import functools
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from synth import graphs as G
+from tests import bruteforce as bf
+
+pytestmark = pytest.mark.gpu
+
+
+def mce():
+    import paper_conf_ipps_geilpo23_b200 as m
+
+    return m
+
+
+@functools.lru_cache(maxsize=None)
+def oracle_answer(key):
+    g = GRAPHS[key]()
+    om, cl = oracle.max_cliques(*g.numpy())
+    return om, cl
+
+
+GRAPHS = {
+    "K1": lambda: G.complete_graph(1),
+    "K2": lambda: G.complete_graph(2),
+    "K7": lambda: G.complete_graph(7),
+    "K64": lambda: G.complete_graph(64),
+    "K65": lambda: G.complete_graph(65),
+    "K130": lambda: G.complete_graph(130),
+    "C5": lambda: G.cycle_graph(5),
+    "C9": lambda: G.cycle_graph(9),
+    "T(12,4)": lambda: G.turan_graph(12, 4),
+    "T(30,6)": lambda: G.turan_graph(30, 6),
+    "T(36,12)": lambda: G.turan_graph(36, 12),
+    "Paley13": lambda: G.paley_graph(13),
+    "Paley17": lambda: G.paley_graph(17),
+    "ER60": lambda: G.erdos_renyi(60, 0.3, seed=4),
+    "ER300": lambda: G.erdos_renyi(300, 0.1, seed=5),
+    "ER150d": lambda: G.erdos_renyi(150, 0.5, seed=6),
+    "ER400d": lambda: G.erdos_renyi(400, 0.35, seed=7),
+    "RMAT11": lambda: G.rmat(11, 8, 0.57, 0.19, 0.19, seed=3),
+    "RMAT13": lambda: G.rmat(13, 8, 0.45, 0.2, 0.2, seed=2),
+    "BA5k": lambda: G.barabasi_albert(5000, 4, seed=2),
+    "planted": lambda: G.plant_cliques(G.erdos_renyi(3000, 0.004, seed=9), 3, 9, seed=9),
+    "er2000": lambda: G.make_config("er2000"),
+}
+
+
+def run_enum(g, **kw):
+    m = mce()
+    gg = m.Graph(g.rowptr, g.col)
+    try:
+        return gg.enumerate(**kw)
+    finally:
+        gg.close()
+
+
+@pytest.mark.parametrize("key", list(GRAPHS))
+def test_enumerate_matches_oracle(key):
+    g = GRAPHS[key]()
+    om, cl = oracle_answer(key)
+    r = run_enum(g)
+    assert r.omega == om
+    assert r.count == len(cl)
+    assert np.array_equal(r.cliques, cl)
+
+
+@pytest.mark.parametrize("bound", ["size", "color"])
+@pytest.mark.parametrize("orientation", ["degeneracy", "degree"])
+@pytest.mark.parametrize("heuristic", ["none", "single_degree", "single_core", "multi_degree", "multi_core"])
+@pytest.mark.parametrize("key", ["ER60", "T(12,4)", "Paley17", "RMAT11", "planted"])
+def test_option_grid(key, heuristic, orientation, bound):
+    if bound == "size" and key in ("RMAT11",):
+        pytest.skip("size bound alone is exponential on the R-MAT hub core")
+    g = GRAPHS[key]()
+    om, cl = oracle_answer(key)
+    r = run_enum(g, heuristic=heuristic, orientation=orientation, bound=bound)
+    assert (r.omega, r.count) == (om, len(cl))
+    assert np.array_equal(r.cliques, cl)
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_random_small_vs_bruteforce(seed):
+    n = 10 + seed
+    rng = np.random.default_rng(seed)
+    edges = [(u, v) for u in range(n) for v in range(u + 1, n) if rng.random() < 0.55]
+    e = np.asarray(edges, np.int64).reshape(-1, 2)
+    g = G.from_edges(n, torch.from_numpy(e[:, 0].copy()), torch.from_numpy(e[:, 1].copy()))
+    bom, bcl = bf.max_cliques(n, edges)
+    r = run_enum(g)
+    assert r.omega == bom and r.cliques.tolist() == bcl
+
+
+def test_empty_and_edgeless():
+    m = mce()
+    g = m.Graph(np.zeros(1, np.int64), np.zeros(0, np.int32))
+    r = g.enumerate()
+    assert r.omega == 0 and r.count == 1
+    g = m.Graph(np.zeros(8, np.int64), np.zeros(0, np.int32))
+    r = g.enumerate()
+    assert r.omega == 1 and r.count == 7 and r.cliques.tolist() == [[v] for v in range(7)]
+    r = g.find_one()
+    assert r.omega == 1 and r.cliques.shape == (1, 1)
+
+
+def test_device_input_and_validation():
+    m = mce()
+    g = GRAPHS["ER300"]()
+    gg = m.Graph(g.rowptr.cuda(), g.col.cuda(), validate=True)
+    om, cl = oracle_answer("ER300")
+    r = gg.enumerate()
+    assert r.omega == om and np.array_equal(r.cliques, cl)
+    bad_col = g.col.clone()
+    bad_col[0], bad_col[1] = bad_col[1].item(), bad_col[0].item()  # unsorted row
+    with pytest.raises(m.MCEError):
+        m.Graph(g.rowptr, bad_col, validate=True)
+
+
+@pytest.mark.parametrize("key", ["ER300", "RMAT11", "BA5k", "T(30,6)", "ER400d"])
+def test_core_numbers_and_orientation(key):
+    g = GRAPHS[key]()
+    rp, col = g.numpy()
+    core_o, _, d_o = oracle.core_numbers(rp, col)
+    m = mce()
+    gg = m.Graph(g.rowptr, g.col)
+    for orientation in ("degeneracy", "degree"):
+        gg.clear_cache()
+        core, order, d = gg.preprocess(orientation)
+        assert np.array_equal(core, core_o) and d == d_o
+        assert sorted(order.tolist()) == list(range(g.n))
+        rank = np.empty(g.n, np.int64)
+        rank[order] = np.arange(g.n)
+        src = np.repeat(np.arange(g.n), np.diff(rp))
+        up = rank[col] > rank[src]
+        outdeg = np.bincount(src[up], minlength=g.n)
+        if orientation == "degeneracy":  # a degeneracy order: out-degree <= core number
+            assert np.all(outdeg <= core_o)
+        else:  # degree order: edges point to vertices of larger or equal degree
+            deg = np.diff(rp)
+            assert np.all(deg[col[up]] >= deg[src[up]])
+
+
+@pytest.mark.parametrize("key", ["ER300", "RMAT11", "BA5k", "planted", "ER150d"])
+@pytest.mark.parametrize("kind", ["degree", "core"])
+def test_heuristic_matches_oracle(key, kind):
+    g = GRAPHS[key]()
+    rp, col = g.numpy()
+    thr = np.diff(rp) if kind == "degree" else oracle.core_numbers(rp, col)[0]
+    m = mce()
+    gg = m.Graph(g.rowptr, g.col)
+    order = np.lexsort((np.arange(g.n), -thr.astype(np.int64)))  # seeds: threshold desc, id asc
+    for h in (1, 7, g.n):
+        w_o, runs_o, best_o = oracle.greedy(rp, col, thr, h)
+        w, clique, runs = gg.heuristic(("single_" if h == 1 else "multi_") + kind, h)
+        assert w == w_o
+        assert clique == best_o.tolist()
+        assert np.array_equal(runs[order[:h]], runs_o)
+        assert np.count_nonzero(runs) == h
+
+
+@pytest.mark.parametrize("window", [1, 3, 64, 0])
+@pytest.mark.parametrize("key", ["ER300", "planted", "ER400d", "RMAT13", "K130", "T(30,6)"])
+def test_find_one(key, window):
+    g = GRAPHS[key]()
+    om, cl = oracle_answer(key)
+    m = mce()
+    gg = m.Graph(g.rowptr, g.col)
+    r = gg.find_one(window=window)
+    assert r.omega == om and r.count == 1 and r.cliques.shape == (1, om)
+    assert oracle.is_clique(*g.numpy(), r.cliques[0])
+    assert len(set(r.cliques[0].tolist())) == om
+
+
+def test_find_one_turan_closed_form():
+    """T(200,20) has 10^20 maximum cliques (omega = 20): only find-one is possible."""
+    g = G.turan_graph(200, 20)
+    m = mce()
+    r = m.Graph(g.rowptr, g.col).find_one(window=16)
+    assert r.omega == 20 and sorted(int(v) % 20 for v in r.cliques[0]) == list(range(20))
+
+
+@pytest.mark.parametrize("key", ["ER400d", "T(30,6)", "RMAT13"])
+def test_small_budget_chunking(key):
+    """A frontier budget far below the peak level forces chunked (recursive
+    windowed) expansion; the answer must not change."""
+    g = GRAPHS[key]()
+    om, cl = oracle_answer(key)
+    r = run_enum(g, budget_bytes=4 << 20, heuristic="none")
+    assert r.omega == om and np.array_equal(r.cliques, cl)
+
+
+def test_max_cliques_truncation():
+    g = G.turan_graph(24, 6)  # parts of 4: 4^6 = 4096 maximum cliques
+    r = run_enum(g, max_cliques=100)
+    assert r.omega == 6 and r.count == 4096 and r.truncated and r.cliques.shape == (100, 6)
+    for c in r.cliques:
+        assert len({int(v) % 6 for v in c}) == 6
+
+
+@pytest.mark.slow
+def test_config_ba1m_full():
+    g = G.make_config("ba1m")
+    om, cl = oracle.max_cliques(*g.numpy())
+    r = run_enum(g)
+    assert r.omega == om and np.array_equal(r.cliques, cl)
+
+
+@pytest.mark.slow
+def test_config_dense800_find_one():
+    g = G.make_config("dense800")
+    m = mce()
+    gg = m.Graph(g.rowptr, g.col)
+    r = gg.find_one(window=32)
+    assert r.omega == 15  # tests/golden/dense800.json (oracle, scripts/make_golden.py)
+    assert oracle.is_clique(*g.numpy(), r.cliques[0])
