@@ -83,6 +83,10 @@ typedef struct {
     int32_t (*bound_sync)(int32_t local_best, int32_t local_active, int32_t *global_active, void *user);
     void *bound_sync_user;
     int32_t verbose;         /* >0: per-level statistics on stderr */
+    int32_t legacy_roots;    /* 0 (default): roots with |N+(r)| <= 64 take the fused root-level
+                                kernel (adjacency build + first expansion in one warp, only
+                                surviving roots materialised); 1: the generic per-level path
+                                for every root (kept for A/B parity tests) */
 } mce_options;
 
 /* Fill `opt` with defaults: degeneracy orientation, multi-run degree heuristic
@@ -151,7 +155,9 @@ mce_status mce_result_levels(const mce_result *r, int64_t *entries, int32_t cap,
 /* Kernel timing of the last run, milliseconds measured with CUDA events on
  * the run's stream: [0] preprocess, [1] heuristic, [2] expansion total,
  * [3] dominant expansion kernel total, [4] number of dominant-kernel launches,
- * [5] algorithmic bytes moved by the dominant kernel, [6] kernels launched. */
+ * [5] algorithmic bytes moved by the dominant kernel, [6] kernels launched,
+ * [7] fused root-level kernel total, [8] its launches, [9] its algorithmic
+ * bytes (16 + 20 L + 4 T per root: row bounds, V, and the out-rows of V). */
 mce_status mce_result_timing(const mce_result *r, double *t, int32_t cap);
 void mce_result_free(mce_result *r);
 

@@ -43,6 +43,7 @@ class Options(ctypes.Structure):
         ("bound_sync", BOUND_SYNC),
         ("bound_sync_user", ctypes.c_void_p),
         ("verbose", ctypes.c_int32),
+        ("legacy_roots", ctypes.c_int32),
     ]
 
 

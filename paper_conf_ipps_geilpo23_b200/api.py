@@ -13,6 +13,7 @@ include/mce.h for every call's contract).
 from __future__ import annotations
 
 import ctypes
+import os
 import dataclasses
 from typing import Callable, List, Optional
 
@@ -58,7 +59,7 @@ def _current_stream(device: int):
 
 def make_options(orientation="degeneracy", heuristic="multi_degree", heuristic_runs=0, bound="color",
                  lower_bound=0, window=0, budget_bytes=0, max_cliques=0, shard_rank=0, shard_count=1,
-                 bound_sync: Optional[Callable[[int, int], tuple]] = None, verbose=0):
+                 bound_sync: Optional[Callable[[int, int], tuple]] = None, verbose=0, legacy_roots=False):
     o = Options()
     lib().mce_default_options(ctypes.byref(o))
     o.orientation = ORIENT[orientation]
@@ -71,7 +72,8 @@ def make_options(orientation="degeneracy", heuristic="multi_degree", heuristic_r
     o.max_cliques = int(max_cliques)
     o.shard_rank = int(shard_rank)
     o.shard_count = int(shard_count)
-    o.verbose = int(verbose)
+    o.verbose = int(verbose) or int(os.environ.get("MCE_VERBOSE", "0") or 0)
+    o.legacy_roots = int(bool(legacy_roots))
     keep = None
     if bound_sync is not None:
         def _cb(local_best, local_active, gactive, _user):
@@ -147,10 +149,11 @@ class Graph:
             nl = ctypes.c_int32()
             ent = (ctypes.c_int64 * 512)()
             check(L.mce_result_levels(handle, ent, 512, ctypes.byref(nl)))
-            tm = (ctypes.c_double * 7)()
-            check(L.mce_result_timing(handle, tm, 7))
+            tm = (ctypes.c_double * 10)()
+            check(L.mce_result_timing(handle, tm, 10))
             timing = dict(preprocess_ms=tm[0], heuristic_ms=tm[1], expand_ms=tm[2], count_kernel_ms=tm[3],
-                          count_launches=int(tm[4]), count_kernel_bytes=tm[5], kernels=int(tm[6]))
+                          count_launches=int(tm[4]), count_kernel_bytes=tm[5], kernels=int(tm[6]),
+                          root_kernel_ms=tm[7], root_launches=int(tm[8]), root_kernel_bytes=tm[9])
             return Result(om.value, cnt.value, cl, bool(tr.value), [int(ent[i]) for i in range(min(nl.value, 512))],
                           timing)
         finally:

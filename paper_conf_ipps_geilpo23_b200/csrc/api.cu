@@ -38,9 +38,14 @@ __global__ void validate_kernel(int64_t n, const int64_t *__restrict__ rowptr, c
         }
     }
 }
+// largest degree: per-thread max, warp max, one atomic per warp
 __global__ void max_deg_kernel(int64_t n, const int64_t *__restrict__ rowptr, unsigned long long *out) {
+    unsigned long long m = 0;
     for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
-        atomicMax(out, (unsigned long long)(rowptr[v + 1] - rowptr[v]));
+        m = max(m, (unsigned long long)(rowptr[v + 1] - rowptr[v]));
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) m = max(m, __shfl_xor_sync(0xffffffffu, m, o));
+    if ((threadIdx.x & 31) == 0 && m) atomicMax(out, m);
 }
 
 
@@ -109,6 +114,7 @@ void mce_default_options(mce_options *o) {
     o->bound_sync = nullptr;
     o->bound_sync_user = nullptr;
     o->verbose = 0;
+    o->legacy_roots = 0;
 }
 
 mce_status mce_load_csr(int32_t device, int64_t n, const int64_t *row_ptr, const int32_t *col_idx, int32_t where,
@@ -146,23 +152,24 @@ mce_status mce_load_csr(int32_t device, int64_t n, const int64_t *row_ptr, const
             if (nnz)
                 MCE_CUDA(cudaMemcpyAsync(g->col.get(), col_idx, sizeof(int32_t) * nnz, kind, g->stream));
             if (n > 0) {
-                DevBuf<unsigned long long> md(1);
-                MCE_CUDA(cudaMemsetAsync(md.get(), 0, md.bytes(), g->stream));
-                max_deg_kernel<<<grid_for(n, 256), 256, 0, g->stream>>>(n, g->rowptr.get(), md.get());
+                g->pool.reset();
+                unsigned long long *md = g->pool.take<unsigned long long>(1);
+                MCE_CUDA(cudaMemsetAsync(md, 0, sizeof(unsigned long long), g->stream));
+                max_deg_kernel<<<grid_for(n, 256), 256, 0, g->stream>>>(n, g->rowptr.get(), md);
                 MCE_LAUNCH_CHECK();
-                unsigned long long h = 0;
-                MCE_CUDA(cudaMemcpyAsync(&h, md.get(), sizeof(h), cudaMemcpyDeviceToHost, g->stream));
+                unsigned long long *h = g->host.get<unsigned long long>(1);
+                MCE_CUDA(cudaMemcpyAsync(h, md, sizeof(unsigned long long), cudaMemcpyDeviceToHost, g->stream));
                 MCE_CUDA(cudaStreamSynchronize(g->stream));
-                g->max_deg = (int64_t)h;
+                g->max_deg = (int64_t)h[0];
                 if (validate) {
-                    DevBuf<int32_t> bad(1);
-                    MCE_CUDA(cudaMemsetAsync(bad.get(), 0, bad.bytes(), g->stream));
-                    validate_kernel<<<grid_for(n, 256), 256, 0, g->stream>>>(n, g->rowptr.get(), g->col.get(),
-                                                                             bad.get());
+                    int32_t *bad = g->pool.take<int32_t>(1);
+                    MCE_CUDA(cudaMemsetAsync(bad, 0, sizeof(int32_t), g->stream));
+                    validate_kernel<<<grid_for(n, 256), 256, 0, g->stream>>>(n, g->rowptr.get(), g->col.get(), bad);
                     MCE_LAUNCH_CHECK();
-                    int32_t hb = 0;
-                    MCE_CUDA(cudaMemcpyAsync(&hb, bad.get(), sizeof(hb), cudaMemcpyDeviceToHost, g->stream));
+                    int32_t *hbp = g->host.get<int32_t>(1);
+                    MCE_CUDA(cudaMemcpyAsync(hbp, bad, sizeof(int32_t), cudaMemcpyDeviceToHost, g->stream));
                     MCE_CUDA(cudaStreamSynchronize(g->stream));
+                    const int32_t hb = hbp[0];
                     if (hb)
                         fail(MCE_ERR_INVALID, "malformed CSR (flags " + std::to_string(hb) +
                                                   ": 1 rowptr, 2 id range, 4 loop, 8 unsorted/dup, 16 asymmetric)");
@@ -299,9 +306,10 @@ mce_status mce_result_levels(const mce_result *r, int64_t *entries, int32_t cap,
 mce_status mce_result_timing(const mce_result *r, double *t, int32_t cap) {
     return run_guarded([&] {
         if (!r || !t) fail(MCE_ERR_INVALID, "NULL argument");
-        double v[7] = {r->t_pre_ms, r->t_heur_ms, r->t_expand_ms, r->t_count_ms, (double)r->count_launches,
-                       r->count_bytes, (double)r->kernels};
-        for (int32_t i = 0; i < std::min(cap, 7); ++i) t[i] = v[i];
+        double v[10] = {r->t_pre_ms,    r->t_heur_ms,     r->t_expand_ms,          r->t_count_ms,
+                        (double)r->count_launches, r->count_bytes, (double)r->kernels, r->t_root_ms,
+                        (double)r->root_launches,  r->root_bytes};
+        for (int32_t i = 0; i < std::min(cap, 10); ++i) t[i] = v[i];
     });
 }
 

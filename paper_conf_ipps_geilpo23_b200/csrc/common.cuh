@@ -3,9 +3,11 @@
 
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cstdint>
 #include <stdexcept>
 #include <string>
+#include <vector>
 
 namespace mce {
 
@@ -53,6 +55,10 @@ struct DevBuf {
         n = count;
         if (count) MCE_CUDA(cudaMalloc(&p, sizeof(T) * count));
     }
+    // keep the current allocation when it is large enough (no cudaMalloc/cudaFree)
+    void ensure(size_t count) {
+        if (n < count || !p) alloc(count);
+    }
     void release() {
         if (p) cudaFree(p);
         p = nullptr;
@@ -62,7 +68,78 @@ struct DevBuf {
     size_t bytes() const { return sizeof(T) * n; }
 };
 
+// pinned host staging buffer (small scalar read-backs without pageable copies)
+struct PinnedBuf {
+    void *p = nullptr;
+    size_t n = 0;
+    PinnedBuf() = default;
+    PinnedBuf(const PinnedBuf &) = delete;
+    PinnedBuf &operator=(const PinnedBuf &) = delete;
+    ~PinnedBuf() {
+        if (p) cudaFreeHost(p);
+    }
+    template <typename T>
+    T *get(size_t count) {
+        if (n < count * sizeof(T)) {
+            if (p) cudaFreeHost(p);
+            p = nullptr;
+            n = std::max<size_t>(count * sizeof(T), 4096);
+            MCE_CUDA(cudaMallocHost(&p, n));
+        }
+        return reinterpret_cast<T *>(p);
+    }
+};
+
 inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+// ---------------------------------------------------------------------------
+// grow-only device scratch pool, stream-ordered: take() bumps a pointer,
+// reset() releases everything taken since the last reset.  A request that
+// does not fit spills to its own cudaMalloc; the next reset() frees the
+// spills and regrows the main block to the high-water mark, so from the
+// second call on a phase runs without any cudaMalloc/cudaFree (both of which
+// serialise the device).
+// ---------------------------------------------------------------------------
+class Pool {
+   public:
+    Pool() = default;
+    Pool(const Pool &) = delete;
+    Pool &operator=(const Pool &) = delete;
+    ~Pool() {
+        for (void *q : spill_) cudaFree(q);
+    }
+    template <typename T>
+    T *take(int64_t count) {
+        const size_t bytes = ((size_t)(count > 0 ? count : 1) * sizeof(T) + 255) / 256 * 256;
+        if (top_ + bytes <= main_.n) {
+            T *q = reinterpret_cast<T *>(main_.p + top_);
+            top_ += bytes;
+            return q;
+        }
+        void *q = nullptr;
+        MCE_CUDA(cudaMalloc(&q, bytes));
+        spill_.push_back(q);
+        spill_bytes_ += bytes;
+        return reinterpret_cast<T *>(q);
+    }
+    void reset() {
+        if (!spill_.empty()) {
+            const size_t want = top_ + spill_bytes_;
+            for (void *q : spill_) cudaFree(q);
+            spill_.clear();
+            spill_bytes_ = 0;
+            if (want > main_.n) main_.alloc(want + want / 4);
+        }
+        top_ = 0;
+    }
+    size_t capacity() const { return main_.n; }
+
+   private:
+    DevBuf<uint8_t> main_;
+    size_t top_ = 0;
+    std::vector<void *> spill_;
+    size_t spill_bytes_ = 0;
+};
 
 // grid size for a grid-stride kernel: a multiple of the SM count
 int grid_for(int64_t work_items, int threads_per_block, int max_blocks_per_sm = 8);

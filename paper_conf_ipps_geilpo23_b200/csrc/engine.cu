@@ -24,21 +24,25 @@ namespace mce {
 namespace {
 constexpr size_t kAlign = 256;
 
+// bump allocator over the graph's persistent workspace, limited to the budget
 struct Arena {
-    DevBuf<uint8_t> buf;
+    uint8_t *base = nullptr;
+    size_t cap = 0;
     size_t top = 0;
-    void init(size_t bytes) {
-        buf.alloc(bytes);
+    void init(DevBuf<uint8_t> &ws, size_t bytes) {
+        ws.ensure(bytes);
+        base = ws.p;
+        cap = bytes;
         top = 0;
     }
-    size_t avail() const { return buf.n > top ? buf.n - top : 0; }
+    size_t avail() const { return cap > top ? cap - top : 0; }
     template <typename T>
     T *alloc(int64_t count) {
         size_t bytes = ((size_t)std::max<int64_t>(count, 1) * sizeof(T) + kAlign - 1) / kAlign * kAlign;
-        if (top + bytes > buf.n)
+        if (top + bytes > cap)
             fail(MCE_ERR_BUDGET, "frontier budget exhausted (need " + std::to_string(bytes) + " more bytes, " +
                                      std::to_string(avail()) + " available)");
-        T *p = reinterpret_cast<T *>(buf.p + top);
+        T *p = reinterpret_cast<T *>(base + top);
         top += bytes;
         return p;
     }
@@ -79,9 +83,57 @@ class Timer {
     bool pending_ = false;
 };
 
+// Per-launch device timing of the expansion kernels without a host sync per
+// launch: event pairs are recorded around each launch and read once the
+// stream has been synchronised (collect()), then reused.
+class LaunchClock {
+   public:
+    explicit LaunchClock(cudaStream_t s) : s_(s) {}
+    ~LaunchClock() {
+        for (auto &e : ev_) {
+            cudaEventDestroy(e.a);
+            cudaEventDestroy(e.b);
+        }
+    }
+    // kind: 0 count pass, 1 write pass, 2 fused root level
+    int start(int kind) {
+        if (used_ == ev_.size()) {
+            Pair p;
+            MCE_CUDA(cudaEventCreate(&p.a));
+            MCE_CUDA(cudaEventCreate(&p.b));
+            ev_.push_back(p);
+        }
+        ev_[used_].kind = kind;
+        MCE_CUDA(cudaEventRecord(ev_[used_].a, s_));
+        return (int)used_++;
+    }
+    void stop(int i) { MCE_CUDA(cudaEventRecord(ev_[i].b, s_)); }
+    // call after a stream sync that covers every recorded pair
+    void collect(double &all_ms, double &count_ms, double &root_ms) {
+        for (size_t i = 0; i < used_; ++i) {
+            float ms = 0;
+            MCE_CUDA(cudaEventElapsedTime(&ms, ev_[i].a, ev_[i].b));
+            all_ms += ms;
+            if (ev_[i].kind == 0) count_ms += ms;
+            if (ev_[i].kind == 2) root_ms += ms;
+        }
+        used_ = 0;
+    }
+
+   private:
+    struct Pair {
+        cudaEvent_t a, b;
+        int kind;
+    };
+    cudaStream_t s_;
+    std::vector<Pair> ev_;
+    size_t used_ = 0;
+};
+
 class Engine {
    public:
-    Engine(mce_graph *g, const mce_options &o, bool find_one) : g_(g), o_(o), find_one_(find_one), s_(g->stream) {}
+    Engine(mce_graph *g, const mce_options &o, bool find_one)
+        : g_(g), o_(o), find_one_(find_one), s_(g->stream), clock_(g->stream) {}
 
     mce_result *run();
 
@@ -89,6 +141,7 @@ class Engine {
     int32_t need() const { return find_one_ ? best_ + 1 : best_; }
     void process(int32_t k, const Level &L);
     void do_class(int32_t cls, const int32_t *list, int64_t count);
+    void do_class_w1(const int32_t *list, int64_t count);
     void handle_leaves(int32_t size, int64_t cnt, ExpandArgs &a);
     void sync_bound(bool active);
     void launch_timed(const ExpandArgs &a, bool write);
@@ -97,22 +150,22 @@ class Engine {
     mce_options o_;
     bool find_one_;
     cudaStream_t s_;
+    LaunchClock clock_;
     Arena arena_;
     int32_t best_ = 0;
     int32_t W_ = 1;
     int64_t stride_ = 1, offset_ = 0;
 
     // leaves
-    DevBuf<unsigned long long> leaf_count_;
-    DevBuf<int32_t> stage_;
+    unsigned long long *leaf_count_ = nullptr;
     int64_t stage_rows_ = 0;
     std::vector<int32_t> rows_;  // host copy of the stored cliques (width res_size_)
     int32_t res_size_ = 0;
     int64_t res_count_ = 0;
     bool truncated_ = false;
 
-    // chain of levels for clique read-out
-    DevBuf<LevelLink> chain_dev_;
+    // chain of levels for clique read-out (device copy in g->misc)
+    LevelLink *chain_dev_ = nullptr;
     int32_t chain_cap_ = 0;
 
     const RootInfo *roots_ = nullptr;
@@ -120,23 +173,17 @@ class Engine {
 
     // stats
     std::vector<int64_t> level_entries_;
-    double t_expand_ms_ = 0.0, t_count_ms_ = 0.0;
-    int64_t count_launches_ = 0, kernels_ = 0;
-    double count_bytes_ = 0.0;
-    DevBuf<unsigned long long> pbits_;  // sum of |P| over counted entries (algorithmic bytes)
+    double t_expand_ms_ = 0.0, t_count_ms_ = 0.0, t_root_ms_ = 0.0;
+    int64_t count_launches_ = 0, kernels_ = 0, root_launches_ = 0;
+    double count_bytes_ = 0.0, root_bytes_ = 0.0;
 };
 
 void Engine::launch_timed(const ExpandArgs &a, bool write) {
-    Timer t(s_);
-    t.start();
+    const int t = clock_.start(write ? 1 : 0);
     launch_expand(a, write, s_);
-    t.stop();
-    MCE_CUDA(cudaStreamSynchronize(s_));
-    double ms = t.collect();
-    t_expand_ms_ += ms;
+    clock_.stop(t);
     ++kernels_;
     if (!write) {
-        t_count_ms_ += ms;
         ++count_launches_;
         const double n = (double)(a.end - a.begin);
         count_bytes_ += n * (8.0 * a.W + 4 + 4 + 4 + sizeof(RootInfo));
@@ -158,7 +205,7 @@ void Engine::handle_leaves(int32_t size, int64_t cnt, ExpandArgs &a) {
         res_size_ = size;
         res_count_ = 1;
         rows_.resize(size);
-        MCE_CUDA(cudaMemcpy(rows_.data(), stage_.get(), sizeof(int32_t) * size, cudaMemcpyDeviceToHost));
+        MCE_CUDA(cudaMemcpy(rows_.data(), g_->stage.get(), sizeof(int32_t) * size, cudaMemcpyDeviceToHost));
         return;
     }
     if (size > res_size_) {
@@ -173,10 +220,10 @@ void Engine::handle_leaves(int32_t size, int64_t cnt, ExpandArgs &a) {
     if (o_.max_cliques > 0) want = std::min<int64_t>(want, std::max<int64_t>(o_.max_cliques - stored, 0));
     if (want > a.leaf_cap) {  // staging too small: grow and replay the count pass (idempotent)
         stage_rows_ = want;
-        stage_.alloc((size_t)want * std::max<int32_t>(g_->max_out + 2, 2));
-        a.leaf_rows = stage_.get();
+        g_->stage.ensure((size_t)want * std::max<int32_t>(g_->max_out + 2, 2));
+        a.leaf_rows = g_->stage.get();
         a.leaf_cap = want;
-        MCE_CUDA(cudaMemsetAsync(leaf_count_.get(), 0, sizeof(unsigned long long), s_));
+        MCE_CUDA(cudaMemsetAsync(leaf_count_, 0, sizeof(unsigned long long), s_));
         launch_expand(a, false, s_);
         ++kernels_;
         MCE_CUDA(cudaStreamSynchronize(s_));
@@ -185,7 +232,8 @@ void Engine::handle_leaves(int32_t size, int64_t cnt, ExpandArgs &a) {
     if (take > 0) {
         size_t old = rows_.size();
         rows_.resize(old + (size_t)take * size);
-        MCE_CUDA(cudaMemcpy(rows_.data() + old, stage_.get(), sizeof(int32_t) * take * size, cudaMemcpyDeviceToHost));
+        MCE_CUDA(cudaMemcpy(rows_.data() + old, g_->stage.get(), sizeof(int32_t) * take * size,
+                            cudaMemcpyDeviceToHost));
     }
     if (take < cnt) truncated_ = true;
     res_count_ += cnt;
@@ -194,16 +242,9 @@ void Engine::handle_leaves(int32_t size, int64_t cnt, ExpandArgs &a) {
 void Engine::process(int32_t k, const Level &L) {
     if ((int64_t)level_entries_.size() <= k) level_entries_.resize(k + 1, 0);
     level_entries_[k] += L.count;
-    if (k + 2 > chain_cap_) {
-        int32_t cap = std::max(256, 2 * (k + 2));
-        DevBuf<LevelLink> nc(cap);
-        if (chain_cap_) MCE_CUDA(cudaMemcpyAsync(nc.get(), chain_dev_.get(), sizeof(LevelLink) * chain_cap_,
-                                                 cudaMemcpyDeviceToDevice, s_));
-        chain_dev_ = std::move(nc);
-        chain_cap_ = cap;
-    }
+    if (k + 2 > chain_cap_) fail(MCE_ERR_INVALID, "clique depth above the supported maximum");
     LevelLink link{L.parent, L.vloc};
-    MCE_CUDA(cudaMemcpyAsync(chain_dev_.get() + k, &link, sizeof(link), cudaMemcpyHostToDevice, s_));
+    MCE_CUDA(cudaMemcpyAsync(chain_dev_ + k, &link, sizeof(link), cudaMemcpyHostToDevice, s_));
 
     const size_t mark = arena_.top;
     const int64_t N = L.count;
@@ -228,20 +269,21 @@ void Engine::process(int32_t k, const Level &L) {
     a.ocol = g_->ocol.get();
     a.order = g_->order.get();
     a.counts = counts;
-    a.leaf_count = leaf_count_.get();
-    a.leaf_rows = stage_.get();
+    a.leaf_count = leaf_count_;
+    a.leaf_rows = g_->stage.get();
     a.leaf_cap = stage_rows_;
-    a.chain = chain_dev_.get();
+    a.chain = chain_dev_;
 
-    MCE_CUDA(cudaMemsetAsync(leaf_count_.get(), 0, sizeof(unsigned long long), s_));
+    MCE_CUDA(cudaMemsetAsync(leaf_count_, 0, sizeof(unsigned long long), s_));
     launch_timed(a, false);
     exclusive_scan_i32(counts, offs, N, tmp, s_);
     kernels_ += 3;
-    int64_t total = 0;
-    unsigned long long leaves = 0;
-    MCE_CUDA(cudaMemcpyAsync(&total, offs + N, sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
-    MCE_CUDA(cudaMemcpyAsync(&leaves, leaf_count_.get(), sizeof(leaves), cudaMemcpyDeviceToHost, s_));
+    int64_t *h = g_->host.get<int64_t>(2);
+    MCE_CUDA(cudaMemcpyAsync(h, offs + N, sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
+    MCE_CUDA(cudaMemcpyAsync(h + 1, leaf_count_, sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
     MCE_CUDA(cudaStreamSynchronize(s_));
+    const int64_t total = h[0];
+    const unsigned long long leaves = (unsigned long long)h[1];
     if (o_.verbose > 0)
         fprintf(stderr, "[mce] level k=%d entries=%lld children=%lld leaves=%llu need=%d\n", k, (long long)N,
                 (long long)total, leaves, a.need);
@@ -259,12 +301,12 @@ void Engine::process(int32_t k, const Level &L) {
         } else {
             launch_find_chunk_end(offs, a0, N, cap, chunk, s_);
             ++kernels_;
-            int64_t h[3];
-            MCE_CUDA(cudaMemcpyAsync(h, chunk, sizeof(h), cudaMemcpyDeviceToHost, s_));
+            int64_t *hc = g_->host.get<int64_t>(3);
+            MCE_CUDA(cudaMemcpyAsync(hc, chunk, 3 * sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
             MCE_CUDA(cudaStreamSynchronize(s_));
-            b = h[0];
-            cnt = h[1];
-            base = h[2];
+            b = hc[0];
+            cnt = hc[1];
+            base = hc[2];
             if (b == a0)
                 fail(MCE_ERR_BUDGET, "the children of one candidate at level " + std::to_string(k) +
                                          " exceed the frontier budget");
@@ -294,61 +336,150 @@ void Engine::process(int32_t k, const Level &L) {
     arena_.top = mark;
 }
 
+// W == 1 roots: the fused root level (roots.cu), then levels >= 2 as usual
+void Engine::do_class_w1(const int32_t *list, int64_t count) {
+    const int64_t mine = count > offset_ ? (count - offset_ + stride_ - 1) / stride_ : 0;
+    if (mine <= 0) return;
+    W_ = 1;
+    const int32_t *base = list + offset_;
+    int32_t *len = arena_.alloc<int32_t>(mine);
+    int64_t *prefix = arena_.alloc<int64_t>(mine + 1);
+    int64_t *tmp = arena_.alloc<int64_t>(scan_tmp_items(mine));
+    int64_t *win = arena_.alloc<int64_t>(2);
+    unsigned long long *ctr = arena_.alloc<unsigned long long>(8);
+    launch_root_lengths(base, mine, stride_, g_->orp.get(), len, s_);
+    exclusive_scan_i32(len, prefix, mine, tmp, s_);
+    kernels_ += 4;
+    // per candidate row: adjacency word + one level-2 entry (P, slot, parent, vloc)
+    const int64_t row_bytes = 8 + 8 + 12;
+    const int64_t per_root = sizeof(RootInfo) + 64;
+    int64_t hi = mine;
+    while (hi > 0) {
+        const size_t mark = arena_.top;
+        const int64_t room = (int64_t)(arena_.avail() / 3);
+        const int64_t maxw = o_.window > 0 ? o_.window : hi;
+        launch_find_window(prefix, hi, std::max<int64_t>(0, hi - maxw), room, row_bytes, per_root, win, s_);
+        ++kernels_;
+        int64_t *hw = g_->host.get<int64_t>(2);
+        MCE_CUDA(cudaMemcpyAsync(hw, win, 2 * sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
+        MCE_CUDA(cudaStreamSynchronize(s_));
+        const int64_t lo = hw[0], rows = hw[1];
+        const int64_t nw = hi - lo;
+        RootArgs ra{};
+        ra.list = base + lo * stride_;
+        ra.count = nw;
+        ra.stride = stride_;
+        ra.orp = g_->orp.get();
+        ra.ocol = g_->ocol.get();
+        ra.order = g_->order.get();
+        ra.need = need();
+        ra.bound = o_.bound;
+        ra.roots = arena_.alloc<RootInfo>(nw);
+        ra.adj = arena_.alloc<uint64_t>(rows);
+        ra.cP = arena_.alloc<uint64_t>(rows);
+        ra.cslot = arena_.alloc<int32_t>(rows);
+        ra.cparent = arena_.alloc<int32_t>(rows);
+        ra.cvloc = arena_.alloc<int32_t>(rows);
+        ra.ctr = ctr;
+        ra.leaf_rows = g_->stage.get();
+        ra.leaf_cap = stage_rows_;
+        unsigned long long *hc = nullptr;
+        for (int attempt = 0; attempt < 2; ++attempt) {
+            MCE_CUDA(cudaMemsetAsync(ctr, 0, 8 * sizeof(unsigned long long), s_));
+            const int t = clock_.start(2);
+            launch_root_expand_w1(ra, s_);
+            clock_.stop(t);
+            ++kernels_;
+            ++root_launches_;
+            hc = g_->host.get<unsigned long long>(8);
+            MCE_CUDA(cudaMemcpyAsync(hc, ctr, 8 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, s_));
+            MCE_CUDA(cudaStreamSynchronize(s_));
+            const int64_t leaves = (int64_t)hc[3];
+            if (attempt == 0 && leaves > ra.leaf_cap && !find_one_) {
+                // staging too small for the size-2 leaves: grow and replay (counters reset)
+                int64_t want = leaves;
+                if (o_.max_cliques > 0) want = std::min<int64_t>(want, o_.max_cliques);
+                if (want > ra.leaf_cap) {
+                    stage_rows_ = want;
+                    g_->stage.ensure((size_t)want * std::max<int32_t>(g_->max_out + 2, 2));
+                    ra.leaf_rows = g_->stage.get();
+                    ra.leaf_cap = want;
+                    continue;
+                }
+            }
+            break;
+        }
+        root_bytes_ += (double)hc[4];
+        if ((int64_t)level_entries_.size() <= 1) level_entries_.resize(2, 0);
+        level_entries_[1] += nw;
+        const int64_t leaves = (int64_t)hc[3];
+        if (leaves > 0) {
+            ExpandArgs la{};
+            la.k = 1;
+            la.leaf_rows = ra.leaf_rows;
+            la.leaf_cap = ra.leaf_cap;
+            la.leaf_count = leaf_count_;
+            handle_leaves(2, leaves, la);
+        }
+        const int64_t entries = (int64_t)hc[2];
+        if (o_.verbose > 0)
+            fprintf(stderr, "[mce] roots=%lld survivors=%llu level2=%lld leaves=%lld need=%d\n", (long long)nw,
+                    hc[0], (long long)entries, (long long)leaves, need());
+        if (entries > 0) {
+            roots_ = ra.roots;
+            adj_ = ra.adj;
+            Level L2;
+            L2.count = entries;
+            L2.P = ra.cP;
+            L2.slot = ra.cslot;
+            L2.parent = ra.cparent;
+            L2.vloc = ra.cvloc;
+            process(2, L2);
+        }
+        sync_bound(true);
+        arena_.top = mark;
+        hi = lo;
+    }
+}
+
 void Engine::do_class(int32_t cls, const int32_t *list, int64_t count) {
+    if (cls == 0 && !o_.legacy_roots) {
+        do_class_w1(list, count);
+        return;
+    }
     // this shard's view: positions offset_, offset_+stride_, ...
     const int64_t mine = count > offset_ ? (count - offset_ + stride_ - 1) / stride_ : 0;
     if (mine <= 0) return;
     W_ = 1 << cls;
     const int32_t *base = list + offset_;
-    // adjacency rows per root -> prefix (host copy, to cut windows)
-    std::vector<int64_t> prefix(mine + 1);
-    {
-        const size_t mark = arena_.top;
-        int32_t *len = arena_.alloc<int32_t>(mine);
-        int64_t *pre = arena_.alloc<int64_t>(mine + 1);
-        int64_t *tmp = arena_.alloc<int64_t>(scan_tmp_items(mine));
-        launch_root_lengths(base, mine, stride_, g_->orp.get(), len, s_);
-        exclusive_scan_i32(len, pre, mine, tmp, s_);
-        kernels_ += 4;
-        MCE_CUDA(cudaMemcpyAsync(prefix.data(), pre, sizeof(int64_t) * (mine + 1), cudaMemcpyDeviceToHost, s_));
-        MCE_CUDA(cudaStreamSynchronize(s_));
-        arena_.top = mark;
-    }
+    // adjacency rows per root -> prefix; it stays on the device and windows
+    // are cut there (one scalar read-back per window)
+    int32_t *len = arena_.alloc<int32_t>(mine);
+    int64_t *prefix = arena_.alloc<int64_t>(mine + 1);
+    int64_t *tmp = arena_.alloc<int64_t>(scan_tmp_items(mine));
+    int64_t *win = arena_.alloc<int64_t>(2);
+    launch_root_lengths(base, mine, stride_, g_->orp.get(), len, s_);
+    exclusive_scan_i32(len, prefix, mine, tmp, s_);
+    kernels_ += 4;
+    const int64_t per_root = sizeof(RootInfo) + 8 * W_ + 12 + 64;
     // windows from the highest ranks down (densest cores first)
     int64_t hi = mine;
     while (hi > 0) {
         const size_t mark = arena_.top;
         const int64_t room = (int64_t)(arena_.avail() / 4);
-        const int64_t per_root = sizeof(RootInfo) + 8 * W_ + 12 + 64;
-        int64_t lo = hi - 1;
-        int64_t maxw = o_.window > 0 ? o_.window : hi;
-        // grow the window while it fits a quarter of the free budget
-        {
-            int64_t l = std::max<int64_t>(0, hi - maxw), h = hi - 1;  // smallest lo that fits
-            while (l < h) {
-                int64_t mid = (l + h) / 2;
-                int64_t bytes = (prefix[hi] - prefix[mid]) * 8 * W_ + (hi - mid) * per_root;
-                if (bytes <= room)
-                    h = mid;
-                else
-                    l = mid + 1;
-            }
-            lo = l;
-        }
+        const int64_t maxw = o_.window > 0 ? o_.window : hi;
+        // smallest lo >= hi - maxw whose rows fit a quarter of the free budget (at least one root)
+        launch_find_window(prefix, hi, std::max<int64_t>(0, hi - maxw), room, 8 * W_, per_root, win, s_);
+        ++kernels_;
+        int64_t *hw = g_->host.get<int64_t>(2);
+        MCE_CUDA(cudaMemcpyAsync(hw, win, 2 * sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
+        MCE_CUDA(cudaStreamSynchronize(s_));
+        const int64_t lo = hw[0], rows = hw[1];
         const int64_t nw = hi - lo;
-        const int64_t rows = prefix[hi] - prefix[lo];
         RootInfo *roots = arena_.alloc<RootInfo>(nw);
-        int64_t *pre = arena_.alloc<int64_t>(nw + 1);
         uint64_t *adj = arena_.alloc<uint64_t>(rows * W_);
-        // row prefix of this window, relative to lo
-        {
-            std::vector<int64_t> rel(nw + 1);
-            for (int64_t i = 0; i <= nw; ++i) rel[i] = prefix[lo + i] - prefix[lo];
-            MCE_CUDA(cudaMemcpyAsync(pre, rel.data(), sizeof(int64_t) * (nw + 1), cudaMemcpyHostToDevice, s_));
-            MCE_CUDA(cudaStreamSynchronize(s_));
-        }
-        launch_make_roots(base + lo * stride_, nw, stride_, W_, g_->orp.get(), pre, roots, s_);
-        launch_build_adj(roots, nw, W_, g_->orp.get(), g_->ocol.get(), adj, s_);
+        launch_make_roots(base + lo * stride_, nw, stride_, W_, g_->orp.get(), prefix + lo, roots, s_);
+        launch_build_adj(roots, nw, W_, g_->orp.get(), g_->ocol.get(), adj, rows * W_, s_);
         kernels_ += 2;
         roots_ = roots;
         adj_ = adj;
@@ -415,61 +546,67 @@ mce_result *Engine::run() {
         sync_bound(true);
     }
 
-    // frontier budget
+    // frontier budget: the graph's workspace is reused across calls, so it
+    // counts as free memory here
     size_t free_b = 0, total_b = 0;
     MCE_CUDA(cudaMemGetInfo(&free_b, &total_b));
+    free_b += g_->ws.n;
     int64_t budget = o_.budget_bytes;
     if (budget <= 0)
         budget = std::min<int64_t>((int64_t)(free_b * 0.8), (int64_t)(1ll << 30) + 48ll * g_->nnz + 64ll * n);
     budget = std::min<int64_t>(budget, (int64_t)(free_b * 0.95));
-    arena_.init((size_t)budget);
-    leaf_count_.alloc(1);
+    if (g_->ws.n < (size_t)budget) g_->ws.release();  // regrow below without holding both blocks
+    arena_.init(g_->ws, (size_t)budget);
+    // leaf counter + level chain (persistent, g->misc)
+    chain_cap_ = 4096;
+    g_->misc.ensure(256 + sizeof(LevelLink) * chain_cap_);
+    leaf_count_ = reinterpret_cast<unsigned long long *>(g_->misc.get());
+    chain_dev_ = reinterpret_cast<LevelLink *>(g_->misc.get() + 256);
     stage_rows_ = find_one_ ? 1 : 4096;
-    stage_.alloc((size_t)stage_rows_ * std::max<int32_t>(g_->max_out + 2, 2));
-    pbits_.alloc(1);
+    g_->stage.ensure((size_t)stage_rows_ * std::max<int32_t>(g_->max_out + 2, 2));
 
     Timer tt(s_);
     tt.start();
-    // roots worth expanding: 1 + |N+(r)| >= need
+    // roots worth expanding: 1 + |N+(r)| >= need, grouped by candidate-set width class
     {
         const size_t mark = arena_.top;
         int32_t *cls = arena_.alloc<int32_t>(n);
         int32_t *flag = arena_.alloc<int32_t>(n);
         int64_t *pos = arena_.alloc<int64_t>(n + 1);
         int64_t *tmp = arena_.alloc<int64_t>(scan_tmp_items(n));
-        launch_classify_roots(n, g_->orp.get(), std::max<int32_t>(need() - 1, 1), cls, s_);
+        int64_t *hist = arena_.alloc<int64_t>(kMaxClass + 1);
+        MCE_CUDA(cudaMemsetAsync(hist, 0, sizeof(int64_t) * (kMaxClass + 1), s_));
+        launch_classify_roots(n, g_->orp.get(), std::max<int32_t>(need() - 1, 1), cls, hist, s_);
         ++kernels_;
+        int64_t *hh = g_->host.get<int64_t>(kMaxClass + 1);
+        MCE_CUDA(cudaMemcpyAsync(hh, hist, sizeof(int64_t) * (kMaxClass + 1), cudaMemcpyDeviceToHost, s_));
+        MCE_CUDA(cudaStreamSynchronize(s_));
+        if (hh[kMaxClass]) fail(MCE_ERR_INVALID, "out-degree above 16384 after orientation is not supported");
+        std::vector<int64_t> counts(hh, hh + kMaxClass);
         std::vector<std::pair<int32_t, int64_t>> classes;
         std::vector<int32_t *> lists;
         for (int32_t c = kMaxClass - 1; c >= 0; --c) {
+            if (counts[c] == 0) continue;
+            int32_t *list = arena_.alloc<int32_t>(counts[c]);
             launch_flag_eq(n, cls, c, flag, s_);
             exclusive_scan_i32(flag, pos, n, tmp, s_);
-            int64_t cnt = 0;
-            MCE_CUDA(cudaMemcpyAsync(&cnt, pos + n, sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
-            MCE_CUDA(cudaStreamSynchronize(s_));
-            kernels_ += 4;
-            if (cnt == 0) continue;
-            int32_t *list = arena_.alloc<int32_t>(cnt);
             launch_compact(n, flag, pos, list, s_);
-            ++kernels_;
-            classes.push_back({c, cnt});
+            kernels_ += 5;
+            classes.push_back({c, counts[c]});
             lists.push_back(list);
         }
-        {  // any root too wide for the kernels?
-            launch_flag_eq(n, cls, 100, flag, s_);
-            exclusive_scan_i32(flag, pos, n, tmp, s_);
-            int64_t cnt = 0;
-            MCE_CUDA(cudaMemcpyAsync(&cnt, pos + n, sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
-            MCE_CUDA(cudaStreamSynchronize(s_));
-            if (cnt) fail(MCE_ERR_INVALID, "out-degree above 16384 after orientation is not supported");
-        }
         // the class lists stay allocated below `mark` while the classes run
-        for (size_t i = 0; i < classes.size(); ++i) do_class(classes[i].first, lists[i], classes[i].second);
+        for (size_t i = 0; i < classes.size(); ++i) {
+            const size_t cmark = arena_.top;
+            do_class(classes[i].first, lists[i], classes[i].second);
+            arena_.top = cmark;
+        }
         arena_.top = mark;
     }
     tt.stop();
     MCE_CUDA(cudaStreamSynchronize(s_));
     res->t_enum_ms = tt.collect();
+    clock_.collect(t_expand_ms_, t_count_ms_, t_root_ms_);
     // keep answering the other shards until everyone is done
     if (o_.bound_sync) {
         int32_t gactive = 1;
@@ -489,6 +626,9 @@ mce_result *Engine::run() {
     res->count_launches = count_launches_;
     res->count_bytes = count_bytes_;
     res->t_expand_ms = t_expand_ms_;
+    res->t_root_ms = t_root_ms_;
+    res->root_launches = root_launches_;
+    res->root_bytes = root_bytes_;
     res->kernels = kernels_;
     return res;
 }

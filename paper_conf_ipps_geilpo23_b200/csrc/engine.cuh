@@ -15,6 +15,8 @@ struct mce_result {
     std::vector<int64_t> level_entries;
     double t_pre_ms = 0, t_heur_ms = 0, t_enum_ms = 0, t_expand_ms = 0, t_count_ms = 0, count_bytes = 0;
     int64_t count_launches = 0, kernels = 0;
+    double t_root_ms = 0, root_bytes = 0;  // fused root-level kernel
+    int64_t root_launches = 0;
 };
 
 namespace mce {

@@ -26,17 +26,6 @@ namespace mce {
 
 namespace {
 
-__device__ __forceinline__ bool adjacent_ranks(const int64_t *__restrict__ orp, const int32_t *__restrict__ ocol,
-                                               int32_t a, int32_t b) {
-    // edges point from lower to higher rank; rows sorted ascending
-    if (a > b) {
-        int32_t t = a;
-        a = b;
-        b = t;
-    }
-    return contains_sorted(ocol, __ldg(orp + a), __ldg(orp + a + 1), b);
-}
-
 // W == 1: one warp per root, lane i builds row i (and i+32) of the 64x64 matrix
 __global__ void build_adj_w1(const RootInfo *__restrict__ roots, int64_t nroots, const int64_t *__restrict__ orp,
                              const int32_t *__restrict__ ocol, uint64_t *__restrict__ adj) {
@@ -66,26 +55,59 @@ __global__ void build_adj_w1(const RootInfo *__restrict__ roots, int64_t nroots,
     }
 }
 
-// W >= 2: one block per root, one warp per row, 32 columns per __ballot_sync
-__global__ void build_adj_wide(const RootInfo *__restrict__ roots, int64_t nroots, int W,
-                               const int64_t *__restrict__ orp, const int32_t *__restrict__ ocol,
-                               uint64_t *__restrict__ adj) {
+// W >= 2: one block per root, warp per row.  Row i of the root-local
+// adjacency is N+(V[i]) ∩ V: the warp reads N+(V[i]) 32 elements at a time
+// (coalesced), every lane binary-searches its element in the staged V
+// (positions > i only: the orientation puts every out-neighbour after V[i]),
+// and a hit at c sets bits (i, c) and (c, i).  The row stops at the first
+// chunk beyond V[L-1].  Bits go to a shared-memory bit matrix when it fits
+// (SMEM), else straight to the (zeroed) global matrix.
+template <bool SMEM>
+__global__ void build_adj_block(const RootInfo *__restrict__ roots, int64_t nroots, int W,
+                                const int64_t *__restrict__ orp, const int32_t *__restrict__ ocol,
+                                uint64_t *__restrict__ adj) {
+    extern __shared__ int32_t dsm[];
     const int lane = threadIdx.x & 31;
     const int wib = threadIdx.x >> 5, nwb = blockDim.x >> 5;
-    uint32_t *adj32 = reinterpret_cast<uint32_t *>(adj);
     for (int64_t j = blockIdx.x; j < nroots; j += gridDim.x) {
         const RootInfo ri = roots[j];
-        const int32_t *V = ocol + ri.vbase;
-        for (int32_t i = wib; i < ri.L; i += nwb) {
-            const int32_t a = __ldg(V + i);
-            uint32_t *row = adj32 + 2 * (ri.abase + (int64_t)i * W);
-            for (int32_t c0 = 0; c0 < 64 * W; c0 += 32) {
-                const int32_t c = c0 + lane;
-                bool e = false;
-                if (c < ri.L && c != i) e = adjacent_ranks(orp, ocol, a, __ldg(V + c));
-                const unsigned m = __ballot_sync(0xffffffffu, e);
-                if (lane == 0) row[c0 >> 5] = m;
+        const int L = ri.L;
+        int32_t *sV = dsm;
+        uint32_t *sA = reinterpret_cast<uint32_t *>(dsm + ((L + 3) & ~3));
+        uint32_t *gA = reinterpret_cast<uint32_t *>(adj + ri.abase);
+        uint32_t *A = SMEM ? sA : gA;
+        for (int i = threadIdx.x; i < L; i += blockDim.x) sV[i] = __ldg(ocol + ri.vbase + i);
+        if (SMEM)
+            for (int64_t w = threadIdx.x; w < (int64_t)L * W * 2; w += blockDim.x) sA[w] = 0u;
+        __syncthreads();
+        const int32_t vmax = sV[L - 1];
+        for (int i = wib; i < L - 1; i += nwb) {
+            const int32_t a = sV[i];
+            const int64_t pb = __ldg(orp + a), pe = __ldg(orp + a + 1);
+            for (int64_t p0 = pb; p0 < pe; p0 += 32) {
+                const int64_t p = p0 + lane;
+                const int32_t u = p < pe ? __ldg(ocol + p) : INT32_MAX;
+                if (__shfl_sync(0xffffffffu, u, 0) > vmax) break;
+                if (u <= vmax) {
+                    int lo = i + 1, hi = L;
+                    while (lo < hi) {
+                        const int mid = (lo + hi) >> 1;
+                        if (sV[mid] < u)
+                            lo = mid + 1;
+                        else
+                            hi = mid;
+                    }
+                    if (lo < L && sV[lo] == u) {
+                        atomicOr(A + (int64_t)i * 2 * W + (lo >> 5), 1u << (lo & 31));
+                        atomicOr(A + (int64_t)lo * 2 * W + (i >> 5), 1u << (i & 31));
+                    }
+                }
             }
+        }
+        __syncthreads();
+        if (SMEM) {
+            for (int64_t w = threadIdx.x; w < (int64_t)L * W * 2; w += blockDim.x) gA[w] = sA[w];
+            __syncthreads();
         }
     }
 }
@@ -375,7 +397,13 @@ __global__ void expand_warp(const ExpandArgs a, int max_l) {
     }
 }
 
-__global__ void classify_roots_kernel(int64_t n, const int64_t *__restrict__ orp, int32_t min_len, int32_t *cls) {
+// cls[r] = width class of root r (-1: cannot reach `need`), hist[c] += 1
+// (hist[kMaxClass] counts roots too wide for the kernels: reported by the host)
+__global__ void classify_roots_kernel(int64_t n, const int64_t *__restrict__ orp, int32_t min_len, int32_t *cls,
+                                      unsigned long long *hist) {
+    __shared__ unsigned int h[kMaxClass + 1];
+    for (int i = threadIdx.x; i <= kMaxClass; i += blockDim.x) h[i] = 0;
+    __syncthreads();
     for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < n; r += (int64_t)gridDim.x * blockDim.x) {
         const int64_t L = orp[r + 1] - orp[r];
         int32_t c = -1;
@@ -383,10 +411,14 @@ __global__ void classify_roots_kernel(int64_t n, const int64_t *__restrict__ orp
             const int64_t words = (L + 63) / 64;
             c = 0;
             while ((1ll << c) < words) ++c;
-            if (c >= kMaxClass) c = 100;  // unsupported size: reported by the host
+            if (c >= kMaxClass) c = kMaxClass;
+            atomicAdd(&h[c], 1u);
         }
         cls[r] = c;
     }
+    __syncthreads();
+    for (int i = threadIdx.x; i <= kMaxClass; i += blockDim.x)
+        if (h[i]) atomicAdd(hist + i, (unsigned long long)h[i]);
 }
 
 __global__ void flag_eq_kernel(int64_t n, const int32_t *__restrict__ cls, int32_t c, int32_t *flag) {
@@ -417,7 +449,7 @@ __global__ void make_roots_kernel(const int32_t *__restrict__ list, int64_t coun
         ri.r = r;
         ri.vbase = orp[r];
         ri.L = (int32_t)(orp[r + 1] - ri.vbase);
-        ri.abase = row_prefix[i] * W;
+        ri.abase = (row_prefix[i] - row_prefix[0]) * W;
         roots[i] = ri;
     }
 }
@@ -437,6 +469,22 @@ __global__ void find_chunk_end_kernel(const int64_t *__restrict__ offsets, int64
     out[0] = lo;
     out[1] = offsets[lo] - base;
     out[2] = base;
+}
+
+// smallest lo in [lo_min, hi) whose roots [lo, hi) fit `room` bytes (at least hi - 1)
+__global__ void find_window_kernel(const int64_t *__restrict__ prefix, int64_t hi, int64_t lo_min, int64_t room,
+                                   int64_t row_bytes, int64_t per_root, int64_t *out) {
+    int64_t l = lo_min, h = hi - 1;
+    while (l < h) {
+        const int64_t mid = (l + h) >> 1;
+        const int64_t bytes = (prefix[hi] - prefix[mid]) * row_bytes + (hi - mid) * per_root;
+        if (bytes <= room)
+            h = mid;
+        else
+            l = mid + 1;
+    }
+    out[0] = l;
+    out[1] = prefix[hi] - prefix[l];
 }
 
 template <int WPL>
@@ -461,12 +509,27 @@ void launch_warp(const ExpandArgs &a, bool write_pass, cudaStream_t s) {
 }  // namespace
 
 void launch_build_adj(const RootInfo *roots, int64_t nroots, int W, const int64_t *orp, const int32_t *ocol,
-                      uint64_t *adj, cudaStream_t s) {
+                      uint64_t *adj, int64_t adj_words, cudaStream_t s) {
     if (nroots <= 0) return;
     if (W == 1) {
         build_adj_w1<<<grid_for(nroots * 32, 256, 16), 256, 0, s>>>(roots, nroots, orp, ocol, adj);
     } else {
-        build_adj_wide<<<grid_for(nroots, 1, 16), 256, 0, s>>>(roots, nroots, W, orp, ocol, adj);
+        // shared-memory bit matrix up to W = 16 (L <= 1024: 128 KB + V)
+        const int64_t Lmax = 64ll * W;
+        const size_t smem = sizeof(int32_t) * (size_t)Lmax + (size_t)Lmax * W * 8;
+        if (W <= 16) {
+            static size_t attr_set = 0;
+            if (smem > 48 * 1024 && attr_set < smem) {
+                MCE_CUDA(cudaFuncSetAttribute(build_adj_block<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                              (int)smem));
+                attr_set = smem;
+            }
+            build_adj_block<true><<<grid_for(nroots, 1, 8), 512, smem, s>>>(roots, nroots, W, orp, ocol, adj);
+        } else {
+            MCE_CUDA(cudaMemsetAsync(adj, 0, sizeof(uint64_t) * (size_t)adj_words, s));
+            build_adj_block<false><<<grid_for(nroots, 1, 8), 512, sizeof(int32_t) * Lmax, s>>>(roots, nroots, W, orp,
+                                                                                                ocol, adj);
+        }
     }
     MCE_LAUNCH_CHECK();
 }
@@ -506,8 +569,14 @@ void launch_expand(const ExpandArgs &a, bool write_pass, cudaStream_t s) {
     }
 }
 
-void launch_classify_roots(int64_t n, const int64_t *orp, int32_t min_len, int32_t *cls, cudaStream_t s) {
-    classify_roots_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, orp, min_len, cls);
+void launch_classify_roots(int64_t n, const int64_t *orp, int32_t min_len, int32_t *cls, int64_t *hist,
+                           cudaStream_t s) {
+    classify_roots_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, orp, min_len, cls, (unsigned long long *)hist);
+    MCE_LAUNCH_CHECK();
+}
+void launch_find_window(const int64_t *prefix, int64_t hi, int64_t lo_min, int64_t room, int64_t row_bytes,
+                        int64_t per_root, int64_t *out, cudaStream_t s) {
+    find_window_kernel<<<1, 1, 0, s>>>(prefix, hi, lo_min, room, row_bytes, per_root, out);
     MCE_LAUNCH_CHECK();
 }
 void launch_flag_eq(int64_t n, const int32_t *cls, int32_t c, int32_t *flag, cudaStream_t s) {

@@ -53,15 +53,39 @@ struct ExpandArgs {
     const LevelLink *chain;  // chain[1..k]
 };
 
+// Fused root level for W == 1 roots (roots.cu): one warp per root builds the
+// induced adjacency of V = N+(r), applies the bound and writes the level-2
+// entries of surviving roots only.
+struct RootArgs {
+    const int32_t *list;  // roots: list[i * stride], i in [0, count)
+    int64_t count, stride;
+    const int64_t *orp;
+    const int32_t *ocol;
+    const int32_t *order;
+    int32_t need, bound;
+    // outputs (appended; ctr = {roots, adjacency rows, level-2 entries, leaves})
+    RootInfo *roots;
+    uint64_t *adj;
+    unsigned long long *ctr;
+    uint64_t *cP;
+    int32_t *cslot, *cparent, *cvloc;
+    int32_t *leaf_rows;  // size-2 leaves (only when need <= 2)
+    int64_t leaf_cap;
+};
+void launch_root_expand_w1(const RootArgs &a, cudaStream_t s);
+
 // W classes: 0 -> 1 word, 1 -> 2, 2 -> 4, ... (W = 1 << class); L <= 64 W
 constexpr int kMaxClass = 9;  // W up to 256 words (L <= 16384)
 
 void launch_build_adj(const RootInfo *roots, int64_t nroots, int W, const int64_t *orp, const int32_t *ocol,
-                      uint64_t *adj, cudaStream_t s);
+                      uint64_t *adj, int64_t adj_words, cudaStream_t s);
 void launch_init_level1(const RootInfo *roots, int64_t nroots, int W, uint64_t *P, int32_t *slot, int32_t *parent,
                         int32_t *vloc, cudaStream_t s);
 void launch_expand(const ExpandArgs &a, bool write_pass, cudaStream_t s);
-void launch_classify_roots(int64_t n, const int64_t *orp, int32_t min_len, int32_t *cls, cudaStream_t s);
+void launch_classify_roots(int64_t n, const int64_t *orp, int32_t min_len, int32_t *cls, int64_t *hist,
+                           cudaStream_t s);
+void launch_find_window(const int64_t *prefix, int64_t hi, int64_t lo_min, int64_t room, int64_t row_bytes,
+                        int64_t per_root, int64_t *out, cudaStream_t s);
 void launch_flag_eq(int64_t n, const int32_t *cls, int32_t c, int32_t *flag, cudaStream_t s);
 void launch_compact(int64_t n, const int32_t *flag, const int64_t *pos, int32_t *out, cudaStream_t s);
 void launch_make_roots(const int32_t *list, int64_t count, int64_t stride, int W, const int64_t *orp,

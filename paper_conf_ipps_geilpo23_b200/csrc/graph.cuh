@@ -25,6 +25,13 @@ struct mce_graph {
     int32_t max_out = 0;           // largest out-degree
     double t_pre_ms = 0.0;         // device time of the last preprocessing
     int64_t kernels = 0;           // kernels launched by the last preprocessing
+
+    // ---- reusable memory (no cudaMalloc/cudaFree on the steady-state path) ----
+    mce::Pool pool;                // per-phase scratch (reset at the start of every phase)
+    mce::DevBuf<uint8_t> ws;       // frontier arena of mce_enumerate / mce_find_one (grow-only)
+    mce::PinnedBuf host;           // pinned staging for small device->host reads
+    mce::DevBuf<uint8_t> misc;     // engine: leaf counter + level chain (persistent)
+    mce::DevBuf<int32_t> stage;    // engine: staged leaf cliques (grow-only)
 };
 
 namespace mce {

@@ -137,6 +137,11 @@ __global__ void compact_kernel(int64_t n, const int32_t *__restrict__ flag, cons
         if (flag[v]) out[pos[v]] = (int32_t)v;
 }
 
+__global__ void strided_gather_kernel(const int32_t *__restrict__ in, int64_t count, int64_t stride, int32_t *out) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < count; i += (int64_t)gridDim.x * blockDim.x)
+        out[i] = in[i * stride];
+}
+
 __global__ void iota_kernel(int64_t n, int32_t *out) {
     for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
         out[v] = (int32_t)v;
@@ -161,33 +166,34 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
     MCE_CUDA(cudaEventRecord(e0, s));
     int64_t kernels = 0;
 
-    DevBuf<int32_t> thr_buf;
+    Pool &pool = g->pool;
+    pool.reset();
     const int32_t *thr;
     if (use_core) {
         thr = g->core.get();
     } else {
-        thr_buf.alloc(n);
-        degree_thr_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(), thr_buf.get());
+        int32_t *tb = pool.take<int32_t>(n);
+        degree_thr_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(), tb);
         MCE_LAUNCH_CHECK();
         ++kernels;
-        thr = thr_buf.get();
+        thr = tb;
     }
     // ---- seeds: the h vertices with the highest threshold (ties: smaller id)
-    DevBuf<int32_t> seeds(n);
+    int32_t *seeds = pool.take<int32_t>(n);
     int64_t nseeds = 0;
     if (h == n) {
-        iota_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, seeds.get());
+        iota_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, seeds);
         MCE_LAUNCH_CHECK();
         ++kernels;
         nseeds = n;
     } else {
         int64_t maxthr = use_core ? g->degeneracy : g->max_deg;
-        DevBuf<int64_t> bins(maxthr + 1);
-        MCE_CUDA(cudaMemsetAsync(bins.get(), 0, bins.bytes(), s));
-        thr_hist_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, thr, bins.get());
+        int64_t *bins = pool.take<int64_t>(maxthr + 1);
+        MCE_CUDA(cudaMemsetAsync(bins, 0, sizeof(int64_t) * (maxthr + 1), s));
+        thr_hist_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, thr, bins);
         MCE_LAUNCH_CHECK();
-        std::vector<int64_t> hb(maxthr + 1);
-        MCE_CUDA(cudaMemcpyAsync(hb.data(), bins.get(), bins.bytes(), cudaMemcpyDeviceToHost, s));
+        int64_t *hb = g->host.get<int64_t>(maxthr + 1);
+        MCE_CUDA(cudaMemcpyAsync(hb, bins, sizeof(int64_t) * (maxthr + 1), cudaMemcpyDeviceToHost, s));
         MCE_CUDA(cudaStreamSynchronize(s));
         int64_t above = 0;
         int32_t tau = 0;
@@ -199,57 +205,55 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
             above += hb[t];
         }
         int64_t quota = h - above;
-        DevBuf<int32_t> flag(n);
-        DevBuf<int64_t> pos(n + 1), tmp(scan_tmp_items(n));
-        tie_flags_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, thr, tau, flag.get());
+        int32_t *flag = pool.take<int32_t>(n);
+        int64_t *pos = pool.take<int64_t>(n + 1), *tmp = pool.take<int64_t>(scan_tmp_items(n));
+        tie_flags_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, thr, tau, flag);
         MCE_LAUNCH_CHECK();
-        exclusive_scan_i32(flag.get(), pos.get(), n, tmp.get(), s);
-        seed_flags_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, thr, tau, pos.get(), quota, flag.get());
+        exclusive_scan_i32(flag, pos, n, tmp, s);
+        seed_flags_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, thr, tau, pos, quota, flag);
         MCE_LAUNCH_CHECK();
-        exclusive_scan_i32(flag.get(), pos.get(), n, tmp.get(), s);
-        compact_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, flag.get(), pos.get(), seeds.get());
+        exclusive_scan_i32(flag, pos, n, tmp, s);
+        compact_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, flag, pos, seeds);
         MCE_LAUNCH_CHECK();
         kernels += 10;
         nseeds = h;
     }
     // ---- shard the runs across ranks (cyclic over the id-ordered seed list)
-    const int32_t *seed_ptr = seeds.get();
-    DevBuf<int32_t> shard_seeds;
-    if (shard_count > 1) {
-        std::vector<int32_t> hs(nseeds);
-        MCE_CUDA(cudaMemcpyAsync(hs.data(), seeds.get(), sizeof(int32_t) * nseeds, cudaMemcpyDeviceToHost, s));
-        MCE_CUDA(cudaStreamSynchronize(s));
-        std::vector<int32_t> mine;
-        for (int64_t i = shard_rank; i < nseeds; i += shard_count) mine.push_back(hs[i]);
-        shard_seeds.alloc(std::max<size_t>(mine.size(), 1));
-        if (!mine.empty())
-            MCE_CUDA(cudaMemcpyAsync(shard_seeds.get(), mine.data(), sizeof(int32_t) * mine.size(),
-                                     cudaMemcpyHostToDevice, s));
-        seed_ptr = shard_seeds.get();
-        nseeds = (int64_t)mine.size();
+    const int32_t *seed_ptr = seeds;
+    if (shard_count > 1) {  // this rank's seeds: positions shard_rank, shard_rank + shard_count, ...
+        const int64_t mine = nseeds > shard_rank ? (nseeds - shard_rank + shard_count - 1) / shard_count : 0;
+        int32_t *sh = pool.take<int32_t>(std::max<int64_t>(mine, 1));
+        if (mine > 0) {
+            strided_gather_kernel<<<grid_for(mine, 256), 256, 0, s>>>(seeds + shard_rank, mine, shard_count, sh);
+            MCE_LAUNCH_CHECK();
+            ++kernels;
+        }
+        seed_ptr = sh;
+        nseeds = mine;
     }
     // ---- the runs
-    DevBuf<int32_t> scratch(std::max<int64_t>(g->nnz, 1)), run_size(n), best(1);
-    DevBuf<unsigned long long> best_key(1);
-    DevBuf<int32_t> clique(g->max_deg + 2);
-    MCE_CUDA(cudaMemsetAsync(run_size.get(), 0, run_size.bytes(), s));
-    MCE_CUDA(cudaMemsetAsync(best.get(), 0, best.bytes(), s));
-    MCE_CUDA(cudaMemsetAsync(best_key.get(), 0, best_key.bytes(), s));
+    int32_t *scratch = pool.take<int32_t>(std::max<int64_t>(g->nnz, 1));
+    int32_t *run_size = pool.take<int32_t>(n), *best = pool.take<int32_t>(1);
+    unsigned long long *best_key = pool.take<unsigned long long>(1);
+    int32_t *clique = pool.take<int32_t>(g->max_deg + 2);
+    MCE_CUDA(cudaMemsetAsync(run_size, 0, sizeof(int32_t) * n, s));
+    MCE_CUDA(cudaMemsetAsync(best, 0, sizeof(int32_t), s));
+    MCE_CUDA(cudaMemsetAsync(best_key, 0, sizeof(unsigned long long), s));
     if (nseeds > 0) {
         greedy_kernel<<<grid_for(nseeds * 32, 256), 256, 0, s>>>(nseeds, seed_ptr, g->rowptr.get(), g->col.get(),
-                                                                  thr, scratch.get(), run_size.get(), best.get());
+                                                                  thr, scratch, run_size, best);
         MCE_LAUNCH_CHECK();
-        best_seed_kernel<<<grid_for(nseeds, 256), 256, 0, s>>>(nseeds, seed_ptr, thr, run_size.get(), best.get(),
-                                                               best_key.get());
+        best_seed_kernel<<<grid_for(nseeds, 256), 256, 0, s>>>(nseeds, seed_ptr, thr, run_size, best, best_key);
         MCE_LAUNCH_CHECK();
-        replay_kernel<<<1, 32, 0, s>>>(best_key.get(), g->rowptr.get(), g->col.get(), thr, scratch.get(),
-                                       clique.get());
+        replay_kernel<<<1, 32, 0, s>>>(best_key, g->rowptr.get(), g->col.get(), thr, scratch, clique);
         MCE_LAUNCH_CHECK();
         kernels += 3;
     }
     MCE_CUDA(cudaEventRecord(e1, s));
-    MCE_CUDA(cudaMemcpyAsync(&res.omega_bar, best.get(), sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+    int32_t *hbest = g->host.get<int32_t>(1);
+    MCE_CUDA(cudaMemcpyAsync(hbest, best, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
     MCE_CUDA(cudaStreamSynchronize(s));
+    res.omega_bar = hbest[0];
     float ms = 0;
     MCE_CUDA(cudaEventElapsedTime(&ms, e0, e1));
     res.ms = ms;
@@ -258,12 +262,11 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
     cudaEventDestroy(e1);
     if (res.omega_bar > 0) {
         res.clique.resize(res.omega_bar);
-        MCE_CUDA(cudaMemcpy(res.clique.data(), clique.get(), sizeof(int32_t) * res.omega_bar,
-                            cudaMemcpyDeviceToHost));
+        MCE_CUDA(cudaMemcpy(res.clique.data(), clique, sizeof(int32_t) * res.omega_bar, cudaMemcpyDeviceToHost));
     }
     if (want_runs) {
         res.run_size.resize(n);
-        MCE_CUDA(cudaMemcpy(res.run_size.data(), run_size.get(), sizeof(int32_t) * n, cudaMemcpyDeviceToHost));
+        MCE_CUDA(cudaMemcpy(res.run_size.data(), run_size, sizeof(int32_t) * n, cudaMemcpyDeviceToHost));
     }
     return res;
 }

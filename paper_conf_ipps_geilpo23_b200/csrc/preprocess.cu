@@ -27,8 +27,23 @@ namespace {
 
 constexpr int kPeelThreads = 512;
 
-// ctrl layout: [0..2] queue append counters (rotating per sub-round),
-//              [3..5] alive-list append counters (rotating per sub-round)
+// ctrl layout (rotating per sub-round s, index s % 3):
+//   [0..2] queue append counters, [3..5] alive-list append counters,
+//   [6..8] smallest degree among the vertices a scan kept alive
+//
+// Level-synchronous peel: a "scan" sub-round queues every alive vertex with
+// degree <= k and compacts the rest into the next alive list; a "cascade"
+// sub-round processes the vertices queued by the previous sub-round (one warp
+// per vertex, lanes over its neighbours) and queues neighbours whose degree
+// falls to k.  All appends are warp-aggregated (one atomicAdd per warp and
+// ballot ranks), so no counter sees more than one atomic per warp.  When a
+// scan queues nothing, k jumps straight to the smallest alive degree it saw.
+__device__ __forceinline__ unsigned long long warp_append(unsigned long long *ctr, unsigned mask, int lane) {
+    unsigned long long base = 0;
+    if (lane == 0 && mask) base = atomicAdd(ctr, (unsigned long long)__popc(mask));
+    return __shfl_sync(0xffffffffu, base, 0);
+}
+
 __global__ void __launch_bounds__(kPeelThreads)
     kcore_peel(int64_t n, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col, int32_t *deg,
                int32_t *core, int32_t *queue, int32_t *alive_a, int32_t *alive_b, uint8_t *dead,
@@ -39,6 +54,7 @@ __global__ void __launch_bounds__(kPeelThreads)
     const int64_t warp = tid >> 5;
     const int64_t nwarps = nthreads >> 5;
     const int lane = threadIdx.x & 31;
+    const unsigned lt = lanemask_lt();
 
     int64_t s = 0;          // sub-round
     int64_t head = 0;       // region to process: [head, region_end)
@@ -50,34 +66,58 @@ __global__ void __launch_bounds__(kPeelThreads)
     while (true) {
         unsigned long long *qcnt = ctrl + (s % 3);
         unsigned long long *acnt = ctrl + 3 + (s % 3);
-        if (tid == 0) {  // zero the counters of sub-round s+1 (last read before this sub-round began)
+        unsigned long long *mind = ctrl + 6 + (s % 3);
+        if (tid == 0) {  // reset the counters of sub-round s+1 (last read before this sub-round began)
             ctrl[(s + 1) % 3] = 0;
             ctrl[3 + (s + 1) % 3] = 0;
+            ctrl[6 + (s + 1) % 3] = ~0ull;
         }
         if (scan) {
-            for (int64_t i = tid; i < n_alive; i += nthreads) {
-                int32_t v = cur[i];
-                if (dead[v]) continue;
-                if (deg[v] <= k) {
-                    unsigned long long p = region_end + atomicAdd(qcnt, 1ull);
-                    queue[p] = v;
+            int32_t dmin = INT32_MAX;
+            for (int64_t i0 = warp * 32; i0 < n_alive; i0 += nwarps * 32) {
+                const int64_t i = i0 + lane;
+                int32_t v = -1, d = 0;
+                bool live = false;
+                if (i < n_alive) {
+                    v = cur[i];
+                    live = !dead[v];
+                    if (live) d = deg[v];
+                }
+                const bool q = live && d <= k;
+                const bool keep = live && d > k;
+                const unsigned qm = __ballot_sync(0xffffffffu, q);
+                const unsigned km = __ballot_sync(0xffffffffu, keep);
+                const unsigned long long qb = warp_append(qcnt, qm, lane);
+                const unsigned long long kb = warp_append(acnt, km, lane);
+                if (q) {
+                    queue[region_end + qb + __popc(qm & lt)] = v;
                     core[v] = k;
                     dead[v] = 1;
-                } else {
-                    unsigned long long p = atomicAdd(acnt, 1ull);
-                    nxt[p] = v;
+                }
+                if (keep) {
+                    nxt[kb + __popc(km & lt)] = v;
+                    dmin = min(dmin, d);
                 }
             }
+            dmin = __reduce_min_sync(0xffffffffu, dmin);
+            if (lane == 0 && dmin != INT32_MAX) atomicMin(mind, (unsigned long long)dmin);
         } else {
-            for (int64_t i = head + warp; i < region_end; i += nwarps) {
-                int32_t v = queue[i];
-                for (int64_t e = rowptr[v] + lane; e < rowptr[v + 1]; e += 32) {
-                    int32_t u = col[e];
-                    if (!dead[u]) {
-                        int32_t old = atomicSub(deg + u, 1);
-                        if (old == k + 1) {
-                            unsigned long long p = region_end + atomicAdd(qcnt, 1ull);
-                            queue[p] = u;
+            for (int64_t qi = head + warp; qi < region_end; qi += nwarps) {
+                const int32_t v = queue[qi];
+                const int64_t eb = rowptr[v], ee = rowptr[v + 1];
+                for (int64_t e0 = eb; e0 < ee; e0 += 32) {
+                    const int64_t e = e0 + lane;
+                    bool fell = false;
+                    int32_t u = -1;
+                    if (e < ee) {
+                        u = col[e];
+                        if (!dead[u]) fell = atomicSub(deg + u, 1) == k + 1;
+                    }
+                    const unsigned fm = __ballot_sync(0xffffffffu, fell);
+                    if (fm) {
+                        const unsigned long long b = warp_append(qcnt, fm, lane);
+                        if (fell) {
+                            queue[region_end + b + __popc(fm & lt)] = u;
                             core[u] = k;
                             dead[u] = 1;
                         }
@@ -87,6 +127,8 @@ __global__ void __launch_bounds__(kPeelThreads)
         }
         grid.sync();
         const int64_t c = (int64_t)(*(volatile unsigned long long *)qcnt);
+        const unsigned long long md = *(volatile unsigned long long *)mind;
+        const bool was_scan = scan;
         if (scan) {
             n_alive = (int64_t)(*(volatile unsigned long long *)acnt);
             int32_t *t = cur;
@@ -97,13 +139,20 @@ __global__ void __launch_bounds__(kPeelThreads)
         region_end += c;
         if (region_end >= n) break;  // every vertex has its core number
         if (c == 0) {
-            ++k;
+            // a scan that queued nothing saw every alive degree: jump to the smallest
+            k = was_scan ? (int32_t)md : k + 1;
             scan = true;
         } else {
             scan = false;
         }
         ++s;
     }
+}
+
+// degeneracy = core number of the last vertex peeled
+__global__ void last_core_kernel(int64_t n, const int32_t *__restrict__ peel, const int32_t *__restrict__ core,
+                                 int32_t *out) {
+    out[0] = core[peel[n - 1]];
 }
 
 __global__ void degrees_kernel(int64_t n, const int64_t *__restrict__ rowptr, int32_t *deg, int32_t *iota) {
@@ -234,13 +283,24 @@ __global__ void sort_rows_block(const int64_t *__restrict__ orp, int32_t *ocol, 
     }
 }
 
+// rows longer than a warp (sorted by one block each) and the largest out-degree
 __global__ void long_rows_kernel(int64_t n, const int64_t *__restrict__ orp, int32_t *rows, int32_t *count,
                                  int32_t *max_out) {
-    for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < n; r += (int64_t)gridDim.x * blockDim.x) {
-        int32_t len = (int32_t)(orp[r + 1] - orp[r]);
-        atomicMax(max_out, len);
-        if (len > 32) rows[atomicAdd(count, 1)] = (int32_t)r;
+    const int lane = threadIdx.x & 31;
+    int32_t mx = 0;
+    for (int64_t r0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) & ~31ll; r0 < n;
+         r0 += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t r = r0 + lane;
+        const int32_t len = r < n ? (int32_t)(orp[r + 1] - orp[r]) : 0;
+        mx = max(mx, len);
+        const unsigned m = __ballot_sync(0xffffffffu, len > 32);
+        int32_t b = 0;
+        if (lane == 0 && m) b = atomicAdd(count, __popc(m));
+        b = __shfl_sync(0xffffffffu, b, 0);
+        if (len > 32) rows[b + __popc(m & lanemask_lt())] = (int32_t)r;
     }
+    mx = __reduce_max_sync(0xffffffffu, mx);
+    if (lane == 0 && mx) atomicMax(max_out, mx);
 }
 
 }  // namespace
@@ -265,38 +325,41 @@ void kcore(mce_graph *g) {
     if (g->have_core) return;
     const int64_t n = g->n;
     cudaStream_t s = g->stream;
-    g->core.alloc(std::max<int64_t>(n, 1));
-    g->peel.alloc(std::max<int64_t>(n, 1));
+    g->core.ensure(std::max<int64_t>(n, 1));
+    g->peel.ensure(std::max<int64_t>(n, 1));
     if (n == 0) {
         g->have_core = true;
         g->degeneracy = 0;
         return;
     }
-    DevBuf<int32_t> deg(n), alive_a(n), alive_b(n);
-    DevBuf<uint8_t> dead(n);
-    DevBuf<unsigned long long> ctrl(8);
-    MCE_CUDA(cudaMemsetAsync(dead.get(), 0, n, s));
-    MCE_CUDA(cudaMemsetAsync(ctrl.get(), 0, ctrl.bytes(), s));
-    degrees_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(), deg.get(), alive_a.get());
+    g->pool.reset();
+    int32_t *deg = g->pool.take<int32_t>(n), *alive_a = g->pool.take<int32_t>(n), *alive_b = g->pool.take<int32_t>(n);
+    uint8_t *dead = g->pool.take<uint8_t>(n);
+    unsigned long long *ctrl = g->pool.take<unsigned long long>(9);
+    MCE_CUDA(cudaMemsetAsync(dead, 0, n, s));
+    MCE_CUDA(cudaMemsetAsync(ctrl, 0, 6 * sizeof(unsigned long long), s));
+    MCE_CUDA(cudaMemsetAsync(ctrl + 6, 0xff, 3 * sizeof(unsigned long long), s));
+    degrees_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(), deg, alive_a);
     MCE_LAUNCH_CHECK();
     int blocks_per_sm = 0;
     MCE_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm, kcore_peel, kPeelThreads, 0));
-    blocks_per_sm = std::max(1, std::min(blocks_per_sm, 4));
+    blocks_per_sm = std::max(1, std::min(blocks_per_sm, 2));
     int grid = num_sms() * blocks_per_sm;
     int64_t n_arg = n;
     const int64_t *rp = g->rowptr.get();
     const int32_t *cl = g->col.get();
-    int32_t *dg = deg.get(), *co = g->core.get(), *qu = g->peel.get(), *aa = alive_a.get(), *ab = alive_b.get();
-    uint8_t *dd = dead.get();
-    unsigned long long *ct = ctrl.get();
+    int32_t *dg = deg, *co = g->core.get(), *qu = g->peel.get(), *aa = alive_a, *ab = alive_b;
+    uint8_t *dd = dead;
+    unsigned long long *ct = ctrl;
     void *args[] = {&n_arg, &rp, &cl, &dg, &co, &qu, &aa, &ab, &dd, &ct};
     MCE_CUDA(cudaLaunchCooperativeKernel((void *)kcore_peel, grid, kPeelThreads, args, 0, s));
     g->kernels += 2;
     // degeneracy = max core (the last queued vertex has it)
-    int32_t last_v = 0;
-    MCE_CUDA(cudaMemcpyAsync(&last_v, g->peel.get() + n - 1, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+    last_core_kernel<<<1, 1, 0, s>>>(n, g->peel.get(), g->core.get(), deg);
+    int32_t *h = g->host.get<int32_t>(1);
+    MCE_CUDA(cudaMemcpyAsync(h, deg, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
     MCE_CUDA(cudaStreamSynchronize(s));
-    MCE_CUDA(cudaMemcpy(&g->degeneracy, g->core.get() + last_v, sizeof(int32_t), cudaMemcpyDeviceToHost));
+    g->degeneracy = h[0];
     g->have_core = true;
 }
 
@@ -304,10 +367,11 @@ void orient(mce_graph *g, int orientation) {
     if (g->orientation == orientation) return;
     const int64_t n = g->n;
     cudaStream_t s = g->stream;
-    g->order.alloc(std::max<int64_t>(n, 1));
-    g->rank.alloc(std::max<int64_t>(n, 1));
-    g->orp.alloc(n + 1);
-    g->ocol.alloc(std::max<int64_t>(g->nnz / 2, 1));
+    g->order.ensure(std::max<int64_t>(n, 1));
+    g->rank.ensure(std::max<int64_t>(n, 1));
+    g->orp.ensure(n + 1);
+    g->ocol.ensure(std::max<int64_t>(g->nnz / 2, 1));
+    g->pool.reset();
     if (n == 0) {
         MCE_CUDA(cudaMemsetAsync(g->orp.get(), 0, sizeof(int64_t), s));
         g->orientation = orientation;
@@ -318,56 +382,51 @@ void orient(mce_graph *g, int orientation) {
         MCE_CUDA(cudaMemcpyAsync(g->order.get(), g->peel.get(), sizeof(int32_t) * n, cudaMemcpyDeviceToDevice, s));
     } else {  // degree order
         int64_t nb = g->max_deg + 1;
-        DevBuf<int32_t> bins(nb);
-        DevBuf<int64_t> cursor(nb + 1), tmp(scan_tmp_items(nb));
-        MCE_CUDA(cudaMemsetAsync(bins.get(), 0, bins.bytes(), s));
-        degree_hist<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(), bins.get());
+        int32_t *bins = g->pool.take<int32_t>(nb);
+        int64_t *cursor = g->pool.take<int64_t>(nb + 1), *tmp = g->pool.take<int64_t>(scan_tmp_items(nb));
+        MCE_CUDA(cudaMemsetAsync(bins, 0, sizeof(int32_t) * nb, s));
+        degree_hist<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(), bins);
         MCE_LAUNCH_CHECK();
-        exclusive_scan_i32(bins.get(), cursor.get(), nb, tmp.get(), s);
-        degree_scatter<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(),
-                                                         (unsigned long long *)cursor.get(), g->order.get());
+        exclusive_scan_i32(bins, cursor, nb, tmp, s);
+        degree_scatter<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(), (unsigned long long *)cursor,
+                                                         g->order.get());
         MCE_LAUNCH_CHECK();
-        MCE_CUDA(cudaStreamSynchronize(s));
         g->kernels += 5;
     }
     invert_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->order.get(), g->rank.get());
     MCE_LAUNCH_CHECK();
-    DevBuf<int32_t> odeg(n);
-    out_degree_kernel<<<grid_for(n * 32, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), g->rank.get(),
-                                                            odeg.get());
+    int32_t *odeg = g->pool.take<int32_t>(n);
+    out_degree_kernel<<<grid_for(n * 32, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), g->rank.get(), odeg);
     MCE_LAUNCH_CHECK();
-    {
-        DevBuf<int64_t> tmp(scan_tmp_items(n));
-        exclusive_scan_i32(odeg.get(), g->orp.get(), n, tmp.get(), s);
-    }
+    exclusive_scan_i32(odeg, g->orp.get(), n, g->pool.take<int64_t>(scan_tmp_items(n)), s);
     orient_fill_kernel<<<grid_for(n * 32, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), g->rank.get(),
                                                              g->orp.get(), g->ocol.get());
     MCE_LAUNCH_CHECK();
     sort_rows_warp<<<grid_for(n * 32, 256), 256, 0, s>>>(n, g->orp.get(), g->ocol.get());
     MCE_LAUNCH_CHECK();
-    DevBuf<int32_t> rows(n), meta(2);
-    MCE_CUDA(cudaMemsetAsync(meta.get(), 0, meta.bytes(), s));
-    long_rows_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->orp.get(), rows.get(), meta.get(), meta.get() + 1);
+    int32_t *rows = g->pool.take<int32_t>(n), *meta = g->pool.take<int32_t>(2);
+    MCE_CUDA(cudaMemsetAsync(meta, 0, 2 * sizeof(int32_t), s));
+    long_rows_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->orp.get(), rows, meta, meta + 1);
     MCE_LAUNCH_CHECK();
-    int32_t hmeta[2];
-    MCE_CUDA(cudaMemcpyAsync(hmeta, meta.get(), sizeof(hmeta), cudaMemcpyDeviceToHost, s));
+    int32_t *hmeta = g->host.get<int32_t>(2);
+    MCE_CUDA(cudaMemcpyAsync(hmeta, meta, 2 * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
     MCE_CUDA(cudaStreamSynchronize(s));
     g->kernels += 8;
     g->max_out = hmeta[1];
-    if (hmeta[0] > 0) {
+    const int32_t n_long = hmeta[0];
+    if (n_long > 0) {
         const int32_t smem_cap = 8192;  // ints (32 KB)
         int32_t p2 = 1;
         while (p2 < g->max_out) p2 <<= 1;
         if (p2 <= smem_cap) {
-            sort_rows_block<<<grid_for(hmeta[0], 1, 16), 256, smem_cap * sizeof(int32_t), s>>>(
-                g->orp.get(), g->ocol.get(), rows.get(), hmeta[0], nullptr, smem_cap);
+            sort_rows_block<<<grid_for(n_long, 1, 16), 256, smem_cap * sizeof(int32_t), s>>>(
+                g->orp.get(), g->ocol.get(), rows, n_long, nullptr, smem_cap);
             MCE_LAUNCH_CHECK();
         } else {  // some row exceeds shared memory: one block, global scratch
-            DevBuf<int32_t> scratch(p2);
-            sort_rows_block<<<1, 1024, smem_cap * sizeof(int32_t), s>>>(g->orp.get(), g->ocol.get(), rows.get(),
-                                                                        hmeta[0], scratch.get(), smem_cap);
+            int32_t *scratch = g->pool.take<int32_t>(p2);
+            sort_rows_block<<<1, 1024, smem_cap * sizeof(int32_t), s>>>(g->orp.get(), g->ocol.get(), rows, n_long,
+                                                                        scratch, smem_cap);
             MCE_LAUNCH_CHECK();
-            MCE_CUDA(cudaStreamSynchronize(s));
         }
         g->kernels += 1;
     }

@@ -67,14 +67,37 @@ def run_enum(g, **kw):
         gg.close()
 
 
+@pytest.mark.parametrize("legacy_roots", [False, True])
 @pytest.mark.parametrize("key", list(GRAPHS))
-def test_enumerate_matches_oracle(key):
+def test_enumerate_matches_oracle(key, legacy_roots):
+    """Fused root-level kernel (default) and the generic per-level path both match the oracle."""
     g = GRAPHS[key]()
     om, cl = oracle_answer(key)
-    r = run_enum(g)
+    r = run_enum(g, legacy_roots=legacy_roots)
     assert r.omega == om
     assert r.count == len(cl)
     assert np.array_equal(r.cliques, cl)
+
+
+@pytest.mark.parametrize("key", ["er2000", "planted", "RMAT11", "BA5k", "C9", "T(36,12)"])
+def test_no_heuristic_size2_leaves(key):
+    """Heuristic 'none' with a lower bound of 2: size-2 leaves come out of the fused root kernel."""
+    g = GRAPHS[key]()
+    om, cl = oracle_answer(key)
+    r = run_enum(g, heuristic="none", bound="size" if key == "C9" else "color")
+    assert (r.omega, r.count) == (om, len(cl)) and np.array_equal(r.cliques, cl)
+
+
+def test_triangle_free_many_leaves():
+    """omega = 2 with more edges than the initial leaf staging (4096 rows): staging grows, replay is exact."""
+    n = 6000
+    i = torch.arange(n, dtype=torch.int64)
+    g = G.from_edges(n, i, (i + 1) % n)  # C_6000: 6000 maximum cliques of size 2
+    r = run_enum(g, heuristic="none")
+    assert r.omega == 2 and r.count == n
+    rows = np.sort(np.stack([i.numpy(), ((i + 1) % n).numpy()], 1), axis=1)
+    rows = rows[np.lexsort(rows.T[::-1])]
+    assert np.array_equal(r.cliques, rows.astype(np.int32))
 
 
 @pytest.mark.parametrize("bound", ["size", "color"])
