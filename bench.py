@@ -40,6 +40,9 @@ def parse():
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
     p.add_argument("--mode", default=None, choices=[None, "enumerate", "find_one"])
     p.add_argument("--window", type=int, default=0)
+    p.add_argument("--max-cliques", type=int, default=-1,
+                   help="stored-clique capacity (multiplicity stays exact); -1: 2^16 for the R-MAT configs "
+                        "(~10^8 maximum cliques of size ~223 there), unbounded otherwise")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
     return p.parse_args()
@@ -184,6 +187,7 @@ def main():
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     mode = args.mode or ("find_one" if args.config == "dense800" else "enumerate")
+    max_cl = args.max_cliques if args.max_cliques >= 0 else (1 << 16 if args.config.startswith("rmat") else 0)
 
     g = build_graph(args.config, f"cuda:{local}")
     edges = g.num_edges
@@ -195,10 +199,10 @@ def main():
         gr.clear_cache()
         if world > 1:
             if mode == "enumerate":
-                return mdist.enumerate_distributed(gr)
+                return mdist.enumerate_distributed(gr, max_cliques=max_cl)
             return mdist.find_one_distributed(gr, window=args.window)
         if mode == "enumerate":
-            return gr.enumerate()
+            return gr.enumerate(max_cliques=max_cl)
         return gr.find_one(window=args.window)
 
     for _ in range(args.warmup):
@@ -254,9 +258,9 @@ def main():
             torch.cuda.synchronize()
             t0 = time.perf_counter()
             gh = mce.Graph(rp_h, col_h, device=local)
-            r2 = mdist.enumerate_distributed(gh) if (world > 1 and mode == "enumerate") else (
+            r2 = mdist.enumerate_distributed(gh, max_cliques=max_cl) if (world > 1 and mode == "enumerate") else (
                 mdist.find_one_distributed(gh, window=args.window) if world > 1 else
-                (gh.enumerate() if mode == "enumerate" else gh.find_one(window=args.window)))
+                (gh.enumerate(max_cliques=max_cl) if mode == "enumerate" else gh.find_one(window=args.window)))
             dt = time.perf_counter() - t0
             gh.close()
             if i:
@@ -290,6 +294,7 @@ def main():
             "data": "synthetic",
             "config": {"workload": args.config, "baseline_config_index": CONFIG_INDEX[args.config],
                        "mode": mode, "n": g.n, "edges": edges, "omega": res.omega, "multiplicity": res.count,
+                       "stored_cliques": int(res.cliques.shape[0]), "max_cliques": max_cl,
                        "parallelism": f"root-shard x{world}", "l2": "flushed (256 MiB write) before every step",
                        "phases_ms": phases, "levels": res.levels},
             "roofline": {"bound": "hbm", "kernel": kname,

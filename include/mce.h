@@ -71,7 +71,8 @@ typedef struct {
     int64_t window;          /* roots per window (PAPER.md IV-E); <=0 = all roots at once */
     int64_t budget_bytes;    /* device bytes the frontier may use; <=0 = 90% of free memory */
     int64_t max_cliques;     /* capacity of the stored clique list; <=0 = unbounded
-                                (still limited by the budget).  The multiplicity is
+                                (still limited: at most max(2^20, rows fitting a quarter
+                                of the budget) are stored).  The multiplicity is
                                 always exact; cliques beyond capacity are counted
                                 but not stored (mce_result_info: truncated). */
     int32_t shard_rank;      /* root sharding for multi-GPU: this process takes the */

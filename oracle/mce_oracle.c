@@ -301,7 +301,7 @@ static void expand(mce_ctx *x, int32_t csize) {
     for (int32_t i = np - 1; i >= 0; --i) {
         if (csize + colr[i] < x->best) return;
         int32_t v = ord[i];
-        x->stack[csize] = x->V[v];
+        x->stack[csize] = x->V[x->L - 1 - v]; /* local index v <-> V[L-1-v] (see oracle_mce) */
         int32_t nonempty = 0;
         for (int32_t j = 0; j < W; ++j) {
             Q[j] = P[j] & x->A[(int64_t)v * W + j];
@@ -403,15 +403,20 @@ int64_t oracle_mce(int64_t n, const int64_t *rowptr, const int32_t *col, int32_t
         }
         const int32_t *V = ocol + orp[r];
         int32_t W = (L + 63) / 64;
-        for (int32_t a = 0; a < L; ++a) loc[V[a]] = a;
+        /* Local index of V[a] is L-1-a: bits run in reverse pi order, so the
+         * greedy colouring meets the high-core vertices first and gives them the
+         * low colours, and the search branches on them last, with the smallest
+         * candidate sets (smallest-last order, reading 5).  The set of
+         * maximum cliques found does not depend on this order, only the run time. */
+        for (int32_t a = 0; a < L; ++a) loc[V[a]] = L - 1 - a;
         memset(A, 0, sizeof(uint64_t) * L * W);
         for (int32_t a = 0; a < L; ++a) {
             int32_t u = V[a];
             for (int64_t e = orp[u]; e < orp[u + 1]; ++e) {
-                int32_t b = loc[ocol[e]];
+                int32_t b = loc[ocol[e]], la = L - 1 - a;
                 if (b >= 0) {
-                    A[(int64_t)a * W + (b >> 6)] |= 1ULL << (b & 63);
-                    A[(int64_t)b * W + (a >> 6)] |= 1ULL << (a & 63);
+                    A[(int64_t)la * W + (b >> 6)] |= 1ULL << (b & 63);
+                    A[(int64_t)b * W + (la >> 6)] |= 1ULL << (la & 63);
                 }
             }
         }

@@ -50,6 +50,7 @@ struct Arena {
 
 struct Level {
     int64_t count = 0;
+    int32_t W = 1;  // words per candidate set (stride of P)
     uint64_t *P = nullptr;
     int32_t *slot = nullptr;
     int32_t *parent = nullptr;
@@ -153,12 +154,15 @@ class Engine {
     LaunchClock clock_;
     Arena arena_;
     int32_t best_ = 0;
-    int32_t W_ = 1;
+    int32_t W_ = 1;   // words per adjacency row of the current root window
     int64_t stride_ = 1, offset_ = 0;
 
     // leaves
-    unsigned long long *leaf_count_ = nullptr;
+    unsigned long long *leaf_total_ = nullptr;  // g->misc[0]
+    unsigned long long *leaf_slot_ = nullptr;   // g->misc[1]
+    int32_t *maxbit_ = nullptr;                 // g->misc[2]
     int64_t stage_rows_ = 0;
+    int64_t stage_max_rows_ = 0;  // staging never exceeds a quarter of the budget (stored list truncated, count exact)
     std::vector<int32_t> rows_;  // host copy of the stored cliques (width res_size_)
     int32_t res_size_ = 0;
     int64_t res_count_ = 0;
@@ -186,7 +190,7 @@ void Engine::launch_timed(const ExpandArgs &a, bool write) {
     if (!write) {
         ++count_launches_;
         const double n = (double)(a.end - a.begin);
-        count_bytes_ += n * (8.0 * a.W + 4 + 4 + 4 + sizeof(RootInfo));
+        count_bytes_ += n * (8.0 * a.Wp + 4 + 4 + 4 + sizeof(RootInfo));
     }
 }
 
@@ -216,14 +220,15 @@ void Engine::handle_leaves(int32_t size, int64_t cnt, ExpandArgs &a) {
     }
     if (size > best_) best_ = size;
     const int64_t stored = (int64_t)rows_.size() / std::max(res_size_, 1);
-    int64_t want = cnt;
-    if (o_.max_cliques > 0) want = std::min<int64_t>(want, std::max<int64_t>(o_.max_cliques - stored, 0));
+    // stored list capacity: max_cliques, and never more rows than a quarter of the budget holds
+    const int64_t store_cap = o_.max_cliques > 0 ? std::min<int64_t>(o_.max_cliques, stage_max_rows_) : stage_max_rows_;
+    const int64_t want = std::min<int64_t>(cnt, std::max<int64_t>(store_cap - stored, 0));
     if (want > a.leaf_cap) {  // staging too small: grow and replay the count pass (idempotent)
         stage_rows_ = want;
         g_->stage.ensure((size_t)want * std::max<int32_t>(g_->max_out + 2, 2));
         a.leaf_rows = g_->stage.get();
         a.leaf_cap = want;
-        MCE_CUDA(cudaMemsetAsync(leaf_count_, 0, sizeof(unsigned long long), s_));
+        MCE_CUDA(cudaMemsetAsync(leaf_total_, 0, 2 * sizeof(unsigned long long), s_));
         launch_expand(a, false, s_);
         ++kernels_;
         MCE_CUDA(cudaStreamSynchronize(s_));
@@ -263,33 +268,45 @@ void Engine::process(int32_t k, const Level &L) {
     a.k = k;
     a.need = need();
     a.bound = o_.bound;
-    a.W = W_;
+    a.Wp = L.W;
+    a.Wa = W_;
+    a.Wc = L.W;
     a.roots = roots_;
     a.adj = adj_;
     a.ocol = g_->ocol.get();
     a.order = g_->order.get();
     a.counts = counts;
-    a.leaf_count = leaf_count_;
+    a.maxbit = maxbit_;
+    a.leaf_total = leaf_total_;
+    a.leaf_slot = leaf_slot_;
     a.leaf_rows = g_->stage.get();
     a.leaf_cap = stage_rows_;
     a.chain = chain_dev_;
 
-    MCE_CUDA(cudaMemsetAsync(leaf_count_, 0, sizeof(unsigned long long), s_));
+    // misc[0..2] = leaf total, leaf slot, maxbit (-1)
+    MCE_CUDA(cudaMemsetAsync(leaf_total_, 0, 2 * sizeof(unsigned long long), s_));
+    MCE_CUDA(cudaMemsetAsync(maxbit_, 0xff, sizeof(int32_t), s_));
     launch_timed(a, false);
     exclusive_scan_i32(counts, offs, N, tmp, s_);
     kernels_ += 3;
-    int64_t *h = g_->host.get<int64_t>(2);
+    int64_t *h = g_->host.get<int64_t>(4);
     MCE_CUDA(cudaMemcpyAsync(h, offs + N, sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
-    MCE_CUDA(cudaMemcpyAsync(h + 1, leaf_count_, sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
+    MCE_CUDA(cudaMemcpyAsync(h + 1, leaf_total_, 3 * sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
     MCE_CUDA(cudaStreamSynchronize(s_));
     const int64_t total = h[0];
     const unsigned long long leaves = (unsigned long long)h[1];
+    const int32_t maxbit = (int32_t)(uint32_t)(uint64_t)h[3];
+    // children's candidate sets only use bits <= maxbit: shrink their stride
+    // (power of two, so the kernels stay specialised)
+    int32_t Wc = 1;
+    while (Wc * 64 <= maxbit && Wc < L.W) Wc <<= 1;
+    a.Wc = Wc;
     if (o_.verbose > 0)
         fprintf(stderr, "[mce] level k=%d entries=%lld children=%lld leaves=%llu need=%d\n", k, (long long)N,
                 (long long)total, leaves, a.need);
     if (leaves) handle_leaves(k + 1, (int64_t)leaves, a);
 
-    const int64_t per_child = 8 * W_ + 12 + 12 + 16;
+    const int64_t per_child = 8 * Wc + 12 + 12 + 16;
     int64_t a0 = 0;
     while (total > 0 && a0 < N) {
         const int64_t cap = (int64_t)(arena_.avail() / 2) / per_child;
@@ -314,7 +331,8 @@ void Engine::process(int32_t k, const Level &L) {
         const size_t cmark = arena_.top;
         Level C;
         C.count = cnt;
-        C.P = arena_.alloc<uint64_t>(cnt * W_);
+        C.W = Wc;
+        C.P = arena_.alloc<uint64_t>(cnt * Wc);
         C.slot = arena_.alloc<int32_t>(cnt);
         C.parent = arena_.alloc<int32_t>(cnt);
         C.vloc = arena_.alloc<int32_t>(cnt);
@@ -397,7 +415,7 @@ void Engine::do_class_w1(const int32_t *list, int64_t count) {
             const int64_t leaves = (int64_t)hc[3];
             if (attempt == 0 && leaves > ra.leaf_cap && !find_one_) {
                 // staging too small for the size-2 leaves: grow and replay (counters reset)
-                int64_t want = leaves;
+                int64_t want = std::min<int64_t>(leaves, stage_max_rows_);
                 if (o_.max_cliques > 0) want = std::min<int64_t>(want, o_.max_cliques);
                 if (want > ra.leaf_cap) {
                     stage_rows_ = want;
@@ -418,7 +436,8 @@ void Engine::do_class_w1(const int32_t *list, int64_t count) {
             la.k = 1;
             la.leaf_rows = ra.leaf_rows;
             la.leaf_cap = ra.leaf_cap;
-            la.leaf_count = leaf_count_;
+            la.leaf_total = leaf_total_;
+            la.leaf_slot = leaf_slot_;
             handle_leaves(2, leaves, la);
         }
         const int64_t entries = (int64_t)hc[2];
@@ -430,6 +449,7 @@ void Engine::do_class_w1(const int32_t *list, int64_t count) {
             adj_ = ra.adj;
             Level L2;
             L2.count = entries;
+            L2.W = 1;
             L2.P = ra.cP;
             L2.slot = ra.cslot;
             L2.parent = ra.cparent;
@@ -485,6 +505,7 @@ void Engine::do_class(int32_t cls, const int32_t *list, int64_t count) {
         adj_ = adj;
         Level L1;
         L1.count = nw;
+        L1.W = W_;
         L1.P = arena_.alloc<uint64_t>(nw * W_);
         L1.slot = arena_.alloc<int32_t>(nw);
         L1.parent = arena_.alloc<int32_t>(nw);
@@ -560,8 +581,11 @@ mce_result *Engine::run() {
     // leaf counter + level chain (persistent, g->misc)
     chain_cap_ = 4096;
     g_->misc.ensure(256 + sizeof(LevelLink) * chain_cap_);
-    leaf_count_ = reinterpret_cast<unsigned long long *>(g_->misc.get());
+    leaf_total_ = reinterpret_cast<unsigned long long *>(g_->misc.get());
+    leaf_slot_ = leaf_total_ + 1;
+    maxbit_ = reinterpret_cast<int32_t *>(leaf_total_ + 2);
     chain_dev_ = reinterpret_cast<LevelLink *>(g_->misc.get() + 256);
+    stage_max_rows_ = std::max<int64_t>(1ll << 20, budget / 4 / (4ll * std::max<int32_t>(g_->max_out + 2, 2)));
     stage_rows_ = find_one_ ? 1 : 4096;
     g_->stage.ensure((size_t)stage_rows_ * std::max<int32_t>(g_->max_out + 2, 2));
 

@@ -50,7 +50,8 @@ __global__ void build_adj_w1(const RootInfo *__restrict__ roots, int64_t nroots,
                 const int32_t b = __ldg(V + c);
                 if (contains_sorted(ocol, __ldg(orp + b), __ldg(orp + b + 1), a)) row |= 1ull << c;
             }
-            adj[ri.abase + i] = row;
+            // local index = L-1-position (reverse degeneracy order, see expand.cuh)
+            adj[ri.abase + (ri.L - 1 - i)] = __brevll(row) >> (64 - ri.L);
         }
     }
 }
@@ -97,9 +98,10 @@ __global__ void build_adj_block(const RootInfo *__restrict__ roots, int64_t nroo
                         else
                             hi = mid;
                     }
-                    if (lo < L && sV[lo] == u) {
-                        atomicOr(A + (int64_t)i * 2 * W + (lo >> 5), 1u << (lo & 31));
-                        atomicOr(A + (int64_t)lo * 2 * W + (i >> 5), 1u << (i & 31));
+                    if (lo < L && sV[lo] == u) {  // local indices L-1-position (expand.cuh)
+                        const int li = L - 1 - i, lc = L - 1 - lo;
+                        atomicOr(A + (int64_t)li * 2 * W + (lc >> 5), 1u << (lc & 31));
+                        atomicOr(A + (int64_t)lc * 2 * W + (li >> 5), 1u << (li & 31));
                     }
                 }
             }
@@ -127,28 +129,59 @@ __global__ void init_level1_kernel(const RootInfo *__restrict__ roots, int64_t n
     }
 }
 
-__device__ void record_leaf(const ExpandArgs &a, int64_t e, int32_t v, const RootInfo &ri) {
-    const unsigned long long idx = atomicAdd(a.leaf_count, 1ull);
+// Store one leaf clique C + {v} of size k+1 (count pass).  Leaves are counted
+// by the caller (aggregated per warp); a staging slot is taken only while the
+// staging area has room, so a level with 10^8 maximum cliques does not
+// serialise on one counter.
+__device__ void store_leaf(const ExpandArgs &a, int64_t e, int32_t v, const RootInfo &ri) {
+    if (*(volatile unsigned long long *)a.leaf_slot >= (unsigned long long)a.leaf_cap) return;
+    const unsigned long long idx = atomicAdd(a.leaf_slot, 1ull);
     if ((int64_t)idx >= a.leaf_cap) return;
     const int32_t size = a.k + 1;
     int32_t *row = a.leaf_rows + (int64_t)idx * size;
     const int32_t *V = a.ocol + ri.vbase;
-    row[a.k] = a.order[V[v]];
+    row[a.k] = a.order[V[ri.L - 1 - v]];
     int64_t cur = e;
     for (int32_t lev = a.k; lev >= 2; --lev) {
-        row[lev - 1] = a.order[V[a.chain[lev].vloc[cur]]];
+        row[lev - 1] = a.order[V[ri.L - 1 - a.chain[lev].vloc[cur]]];
         cur = a.chain[lev].parent[cur];
     }
     row[0] = a.order[ri.r];
 }
 
+// highest set bit of a W-word set (-1 if empty)
+template <int W>
+__device__ __forceinline__ int top_bit(const uint64_t (&C)[W]) {
+    int hb = -1;
+#pragma unroll
+    for (int w = 0; w < W; ++w)
+        if (C[w]) hb = w * 64 + 63 - __clzll((long long)C[w]);
+    return hb;
+}
+
+// end-of-kernel reductions of the count pass: leaves (sum) and the highest
+// candidate bit of any surviving child (max) -> the children's word stride
+__device__ __forceinline__ void flush_counters(const ExpandArgs &a, unsigned long long nleaf, int hb) {
+    nleaf = __reduce_add_sync(0xffffffffu, (unsigned)nleaf) ;
+    hb = __reduce_max_sync(0xffffffffu, hb + 1) - 1;
+    if ((threadIdx.x & 31) == 0) {
+        if (nleaf) atomicAdd(a.leaf_total, nleaf);
+        if (hb >= 0) atomicMax(a.maxbit, hb);
+    }
+}
+
 // ---------------------------------------------------------------------------
-// thread per candidate, W <= 2 words (|V| <= 128): the sparse-graph workhorse
+// thread per candidate, W <= 4 words (|P| bits < 256): P, the running set R
+// and the child set C live in registers; the colouring order in local memory
 // ---------------------------------------------------------------------------
 template <int W, bool WRITE>
 __global__ void __launch_bounds__(256) expand_thread(const ExpandArgs a) {
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    for (int64_t e = a.begin + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < a.end; e += stride) {
+    unsigned nleaf = 0;
+    int hb = -1;
+    const int64_t e_end = a.begin + (a.end - a.begin + stride - 1) / stride * stride;  // warp-uniform trip count
+    for (int64_t e = a.begin + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < e_end; e += stride) {
+        if (e >= a.end) continue;
         int64_t out = 0;
         if (WRITE) {
             out = a.offsets[e];
@@ -160,6 +193,7 @@ __global__ void __launch_bounds__(256) expand_thread(const ExpandArgs a) {
         for (int w = 0; w < W; ++w) P[w] = a.P[e * W + w];
         const RootInfo ri = a.roots[a.slot[e]];
         const uint64_t *A = a.adj + ri.abase;
+        const int Wa = a.Wa;
         uint8_t ord[64 * W];
         uint8_t colr[64 * W];
         int np = 0;
@@ -182,7 +216,7 @@ __global__ void __launch_bounds__(256) expand_thread(const ExpandArgs a) {
                     while (Q[w]) {
                         const int b = __ffsll((long long)Q[w]) - 1;
                         const int v = w * 64 + b;
-                        const uint64_t *row = A + (int64_t)v * W;
+                        const uint64_t *row = A + (int64_t)v * Wa;
 #pragma unroll
                         for (int x = 0; x < W; ++x) Q[x] &= ~__ldg(row + x);
                         Q[w] &= ~(1ull << b);
@@ -215,7 +249,7 @@ __global__ void __launch_bounds__(256) expand_thread(const ExpandArgs a) {
             for (int i = np - 1; i >= 0; --i) {
                 if (a.k + colr[i] < a.need) break;
                 const int v = ord[i];
-                const uint64_t *row = A + (int64_t)v * W;
+                const uint64_t *row = A + (int64_t)v * Wa;
                 uint64_t C[W];
                 int pc = 0;
 #pragma unroll
@@ -225,15 +259,21 @@ __global__ void __launch_bounds__(256) expand_thread(const ExpandArgs a) {
                 }
                 R[v >> 6] &= ~(1ull << (v & 63));
                 if (pc == 0) {
-                    if (!WRITE && a.k + 1 >= a.need) record_leaf(a, e, v, ri);
+                    if (!WRITE && a.k + 1 >= a.need) {
+                        ++nleaf;
+                        store_leaf(a, e, v, ri);
+                    }
                 } else if (a.k + 1 + pc >= a.need) {
                     if (WRITE) {
                         const int64_t c = out + cnt;
 #pragma unroll
-                        for (int w = 0; w < W; ++w) a.cP[c * W + w] = C[w];
+                        for (int w = 0; w < W; ++w)
+                            if (w < a.Wc) a.cP[c * a.Wc + w] = C[w];
                         a.cslot[c] = a.slot[e];
                         a.cparent[c] = (int32_t)e;
                         a.cvloc[c] = v;
+                    } else {
+                        hb = max(hb, top_bit<W>(C));
                     }
                     ++cnt;
                 }
@@ -241,10 +281,11 @@ __global__ void __launch_bounds__(256) expand_thread(const ExpandArgs a) {
         }
         if (!WRITE) a.counts[e] = cnt;
     }
+    if (!WRITE) flush_counters(a, nleaf, hb);
 }
 
 // ---------------------------------------------------------------------------
-// warp per candidate, W >= 4 words: lanes own words (WPL words per lane)
+// warp per candidate, 4 < W <= 256 words: lanes own words (WPL words per lane)
 // ---------------------------------------------------------------------------
 template <int WPL, bool WRITE>
 __global__ void expand_warp(const ExpandArgs a, int max_l) {
@@ -255,7 +296,9 @@ __global__ void expand_warp(const ExpandArgs a, int max_l) {
     uint16_t *colr = ord + max_l;
     const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    const int W = a.W;
+    const int W = a.Wp, Wa = a.Wa;
+    unsigned nleaf = 0;
+    int hb = -1;
     for (int64_t e = a.begin + warp; e < a.end; e += nwarps) {
         int64_t out = 0;
         if (WRITE) {
@@ -299,7 +342,7 @@ __global__ void expand_warp(const ExpandArgs a, int max_l) {
                         }
                     }
                     if (v < 0) break;
-                    const uint64_t *row = A + (int64_t)v * W;
+                    const uint64_t *row = A + (int64_t)v * Wa;
 #pragma unroll
                     for (int t = 0; t < WPL; ++t) {
                         const int j = lane + 32 * t;
@@ -356,7 +399,7 @@ __global__ void expand_warp(const ExpandArgs a, int max_l) {
             for (int i = np - 1; i >= 0; --i) {
                 if (a.k + colr[i] < a.need) break;
                 const int v = ord[i];
-                const uint64_t *row = A + (int64_t)v * W;
+                const uint64_t *row = A + (int64_t)v * Wa;
                 uint64_t C[WPL];
                 int pc = 0;
 #pragma unroll
@@ -373,20 +416,27 @@ __global__ void expand_warp(const ExpandArgs a, int max_l) {
                         if (t == (jv >> 5)) R[t] &= ~(1ull << (v & 63));
                 }
                 if (pc == 0) {
-                    if (!WRITE && lane == 0 && a.k + 1 >= a.need) record_leaf(a, e, v, ri);
+                    if (!WRITE && a.k + 1 >= a.need && lane == 0) {
+                        ++nleaf;
+                        store_leaf(a, e, v, ri);
+                    }
                 } else if (a.k + 1 + pc >= a.need) {
                     if (WRITE) {
                         const int64_t c = out + cnt;
 #pragma unroll
                         for (int t = 0; t < WPL; ++t) {
                             const int j = lane + 32 * t;
-                            if (j < W) a.cP[c * W + j] = C[t];
+                            if (j < a.Wc) a.cP[c * a.Wc + j] = C[t];
                         }
                         if (lane == 0) {
                             a.cslot[c] = a.slot[e];
                             a.cparent[c] = (int32_t)e;
                             a.cvloc[c] = v;
                         }
+                    } else {
+#pragma unroll
+                        for (int t = 0; t < WPL; ++t)
+                            if (C[t]) hb = max(hb, (lane + 32 * t) * 64 + 63 - __clzll((long long)C[t]));
                     }
                     ++cnt;
                 }
@@ -395,10 +445,9 @@ __global__ void expand_warp(const ExpandArgs a, int max_l) {
         if (!WRITE && lane == 0) a.counts[e] = cnt;
         __syncwarp();
     }
+    if (!WRITE) flush_counters(a, nleaf, hb);
 }
 
-// cls[r] = width class of root r (-1: cannot reach `need`), hist[c] += 1
-// (hist[kMaxClass] counts roots too wide for the kernels: reported by the host)
 __global__ void classify_roots_kernel(int64_t n, const int64_t *__restrict__ orp, int32_t min_len, int32_t *cls,
                                       unsigned long long *hist) {
     __shared__ unsigned int h[kMaxClass + 1];
@@ -489,7 +538,7 @@ __global__ void find_window_kernel(const int64_t *__restrict__ prefix, int64_t h
 
 template <int WPL>
 void launch_warp(const ExpandArgs &a, bool write_pass, cudaStream_t s) {
-    const int max_l = 64 * a.W;
+    const int max_l = 64 * a.Wp;
     const int warps = WPL >= 4 ? 1 : (WPL == 2 ? 2 : 4);
     const size_t smem = (size_t)warps * 2 * max_l * sizeof(uint16_t);
     const int64_t items = a.end - a.begin;
@@ -541,28 +590,30 @@ void launch_init_level1(const RootInfo *roots, int64_t nroots, int W, uint64_t *
     MCE_LAUNCH_CHECK();
 }
 
+template <int W>
+void launch_thread(const ExpandArgs &a, bool write_pass, cudaStream_t s) {
+    const int grid = grid_for(a.end - a.begin, 256, 8);
+    if (write_pass)
+        expand_thread<W, true><<<grid, 256, 0, s>>>(a);
+    else
+        expand_thread<W, false><<<grid, 256, 0, s>>>(a);
+    MCE_LAUNCH_CHECK();
+}
+
 void launch_expand(const ExpandArgs &a, bool write_pass, cudaStream_t s) {
     const int64_t items = a.end - a.begin;
     if (items <= 0) return;
-    if (a.W == 1 || a.W == 2) {
-        const int grid = grid_for(items, 256, 8);
-        if (a.W == 1) {
-            if (write_pass)
-                expand_thread<1, true><<<grid, 256, 0, s>>>(a);
-            else
-                expand_thread<1, false><<<grid, 256, 0, s>>>(a);
-        } else {
-            if (write_pass)
-                expand_thread<2, true><<<grid, 256, 0, s>>>(a);
-            else
-                expand_thread<2, false><<<grid, 256, 0, s>>>(a);
-        }
-        MCE_LAUNCH_CHECK();
-    } else if (a.W <= 32) {
+    if (a.Wp == 1) {
+        launch_thread<1>(a, write_pass, s);
+    } else if (a.Wp == 2) {
+        launch_thread<2>(a, write_pass, s);
+    } else if (a.Wp == 4) {
+        launch_thread<4>(a, write_pass, s);
+    } else if (a.Wp <= 32) {
         launch_warp<1>(a, write_pass, s);
-    } else if (a.W <= 64) {
+    } else if (a.Wp <= 64) {
         launch_warp<2>(a, write_pass, s);
-    } else if (a.W <= 128) {
+    } else if (a.Wp <= 128) {
         launch_warp<4>(a, write_pass, s);
     } else {
         launch_warp<8>(a, write_pass, s);

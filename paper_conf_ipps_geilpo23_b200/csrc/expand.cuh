@@ -6,7 +6,13 @@
 namespace mce {
 
 // One root of the current window.  Its candidate space is V = the root's
-// out-neighbours (oriented CSR row, ranks ascending); local index i <-> V[i].
+// out-neighbours (oriented CSR row, ranks ascending); local index i <-> V[L-1-i],
+// i.e. bit order is REVERSE degeneracy order.  The colouring bound colours P
+// in bit order and branches from the highest colour down (Tomita-Seki MCQ), so
+// the high-core vertices get the low colours and are branched last, with the
+// smallest candidate sets (the "smallest-last" initial order of Matula-Beck,
+// DESIGN.md reading 5).  In ascending rank order the hub vertices took the
+// highest colours and the R-MAT searches exploded.
 struct RootInfo {
     int32_t r;      // rank of the root
     int32_t L;      // |V| = out-degree
@@ -32,7 +38,9 @@ struct ExpandArgs {
     int32_t k;           // |C|
     int32_t need;        // smallest clique size still of interest
     int32_t bound;       // 0: |C|+|P|, 1: colouring
-    int32_t W;           // words per candidate set (runtime, warp kernels)
+    int32_t Wp;          // words per candidate set of this level (its P stride; 1, 2, 4, 8, ...)
+    int32_t Wa;          // words per adjacency row of the root window (>= Wp)
+    int32_t Wc;          // write pass: words per child candidate set (<= Wp, from *maxbit)
     const RootInfo *roots;
     const uint64_t *adj;
     const int32_t *ocol;
@@ -46,8 +54,11 @@ struct ExpandArgs {
     int32_t *cslot;
     int32_t *cparent;
     int32_t *cvloc;
-    // leaves of size k+1 (count pass only)
-    unsigned long long *leaf_count;
+    // count pass: highest candidate bit of any surviving child (atomicMax)
+    int32_t *maxbit;
+    // leaves of size k+1 (count pass only): total (exact) and staged rows
+    unsigned long long *leaf_total;
+    unsigned long long *leaf_slot;
     int32_t *leaf_rows;
     int64_t leaf_cap;  // rows
     const LevelLink *chain;  // chain[1..k]

@@ -38,58 +38,95 @@ __device__ __forceinline__ unsigned long long pick_key(const int32_t *__restrict
     return ((unsigned long long)(uint32_t)__ldg(thr + x) << 32) | (unsigned long long)(0x7fffffffu - (uint32_t)x);
 }
 
-// One greedy run for seed s by the calling warp.  Writes the clique (in order
-// added) to `clique` when non-null.  Returns the clique size.
+// One greedy run for seed s by a tile of G lanes (G = 8 or 32) of the calling
+// warp.  Writes the clique (in order added) to `clique` when non-null.
+// Returns the clique size.
+template <int G>
 __device__ int32_t greedy_run(int32_t s, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
                               const int32_t *__restrict__ thr, int32_t *__restrict__ scratch, int32_t *clique) {
     const int lane = threadIdx.x & 31;
+    const int gl = lane & (G - 1);
+    const int gbase = lane & ~(G - 1);
+    const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << gbase);
     const int64_t base = rowptr[s];
     int64_t len = rowptr[s + 1] - base;
     const int32_t *src = col + base;  // first round reads the CSR row directly
     int32_t *buf = scratch + base;    // later rounds work in place in the seed's segment
     int32_t csize = 1;
-    if (clique && lane == 0) clique[0] = s;
+    if (clique && gl == 0) clique[0] = s;
     while (len > 0) {
         unsigned long long key = 0;
-        for (int64_t i = lane; i < len; i += 32) {
+        for (int64_t i = gl; i < len; i += G) {
             unsigned long long k2 = pick_key(thr, src[i]);
             key = k2 > key ? k2 : key;
         }
-        key = warp_max_u64(key);
+#pragma unroll
+        for (int o = G / 2; o > 0; o >>= 1) {
+            unsigned long long y = __shfl_xor_sync(gmask, key, o, G);
+            key = y > key ? y : key;
+        }
         const int32_t w = (int32_t)(0x7fffffffu - (uint32_t)(key & 0xffffffffull));
-        if (clique && lane == 0) clique[csize] = w;
+        if (clique && gl == 0) clique[csize] = w;
         ++csize;
         const int64_t wb = rowptr[w], we = rowptr[w + 1];
         int64_t out = 0;
-        for (int64_t i0 = 0; i0 < len; i0 += 32) {
-            int64_t i = i0 + lane;
+        for (int64_t i0 = 0; i0 < len; i0 += G) {
+            int64_t i = i0 + gl;
             int32_t x = i < len ? src[i] : -1;
             bool keep = i < len && x != w && contains_sorted(col, wb, we, x);
-            unsigned m = __ballot_sync(0xffffffffu, keep);
-            if (keep) buf[out + __popc(m & lanemask_lt())] = x;
+            const unsigned m = (__ballot_sync(gmask, keep) & gmask) >> gbase;
+            if (keep) buf[out + __popc(m & ((1u << gl) - 1u))] = x;
             out += __popc(m);
         }
-        __syncwarp();
+        __syncwarp(gmask);
         src = buf;
         len = out;
     }
     return csize;
 }
 
-__global__ void greedy_kernel(int64_t nseeds, const int32_t *__restrict__ seeds, const int64_t *__restrict__ rowptr,
-                              const int32_t *__restrict__ col, const int32_t *__restrict__ thr,
-                              int32_t *__restrict__ scratch, int32_t *__restrict__ run_size, int32_t *best_size) {
+// Warp w takes seeds [4w, 4w+4): when all four have degree <= 64 they run in
+// parallel on 8-lane tiles (low-degree seeds leave most of a warp idle),
+// otherwise one after another on the whole warp.  The best size is reduced
+// per block before one atomicMax per block.
+__global__ void __launch_bounds__(256) greedy_kernel(int64_t nseeds, const int32_t *__restrict__ seeds,
+                                                     const int64_t *__restrict__ rowptr,
+                                                     const int32_t *__restrict__ col, const int32_t *__restrict__ thr,
+                                                     int32_t *__restrict__ scratch, int32_t *__restrict__ run_size,
+                                                     int32_t *best_size) {
+    __shared__ int32_t block_best;
+    if (threadIdx.x == 0) block_best = 0;
+    __syncthreads();
     const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     const int lane = threadIdx.x & 31;
-    for (int64_t i = warp; i < nseeds; i += nwarps) {
-        int32_t s = seeds[i];
-        int32_t c = greedy_run(s, rowptr, col, thr, scratch, nullptr);
-        if (lane == 0) {
-            run_size[s] = c;
-            atomicMax(best_size, c);
+    int32_t mybest = 0;
+    for (int64_t i0 = warp * 4; i0 < nseeds; i0 += nwarps * 4) {
+        const int64_t my = i0 + (lane >> 3);
+        const int32_t s_mine = my < nseeds ? seeds[my] : -1;
+        const int64_t d_mine = s_mine >= 0 ? rowptr[s_mine + 1] - rowptr[s_mine] : 0;
+        const bool small = __all_sync(0xffffffffu, d_mine <= 64);
+        if (small) {
+            if (s_mine >= 0) {
+                const int32_t c = greedy_run<8>(s_mine, rowptr, col, thr, scratch, nullptr);
+                if ((lane & 7) == 0) run_size[s_mine] = c;
+                mybest = max(mybest, c);
+            }
+        } else {
+            for (int t = 0; t < 4; ++t) {
+                const int32_t s = __shfl_sync(0xffffffffu, s_mine, 8 * t);
+                if (s < 0) break;
+                const int32_t c = greedy_run<32>(s, rowptr, col, thr, scratch, nullptr);
+                if (lane == 0) run_size[s] = c;
+                mybest = max(mybest, c);
+            }
         }
+        __syncwarp();
     }
+    mybest = __reduce_max_sync(0xffffffffu, mybest);
+    if (lane == 0 && mybest) atomicMax(&block_best, mybest);
+    __syncthreads();
+    if (threadIdx.x == 0 && block_best) atomicMax(best_size, block_best);
 }
 
 // among seeds whose run reached best, the first in seed order (threshold desc, id asc)
@@ -102,11 +139,67 @@ __global__ void best_seed_kernel(int64_t nseeds, const int32_t *__restrict__ see
     }
 }
 
-__global__ void replay_kernel(const unsigned long long *best_key, const int64_t *__restrict__ rowptr,
-                              const int32_t *__restrict__ col, const int32_t *__restrict__ thr,
-                              int32_t *__restrict__ scratch, int32_t *clique) {
-    int32_t s = (int32_t)(0x7fffffffu - (uint32_t)(*best_key & 0xffffffffull));
-    greedy_run(s, rowptr, col, thr, scratch, clique);
+// Replay of the winning run to recover its clique: the same greedy steps as
+// greedy_run, by one block of kReplay threads (block-wide argmax and an
+// order-preserving in-place compaction), since a single run on a hub seed is
+// long and nothing else is running.
+constexpr int kReplay = 1024;
+__global__ void __launch_bounds__(kReplay) replay_kernel(const unsigned long long *best_key,
+                                                         const int64_t *__restrict__ rowptr,
+                                                         const int32_t *__restrict__ col,
+                                                         const int32_t *__restrict__ thr,
+                                                         int32_t *__restrict__ scratch, int32_t *clique) {
+    __shared__ unsigned long long wkey[kReplay / 32];
+    __shared__ int32_t wcnt[kReplay / 32];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int32_t s = (int32_t)(0x7fffffffu - (uint32_t)(*best_key & 0xffffffffull));
+    const int64_t base = rowptr[s];
+    int64_t len = rowptr[s + 1] - base;
+    const int32_t *src = col + base;
+    int32_t *buf = scratch + base;
+    int32_t csize = 1;
+    if (threadIdx.x == 0) clique[0] = s;
+    while (len > 0) {
+        unsigned long long key = 0;
+        for (int64_t i = threadIdx.x; i < len; i += kReplay) {
+            const unsigned long long k2 = pick_key(thr, src[i]);
+            key = k2 > key ? k2 : key;
+        }
+        key = warp_max_u64(key);
+        if (lane == 0) wkey[wid] = key;
+        __syncthreads();
+        if (wid == 0) {
+            key = warp_max_u64(wkey[lane]);
+            if (lane == 0) wkey[0] = key;
+        }
+        __syncthreads();
+        key = wkey[0];
+        const int32_t w = (int32_t)(0x7fffffffu - (uint32_t)(key & 0xffffffffull));
+        if (threadIdx.x == 0) clique[csize] = w;
+        ++csize;
+        const int64_t wb = rowptr[w], we = rowptr[w + 1];
+        int64_t out = 0;
+        for (int64_t i0 = 0; i0 < len; i0 += kReplay) {
+            const int64_t i = i0 + threadIdx.x;
+            const int32_t x = i < len ? src[i] : -1;
+            const bool keep = i < len && x != w && contains_sorted(col, wb, we, x);
+            const unsigned m = __ballot_sync(0xffffffffu, keep);
+            __syncthreads();  // wkey/wcnt reuse, and every read of this chunk precedes its writes
+            if (lane == 0) wcnt[wid] = __popc(m);
+            __syncthreads();
+            int32_t before = 0, total = 0;
+            for (int j = 0; j < kReplay / 32; ++j) {
+                const int32_t c = wcnt[j];
+                before += j < wid ? c : 0;
+                total += c;
+            }
+            if (keep) buf[out + before + __popc(m & lanemask_lt())] = x;
+            out += total;
+        }
+        __syncthreads();
+        src = buf;
+        len = out;
+    }
 }
 
 __global__ void degree_thr_kernel(int64_t n, const int64_t *__restrict__ rowptr, int32_t *thr) {
@@ -240,12 +333,12 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
     MCE_CUDA(cudaMemsetAsync(best, 0, sizeof(int32_t), s));
     MCE_CUDA(cudaMemsetAsync(best_key, 0, sizeof(unsigned long long), s));
     if (nseeds > 0) {
-        greedy_kernel<<<grid_for(nseeds * 32, 256), 256, 0, s>>>(nseeds, seed_ptr, g->rowptr.get(), g->col.get(),
+        greedy_kernel<<<grid_for(nseeds * 8, 256), 256, 0, s>>>(nseeds, seed_ptr, g->rowptr.get(), g->col.get(),
                                                                   thr, scratch, run_size, best);
         MCE_LAUNCH_CHECK();
         best_seed_kernel<<<grid_for(nseeds, 256), 256, 0, s>>>(nseeds, seed_ptr, thr, run_size, best, best_key);
         MCE_LAUNCH_CHECK();
-        replay_kernel<<<1, 32, 0, s>>>(best_key, g->rowptr.get(), g->col.get(), thr, scratch, clique);
+        replay_kernel<<<1, kReplay, 0, s>>>(best_key, g->rowptr.get(), g->col.get(), thr, scratch, clique);
         MCE_LAUNCH_CHECK();
         kernels += 3;
     }

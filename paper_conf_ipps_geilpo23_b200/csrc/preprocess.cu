@@ -44,6 +44,39 @@ __device__ __forceinline__ unsigned long long warp_append(unsigned long long *ct
     return __shfl_sync(0xffffffffu, base, 0);
 }
 
+// cascade step for one queued vertex v by a tile of G lanes: decrement the
+// alive neighbours, queue those that fall to k (one atomicAdd per tile chunk)
+template <int G>
+__device__ __forceinline__ void peel_neighbours(int32_t v, const int64_t *__restrict__ rowptr,
+                                                const int32_t *__restrict__ col, int32_t *deg, int32_t *core,
+                                                int32_t *queue, uint8_t *dead, unsigned long long *qcnt,
+                                                int64_t region_end, int32_t k) {
+    const int lane = threadIdx.x & 31;
+    const int gl = lane & (G - 1), gbase = lane & ~(G - 1);
+    const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << gbase);
+    const int64_t eb = rowptr[v], ee = rowptr[v + 1];
+    for (int64_t e0 = eb; e0 < ee; e0 += G) {
+        const int64_t e = e0 + gl;
+        bool fell = false;
+        int32_t u = -1;
+        if (e < ee) {
+            u = col[e];
+            if (!dead[u]) fell = atomicSub(deg + u, 1) == k + 1;
+        }
+        const unsigned fm = (__ballot_sync(gmask, fell) & gmask) >> gbase;
+        if (fm) {
+            unsigned long long b = 0;
+            if (gl == 0) b = atomicAdd(qcnt, (unsigned long long)__popc(fm));
+            b = __shfl_sync(gmask, b, 0, G);
+            if (fell) {
+                queue[region_end + b + __popc(fm & ((1u << gl) - 1u))] = u;
+                core[u] = k;
+                dead[u] = 1;
+            }
+        }
+    }
+}
+
 __global__ void __launch_bounds__(kPeelThreads)
     kcore_peel(int64_t n, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col, int32_t *deg,
                int32_t *core, int32_t *queue, int32_t *alive_a, int32_t *alive_b, uint8_t *dead,
@@ -102,27 +135,21 @@ __global__ void __launch_bounds__(kPeelThreads)
             dmin = __reduce_min_sync(0xffffffffu, dmin);
             if (lane == 0 && dmin != INT32_MAX) atomicMin(mind, (unsigned long long)dmin);
         } else {
-            for (int64_t qi = head + warp; qi < region_end; qi += nwarps) {
-                const int32_t v = queue[qi];
-                const int64_t eb = rowptr[v], ee = rowptr[v + 1];
-                for (int64_t e0 = eb; e0 < ee; e0 += 32) {
-                    const int64_t e = e0 + lane;
-                    bool fell = false;
-                    int32_t u = -1;
-                    if (e < ee) {
-                        u = col[e];
-                        if (!dead[u]) fell = atomicSub(deg + u, 1) == k + 1;
-                    }
-                    const unsigned fm = __ballot_sync(0xffffffffu, fell);
-                    if (fm) {
-                        const unsigned long long b = warp_append(qcnt, fm, lane);
-                        if (fell) {
-                            queue[region_end + b + __popc(fm & lt)] = u;
-                            core[u] = k;
-                            dead[u] = 1;
-                        }
+            // warp takes four queued vertices: 8-lane tiles when all have degree <= 64
+            for (int64_t q0 = head + warp * 4; q0 < region_end; q0 += nwarps * 4) {
+                const int64_t qi = q0 + (lane >> 3);
+                const int32_t v = qi < region_end ? queue[qi] : -1;
+                const int64_t d = v >= 0 ? rowptr[v + 1] - rowptr[v] : 0;
+                if (__all_sync(0xffffffffu, d <= 64)) {
+                    if (v >= 0) peel_neighbours<8>(v, rowptr, col, deg, core, queue, dead, qcnt, region_end, k);
+                } else {
+                    for (int t = 0; t < 4; ++t) {
+                        const int32_t vt = __shfl_sync(0xffffffffu, v, 8 * t);
+                        if (vt < 0) break;
+                        peel_neighbours<32>(vt, rowptr, col, deg, core, queue, dead, qcnt, region_end, k);
                     }
                 }
+                __syncwarp();
             }
         }
         grid.sync();
@@ -180,55 +207,98 @@ __global__ void degree_scatter(int64_t n, const int64_t *__restrict__ rowptr, un
     }
 }
 
-// out-degree of every rank: warp per vertex, ballot over neighbour chunks
-__global__ void out_degree_kernel(int64_t n, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
-                                  const int32_t *__restrict__ rank, int32_t *odeg) {
-    const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    const int lane = threadIdx.x & 31;
-    for (int64_t v = warp; v < n; v += nwarps) {
-        const int32_t r = rank[v];
-        int32_t cnt = 0;
-        for (int64_t e0 = rowptr[v]; e0 < rowptr[v + 1]; e0 += 32) {
-            int64_t e = e0 + lane;
-            bool up = e < rowptr[v + 1] && rank[col[e]] > r;
-            cnt += __popc(__ballot_sync(0xffffffffu, up));
-        }
-        if (lane == 0) odeg[r] = cnt;
+// Tile of G lanes (8 or 32) inside a warp: lane index, first lane, member mask.
+template <int G>
+struct Tile {
+    int gl, gbase;
+    unsigned mask;
+    __device__ Tile() {
+        const int lane = threadIdx.x & 31;
+        gl = lane & (G - 1);
+        gbase = lane & ~(G - 1);
+        mask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << gbase);
+    }
+    __device__ unsigned ballot(bool p) const { return (__ballot_sync(mask, p) & mask) >> gbase; }
+    __device__ unsigned lt() const { return (1u << gl) - 1u; }
+};
+
+// out-degree of vertex v's rank (tile of G lanes over v's neighbours)
+template <int G>
+__device__ void out_degree_one(int64_t v, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
+                               const int32_t *__restrict__ rank, int32_t *odeg) {
+    Tile<G> t;
+    const int32_t r = rank[v];
+    int32_t cnt = 0;
+    const int64_t eb = rowptr[v], ee = rowptr[v + 1];
+    for (int64_t e0 = eb; e0 < ee; e0 += G) {
+        const int64_t e = e0 + t.gl;
+        cnt += __popc(t.ballot(e < ee && rank[col[e]] > r));
+    }
+    if (t.gl == 0) odeg[r] = cnt;
+}
+
+// oriented row of v (in CSR order of the source; sorted afterwards)
+template <int G>
+__device__ void orient_fill_one(int64_t v, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
+                                const int32_t *__restrict__ rank, const int64_t *__restrict__ orp, int32_t *ocol) {
+    Tile<G> t;
+    const int32_t r = rank[v];
+    int64_t out = orp[r];
+    const int64_t eb = rowptr[v], ee = rowptr[v + 1];
+    for (int64_t e0 = eb; e0 < ee; e0 += G) {
+        const int64_t e = e0 + t.gl;
+        const int32_t ru = e < ee ? rank[col[e]] : -1;
+        const bool up = ru > r;
+        const unsigned m = t.ballot(up);
+        if (up) ocol[out + __popc(m & t.lt())] = ru;
+        out += __popc(m);
     }
 }
 
-// fill the oriented rows (in CSR order of the source; sorted afterwards)
-__global__ void orient_fill_kernel(int64_t n, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
-                                   const int32_t *__restrict__ rank, const int64_t *__restrict__ orp,
-                                   int32_t *ocol) {
+// Warp w takes vertices [4w, 4w+4): 8-lane tiles when all four have degree
+// <= 64 (sparse graphs: a warp per vertex would leave most lanes idle),
+// otherwise one vertex after another on the whole warp.
+template <bool FILL>
+__global__ void __launch_bounds__(256) orient_kernel(int64_t n, const int64_t *__restrict__ rowptr,
+                                                     const int32_t *__restrict__ col, const int32_t *__restrict__ rank,
+                                                     int32_t *odeg, const int64_t *__restrict__ orp, int32_t *ocol) {
     const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     const int lane = threadIdx.x & 31;
-    for (int64_t v = warp; v < n; v += nwarps) {
-        const int32_t r = rank[v];
-        int64_t out = orp[r];
-        for (int64_t e0 = rowptr[v]; e0 < rowptr[v + 1]; e0 += 32) {
-            int64_t e = e0 + lane;
-            int32_t ru = e < rowptr[v + 1] ? rank[col[e]] : -1;
-            bool up = ru > r;
-            unsigned m = __ballot_sync(0xffffffffu, up);
-            if (up) ocol[out + __popc(m & lanemask_lt())] = ru;
-            out += __popc(m);
+    for (int64_t v0 = warp * 4; v0 < n; v0 += nwarps * 4) {
+        const int64_t v = v0 + (lane >> 3);
+        const int64_t d = v < n ? rowptr[v + 1] - rowptr[v] : 0;
+        if (__all_sync(0xffffffffu, d <= 64)) {
+            if (v < n) {
+                if (FILL)
+                    orient_fill_one<8>(v, rowptr, col, rank, orp, ocol);
+                else
+                    out_degree_one<8>(v, rowptr, col, rank, odeg);
+            }
+        } else {
+            for (int t = 0; t < 4 && v0 + t < n; ++t) {
+                if (FILL)
+                    orient_fill_one<32>(v0 + t, rowptr, col, rank, orp, ocol);
+                else
+                    out_degree_one<32>(v0 + t, rowptr, col, rank, odeg);
+            }
         }
+        __syncwarp();
     }
 }
 
 // ---- row sorts (rows of the oriented CSR) ----
-__device__ __forceinline__ int32_t warp_bitonic_sort(int32_t x) {
-    const int lane = threadIdx.x & 31;
+// bitonic sort of G values held one per lane of a G-lane tile (ascending)
+template <int G>
+__device__ __forceinline__ int32_t tile_bitonic_sort(int32_t x, unsigned mask) {
+    const int gl = threadIdx.x & (G - 1);
 #pragma unroll
-    for (int size = 2; size <= 32; size <<= 1) {
+    for (int size = 2; size <= G; size <<= 1) {
 #pragma unroll
         for (int stride = size >> 1; stride > 0; stride >>= 1) {
-            int32_t y = __shfl_xor_sync(0xffffffffu, x, stride);
-            bool up = ((lane & size) == 0);
-            bool lower = ((lane & stride) == 0);
+            int32_t y = __shfl_xor_sync(mask, x, stride, G);
+            bool up = ((gl & size) == 0);
+            bool lower = ((gl & stride) == 0);
             int32_t lo = min(x, y), hi = max(x, y);
             x = (lower == up) ? lo : hi;
         }
@@ -236,16 +306,30 @@ __device__ __forceinline__ int32_t warp_bitonic_sort(int32_t x) {
     return x;
 }
 
-__global__ void sort_rows_warp(int64_t n, const int64_t *__restrict__ orp, int32_t *ocol) {
+// rows of length <= 32: 8-lane tiles for four rows of length <= 8, else a warp per row
+__global__ void __launch_bounds__(256) sort_rows_warp(int64_t n, const int64_t *__restrict__ orp, int32_t *ocol) {
     const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     const int lane = threadIdx.x & 31;
-    for (int64_t r = warp; r < n; r += nwarps) {
-        int64_t b = orp[r], len = orp[r + 1] - b;
-        if (len <= 1 || len > 32) continue;
-        int32_t x = lane < len ? ocol[b + lane] : INT32_MAX;
-        x = warp_bitonic_sort(x);
-        if (lane < len) ocol[b + lane] = x;
+    for (int64_t r0 = warp * 4; r0 < n; r0 += nwarps * 4) {
+        const int64_t r = r0 + (lane >> 3);
+        const int64_t b = r < n ? orp[r] : 0, len = r < n ? orp[r + 1] - b : 0;
+        if (__all_sync(0xffffffffu, len <= 8)) {
+            Tile<8> t;
+            int32_t x = t.gl < len ? ocol[b + t.gl] : INT32_MAX;
+            x = tile_bitonic_sort<8>(x, t.mask);
+            if (t.gl < len && len > 1) ocol[b + t.gl] = x;
+        } else {
+            for (int q = 0; q < 4; ++q) {
+                const int64_t bb = __shfl_sync(0xffffffffu, b, 8 * q);
+                const int64_t ll = __shfl_sync(0xffffffffu, len, 8 * q);
+                if (ll <= 1 || ll > 32) continue;
+                int32_t x = lane < ll ? ocol[bb + lane] : INT32_MAX;
+                x = tile_bitonic_sort<32>(x, 0xffffffffu);
+                if (lane < ll) ocol[bb + lane] = x;
+            }
+        }
+        __syncwarp();
     }
 }
 
@@ -396,13 +480,14 @@ void orient(mce_graph *g, int orientation) {
     invert_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->order.get(), g->rank.get());
     MCE_LAUNCH_CHECK();
     int32_t *odeg = g->pool.take<int32_t>(n);
-    out_degree_kernel<<<grid_for(n * 32, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), g->rank.get(), odeg);
+    orient_kernel<false><<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), g->rank.get(), odeg,
+                                                               nullptr, nullptr);
     MCE_LAUNCH_CHECK();
     exclusive_scan_i32(odeg, g->orp.get(), n, g->pool.take<int64_t>(scan_tmp_items(n)), s);
-    orient_fill_kernel<<<grid_for(n * 32, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), g->rank.get(),
-                                                             g->orp.get(), g->ocol.get());
+    orient_kernel<true><<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), g->rank.get(),
+                                                              nullptr, g->orp.get(), g->ocol.get());
     MCE_LAUNCH_CHECK();
-    sort_rows_warp<<<grid_for(n * 32, 256), 256, 0, s>>>(n, g->orp.get(), g->ocol.get());
+    sort_rows_warp<<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->orp.get(), g->ocol.get());
     MCE_LAUNCH_CHECK();
     int32_t *rows = g->pool.take<int32_t>(n), *meta = g->pool.take<int32_t>(2);
     MCE_CUDA(cudaMemsetAsync(meta, 0, 2 * sizeof(int32_t), s));

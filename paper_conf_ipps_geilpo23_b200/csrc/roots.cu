@@ -4,7 +4,8 @@
 // out-neighbours under the orientation) and IV-D / Algorithm 2 expands it.
 // Here the whole first expansion step of a root r runs inside one warp:
 //
-//   1. V = N+(r) (|V| = L <= 64) is staged in shared memory;
+//   1. V = N+(r) (|V| = L <= 64) is staged in shared memory (rank order;
+//      local index = L-1-position, the reverse degeneracy order of expand.cuh);
 //   2. the induced adjacency of V is built by a flattened, warp-cooperative
 //      sorted-list intersection: the out-rows N+(v) of every v in V are read
 //      32 elements at a time (coalesced within a row), each lane binary-searches
@@ -116,9 +117,10 @@ __global__ void __launch_bounds__(kRootWarps * 32) root_expand_w1(const RootArgs
                 }
                 const int32_t u = __ldg(a.ocol + sm.start[lo] + (t - sm.off[lo]));
                 const int c = lower_bound_smem(sm.V, L, u);
-                if (c < L && sm.V[c] == u) {
-                    atomicOr(&sm.adj[lo][c >> 5], 1u << (c & 31));
-                    atomicOr(&sm.adj[c][lo >> 5], 1u << (lo & 31));
+                if (c < L && sm.V[c] == u) {  // local indices L-1-position (expand.cuh)
+                    const int li = L - 1 - lo, lc = L - 1 - c;
+                    atomicOr(&sm.adj[li][lc >> 5], 1u << (lc & 31));
+                    atomicOr(&sm.adj[lc][li >> 5], 1u << (li & 31));
                 }
             }
         }
@@ -173,7 +175,7 @@ __global__ void __launch_bounds__(kRootWarps * 32) root_expand_w1(const RootArgs
                         const unsigned long long idx = atomicAdd(a.ctr + 3, 1ull);
                         if ((int64_t)idx < a.leaf_cap) {
                             a.leaf_rows[idx * 2] = __ldg(a.order + r);
-                            a.leaf_rows[idx * 2 + 1] = __ldg(a.order + sm.V[v]);
+                            a.leaf_rows[idx * 2 + 1] = __ldg(a.order + sm.V[L - 1 - v]);
                         }
                     }
                 } else if (2 + pc >= a.need) {
