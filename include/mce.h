@@ -162,6 +162,12 @@ mce_status mce_result_levels(const mce_result *r, int64_t *entries, int32_t cap,
 mce_status mce_result_timing(const mce_result *r, double *t, int32_t cap);
 void mce_result_free(mce_result *r);
 
+/* Device memory freed by the library (graph handles, regrown workspaces) is
+ * cached per device and reused by later calls, so a new graph or a new call
+ * does not pay cudaMalloc/cudaFree.  This returns the cached blocks of
+ * `device` to the driver.  MCE_ERR_INVALID for a bad device index. */
+mce_status mce_empty_cache(int32_t device);
+
 const char *mce_last_error(void);
 const char *mce_version(void);
 

@@ -65,7 +65,7 @@ def build(force: bool = False, jobs: int = 8) -> str:
 EXPORTS = [
     "mce_default_options", "mce_load_csr", "mce_graph_free", "mce_graph_clear_cache", "mce_preprocess", "mce_heuristic", "mce_enumerate",
     "mce_find_one", "mce_result_info", "mce_result_cliques", "mce_result_levels", "mce_result_timing",
-    "mce_result_free", "mce_last_error", "mce_version",
+    "mce_result_free", "mce_empty_cache", "mce_last_error", "mce_version",
 ]
 
 _lib = None
@@ -108,6 +108,8 @@ def lib():
     L.mce_result_timing.argtypes = [vp, ctypes.POINTER(ctypes.c_double), i32]
     L.mce_result_free.restype = None
     L.mce_result_free.argtypes = [vp]
+    L.mce_empty_cache.restype = i32
+    L.mce_empty_cache.argtypes = [i32]
     L.mce_last_error.restype = ctypes.c_char_p
     L.mce_last_error.argtypes = []
     L.mce_version.restype = ctypes.c_char_p

@@ -174,5 +174,10 @@ class Graph:
         return self._result(h)
 
 
+def empty_cache(device: int = 0) -> None:
+    """Return the library's cached device memory of `device` to the driver (mce_empty_cache)."""
+    check(lib().mce_empty_cache(int(device)))
+
+
 def version() -> str:
     return lib().mce_version().decode()

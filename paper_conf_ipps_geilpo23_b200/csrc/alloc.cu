@@ -1,0 +1,131 @@
+// Per-device caching allocator and pinned staging (see common.cuh).
+//
+// Safety: a block is handed back to the cache only when no kernel can still
+// touch it.  Every public call of the library synchronises its stream before
+// returning, and the internal frees (Pool::reset at the start of a phase, a
+// workspace regrow) happen after such a synchronisation, so a cached block is
+// never reused while in flight, whichever stream the next user runs on.
+#include <map>
+#include <mutex>
+#include <unordered_map>
+
+#include "common.cuh"
+#include "mce.h"
+
+namespace mce {
+
+namespace {
+
+struct DeviceCache {
+    std::multimap<size_t, void *> free_blocks;  // rounded size -> block
+    size_t cached = 0;
+    void *pinned = nullptr;
+    size_t pinned_bytes = 0;
+};
+
+std::mutex g_mu;
+std::unordered_map<int, DeviceCache> g_cache;
+
+int current_device() {
+    int d = 0;
+    MCE_CUDA(cudaGetDevice(&d));
+    return d;
+}
+
+size_t round_size(size_t bytes) {
+    if (bytes <= (1u << 20)) return (bytes + 4095) / 4096 * 4096;
+    return (bytes + (2u << 20) - 1) / (2u << 20) * (2u << 20);
+}
+
+void release_all(DeviceCache &c) {
+    for (auto &b : c.free_blocks) cudaFree(b.second);
+    c.free_blocks.clear();
+    c.cached = 0;
+}
+
+}  // namespace
+
+void *dev_alloc(size_t bytes) {
+    const size_t r = round_size(bytes);
+    const int dev = current_device();
+    {
+        std::lock_guard<std::mutex> lk(g_mu);
+        DeviceCache &c = g_cache[dev];
+        auto it = c.free_blocks.lower_bound(r);
+        // reuse a block of at most 4/3 of the request.  The caller frees with its
+        // own size, so the block may come back under a smaller key than its real
+        // size: always safe (it is only ever handed out for smaller requests).
+        if (it != c.free_blocks.end() && it->first - it->first / 4 <= r) {
+            void *p = it->second;
+            c.cached -= it->first;
+            c.free_blocks.erase(it);
+            return p;
+        }
+    }
+    void *p = nullptr;
+    cudaError_t e = cudaMalloc(&p, r);
+    if (e == cudaErrorMemoryAllocation) {  // drop the cache and retry once
+        cudaGetLastError();
+        dev_empty_cache();
+        e = cudaMalloc(&p, r);
+    }
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        fail(e == cudaErrorMemoryAllocation ? MCE_ERR_NOMEM : MCE_ERR_CUDA,
+             std::string("cudaMalloc(") + std::to_string(r) + "): " + cudaGetErrorString(e));
+    }
+    return p;
+}
+
+void dev_free(void *p, size_t bytes) {
+    if (!p) return;
+    const size_t r = round_size(bytes);
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) return;
+    std::lock_guard<std::mutex> lk(g_mu);
+    DeviceCache &c = g_cache[dev];
+    c.free_blocks.emplace(r, p);
+    c.cached += r;
+}
+
+size_t dev_cached_bytes() {
+    const int dev = current_device();
+    std::lock_guard<std::mutex> lk(g_mu);
+    return g_cache[dev].cached;
+}
+
+void dev_empty_cache() {
+    const int dev = current_device();
+    std::lock_guard<std::mutex> lk(g_mu);
+    release_all(g_cache[dev]);
+}
+
+void *host_pinned(size_t bytes) {
+    const int dev = current_device();
+    std::lock_guard<std::mutex> lk(g_mu);
+    DeviceCache &c = g_cache[dev];
+    if (c.pinned_bytes < bytes) {
+        if (c.pinned) cudaFreeHost(c.pinned);
+        c.pinned = nullptr;
+        c.pinned_bytes = std::max<size_t>(bytes, 1 << 16);
+        MCE_CUDA(cudaMallocHost(&c.pinned, c.pinned_bytes));
+    }
+    return c.pinned;
+}
+
+}  // namespace mce
+
+extern "C" mce_status mce_empty_cache(int32_t device) {
+    try {
+        int ndev = 0;
+        if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) return MCE_ERR_INVALID;
+        int prev = 0;
+        cudaGetDevice(&prev);
+        cudaSetDevice(device);
+        mce::dev_empty_cache();
+        cudaSetDevice(prev);
+        return MCE_OK;
+    } catch (...) {
+        return MCE_ERR_CUDA;
+    }
+}

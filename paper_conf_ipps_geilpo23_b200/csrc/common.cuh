@@ -34,6 +34,19 @@ struct Error : std::runtime_error {
 #define MCE_LAUNCH_CHECK() MCE_CUDA(cudaGetLastError())
 
 // ---------------------------------------------------------------------------
+// per-device caching allocator (alloc.cu): freed blocks are kept and handed
+// out again, so a new graph handle, a new phase or a regrown buffer does not
+// pay cudaMalloc/cudaFree (cudaFree serialises the whole device).  Sizes are
+// rounded (4 KiB below 1 MiB, 2 MiB above); a cached block is reused for a
+// request of at least 3/4 of its size.  mce_empty_cache() returns it all.
+// ---------------------------------------------------------------------------
+void *dev_alloc(size_t bytes);           // throws MCE_ERR_NOMEM / MCE_ERR_CUDA
+void dev_free(void *p, size_t bytes);    // bytes = the size passed to dev_alloc
+size_t dev_cached_bytes();               // free bytes held by the cache on this device
+void dev_empty_cache();
+void *host_pinned(size_t bytes);         // per-device pinned staging (grow-only, shared)
+
+// ---------------------------------------------------------------------------
 // owning device buffer
 // ---------------------------------------------------------------------------
 template <typename T>
@@ -52,15 +65,15 @@ struct DevBuf {
     ~DevBuf() { release(); }
     void alloc(size_t count) {
         release();
+        if (count) p = static_cast<T *>(dev_alloc(sizeof(T) * count));
         n = count;
-        if (count) MCE_CUDA(cudaMalloc(&p, sizeof(T) * count));
     }
     // keep the current allocation when it is large enough (no cudaMalloc/cudaFree)
     void ensure(size_t count) {
         if (n < count || !p) alloc(count);
     }
     void release() {
-        if (p) cudaFree(p);
+        if (p) dev_free(p, sizeof(T) * n);
         p = nullptr;
         n = 0;
     }
@@ -68,25 +81,12 @@ struct DevBuf {
     size_t bytes() const { return sizeof(T) * n; }
 };
 
-// pinned host staging buffer (small scalar read-backs without pageable copies)
+// pinned host staging (small scalar read-backs without pageable copies);
+// the memory is the device's shared staging block (host_pinned)
 struct PinnedBuf {
-    void *p = nullptr;
-    size_t n = 0;
-    PinnedBuf() = default;
-    PinnedBuf(const PinnedBuf &) = delete;
-    PinnedBuf &operator=(const PinnedBuf &) = delete;
-    ~PinnedBuf() {
-        if (p) cudaFreeHost(p);
-    }
     template <typename T>
     T *get(size_t count) {
-        if (n < count * sizeof(T)) {
-            if (p) cudaFreeHost(p);
-            p = nullptr;
-            n = std::max<size_t>(count * sizeof(T), 4096);
-            MCE_CUDA(cudaMallocHost(&p, n));
-        }
-        return reinterpret_cast<T *>(p);
+        return reinterpret_cast<T *>(host_pinned(count * sizeof(T)));
     }
 };
 
@@ -106,7 +106,7 @@ class Pool {
     Pool(const Pool &) = delete;
     Pool &operator=(const Pool &) = delete;
     ~Pool() {
-        for (void *q : spill_) cudaFree(q);
+        for (auto &q : spill_) dev_free(q.first, q.second);
     }
     template <typename T>
     T *take(int64_t count) {
@@ -116,16 +116,15 @@ class Pool {
             top_ += bytes;
             return q;
         }
-        void *q = nullptr;
-        MCE_CUDA(cudaMalloc(&q, bytes));
-        spill_.push_back(q);
+        void *q = dev_alloc(bytes);
+        spill_.push_back({q, bytes});
         spill_bytes_ += bytes;
         return reinterpret_cast<T *>(q);
     }
     void reset() {
         if (!spill_.empty()) {
             const size_t want = top_ + spill_bytes_;
-            for (void *q : spill_) cudaFree(q);
+            for (auto &q : spill_) dev_free(q.first, q.second);
             spill_.clear();
             spill_bytes_ = 0;
             if (want > main_.n) main_.alloc(want + want / 4);
@@ -137,7 +136,7 @@ class Pool {
    private:
     DevBuf<uint8_t> main_;
     size_t top_ = 0;
-    std::vector<void *> spill_;
+    std::vector<std::pair<void *, size_t>> spill_;
     size_t spill_bytes_ = 0;
 };
 

@@ -274,7 +274,7 @@ void Engine::process(int32_t k, const Level &L) {
     a.roots = roots_;
     a.adj = adj_;
     a.ocol = g_->ocol.get();
-    a.order = g_->order.get();
+    a.order = g_->vid.get();
     a.counts = counts;
     a.maxbit = maxbit_;
     a.leaf_total = leaf_total_;
@@ -285,7 +285,7 @@ void Engine::process(int32_t k, const Level &L) {
 
     // misc[0..2] = leaf total, leaf slot, maxbit (-1)
     MCE_CUDA(cudaMemsetAsync(leaf_total_, 0, 2 * sizeof(unsigned long long), s_));
-    MCE_CUDA(cudaMemsetAsync(maxbit_, 0xff, sizeof(int32_t), s_));
+    MCE_CUDA(cudaMemsetAsync(maxbit_, 0xff, 2 * sizeof(int32_t), s_));
     launch_timed(a, false);
     exclusive_scan_i32(counts, offs, N, tmp, s_);
     kernels_ += 3;
@@ -296,6 +296,7 @@ void Engine::process(int32_t k, const Level &L) {
     const int64_t total = h[0];
     const unsigned long long leaves = (unsigned long long)h[1];
     const int32_t maxbit = (int32_t)(uint32_t)(uint64_t)h[3];
+    const int32_t maxub = (int32_t)(uint32_t)((uint64_t)h[3] >> 32);  // deepest reachable level
     // children's candidate sets only use bits <= maxbit: shrink their stride
     // (power of two, so the kernels stay specialised)
     int32_t Wc = 1;
@@ -307,9 +308,15 @@ void Engine::process(int32_t k, const Level &L) {
     if (leaves) handle_leaves(k + 1, (int64_t)leaves, a);
 
     const int64_t per_child = 8 * Wc + 12 + 12 + 16;
+    // When the children do not fit they are produced in chunks.  Each chunk may
+    // take 1/(levels still reachable below it + 1) of the free arena, so a
+    // frontier that keeps growing for many levels (R-MAT: 2x per level over the
+    // last ~30 levels) is chunked evenly instead of halving the budget per level.
+    const int64_t depth_left = std::max<int64_t>(1, (int64_t)maxub - (k + 1));
     int64_t a0 = 0;
     while (total > 0 && a0 < N) {
-        const int64_t cap = (int64_t)(arena_.avail() / 2) / per_child;
+        const int64_t share = total * per_child <= (int64_t)(arena_.avail() / 2) ? 2 : depth_left + 1;
+        const int64_t cap = (int64_t)(arena_.avail() / share) / per_child;
         int64_t b, cnt, base;
         if (a0 == 0 && total <= cap) {
             b = N;
@@ -389,7 +396,7 @@ void Engine::do_class_w1(const int32_t *list, int64_t count) {
         ra.stride = stride_;
         ra.orp = g_->orp.get();
         ra.ocol = g_->ocol.get();
-        ra.order = g_->order.get();
+        ra.order = g_->vid.get();
         ra.need = need();
         ra.bound = o_.bound;
         ra.roots = arena_.alloc<RootInfo>(nw);
@@ -571,7 +578,7 @@ mce_result *Engine::run() {
     // counts as free memory here
     size_t free_b = 0, total_b = 0;
     MCE_CUDA(cudaMemGetInfo(&free_b, &total_b));
-    free_b += g_->ws.n;
+    free_b += g_->ws.n + dev_cached_bytes();
     int64_t budget = o_.budget_bytes;
     if (budget <= 0)
         budget = std::min<int64_t>((int64_t)(free_b * 0.8), (int64_t)(1ll << 30) + 48ll * g_->nnz + 64ll * n);

@@ -38,17 +38,19 @@ __global__ void build_adj_w1(const RootInfo *__restrict__ roots, int64_t nroots,
         for (int32_t i = lane; i < ri.L; i += 32) {
             const int32_t a = __ldg(V + i);
             uint64_t row = 0;
-            // j > i: V[j] in N+(a) -- one merge pass over two sorted lists
+            // V and every out-row are sorted by CSR id, which need not follow
+            // the orientation (rank) order, so both directions are checked for
+            // every c: V[c] in N+(a) by one merge pass over the two sorted lists,
+            // a in N+(V[c]) by binary search
             int64_t p = __ldg(orp + a), pe = __ldg(orp + a + 1);
-            for (int32_t c = i + 1; c < ri.L && p < pe; ++c) {
+            for (int32_t c = 0; c < ri.L && p < pe; ++c) {
                 const int32_t b = __ldg(V + c);
                 while (p < pe && __ldg(ocol + p) < b) ++p;
                 if (p < pe && __ldg(ocol + p) == b) row |= 1ull << c;
             }
-            // j < i: a in N+(V[j])
-            for (int32_t c = 0; c < i; ++c) {
+            for (int32_t c = 0; c < ri.L; ++c) {
                 const int32_t b = __ldg(V + c);
-                if (contains_sorted(ocol, __ldg(orp + b), __ldg(orp + b + 1), a)) row |= 1ull << c;
+                if (c != i && contains_sorted(ocol, __ldg(orp + b), __ldg(orp + b + 1), a)) row |= 1ull << c;
             }
             // local index = L-1-position (reverse degeneracy order, see expand.cuh)
             adj[ri.abase + (ri.L - 1 - i)] = __brevll(row) >> (64 - ri.L);
@@ -59,7 +61,7 @@ __global__ void build_adj_w1(const RootInfo *__restrict__ roots, int64_t nroots,
 // W >= 2: one block per root, warp per row.  Row i of the root-local
 // adjacency is N+(V[i]) ∩ V: the warp reads N+(V[i]) 32 elements at a time
 // (coalesced), every lane binary-searches its element in the staged V
-// (positions > i only: the orientation puts every out-neighbour after V[i]),
+// (CSR ids order V but need not follow the orientation, so all of V),
 // and a hit at c sets bits (i, c) and (c, i).  The row stops at the first
 // chunk beyond V[L-1].  Bits go to a shared-memory bit matrix when it fits
 // (SMEM), else straight to the (zeroed) global matrix.
@@ -82,7 +84,7 @@ __global__ void build_adj_block(const RootInfo *__restrict__ roots, int64_t nroo
             for (int64_t w = threadIdx.x; w < (int64_t)L * W * 2; w += blockDim.x) sA[w] = 0u;
         __syncthreads();
         const int32_t vmax = sV[L - 1];
-        for (int i = wib; i < L - 1; i += nwb) {
+        for (int i = wib; i < L; i += nwb) {
             const int32_t a = sV[i];
             const int64_t pb = __ldg(orp + a), pe = __ldg(orp + a + 1);
             for (int64_t p0 = pb; p0 < pe; p0 += 32) {
@@ -90,7 +92,7 @@ __global__ void build_adj_block(const RootInfo *__restrict__ roots, int64_t nroo
                 const int32_t u = p < pe ? __ldg(ocol + p) : INT32_MAX;
                 if (__shfl_sync(0xffffffffu, u, 0) > vmax) break;
                 if (u <= vmax) {
-                    int lo = i + 1, hi = L;
+                    int lo = 0, hi = L;  // CSR-id order need not follow the orientation
                     while (lo < hi) {
                         const int mid = (lo + hi) >> 1;
                         if (sV[mid] < u)
@@ -161,12 +163,15 @@ __device__ __forceinline__ int top_bit(const uint64_t (&C)[W]) {
 
 // end-of-kernel reductions of the count pass: leaves (sum) and the highest
 // candidate bit of any surviving child (max) -> the children's word stride
-__device__ __forceinline__ void flush_counters(const ExpandArgs &a, unsigned long long nleaf, int hb) {
-    nleaf = __reduce_add_sync(0xffffffffu, (unsigned)nleaf) ;
+// ... and the deepest level any descendant can reach (max of k + 1 + |P'|)
+__device__ __forceinline__ void flush_counters(const ExpandArgs &a, unsigned long long nleaf, int hb, int ub) {
+    nleaf = __reduce_add_sync(0xffffffffu, (unsigned)nleaf);
     hb = __reduce_max_sync(0xffffffffu, hb + 1) - 1;
+    ub = __reduce_max_sync(0xffffffffu, ub);
     if ((threadIdx.x & 31) == 0) {
         if (nleaf) atomicAdd(a.leaf_total, nleaf);
         if (hb >= 0) atomicMax(a.maxbit, hb);
+        if (ub > 0) atomicMax(a.maxbit + 1, ub);
     }
 }
 
@@ -178,7 +183,7 @@ template <int W, bool WRITE>
 __global__ void __launch_bounds__(256) expand_thread(const ExpandArgs a) {
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     unsigned nleaf = 0;
-    int hb = -1;
+    int hb = -1, ub = 0;
     const int64_t e_end = a.begin + (a.end - a.begin + stride - 1) / stride * stride;  // warp-uniform trip count
     for (int64_t e = a.begin + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < e_end; e += stride) {
         if (e >= a.end) continue;
@@ -274,6 +279,7 @@ __global__ void __launch_bounds__(256) expand_thread(const ExpandArgs a) {
                         a.cvloc[c] = v;
                     } else {
                         hb = max(hb, top_bit<W>(C));
+                        ub = max(ub, a.k + 1 + pc);
                     }
                     ++cnt;
                 }
@@ -281,7 +287,7 @@ __global__ void __launch_bounds__(256) expand_thread(const ExpandArgs a) {
         }
         if (!WRITE) a.counts[e] = cnt;
     }
-    if (!WRITE) flush_counters(a, nleaf, hb);
+    if (!WRITE) flush_counters(a, nleaf, hb, ub);
 }
 
 // ---------------------------------------------------------------------------
@@ -298,7 +304,7 @@ __global__ void expand_warp(const ExpandArgs a, int max_l) {
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     const int W = a.Wp, Wa = a.Wa;
     unsigned nleaf = 0;
-    int hb = -1;
+    int hb = -1, ub = 0;
     for (int64_t e = a.begin + warp; e < a.end; e += nwarps) {
         int64_t out = 0;
         if (WRITE) {
@@ -437,6 +443,7 @@ __global__ void expand_warp(const ExpandArgs a, int max_l) {
 #pragma unroll
                         for (int t = 0; t < WPL; ++t)
                             if (C[t]) hb = max(hb, (lane + 32 * t) * 64 + 63 - __clzll((long long)C[t]));
+                        ub = max(ub, a.k + 1 + pc);
                     }
                     ++cnt;
                 }
@@ -445,7 +452,7 @@ __global__ void expand_warp(const ExpandArgs a, int max_l) {
         if (!WRITE && lane == 0) a.counts[e] = cnt;
         __syncwarp();
     }
-    if (!WRITE) flush_counters(a, nleaf, hb);
+    if (!WRITE) flush_counters(a, nleaf, hb, ub);
 }
 
 __global__ void classify_roots_kernel(int64_t n, const int64_t *__restrict__ orp, int32_t min_len, int32_t *cls,

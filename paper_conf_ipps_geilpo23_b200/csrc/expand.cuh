@@ -54,7 +54,8 @@ struct ExpandArgs {
     int32_t *cslot;
     int32_t *cparent;
     int32_t *cvloc;
-    // count pass: highest candidate bit of any surviving child (atomicMax)
+    // count pass (atomicMax): maxbit[0] = highest candidate bit of any surviving
+    // child, maxbit[1] = deepest level a descendant can reach (k + 1 + |P'|)
     int32_t *maxbit;
     // leaves of size k+1 (count pass only): total (exact) and staged rows
     unsigned long long *leaf_total;

@@ -20,8 +20,10 @@ struct mce_graph {
     int32_t degeneracy = 0;
     mce::DevBuf<int32_t> order;    // [n] rank -> vertex (orientation order)
     mce::DevBuf<int32_t> rank;     // [n] vertex -> rank
-    mce::DevBuf<int64_t> orp;      // [n+1] oriented CSR over ranks
-    mce::DevBuf<int32_t> ocol;     // [nnz/2] out-neighbour ranks, rows ascending
+    mce::DevBuf<int32_t> vid;      // [n] CSR id -> vertex (ids of orp/ocol: (core, degree) order, or the rank)
+    mce::DevBuf<int32_t> pid;      // [n] vertex -> CSR id
+    mce::DevBuf<int64_t> orp;      // [n+1] oriented CSR (edges to higher rank), indexed by CSR id
+    mce::DevBuf<int32_t> ocol;     // [nnz/2] out-neighbour CSR ids, rows ascending
     int32_t max_out = 0;           // largest out-degree
     double t_pre_ms = 0.0;         // device time of the last preprocessing
     int64_t kernels = 0;           // kernels launched by the last preprocessing
@@ -29,7 +31,7 @@ struct mce_graph {
     // ---- reusable memory (no cudaMalloc/cudaFree on the steady-state path) ----
     mce::Pool pool;                // per-phase scratch (reset at the start of every phase)
     mce::DevBuf<uint8_t> ws;       // frontier arena of mce_enumerate / mce_find_one (grow-only)
-    mce::PinnedBuf host;           // pinned staging for small device->host reads
+    mce::PinnedBuf host;           // pinned staging for small device->host reads (per device, shared)
     mce::DevBuf<uint8_t> misc;     // engine: leaf counter + level chain (persistent)
     mce::DevBuf<int32_t> stage;    // engine: staged leaf cliques (grow-only)
 };

@@ -1,18 +1,24 @@
 // Preprocessing on the device (north star: "k-core/degeneracy ordering and
 // edge orientation, done on device").
 //
-//  * kcore(): core numbers (PAPER.md II-B-2, line 61) by parallel peeling in
-//    ONE cooperative persistent launch: at level k every alive vertex with
-//    degree <= k is queued (core = k); processing a queued vertex decrements
-//    its alive neighbours and queues those that fall to k.  The queue order is
-//    a degeneracy order: when v is queued its remaining degree (<= k) counts
-//    every neighbour queued after it, so orienting edges along the queue gives
-//    out-degree <= core(v) <= degeneracy.
-//  * orient(): ranks (degeneracy = queue order, or degree order = PAPER.md
-//    IV-C line 131 "keep the edge where the source vertex has lower degree"),
-//    and the oriented CSR over ranks with every row sorted ascending, so that
-//    "the candidates after v" are exactly v's out-neighbours (IV-C line 133).
+//  * kcore(): core numbers (PAPER.md II-B-2, line 61) by level peeling in ONE
+//    cooperative persistent launch (kcore_async below): at level k every alive
+//    vertex with degree <= k is appended to the peel order (core = k) and its
+//    edges drained asynchronously, appending neighbours that fall to k.  The
+//    peel order is a degeneracy order: when v is appended its remaining degree
+//    (<= k) counts every neighbour appended after it, so orienting edges along
+//    the order gives out-degree <= core(v) <= degeneracy.
+//  * orient(): ranks (degeneracy = peel order, or degree order = PAPER.md IV-C
+//    line 131 "keep the edge where the source vertex has lower degree") decide
+//    the direction of every edge; the oriented CSR is stored in a second id
+//    space ("CSR ids": vertices sorted by (core, degree) for the degeneracy
+//    orientation, the rank itself for the degree orientation) with every row
+//    sorted ascending.  The search colours candidates in reverse CSR-id order
+//    (expand.cuh), i.e. high core first and, inside one core shell (where the
+//    peel order is arbitrary), high degree first.
 #include <cooperative_groups.h>
+
+#include <cub/device/device_radix_sort.cuh>
 
 #include <algorithm>
 #include <vector>
@@ -27,154 +33,241 @@ namespace {
 
 constexpr int kPeelThreads = 512;
 
-// ctrl layout (rotating per sub-round s, index s % 3):
-//   [0..2] queue append counters, [3..5] alive-list append counters,
-//   [6..8] smallest degree among the vertices a scan kept alive
+// ---------------------------------------------------------------------------
+// k-core numbers and a degeneracy order: asynchronous level peel.  Within a level k the order in which
+// queued vertices are processed does not matter: a vertex is appended to the
+// peel order when its degree falls to <= k, and every neighbour appended after
+// it was still unprocessed then, hence counted in that degree, so out-degrees
+// along the order stay <= k (= its core number).  So a level runs as one
+// asynchronous work list instead of one grid barrier per cascade round:
 //
-// Level-synchronous peel: a "scan" sub-round queues every alive vertex with
-// degree <= k and compacts the rest into the next alive list; a "cascade"
-// sub-round processes the vertices queued by the previous sub-round (one warp
-// per vertex, lanes over its neighbours) and queues neighbours whose degree
-// falls to k.  All appends are warp-aggregated (one atomicAdd per warp and
-// ballot ranks), so no counter sees more than one atomic per warp.  When a
-// scan queues nothing, k jumps straight to the smallest alive degree it saw.
-__device__ __forceinline__ unsigned long long warp_append(unsigned long long *ctr, unsigned mask, int lane) {
-    unsigned long long base = 0;
-    if (lane == 0 && mask) base = atomicAdd(ctr, (unsigned long long)__popc(mask));
-    return __shfl_sync(0xffffffffu, base, 0);
+//   scan   : every alive vertex with degree <= k is appended (peel order,
+//            core = k) and its edges are cut into work items of kChunk edges;
+//            the rest is compacted into the next alive list
+//   barrier
+//   drain  : warps grab four work-list slots at a time (one atomicAdd), an
+//            8-lane tile per item decrements the item's alive neighbours and
+//            appends those that fall to k (tile-aggregated atomics); a slot
+//            that is not yet written is polled until it is, or until every
+//            reserved item is processed (done == tail: nothing can follow)
+//   barrier, clear the level's work list, next level (k jumps to the
+//            smallest alive degree when a scan appends nothing)
+//
+// Work items are int64 (vertex | chunk << 32), -1 = empty; levels alternate
+// between two lists so one can be cleared while the other fills.
+// ---------------------------------------------------------------------------
+constexpr int64_t kChunk = 128;  // edges per work item
+
+__device__ __forceinline__ unsigned long long ld_relaxed(const unsigned long long *p) {
+    unsigned long long v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
 }
 
-// cascade step for one queued vertex v by a tile of G lanes: decrement the
-// alive neighbours, queue those that fall to k (one atomicAdd per tile chunk)
+// append the vertices whose flag is set (tile of G lanes): peel order, core,
+// dead, and ceil(deg / kChunk) work items each
 template <int G>
-__device__ __forceinline__ void peel_neighbours(int32_t v, const int64_t *__restrict__ rowptr,
-                                                const int32_t *__restrict__ col, int32_t *deg, int32_t *core,
-                                                int32_t *queue, uint8_t *dead, unsigned long long *qcnt,
-                                                int64_t region_end, int32_t k) {
+__device__ __forceinline__ void async_append(bool take, int32_t u, const int64_t *__restrict__ rowptr, int32_t *core,
+                                             int32_t *order, uint8_t *dead, long long *work,
+                                             unsigned long long *otail, unsigned long long *wtail, int32_t k) {
     const int lane = threadIdx.x & 31;
     const int gl = lane & (G - 1), gbase = lane & ~(G - 1);
     const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << gbase);
-    const int64_t eb = rowptr[v], ee = rowptr[v + 1];
-    for (int64_t e0 = eb; e0 < ee; e0 += G) {
-        const int64_t e = e0 + gl;
-        bool fell = false;
-        int32_t u = -1;
-        if (e < ee) {
-            u = col[e];
-            if (!dead[u]) fell = atomicSub(deg + u, 1) == k + 1;
-        }
-        const unsigned fm = (__ballot_sync(gmask, fell) & gmask) >> gbase;
-        if (fm) {
-            unsigned long long b = 0;
-            if (gl == 0) b = atomicAdd(qcnt, (unsigned long long)__popc(fm));
-            b = __shfl_sync(gmask, b, 0, G);
-            if (fell) {
-                queue[region_end + b + __popc(fm & ((1u << gl) - 1u))] = u;
-                core[u] = k;
-                dead[u] = 1;
-            }
-        }
+    const unsigned m = (__ballot_sync(gmask, take) & gmask) >> gbase;
+    if (!m) return;
+    int items = 0;
+    if (take) {
+        const int64_t d = rowptr[u + 1] - rowptr[u];
+        items = (int)((d + kChunk - 1) / kChunk);
+    }
+    int inc = items;  // tile inclusive scan of item counts
+#pragma unroll
+    for (int o = 1; o < G; o <<= 1) {
+        const int y = __shfl_up_sync(gmask, inc, o, G);
+        if (gl >= o) inc += y;
+    }
+    const int total = __shfl_sync(gmask, inc, G - 1, G);
+    unsigned long long ob = 0, wb = 0;
+    if (gl == 0) {
+        ob = atomicAdd(otail, (unsigned long long)__popc(m));
+        if (total) wb = atomicAdd(wtail, (unsigned long long)total);
+    }
+    ob = __shfl_sync(gmask, ob, 0, G);
+    wb = __shfl_sync(gmask, wb, 0, G);
+    if (take) {
+        order[ob + __popc(m & ((1u << gl) - 1u))] = u;
+        core[u] = k;
+        dead[u] = 1;
+        for (int c = 0; c < items; ++c) work[wb + inc - items + c] = (long long)(uint32_t)u | ((long long)c << 32);
     }
 }
 
+// ctrl (u64, one counter per 128-byte line so the hot counters do not share an
+// L2 sector / slice): line 0 peel-order tail; lines 1..3 + 3 * (L % 2): work
+// head, tail, done of level L; lines 8..10 + 3 * (s % 3): scan s appended /
+// kept-alive count / min kept degree
+constexpr int kLine = 16;  // u64 per counter line
 __global__ void __launch_bounds__(kPeelThreads)
-    kcore_peel(int64_t n, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col, int32_t *deg,
-               int32_t *core, int32_t *queue, int32_t *alive_a, int32_t *alive_b, uint8_t *dead,
-               unsigned long long *ctrl) {
+    kcore_async(int64_t n, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col, int32_t *deg,
+                int32_t *core, int32_t *order, int32_t *alive_a, int32_t *alive_b, uint8_t *dead,
+                long long *work0, long long *work1, int64_t witems, unsigned long long *ctrl) {
     cg::grid_group grid = cg::this_grid();
+    __shared__ unsigned long long sh[6];
     const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const int64_t nthreads = (int64_t)gridDim.x * blockDim.x;
     const int64_t warp = tid >> 5;
     const int64_t nwarps = nthreads >> 5;
     const int lane = threadIdx.x & 31;
-    const unsigned lt = lanemask_lt();
+    unsigned long long *otail = ctrl;
+#define CTR(i) (ctrl + kLine * (i))
 
-    int64_t s = 0;          // sub-round
-    int64_t head = 0;       // region to process: [head, region_end)
-    int64_t region_end = 0;
+    int64_t s = 0, L = 0;
     int64_t n_alive = n;
     int32_t *cur = alive_a, *nxt = alive_b;
     int32_t k = 0;
-    bool scan = true;
     while (true) {
-        unsigned long long *qcnt = ctrl + (s % 3);
-        unsigned long long *acnt = ctrl + 3 + (s % 3);
-        unsigned long long *mind = ctrl + 6 + (s % 3);
-        if (tid == 0) {  // reset the counters of sub-round s+1 (last read before this sub-round began)
-            ctrl[(s + 1) % 3] = 0;
-            ctrl[3 + (s + 1) % 3] = 0;
-            ctrl[6 + (s + 1) % 3] = ~0ull;
+        unsigned long long *head = CTR(1 + 3 * (L & 1)), *tail = CTR(2 + 3 * (L & 1)), *done = CTR(3 + 3 * (L & 1));
+        unsigned long long *sapp = CTR(8 + 3 * (s % 3)), *skept = CTR(9 + 3 * (s % 3)), *smin = CTR(10 + 3 * (s % 3));
+        long long *work = (L & 1) ? work1 : work0;
+        if (tid == 0) {  // scan counters of s+1 (last read before scan s began)
+            *CTR(8 + 3 * ((s + 1) % 3)) = 0;
+            *CTR(9 + 3 * ((s + 1) % 3)) = 0;
+            *CTR(10 + 3 * ((s + 1) % 3)) = ~0ull;
         }
-        if (scan) {
-            int32_t dmin = INT32_MAX;
-            for (int64_t i0 = warp * 32; i0 < n_alive; i0 += nwarps * 32) {
-                const int64_t i = i0 + lane;
-                int32_t v = -1, d = 0;
-                bool live = false;
-                if (i < n_alive) {
-                    v = cur[i];
-                    live = !dead[v];
-                    if (live) d = deg[v];
-                }
-                const bool q = live && d <= k;
-                const bool keep = live && d > k;
-                const unsigned qm = __ballot_sync(0xffffffffu, q);
-                const unsigned km = __ballot_sync(0xffffffffu, keep);
-                const unsigned long long qb = warp_append(qcnt, qm, lane);
-                const unsigned long long kb = warp_append(acnt, km, lane);
-                if (q) {
-                    queue[region_end + qb + __popc(qm & lt)] = v;
-                    core[v] = k;
-                    dead[v] = 1;
-                }
-                if (keep) {
-                    nxt[kb + __popc(km & lt)] = v;
-                    dmin = min(dmin, d);
-                }
+        // ---- scan: append every alive vertex of degree <= k, compact the rest
+        int32_t dmin = INT32_MAX;
+        for (int64_t i0 = warp * 32; i0 < n_alive; i0 += nwarps * 32) {
+            const int64_t i = i0 + lane;
+            int32_t v = -1, d = 0;
+            bool live = false;
+            if (i < n_alive) {
+                v = cur[i];
+                live = !dead[v];
+                if (live) d = deg[v];
             }
-            dmin = __reduce_min_sync(0xffffffffu, dmin);
-            if (lane == 0 && dmin != INT32_MAX) atomicMin(mind, (unsigned long long)dmin);
-        } else {
-            // warp takes four queued vertices: 8-lane tiles when all have degree <= 64
-            for (int64_t q0 = head + warp * 4; q0 < region_end; q0 += nwarps * 4) {
-                const int64_t qi = q0 + (lane >> 3);
-                const int32_t v = qi < region_end ? queue[qi] : -1;
-                const int64_t d = v >= 0 ? rowptr[v + 1] - rowptr[v] : 0;
-                if (__all_sync(0xffffffffu, d <= 64)) {
-                    if (v >= 0) peel_neighbours<8>(v, rowptr, col, deg, core, queue, dead, qcnt, region_end, k);
-                } else {
-                    for (int t = 0; t < 4; ++t) {
-                        const int32_t vt = __shfl_sync(0xffffffffu, v, 8 * t);
-                        if (vt < 0) break;
-                        peel_neighbours<32>(vt, rowptr, col, deg, core, queue, dead, qcnt, region_end, k);
-                    }
-                }
-                __syncwarp();
+            const bool q = live && d <= k;
+            const bool keep = live && d > k;
+            const unsigned qm = __ballot_sync(0xffffffffu, q);
+            if (lane == 0 && qm) atomicAdd(sapp, (unsigned long long)__popc(qm));
+            async_append<32>(q, v, rowptr, core, order, dead, work, otail, tail, k);
+            const unsigned km = __ballot_sync(0xffffffffu, keep);
+            unsigned long long kb = 0;
+            if (lane == 0 && km) kb = atomicAdd(skept, (unsigned long long)__popc(km));
+            kb = __shfl_sync(0xffffffffu, kb, 0);
+            if (keep) {
+                nxt[kb + __popc(km & lanemask_lt())] = v;
+                dmin = min(dmin, d);
             }
         }
+        dmin = __reduce_min_sync(0xffffffffu, dmin);
+        if (lane == 0 && dmin != INT32_MAX) atomicMin(smin, (unsigned long long)dmin);
         grid.sync();
-        const int64_t c = (int64_t)(*(volatile unsigned long long *)qcnt);
-        const unsigned long long md = *(volatile unsigned long long *)mind;
-        const bool was_scan = scan;
-        if (scan) {
-            n_alive = (int64_t)(*(volatile unsigned long long *)acnt);
+        if (threadIdx.x == 0) {
+            sh[0] = __ldcg(sapp);
+            sh[1] = __ldcg(skept);
+            sh[2] = __ldcg(smin);
+            sh[3] = __ldcg(otail);
+        }
+        __syncthreads();
+        const unsigned long long appended = sh[0], kept = sh[1], md = sh[2], placed = sh[3];
+        __syncthreads();
+        n_alive = (int64_t)kept;
+        {
             int32_t *t = cur;
             cur = nxt;
             nxt = t;
         }
-        head = region_end;
-        region_end += c;
-        if (region_end >= n) break;  // every vertex has its core number
-        if (c == 0) {
-            // a scan that queued nothing saw every alive degree: jump to the smallest
-            k = was_scan ? (int32_t)md : k + 1;
-            scan = true;
-        } else {
-            scan = false;
-        }
         ++s;
+        if ((int64_t)placed >= n) break;  // every vertex has its core number
+        if (appended == 0) {              // nothing of degree <= k: jump to the smallest alive degree
+            k = (int32_t)md;
+            continue;
+        }
+        if (tid == 0) {  // counters of level L+1 (last read right after level L-1's drain)
+            *CTR(1 + 3 * ((L + 1) & 1)) = 0;
+            *CTR(2 + 3 * ((L + 1) & 1)) = 0;
+            *CTR(3 + 3 * ((L + 1) & 1)) = 0;
+        }
+        // ---- drain the level's work list asynchronously.  A warp reserves four
+        // slots (one per 8-lane tile) and polls them without blocking: an
+        // unwritten slot may be waiting for an item that a sibling tile's item
+        // appends.  The tiles' edge loops run in warp lock-step so appends and
+        // done counts are aggregated over the whole warp (one atomic each).
+        while (true) {
+            unsigned long long base = 0;
+            if (lane == 0) base = atomicAdd(head, 4ull);
+            base = __shfl_sync(0xffffffffu, base, 0);
+            const unsigned long long slot = base + (lane >> 3);
+            const int leader = lane & ~7;
+            bool resolved = false, over = false;
+            while (true) {
+                long long item = -1;
+                bool dead_slot = false;
+                if (!resolved && (lane & 7) == 0) {
+                    if (slot >= (unsigned long long)witems) {
+                        dead_slot = true;  // beyond the list: can never be filled
+                    } else {
+                        item = (long long)ld_relaxed((const unsigned long long *)(work + slot));
+                        if (item == -1) {
+                            const unsigned long long dn = ld_relaxed(done);
+                            const unsigned long long tl = ld_relaxed(tail);
+                            dead_slot = dn == tl && slot >= tl;
+                        }
+                    }
+                }
+                item = __shfl_sync(0xffffffffu, item, leader);
+                dead_slot = __shfl_sync(0xffffffffu, dead_slot, leader);
+                const bool work_now = !resolved && item != -1;
+                int64_t eb = 0, ee = 0;
+                if (work_now) {
+                    const int32_t v = (int32_t)(item & 0xffffffffll);
+                    const int64_t c = item >> 32;
+                    eb = rowptr[v] + c * kChunk;
+                    ee = min(rowptr[v + 1], eb + kChunk);
+                }
+                const int iters = __reduce_max_sync(0xffffffffu, (unsigned)((ee - eb + 7) >> 3));
+                for (int it = 0; it < iters; ++it) {
+                    const int64_t e = eb + it * 8 + (lane & 7);
+                    bool fell = false;
+                    int32_t u = -1;
+                    if (e < ee) {
+                        u = col[e];
+                        if (!dead[u]) fell = atomicSub(deg + u, 1) == k + 1;
+                    }
+                    async_append<32>(fell, u, rowptr, core, order, dead, work, otail, tail, k);
+                }
+                const unsigned done_m = __ballot_sync(0xffffffffu, work_now && (lane & 7) == 0);
+                if (lane == 0 && done_m) {
+                    __threadfence();  // this warp's appends before its done count
+                    atomicAdd(done, (unsigned long long)__popc(done_m));
+                }
+                if (work_now) resolved = true;
+                if (!resolved && dead_slot) {
+                    resolved = true;
+                    over = true;
+                }
+                if (__all_sync(0xffffffffu, resolved)) break;
+                if (!done_m) __nanosleep(64);
+            }
+            if (__all_sync(0xffffffffu, over)) break;
+        }
+        grid.sync();
+        // ---- clear this level's work list (the next level fills the other one)
+        if (threadIdx.x == 0) {
+            sh[4] = __ldcg(head);
+            sh[5] = __ldcg(tail);
+        }
+        __syncthreads();
+        const int64_t extent = min((int64_t)max(sh[4], sh[5]), witems);
+        const int64_t placed2 = (int64_t)__ldcg(otail);
+        __syncthreads();
+        for (int64_t i = tid; i < extent; i += nthreads) work[i] = -1;
+        ++L;
+        ++k;
+        if (placed2 >= n) break;
     }
 }
+#undef CTR
 
 // degeneracy = core number of the last vertex peeled
 __global__ void last_core_kernel(int64_t n, const int32_t *__restrict__ peel, const int32_t *__restrict__ core,
@@ -186,6 +279,15 @@ __global__ void degrees_kernel(int64_t n, const int64_t *__restrict__ rowptr, in
     for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
         deg[v] = (int32_t)(rowptr[v + 1] - rowptr[v]);
         iota[v] = (int32_t)v;
+    }
+}
+
+// sort key of the CSR id space: core number (high word), degree (low word)
+__global__ void priority_keys_kernel(int64_t n, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ core,
+                                     uint64_t *keys, int32_t *vals) {
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+        keys[v] = ((uint64_t)(uint32_t)core[v] << 32) | (uint64_t)(rowptr[v + 1] - rowptr[v]);
+        vals[v] = (int32_t)v;
     }
 }
 
@@ -225,7 +327,7 @@ struct Tile {
 // out-degree of vertex v's rank (tile of G lanes over v's neighbours)
 template <int G>
 __device__ void out_degree_one(int64_t v, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
-                               const int32_t *__restrict__ rank, int32_t *odeg) {
+                               const int32_t *__restrict__ rank, const int32_t *__restrict__ pid, int32_t *odeg) {
     Tile<G> t;
     const int32_t r = rank[v];
     int32_t cnt = 0;
@@ -234,23 +336,25 @@ __device__ void out_degree_one(int64_t v, const int64_t *__restrict__ rowptr, co
         const int64_t e = e0 + t.gl;
         cnt += __popc(t.ballot(e < ee && rank[col[e]] > r));
     }
-    if (t.gl == 0) odeg[r] = cnt;
+    if (t.gl == 0) odeg[pid[v]] = cnt;
 }
 
 // oriented row of v (in CSR order of the source; sorted afterwards)
 template <int G>
 __device__ void orient_fill_one(int64_t v, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
-                                const int32_t *__restrict__ rank, const int64_t *__restrict__ orp, int32_t *ocol) {
+                                const int32_t *__restrict__ rank, const int32_t *__restrict__ pid,
+                                const int64_t *__restrict__ orp, int32_t *ocol) {
     Tile<G> t;
     const int32_t r = rank[v];
-    int64_t out = orp[r];
+    int64_t out = orp[pid[v]];
     const int64_t eb = rowptr[v], ee = rowptr[v + 1];
     for (int64_t e0 = eb; e0 < ee; e0 += G) {
         const int64_t e = e0 + t.gl;
-        const int32_t ru = e < ee ? rank[col[e]] : -1;
+        const int32_t u = e < ee ? col[e] : 0;
+        const int32_t ru = e < ee ? rank[u] : -1;
         const bool up = ru > r;
         const unsigned m = t.ballot(up);
-        if (up) ocol[out + __popc(m & t.lt())] = ru;
+        if (up) ocol[out + __popc(m & t.lt())] = pid[u];
         out += __popc(m);
     }
 }
@@ -261,7 +365,8 @@ __device__ void orient_fill_one(int64_t v, const int64_t *__restrict__ rowptr, c
 template <bool FILL>
 __global__ void __launch_bounds__(256) orient_kernel(int64_t n, const int64_t *__restrict__ rowptr,
                                                      const int32_t *__restrict__ col, const int32_t *__restrict__ rank,
-                                                     int32_t *odeg, const int64_t *__restrict__ orp, int32_t *ocol) {
+                                                     const int32_t *__restrict__ pid, int32_t *odeg,
+                                                     const int64_t *__restrict__ orp, int32_t *ocol) {
     const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     const int lane = threadIdx.x & 31;
@@ -271,16 +376,16 @@ __global__ void __launch_bounds__(256) orient_kernel(int64_t n, const int64_t *_
         if (__all_sync(0xffffffffu, d <= 64)) {
             if (v < n) {
                 if (FILL)
-                    orient_fill_one<8>(v, rowptr, col, rank, orp, ocol);
+                    orient_fill_one<8>(v, rowptr, col, rank, pid, orp, ocol);
                 else
-                    out_degree_one<8>(v, rowptr, col, rank, odeg);
+                    out_degree_one<8>(v, rowptr, col, rank, pid, odeg);
             }
         } else {
             for (int t = 0; t < 4 && v0 + t < n; ++t) {
                 if (FILL)
-                    orient_fill_one<32>(v0 + t, rowptr, col, rank, orp, ocol);
+                    orient_fill_one<32>(v0 + t, rowptr, col, rank, pid, orp, ocol);
                 else
-                    out_degree_one<32>(v0 + t, rowptr, col, rank, odeg);
+                    out_degree_one<32>(v0 + t, rowptr, col, rank, pid, odeg);
             }
         }
         __syncwarp();
@@ -419,14 +524,20 @@ void kcore(mce_graph *g) {
     g->pool.reset();
     int32_t *deg = g->pool.take<int32_t>(n), *alive_a = g->pool.take<int32_t>(n), *alive_b = g->pool.take<int32_t>(n);
     uint8_t *dead = g->pool.take<uint8_t>(n);
-    unsigned long long *ctrl = g->pool.take<unsigned long long>(9);
+    // work items: at most one per vertex plus one per kChunk edges, per level list
+    const int64_t witems = n + g->nnz / kChunk + 1;
+    long long *work0 = g->pool.take<long long>(witems), *work1 = g->pool.take<long long>(witems);
+    unsigned long long *ctrl = g->pool.take<unsigned long long>(kLine * 20);
     MCE_CUDA(cudaMemsetAsync(dead, 0, n, s));
-    MCE_CUDA(cudaMemsetAsync(ctrl, 0, 6 * sizeof(unsigned long long), s));
-    MCE_CUDA(cudaMemsetAsync(ctrl + 6, 0xff, 3 * sizeof(unsigned long long), s));
+    MCE_CUDA(cudaMemsetAsync(work0, 0xff, sizeof(long long) * witems, s));
+    MCE_CUDA(cudaMemsetAsync(work1, 0xff, sizeof(long long) * witems, s));
+    MCE_CUDA(cudaMemsetAsync(ctrl, 0, kLine * 20 * sizeof(unsigned long long), s));
+    for (int i = 0; i < 3; ++i)
+        MCE_CUDA(cudaMemsetAsync(ctrl + kLine * (10 + 3 * i), 0xff, sizeof(unsigned long long), s));
     degrees_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(), deg, alive_a);
     MCE_LAUNCH_CHECK();
     int blocks_per_sm = 0;
-    MCE_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm, kcore_peel, kPeelThreads, 0));
+    MCE_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm, kcore_async, kPeelThreads, 0));
     blocks_per_sm = std::max(1, std::min(blocks_per_sm, 2));
     int grid = num_sms() * blocks_per_sm;
     int64_t n_arg = n;
@@ -434,9 +545,11 @@ void kcore(mce_graph *g) {
     const int32_t *cl = g->col.get();
     int32_t *dg = deg, *co = g->core.get(), *qu = g->peel.get(), *aa = alive_a, *ab = alive_b;
     uint8_t *dd = dead;
+    long long *w0 = work0, *w1 = work1;
+    int64_t wi = witems;
     unsigned long long *ct = ctrl;
-    void *args[] = {&n_arg, &rp, &cl, &dg, &co, &qu, &aa, &ab, &dd, &ct};
-    MCE_CUDA(cudaLaunchCooperativeKernel((void *)kcore_peel, grid, kPeelThreads, args, 0, s));
+    void *args[] = {&n_arg, &rp, &cl, &dg, &co, &qu, &aa, &ab, &dd, &w0, &w1, &wi, &ct};
+    MCE_CUDA(cudaLaunchCooperativeKernel((void *)kcore_async, grid, kPeelThreads, args, 0, s));
     g->kernels += 2;
     // degeneracy = max core (the last queued vertex has it)
     last_core_kernel<<<1, 1, 0, s>>>(n, g->peel.get(), g->core.get(), deg);
@@ -453,6 +566,8 @@ void orient(mce_graph *g, int orientation) {
     cudaStream_t s = g->stream;
     g->order.ensure(std::max<int64_t>(n, 1));
     g->rank.ensure(std::max<int64_t>(n, 1));
+    g->vid.ensure(std::max<int64_t>(n, 1));
+    g->pid.ensure(std::max<int64_t>(n, 1));
     g->orp.ensure(n + 1);
     g->ocol.ensure(std::max<int64_t>(g->nnz / 2, 1));
     g->pool.reset();
@@ -479,13 +594,36 @@ void orient(mce_graph *g, int orientation) {
     }
     invert_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->order.get(), g->rank.get());
     MCE_LAUNCH_CHECK();
+    // id space of the oriented CSR (reading 5): degeneracy -> vertices
+    // sorted by (core, degree) ascending, so the reverse local order of a root
+    // meets high-core, then high-degree vertices first; degree -> the rank itself
+    if (orientation == 0) {
+        uint64_t *keys = g->pool.take<uint64_t>(n), *keys_out = g->pool.take<uint64_t>(n);
+        int32_t *vals = g->pool.take<int32_t>(n);
+        priority_keys_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(), g->core.get(), keys, vals);
+        MCE_LAUNCH_CHECK();
+        int end_bit = 32;
+        while (end_bit < 64 && (1ll << (end_bit - 32)) <= (int64_t)g->degeneracy) ++end_bit;
+        size_t tmp_bytes = 0;
+        MCE_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tmp_bytes, keys, keys_out, vals, g->vid.get(), (int)n, 0,
+                                                 end_bit, s));
+        void *tmp = g->pool.take<uint8_t>((int64_t)tmp_bytes);
+        MCE_CUDA(cub::DeviceRadixSort::SortPairs(tmp, tmp_bytes, keys, keys_out, vals, g->vid.get(), (int)n, 0,
+                                                 end_bit, s));
+        invert_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->vid.get(), g->pid.get());
+        MCE_LAUNCH_CHECK();
+        g->kernels += 4;
+    } else {
+        MCE_CUDA(cudaMemcpyAsync(g->vid.get(), g->order.get(), sizeof(int32_t) * n, cudaMemcpyDeviceToDevice, s));
+        MCE_CUDA(cudaMemcpyAsync(g->pid.get(), g->rank.get(), sizeof(int32_t) * n, cudaMemcpyDeviceToDevice, s));
+    }
     int32_t *odeg = g->pool.take<int32_t>(n);
-    orient_kernel<false><<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), g->rank.get(), odeg,
-                                                               nullptr, nullptr);
+    orient_kernel<false><<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), g->rank.get(),
+                                                               g->pid.get(), odeg, nullptr, nullptr);
     MCE_LAUNCH_CHECK();
     exclusive_scan_i32(odeg, g->orp.get(), n, g->pool.take<int64_t>(scan_tmp_items(n)), s);
     orient_kernel<true><<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), g->rank.get(),
-                                                              nullptr, g->orp.get(), g->ocol.get());
+                                                              g->pid.get(), nullptr, g->orp.get(), g->ocol.get());
     MCE_LAUNCH_CHECK();
     sort_rows_warp<<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->orp.get(), g->ocol.get());
     MCE_LAUNCH_CHECK();

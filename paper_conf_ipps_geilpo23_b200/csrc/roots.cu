@@ -30,14 +30,16 @@ namespace {
 
 constexpr int kRootWarps = 8;  // warps per block
 
+// per-tile scratch for one root of up to M = G * RPL candidates
+template <int M>
 struct RootSmem {
-    int32_t V[64];
-    int32_t off[65];       // flattened row offsets
-    int64_t start[64];     // orp[V[i]]
-    uint32_t adj[64][2];   // row i, 64 columns as two words
-    uint8_t ord[64], colr[64];
-    uint8_t chv[64];       // children: local vertex
-    uint64_t chP[64];      // children: candidate set
+    int32_t V[M];
+    int32_t off[M + 1];    // flattened row offsets
+    int64_t start[M];      // orp[V[i]]
+    uint32_t adj[M][2];    // row of local index i, 64 columns as two words
+    uint8_t ord[M], colr[M];
+    uint8_t chv[M];        // children: local vertex
+    uint64_t chP[M];       // children: candidate set
 };
 
 __device__ __forceinline__ int lower_bound_smem(const int32_t *a, int n, int32_t key) {
@@ -52,172 +54,205 @@ __device__ __forceinline__ int lower_bound_smem(const int32_t *a, int n, int32_t
     return lo;
 }
 
-__global__ void __launch_bounds__(kRootWarps * 32) root_expand_w1(const RootArgs a) {
-    __shared__ RootSmem sm_all[kRootWarps];
+// The whole first expansion step of root r (|N+(r)| = L <= G * RPL) by a tile
+// of G lanes; lane gl owns local rows gl, gl + G, ... (RPL of them).
+template <int G, int RPL>
+__device__ void root_step(const RootArgs &a, int32_t r, RootSmem<G * RPL> &sm, unsigned long long &bytes) {
+    constexpr int M = G * RPL;
     const int lane = threadIdx.x & 31;
-    RootSmem &sm = sm_all[threadIdx.x >> 5];
+    const int gl = lane & (G - 1), gbase = lane & ~(G - 1);
+    const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << gbase);
+    const int64_t vb = __ldg(a.orp + r);
+    const int L = (int)(__ldg(a.orp + r + 1) - vb);
+    // 1. stage V (rank order), row starts and lengths; zero the bit matrix
+    int len[RPL];
+#pragma unroll
+    for (int q = 0; q < RPL; ++q) {
+        const int p = gl + q * G;
+        len[q] = 0;
+        if (p < L) {
+            const int32_t v = __ldg(a.ocol + vb + p);
+            sm.V[p] = v;
+            const int64_t s0 = __ldg(a.orp + v);
+            sm.start[p] = s0;
+            len[q] = (int)(__ldg(a.orp + v + 1) - s0);
+        }
+        sm.adj[p][0] = sm.adj[p][1] = 0u;
+    }
+    // exclusive offsets of rows 0..M-1 in position order
+    int carry = 0;
+#pragma unroll
+    for (int q = 0; q < RPL; ++q) {
+        int inc = len[q];
+#pragma unroll
+        for (int o = 1; o < G; o <<= 1) {
+            const int y = __shfl_up_sync(gmask, inc, o, G);
+            if (gl >= o) inc += y;
+        }
+        sm.off[gl + q * G] = carry + inc - len[q];
+        carry += __shfl_sync(gmask, inc, G - 1, G);
+    }
+    const int T = carry;
+    if (gl == 0) {
+        sm.off[M] = T;
+        // root row bounds + V + (row bounds + out-row) of every v in V
+        bytes += 16ull + 20ull * (unsigned long long)L + 4ull * (unsigned long long)T;
+    }
+    __syncwarp(gmask);
+    // 2. flattened intersection: element t of the concatenated out-rows
+    for (int t0 = 0; t0 < T; t0 += G) {
+        const int t = t0 + gl;
+        if (t < T) {
+            int lo = 0, hi = L - 1;  // row: last i with off[i] <= t
+            while (lo < hi) {
+                const int mid = (lo + hi + 1) >> 1;
+                if (sm.off[mid] <= t)
+                    lo = mid;
+                else
+                    hi = mid - 1;
+            }
+            const int32_t u = __ldg(a.ocol + sm.start[lo] + (t - sm.off[lo]));
+            const int c = lower_bound_smem(sm.V, L, u);
+            if (c < L && sm.V[c] == u) {  // local indices L-1-position (expand.cuh)
+                const int li = L - 1 - lo, lc = L - 1 - c;
+                atomicOr(&sm.adj[li][lc >> 5], 1u << (lc & 31));
+                atomicOr(&sm.adj[lc][li >> 5], 1u << (li & 31));
+            }
+        }
+    }
+    __syncwarp(gmask);
+    uint64_t row[RPL];
+#pragma unroll
+    for (int q = 0; q < RPL; ++q) {
+        const int p = gl + q * G;
+        row[q] = ((uint64_t)sm.adj[p][1] << 32) | sm.adj[p][0];
+    }
+    const uint64_t P = L >= 64 ? ~0ull : ((1ull << L) - 1);
+    auto fetch = [&](int v) -> uint64_t {  // row of local v, from the lane that owns it
+        uint64_t x = 0;
+#pragma unroll
+        for (int q = 0; q < RPL; ++q) {
+            const uint64_t y = __shfl_sync(gmask, row[q], v & (G - 1), G);
+            if (v / G == q) x = y;
+        }
+        return x;
+    };
+    // 3. bound + children (|C| = 1)
+    int np = 0, ncol = 0;
+    if (a.bound == 1) {
+        uint64_t U = P;
+        while (U) {
+            ++ncol;
+            uint64_t Q = U;
+            while (Q) {
+                const int v = __ffsll((long long)Q) - 1;
+                Q &= ~fetch(v);
+                Q &= ~(1ull << v);
+                U &= ~(1ull << v);
+                if (gl == 0) {
+                    sm.ord[np] = (uint8_t)v;
+                    sm.colr[np] = (uint8_t)ncol;
+                }
+                ++np;
+            }
+        }
+    } else {
+        if (gl == 0)
+            for (int j = 0; j < L; ++j) {
+                sm.ord[j] = (uint8_t)j;
+                sm.colr[j] = (uint8_t)(j + 1);
+            }
+        np = ncol = L;
+    }
+    __syncwarp(gmask);
+    int cnt = 0;
+    if (1 + ncol >= a.need) {
+        uint64_t R = P;
+        for (int j = np - 1; j >= 0; --j) {
+            if (1 + sm.colr[j] < a.need) break;
+            const int v = sm.ord[j];
+            const uint64_t C = R & fetch(v);
+            R &= ~(1ull << v);
+            const int pc = __popcll(C);
+            if (pc == 0) {
+                if (2 >= a.need && gl == 0) {  // {r, v} is a leaf clique of interest
+                    const unsigned long long idx = atomicAdd(a.ctr + 3, 1ull);
+                    if ((int64_t)idx < a.leaf_cap) {
+                        a.leaf_rows[idx * 2] = __ldg(a.order + r);
+                        a.leaf_rows[idx * 2 + 1] = __ldg(a.order + sm.V[L - 1 - v]);
+                    }
+                }
+            } else if (2 + pc >= a.need) {
+                if (gl == 0) {
+                    sm.chv[cnt] = (uint8_t)v;
+                    sm.chP[cnt] = C;
+                }
+                ++cnt;
+            }
+        }
+    }
+    // 4. materialise a surviving root: record, adjacency rows, level-2 entries
+    if (cnt > 0) {
+        unsigned long long s = 0, ab = 0, e0 = 0;
+        if (gl == 0) {
+            s = atomicAdd(a.ctr + 0, 1ull);
+            ab = atomicAdd(a.ctr + 1, (unsigned long long)L);
+            e0 = atomicAdd(a.ctr + 2, (unsigned long long)cnt);
+        }
+        s = __shfl_sync(gmask, s, 0, G);
+        ab = __shfl_sync(gmask, ab, 0, G);
+        e0 = __shfl_sync(gmask, e0, 0, G);
+        __syncwarp(gmask);
+        if (gl == 0) {
+            RootInfo ri;
+            ri.r = r;
+            ri.L = L;
+            ri.vbase = vb;
+            ri.abase = (int64_t)ab;
+            a.roots[s] = ri;
+        }
+#pragma unroll
+        for (int q = 0; q < RPL; ++q)
+            if (gl + q * G < L) a.adj[ab + gl + q * G] = row[q];
+        for (int j = gl; j < cnt; j += G) {
+            a.cP[e0 + j] = sm.chP[j];
+            a.cslot[e0 + j] = (int32_t)s;
+            a.cparent[e0 + j] = -1;
+            a.cvloc[e0 + j] = sm.chv[j];
+        }
+    }
+    __syncwarp(gmask);
+}
+
+// Warp w takes roots [4w, 4w+4): four 8-lane tiles when all four have
+// |N+(r)| <= 8 (the sparse case: BA m=4 roots have 4), else one root after
+// another on the whole warp (|N+(r)| <= 64).
+__global__ void __launch_bounds__(kRootWarps * 32) root_expand_w1(const RootArgs a) {
+    __shared__ RootSmem<64> sm_all[kRootWarps];
+    const int lane = threadIdx.x & 31;
+    RootSmem<64> &sm = sm_all[threadIdx.x >> 5];
+    RootSmem<8> *tiles = reinterpret_cast<RootSmem<8> *>(&sm);  // 4 x RootSmem<8> fit in one RootSmem<64>
+    static_assert(4 * sizeof(RootSmem<8>) <= sizeof(RootSmem<64>), "tile scratch");
     const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    unsigned long long bytes = 0;  // algorithmic bytes read, lane 0
-    for (int64_t i = warp; i < a.count; i += nwarps) {
-        const int32_t r = __ldg(a.list + i * a.stride);
-        const int64_t vb = __ldg(a.orp + r);
-        const int L = (int)(__ldg(a.orp + r + 1) - vb);
-        // 1. stage V, row starts and lengths
-        int len0 = 0, len1 = 0;
-        if (lane < L) {
-            const int32_t v = __ldg(a.ocol + vb + lane);
-            sm.V[lane] = v;
-            const int64_t s0 = __ldg(a.orp + v);
-            sm.start[lane] = s0;
-            len0 = (int)(__ldg(a.orp + v + 1) - s0);
-        }
-        if (lane + 32 < L) {
-            const int32_t v = __ldg(a.ocol + vb + lane + 32);
-            sm.V[lane + 32] = v;
-            const int64_t s1 = __ldg(a.orp + v);
-            sm.start[lane + 32] = s1;
-            len1 = (int)(__ldg(a.orp + v + 1) - s1);
-        }
-        sm.adj[lane][0] = sm.adj[lane][1] = 0u;
-        sm.adj[lane + 32][0] = sm.adj[lane + 32][1] = 0u;
-        // exclusive offsets of rows 0..63 (row lane, then row lane + 32)
-        int inc0 = len0, inc1 = len1;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const int y0 = __shfl_up_sync(0xffffffffu, inc0, o);
-            const int y1 = __shfl_up_sync(0xffffffffu, inc1, o);
-            if (lane >= o) {
-                inc0 += y0;
-                inc1 += y1;
-            }
-        }
-        const int tot0 = __shfl_sync(0xffffffffu, inc0, 31);
-        sm.off[lane] = inc0 - len0;
-        sm.off[lane + 32] = tot0 + inc1 - len1;
-        const int T = tot0 + __shfl_sync(0xffffffffu, inc1, 31);
-        if (lane == 0) {
-            sm.off[64] = T;
-            // root row bounds + V + (row bounds + out-row) of every v in V
-            bytes += 16ull + 20ull * (unsigned long long)L + 4ull * (unsigned long long)T;
-        }
-        __syncwarp();
-        // 2. flattened intersection: element t of the concatenated rows
-        for (int t0 = 0; t0 < T; t0 += 32) {
-            const int t = t0 + lane;
-            if (t < T) {
-                // row: last i with off[i] <= t (rows past L have length 0 and off == T)
-                int lo = 0, hi = L - 1;
-                while (lo < hi) {
-                    const int mid = (lo + hi + 1) >> 1;
-                    if (sm.off[mid] <= t)
-                        lo = mid;
-                    else
-                        hi = mid - 1;
-                }
-                const int32_t u = __ldg(a.ocol + sm.start[lo] + (t - sm.off[lo]));
-                const int c = lower_bound_smem(sm.V, L, u);
-                if (c < L && sm.V[c] == u) {  // local indices L-1-position (expand.cuh)
-                    const int li = L - 1 - lo, lc = L - 1 - c;
-                    atomicOr(&sm.adj[li][lc >> 5], 1u << (lc & 31));
-                    atomicOr(&sm.adj[lc][li >> 5], 1u << (li & 31));
-                }
-            }
-        }
-        __syncwarp();
-        const uint64_t row0 = ((uint64_t)sm.adj[lane][1] << 32) | sm.adj[lane][0];
-        const uint64_t row1 = ((uint64_t)sm.adj[lane + 32][1] << 32) | sm.adj[lane + 32][0];
-        const uint64_t P = L >= 64 ? ~0ull : ((1ull << L) - 1);
-        // 3. bound + children (|C| = 1)
-        int np = 0, ncol = 0;
-        if (a.bound == 1) {
-            uint64_t U = P;
-            while (U) {
-                ++ncol;
-                uint64_t Q = U;
-                while (Q) {
-                    const int v = __ffsll((long long)Q) - 1;
-                    const uint64_t rv0 = __shfl_sync(0xffffffffu, row0, v & 31);
-                    const uint64_t rv1 = __shfl_sync(0xffffffffu, row1, v & 31);
-                    const uint64_t rv = v < 32 ? rv0 : rv1;
-                    Q &= ~rv;
-                    Q &= ~(1ull << v);
-                    U &= ~(1ull << v);
-                    if (lane == 0) {
-                        sm.ord[np] = (uint8_t)v;
-                        sm.colr[np] = (uint8_t)ncol;
-                    }
-                    ++np;
-                }
-            }
+    unsigned long long bytes = 0;  // algorithmic bytes read, tile leaders
+    for (int64_t i0 = warp * 4; i0 < a.count; i0 += nwarps * 4) {
+        const int64_t i = i0 + (lane >> 3);
+        const int32_t r = i < a.count ? __ldg(a.list + i * a.stride) : -1;
+        const int L = r >= 0 ? (int)(__ldg(a.orp + r + 1) - __ldg(a.orp + r)) : 0;
+        if (__all_sync(0xffffffffu, L <= 8)) {
+            if (r >= 0) root_step<8, 1>(a, r, tiles[lane >> 3], bytes);
         } else {
-            if (lane == 0)
-                for (int j = 0; j < L; ++j) {
-                    sm.ord[j] = (uint8_t)j;
-                    sm.colr[j] = (uint8_t)(j + 1);
-                }
-            np = ncol = L;
-        }
-        __syncwarp();
-        int cnt = 0;
-        if (1 + ncol >= a.need) {
-            uint64_t R = P;
-            for (int j = np - 1; j >= 0; --j) {
-                if (1 + sm.colr[j] < a.need) break;
-                const int v = sm.ord[j];
-                const uint64_t rv0 = __shfl_sync(0xffffffffu, row0, v & 31);
-                const uint64_t rv1 = __shfl_sync(0xffffffffu, row1, v & 31);
-                const uint64_t C = R & (v < 32 ? rv0 : rv1);
-                R &= ~(1ull << v);
-                const int pc = __popcll(C);
-                if (pc == 0) {
-                    if (2 >= a.need && lane == 0) {  // {r, v} is a leaf clique of interest
-                        const unsigned long long idx = atomicAdd(a.ctr + 3, 1ull);
-                        if ((int64_t)idx < a.leaf_cap) {
-                            a.leaf_rows[idx * 2] = __ldg(a.order + r);
-                            a.leaf_rows[idx * 2 + 1] = __ldg(a.order + sm.V[L - 1 - v]);
-                        }
-                    }
-                } else if (2 + pc >= a.need) {
-                    if (lane == 0) {
-                        sm.chv[cnt] = (uint8_t)v;
-                        sm.chP[cnt] = C;
-                    }
-                    ++cnt;
-                }
-            }
-        }
-        // 4. materialise surviving roots
-        if (cnt > 0) {
-            unsigned long long s = 0, ab = 0, e0 = 0;
-            if (lane == 0) {
-                s = atomicAdd(a.ctr + 0, 1ull);
-                ab = atomicAdd(a.ctr + 1, (unsigned long long)L);
-                e0 = atomicAdd(a.ctr + 2, (unsigned long long)cnt);
-            }
-            s = __shfl_sync(0xffffffffu, s, 0);
-            ab = __shfl_sync(0xffffffffu, ab, 0);
-            e0 = __shfl_sync(0xffffffffu, e0, 0);
-            __syncwarp();
-            if (lane == 0) {
-                RootInfo ri;
-                ri.r = r;
-                ri.L = L;
-                ri.vbase = vb;
-                ri.abase = (int64_t)ab;
-                a.roots[s] = ri;
-            }
-            if (lane < L) a.adj[ab + lane] = row0;
-            if (lane + 32 < L) a.adj[ab + lane + 32] = row1;
-            for (int j = lane; j < cnt; j += 32) {
-                a.cP[e0 + j] = sm.chP[j];
-                a.cslot[e0 + j] = (int32_t)s;
-                a.cparent[e0 + j] = -1;
-                a.cvloc[e0 + j] = sm.chv[j];
+            for (int t = 0; t < 4; ++t) {
+                const int32_t rt = __shfl_sync(0xffffffffu, r, 8 * t);
+                if (rt < 0) break;
+                root_step<32, 2>(a, rt, sm, bytes);
             }
         }
         __syncwarp();
     }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) bytes += __shfl_xor_sync(0xffffffffu, bytes, o);
     if (lane == 0 && bytes) atomicAdd(a.ctr + 4, bytes);
 }
 
@@ -225,7 +260,7 @@ __global__ void __launch_bounds__(kRootWarps * 32) root_expand_w1(const RootArgs
 
 void launch_root_expand_w1(const RootArgs &a, cudaStream_t s) {
     if (a.count <= 0) return;
-    root_expand_w1<<<grid_for(a.count * 32, kRootWarps * 32, 8), kRootWarps * 32, 0, s>>>(a);
+    root_expand_w1<<<grid_for(a.count * 8, kRootWarps * 32, 8), kRootWarps * 32, 0, s>>>(a);
     MCE_LAUNCH_CHECK();
 }
 
