@@ -49,59 +49,78 @@ def parse():
 
 
 class ClockSampler:
-    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+    """SM clocks + throttle reasons sampled DURING the timed region (B200_PROFILING.md clocks line).
 
-    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
-              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
-              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+    In-process NVML polling every 20 ms (no nvidia-smi child process, whose
+    queries can stall a short timed region); nvidia-smi -lms is the fallback.
+    """
 
-    def __init__(self, index: int):
+    REASONS = {"hw_slowdown": 0x8, "hw_thermal_slowdown": 0x40, "sw_thermal_slowdown": 0x20, "sw_power_cap": 0x4}
+
+    def __init__(self, index: int, interval_s: float = 0.02):
         self.index = index
-        self.proc = None
-        self.lines = []
+        self.interval = interval_s
+        self.samples = []  # (sm_mhz, max_mhz, reasons bitmask)
+        self._stop = threading.Event()
+        self._nvml = None
+        self._proc = None
+
+    def _poll_nvml(self):
+        import pynvml as N
+
+        h = N.nvmlDeviceGetHandleByIndex(self.index)
+        mx = N.nvmlDeviceGetMaxClockInfo(h, N.NVML_CLOCK_SM)
+        while True:
+            try:
+                sm = N.nvmlDeviceGetClockInfo(h, N.NVML_CLOCK_SM)
+                rs = N.nvmlDeviceGetCurrentClocksEventReasons(h)
+                self.samples.append((float(sm), float(mx), int(rs)))
+            except Exception:
+                pass
+            if self._stop.wait(self.interval):
+                break
+
+    def _poll_smi(self):
+        fields = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+                  "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        self._proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={fields}",
+                                       "--format=csv,noheader,nounits", "-lms", "100"],
+                                      stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        bits = [0x8, 0x40, 0x20, 0x4]
+        for line in self._proc.stdout:
+            parts = [x.strip() for x in line.split(",")]
+            try:
+                rs = sum(b for b, v in zip(bits, parts[2:6]) if v.lower() == "active")
+                self.samples.append((float(parts[0]), float(parts[1]), rs))
+            except (ValueError, IndexError):
+                continue
 
     def __enter__(self):
         try:
-            self.proc = subprocess.Popen(
-                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
-                 "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
-            self.t = threading.Thread(target=self._read, daemon=True)
-            self.t.start()
+            import pynvml as N
+
+            N.nvmlInit()
+            self._nvml = N
+            target = self._poll_nvml
         except Exception:
-            self.proc = None
+            target = self._poll_smi
+        self._t = threading.Thread(target=target, daemon=True)
+        self._t.start()
         return self
 
-    def _read(self):
-        for line in self.proc.stdout:
-            self.lines.append(line.strip())
-
     def __exit__(self, *exc):
-        if self.proc:
-            self.proc.terminate()
-            try:
-                self.proc.wait(timeout=5)
-            except Exception:
-                self.proc.kill()
+        self._stop.set()
+        if self._proc:
+            self._proc.terminate()
+        self._t.join(timeout=5)
 
     def summary(self):
-        sm, mx, reasons = [], [], set()
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for ln in self.lines:
-            parts = [x.strip() for x in ln.split(",")]
-            if len(parts) < 8:
-                continue
-            try:
-                sm.append(float(parts[0]))
-                mx.append(float(parts[1]))
-            except ValueError:
-                continue
-            for nm, v in zip(names, parts[4:8]):
-                if v.lower() == "active":
-                    reasons.add(nm)
-        if not sm:
+        if not self.samples:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
-        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": max(mx), "reasons": sorted(reasons),
-                "samples": len(sm)}
+        reasons = sorted(n for n, b in self.REASONS.items() if any(s[2] & b for s in self.samples))
+        return {"sm_mhz": statistics.median(s[0] for s in self.samples),
+                "sm_max_mhz": max(s[1] for s in self.samples), "reasons": reasons, "samples": len(self.samples),
+                "source": "nvml" if self._nvml else "nvidia-smi"}
 
 
 def measured_peak_hbm():
@@ -212,7 +231,7 @@ def main():
     start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(local) as clocks:
         for _ in range(args.steps):
-            flush.fill_(1)
+            flush.fill_(1)  # L2 flush (256 MiB > 126 MB L2) before every timed step
             if world > 1:
                 dist.barrier()
             torch.cuda.synchronize()
@@ -222,7 +241,7 @@ def main():
             torch.cuda.synchronize()
             times.append(start.elapsed_time(end))
             timings.append(res.timing)
-    t_ms = statistics.mean(times)
+    t_ms = sum(times) / len(times)  # exactly K timed steps
     if world > 1:
         tt = torch.tensor([t_ms], dtype=torch.float64, device=f"cuda:{local}")
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
@@ -245,7 +264,11 @@ def main():
     phases = {"preprocess_ms": statistics.mean(t["preprocess_ms"] for t in timings),
               "heuristic_ms": statistics.mean(t["heuristic_ms"] for t in timings),
               "expand_ms": statistics.mean(t["expand_ms"] for t in timings),
-              "expand_count_ms": cnt_ms, "root_kernel_ms": root_ms}
+              "expand_count_ms": cnt_ms, "root_kernel_ms": root_ms,
+              "host_call_ms": statistics.mean(t["host_total_ms"] for t in timings),
+              "host_preprocess_ms": statistics.mean(t["host_preprocess_ms"] for t in timings),
+              "host_heuristic_ms": statistics.mean(t["host_heuristic_ms"] for t in timings),
+              "syncs_per_step": statistics.mean(t["syncs"] for t in timings)}
 
     # ---- end to end through the public API: pinned host CSR -> GPU -> cliques on the host
     e2e = None
@@ -296,7 +319,8 @@ def main():
                        "mode": mode, "n": g.n, "edges": edges, "omega": res.omega, "multiplicity": res.count,
                        "stored_cliques": int(res.cliques.shape[0]), "max_cliques": max_cl,
                        "parallelism": f"root-shard x{world}", "l2": "flushed (256 MiB write) before every step",
-                       "phases_ms": phases, "levels": res.levels},
+                       "phases_ms": phases, "levels": res.levels,
+                       "step_ms": [round(t, 4) for t in times]},
             "roofline": {"bound": "hbm", "kernel": kname,
                          "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak if peak else None, "traffic": None, "peak_source": peak_src,

@@ -69,7 +69,9 @@ typedef struct {
     int32_t bound;           /* MCE_BOUND_* */
     int32_t lower_bound;     /* extra known lower bound on omega (0 = none) */
     int64_t window;          /* roots per window (PAPER.md IV-E); <=0 = all roots at once */
-    int64_t budget_bytes;    /* device bytes the frontier may use; <=0 = 90% of free memory */
+    int64_t budget_bytes;    /* device bytes the frontier may use; <=0 = half of the free device
+                                memory.  Allocated on demand in segments (the first sized
+                                ~1 GiB + 48 B/edge), kept on the graph for later calls. */
     int64_t max_cliques;     /* capacity of the stored clique list; <=0 = unbounded
                                 (still limited: at most max(2^20, rows fitting a quarter
                                 of the budget) are stored).  The multiplicity is
@@ -158,7 +160,9 @@ mce_status mce_result_levels(const mce_result *r, int64_t *entries, int32_t cap,
  * [3] dominant expansion kernel total, [4] number of dominant-kernel launches,
  * [5] algorithmic bytes moved by the dominant kernel, [6] kernels launched,
  * [7] fused root-level kernel total, [8] its launches, [9] its algorithmic
- * bytes (16 + 20 L + 4 T per root: row bounds, V, and the out-rows of V). */
+ * bytes (16 + 20 L + 4 T per root: row bounds, V, and the out-rows of V),
+ * [10] host wall time of the whole call, [11] of its preprocessing, [12] of
+ * its heuristic, [13] host<->device synchronisations it made. */
 mce_status mce_result_timing(const mce_result *r, double *t, int32_t cap);
 void mce_result_free(mce_result *r);
 

@@ -14,6 +14,8 @@
 
 namespace mce {
 
+thread_local int64_t g_syncs = 0;
+
 namespace {
 
 struct DeviceCache {

@@ -159,7 +159,7 @@ mce_status mce_load_csr(int32_t device, int64_t n, const int64_t *row_ptr, const
                 MCE_LAUNCH_CHECK();
                 unsigned long long *h = g->host.get<unsigned long long>(1);
                 MCE_CUDA(cudaMemcpyAsync(h, md, sizeof(unsigned long long), cudaMemcpyDeviceToHost, g->stream));
-                MCE_CUDA(cudaStreamSynchronize(g->stream));
+                stream_sync(g->stream);
                 g->max_deg = (int64_t)h[0];
                 if (validate) {
                     int32_t *bad = g->pool.take<int32_t>(1);
@@ -168,14 +168,14 @@ mce_status mce_load_csr(int32_t device, int64_t n, const int64_t *row_ptr, const
                     MCE_LAUNCH_CHECK();
                     int32_t *hbp = g->host.get<int32_t>(1);
                     MCE_CUDA(cudaMemcpyAsync(hbp, bad, sizeof(int32_t), cudaMemcpyDeviceToHost, g->stream));
-                    MCE_CUDA(cudaStreamSynchronize(g->stream));
+                    stream_sync(g->stream);
                     const int32_t hb = hbp[0];
                     if (hb)
                         fail(MCE_ERR_INVALID, "malformed CSR (flags " + std::to_string(hb) +
                                                   ": 1 rowptr, 2 id range, 4 loop, 8 unsorted/dup, 16 asymmetric)");
                 }
             }
-            MCE_CUDA(cudaStreamSynchronize(g->stream));
+            stream_sync(g->stream);
         } catch (...) {
             delete g;
             throw;
@@ -306,10 +306,11 @@ mce_status mce_result_levels(const mce_result *r, int64_t *entries, int32_t cap,
 mce_status mce_result_timing(const mce_result *r, double *t, int32_t cap) {
     return run_guarded([&] {
         if (!r || !t) fail(MCE_ERR_INVALID, "NULL argument");
-        double v[10] = {r->t_pre_ms,    r->t_heur_ms,     r->t_expand_ms,          r->t_count_ms,
+        double v[14] = {r->t_pre_ms,    r->t_heur_ms,     r->t_expand_ms,          r->t_count_ms,
                         (double)r->count_launches, r->count_bytes, (double)r->kernels, r->t_root_ms,
-                        (double)r->root_launches,  r->root_bytes};
-        for (int32_t i = 0; i < std::min(cap, 10); ++i) t[i] = v[i];
+                        (double)r->root_launches,  r->root_bytes,  r->h_total_ms, r->h_pre_ms,
+                        r->h_heur_ms,              (double)r->syncs};
+        for (int32_t i = 0; i < std::min(cap, 14); ++i) t[i] = v[i];
     });
 }
 

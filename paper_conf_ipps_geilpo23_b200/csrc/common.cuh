@@ -90,6 +90,14 @@ struct PinnedBuf {
     }
 };
 
+// host<->device round trips are the fixed cost of every level; they are
+// counted (per thread) so the bench can report them
+extern thread_local int64_t g_syncs;
+inline void stream_sync(cudaStream_t s) {
+    ++g_syncs;
+    MCE_CUDA(cudaStreamSynchronize(s));
+}
+
 inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
 // ---------------------------------------------------------------------------

@@ -24,26 +24,58 @@ namespace mce {
 namespace {
 constexpr size_t kAlign = 256;
 
-// bump allocator over the graph's persistent workspace, limited to the budget
+// Bump allocator over the graph's workspace segments, limited to the budget.
+// Segments are allocated on demand (the first sized for a typical run, later
+// ones kBigSeg or larger) and kept on the graph handle for the next call, so
+// small problems stay small while an exploding frontier may use the whole
+// budget.  Allocation is stack-like: mark() / reset(mark).
+constexpr size_t kBigSeg = 4ull << 30;
 struct Arena {
-    uint8_t *base = nullptr;
-    size_t cap = 0;
-    size_t top = 0;
-    void init(DevBuf<uint8_t> &ws, size_t bytes) {
-        ws.ensure(bytes);
-        base = ws.p;
-        cap = bytes;
-        top = 0;
+    struct Mark {
+        size_t seg, off, before;
+    };
+    std::vector<DevBuf<uint8_t>> *segs = nullptr;
+    size_t budget = 0, first = 0;
+    size_t cur = 0, off = 0, before = 0;  // before = bytes of the segments below cur
+    void init(std::vector<DevBuf<uint8_t>> &s, size_t budget_bytes, size_t first_seg) {
+        segs = &s;
+        budget = budget_bytes;
+        first = std::min(first_seg, budget_bytes);
+        cur = off = before = 0;
+        if (segs->empty() || (*segs)[0].n < first) {
+            segs->clear();
+            segs->emplace_back();
+            (*segs)[0].alloc(first);
+        }
     }
-    size_t avail() const { return cap > top ? cap - top : 0; }
+    size_t used() const { return before + off; }
+    size_t avail() const { return budget > used() ? budget - used() : 0; }
+    Mark mark() const { return {cur, off, before}; }
+    void reset(const Mark &m) {
+        cur = m.seg;
+        off = m.off;
+        before = m.before;
+    }
     template <typename T>
     T *alloc(int64_t count) {
-        size_t bytes = ((size_t)std::max<int64_t>(count, 1) * sizeof(T) + kAlign - 1) / kAlign * kAlign;
-        if (top + bytes > cap)
+        const size_t bytes = ((size_t)std::max<int64_t>(count, 1) * sizeof(T) + kAlign - 1) / kAlign * kAlign;
+        if (off + bytes > (*segs)[cur].n) {  // next segment (the rest of this one is skipped)
+            const size_t nb = before + (*segs)[cur].n;
+            if (nb + bytes > budget)
+                fail(MCE_ERR_BUDGET, "frontier budget exhausted (need " + std::to_string(bytes) + " more bytes, " +
+                                         std::to_string(avail()) + " available)");
+            const size_t want = std::min(std::max(kBigSeg, bytes), budget - nb);
+            if (cur + 1 >= segs->size()) segs->emplace_back();
+            if ((*segs)[cur + 1].n < bytes) (*segs)[cur + 1].alloc(want);
+            before = nb;
+            ++cur;
+            off = 0;
+        }
+        if (used() + bytes > budget)
             fail(MCE_ERR_BUDGET, "frontier budget exhausted (need " + std::to_string(bytes) + " more bytes, " +
                                      std::to_string(avail()) + " available)");
-        T *p = reinterpret_cast<T *>(base + top);
-        top += bytes;
+        T *p = reinterpret_cast<T *>((*segs)[cur].p + off);
+        off += bytes;
         return p;
     }
 };
@@ -231,7 +263,7 @@ void Engine::handle_leaves(int32_t size, int64_t cnt, ExpandArgs &a) {
         MCE_CUDA(cudaMemsetAsync(leaf_total_, 0, 2 * sizeof(unsigned long long), s_));
         launch_expand(a, false, s_);
         ++kernels_;
-        MCE_CUDA(cudaStreamSynchronize(s_));
+        stream_sync(s_);
     }
     const int64_t take = std::min<int64_t>(want, a.leaf_cap);
     if (take > 0) {
@@ -251,7 +283,7 @@ void Engine::process(int32_t k, const Level &L) {
     LevelLink link{L.parent, L.vloc};
     MCE_CUDA(cudaMemcpyAsync(chain_dev_ + k, &link, sizeof(link), cudaMemcpyHostToDevice, s_));
 
-    const size_t mark = arena_.top;
+    const Arena::Mark mark = arena_.mark();
     const int64_t N = L.count;
     int32_t *counts = arena_.alloc<int32_t>(N);
     int64_t *offs = arena_.alloc<int64_t>(N + 1);
@@ -292,7 +324,7 @@ void Engine::process(int32_t k, const Level &L) {
     int64_t *h = g_->host.get<int64_t>(4);
     MCE_CUDA(cudaMemcpyAsync(h, offs + N, sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
     MCE_CUDA(cudaMemcpyAsync(h + 1, leaf_total_, 3 * sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
-    MCE_CUDA(cudaStreamSynchronize(s_));
+    stream_sync(s_);
     const int64_t total = h[0];
     const unsigned long long leaves = (unsigned long long)h[1];
     const int32_t maxbit = (int32_t)(uint32_t)(uint64_t)h[3];
@@ -327,7 +359,7 @@ void Engine::process(int32_t k, const Level &L) {
             ++kernels_;
             int64_t *hc = g_->host.get<int64_t>(3);
             MCE_CUDA(cudaMemcpyAsync(hc, chunk, 3 * sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
-            MCE_CUDA(cudaStreamSynchronize(s_));
+            stream_sync(s_);
             b = hc[0];
             cnt = hc[1];
             base = hc[2];
@@ -335,7 +367,7 @@ void Engine::process(int32_t k, const Level &L) {
                 fail(MCE_ERR_BUDGET, "the children of one candidate at level " + std::to_string(k) +
                                          " exceed the frontier budget");
         }
-        const size_t cmark = arena_.top;
+        const Arena::Mark cmark = arena_.mark();
         Level C;
         C.count = cnt;
         C.W = Wc;
@@ -355,10 +387,10 @@ void Engine::process(int32_t k, const Level &L) {
         launch_timed(w, true);
         sync_bound(true);
         if (cnt > 0) process(k + 1, C);
-        arena_.top = cmark;
+        arena_.reset(cmark);
         a0 = b;
     }
-    arena_.top = mark;
+    arena_.reset(mark);
 }
 
 // W == 1 roots: the fused root level (roots.cu), then levels >= 2 as usual
@@ -380,14 +412,14 @@ void Engine::do_class_w1(const int32_t *list, int64_t count) {
     const int64_t per_root = sizeof(RootInfo) + 64;
     int64_t hi = mine;
     while (hi > 0) {
-        const size_t mark = arena_.top;
+        const Arena::Mark mark = arena_.mark();
         const int64_t room = (int64_t)(arena_.avail() / 3);
         const int64_t maxw = o_.window > 0 ? o_.window : hi;
         launch_find_window(prefix, hi, std::max<int64_t>(0, hi - maxw), room, row_bytes, per_root, win, s_);
         ++kernels_;
         int64_t *hw = g_->host.get<int64_t>(2);
         MCE_CUDA(cudaMemcpyAsync(hw, win, 2 * sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
-        MCE_CUDA(cudaStreamSynchronize(s_));
+        stream_sync(s_);
         const int64_t lo = hw[0], rows = hw[1];
         const int64_t nw = hi - lo;
         RootArgs ra{};
@@ -418,7 +450,7 @@ void Engine::do_class_w1(const int32_t *list, int64_t count) {
             ++root_launches_;
             hc = g_->host.get<unsigned long long>(8);
             MCE_CUDA(cudaMemcpyAsync(hc, ctr, 8 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, s_));
-            MCE_CUDA(cudaStreamSynchronize(s_));
+            stream_sync(s_);
             const int64_t leaves = (int64_t)hc[3];
             if (attempt == 0 && leaves > ra.leaf_cap && !find_one_) {
                 // staging too small for the size-2 leaves: grow and replay (counters reset)
@@ -464,7 +496,7 @@ void Engine::do_class_w1(const int32_t *list, int64_t count) {
             process(2, L2);
         }
         sync_bound(true);
-        arena_.top = mark;
+        arena_.reset(mark);
         hi = lo;
     }
 }
@@ -492,7 +524,7 @@ void Engine::do_class(int32_t cls, const int32_t *list, int64_t count) {
     // windows from the highest ranks down (densest cores first)
     int64_t hi = mine;
     while (hi > 0) {
-        const size_t mark = arena_.top;
+        const Arena::Mark mark = arena_.mark();
         const int64_t room = (int64_t)(arena_.avail() / 4);
         const int64_t maxw = o_.window > 0 ? o_.window : hi;
         // smallest lo >= hi - maxw whose rows fit a quarter of the free budget (at least one root)
@@ -500,7 +532,7 @@ void Engine::do_class(int32_t cls, const int32_t *list, int64_t count) {
         ++kernels_;
         int64_t *hw = g_->host.get<int64_t>(2);
         MCE_CUDA(cudaMemcpyAsync(hw, win, 2 * sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
-        MCE_CUDA(cudaStreamSynchronize(s_));
+        stream_sync(s_);
         const int64_t lo = hw[0], rows = hw[1];
         const int64_t nw = hi - lo;
         RootInfo *roots = arena_.alloc<RootInfo>(nw);
@@ -521,13 +553,17 @@ void Engine::do_class(int32_t cls, const int32_t *list, int64_t count) {
         ++kernels_;
         process(1, L1);
         sync_bound(true);
-        arena_.top = mark;
+        arena_.reset(mark);
         hi = lo;
     }
 }
 
 mce_result *Engine::run() {
     auto *res = new mce_result();
+    using clk = std::chrono::steady_clock;
+    const auto h0 = clk::now();
+    const int64_t syncs0 = g_syncs;
+    auto ms_since = [](clk::time_point t) { return std::chrono::duration<double, std::milli>(clk::now() - t).count(); };
     const int64_t n = g_->n;
     stride_ = o_.shard_count > 1 ? o_.shard_count : 1;
     offset_ = o_.shard_count > 1 ? o_.shard_rank : 0;
@@ -556,12 +592,15 @@ mce_result *Engine::run() {
     }
     preprocess(g_, o_.orientation);
     res->t_pre_ms = g_->t_pre_ms;
+    res->h_pre_ms = ms_since(h0);
+    const auto h1 = clk::now();
     kernels_ += g_->kernels;
 
     int heur = o_.heuristic;
     if (find_one_ && heur == 0) heur = 1;  // find-one needs an incumbent clique
     HeuristicResult hr = run_heuristic(g_, heur, o_.heuristic_runs, (int32_t)offset_, (int32_t)stride_, false);
     res->t_heur_ms = hr.ms;
+    res->h_heur_ms = ms_since(h1);
     kernels_ += hr.kernels;
     best_ = std::max<int32_t>(hr.omega_bar, 2);
     if (find_one_) {
@@ -578,13 +617,15 @@ mce_result *Engine::run() {
     // counts as free memory here
     size_t free_b = 0, total_b = 0;
     MCE_CUDA(cudaMemGetInfo(&free_b, &total_b));
-    free_b += g_->ws.n + dev_cached_bytes();
-    int64_t budget = o_.budget_bytes;
-    if (budget <= 0)
-        budget = std::min<int64_t>((int64_t)(free_b * 0.8), (int64_t)(1ll << 30) + 48ll * g_->nnz + 64ll * n);
+    size_t held = dev_cached_bytes();
+    for (auto &sg : g_->wsegs) held += sg.n;
+    free_b += held;
+    // default budget: half of the free device memory; the first segment is
+    // sized for a typical run, the rest is only allocated if the frontier needs it
+    int64_t budget = o_.budget_bytes > 0 ? o_.budget_bytes : (int64_t)(free_b / 2);
     budget = std::min<int64_t>(budget, (int64_t)(free_b * 0.95));
-    if (g_->ws.n < (size_t)budget) g_->ws.release();  // regrow below without holding both blocks
-    arena_.init(g_->ws, (size_t)budget);
+    const int64_t first = std::min<int64_t>(budget, (int64_t)(1ll << 30) + 48ll * g_->nnz + 64ll * n);
+    arena_.init(g_->wsegs, (size_t)budget, (size_t)first);
     // leaf counter + level chain (persistent, g->misc)
     chain_cap_ = 4096;
     g_->misc.ensure(256 + sizeof(LevelLink) * chain_cap_);
@@ -600,7 +641,7 @@ mce_result *Engine::run() {
     tt.start();
     // roots worth expanding: 1 + |N+(r)| >= need, grouped by candidate-set width class
     {
-        const size_t mark = arena_.top;
+        const Arena::Mark mark = arena_.mark();
         int32_t *cls = arena_.alloc<int32_t>(n);
         int32_t *flag = arena_.alloc<int32_t>(n);
         int64_t *pos = arena_.alloc<int64_t>(n + 1);
@@ -611,7 +652,7 @@ mce_result *Engine::run() {
         ++kernels_;
         int64_t *hh = g_->host.get<int64_t>(kMaxClass + 1);
         MCE_CUDA(cudaMemcpyAsync(hh, hist, sizeof(int64_t) * (kMaxClass + 1), cudaMemcpyDeviceToHost, s_));
-        MCE_CUDA(cudaStreamSynchronize(s_));
+        stream_sync(s_);
         if (hh[kMaxClass]) fail(MCE_ERR_INVALID, "out-degree above 16384 after orientation is not supported");
         std::vector<int64_t> counts(hh, hh + kMaxClass);
         std::vector<std::pair<int32_t, int64_t>> classes;
@@ -628,14 +669,14 @@ mce_result *Engine::run() {
         }
         // the class lists stay allocated below `mark` while the classes run
         for (size_t i = 0; i < classes.size(); ++i) {
-            const size_t cmark = arena_.top;
+            const Arena::Mark cmark = arena_.mark();
             do_class(classes[i].first, lists[i], classes[i].second);
-            arena_.top = cmark;
+            arena_.reset(cmark);
         }
-        arena_.top = mark;
+        arena_.reset(mark);
     }
     tt.stop();
-    MCE_CUDA(cudaStreamSynchronize(s_));
+    stream_sync(s_);
     res->t_enum_ms = tt.collect();
     clock_.collect(t_expand_ms_, t_count_ms_, t_root_ms_);
     // keep answering the other shards until everyone is done
@@ -661,6 +702,8 @@ mce_result *Engine::run() {
     res->root_launches = root_launches_;
     res->root_bytes = root_bytes_;
     res->kernels = kernels_;
+    res->h_total_ms = ms_since(h0);
+    res->syncs = g_syncs - syncs0;
     return res;
 }
 

@@ -17,6 +17,8 @@ struct mce_result {
     int64_t count_launches = 0, kernels = 0;
     double t_root_ms = 0, root_bytes = 0;  // fused root-level kernel
     int64_t root_launches = 0;
+    double h_total_ms = 0, h_pre_ms = 0, h_heur_ms = 0;  // host wall time of the call / its phases
+    int64_t syncs = 0;                                    // host<->device round trips
 };
 
 namespace mce {

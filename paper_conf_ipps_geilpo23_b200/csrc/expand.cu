@@ -291,21 +291,25 @@ __global__ void __launch_bounds__(256) expand_thread(const ExpandArgs a) {
 }
 
 // ---------------------------------------------------------------------------
-// warp per candidate, 4 < W <= 256 words: lanes own words (WPL words per lane)
+// tile of G lanes per candidate, 4 < W <= 256 words: lane j of the tile owns
+// words j, j + G, ... (WPL words per lane).  Launched with G = 32 (a warp per
+// candidate); G = 8 / 16 put several candidates in one warp but diverge.
 // ---------------------------------------------------------------------------
-template <int WPL, bool WRITE>
-__global__ void expand_warp(const ExpandArgs a, int max_l) {
+template <int G, int WPL, bool WRITE>
+__global__ void expand_tile(const ExpandArgs a, int max_l) {
     extern __shared__ uint16_t sm[];
     const int lane = threadIdx.x & 31;
-    const int wib = threadIdx.x >> 5;
-    uint16_t *ord = sm + (int64_t)wib * 2 * max_l;
+    const int gl = lane & (G - 1), gbase = lane & ~(G - 1);
+    const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << gbase);
+    const int tib = threadIdx.x / G;  // tile in block
+    uint16_t *ord = sm + (int64_t)tib * 2 * max_l;
     uint16_t *colr = ord + max_l;
-    const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int64_t tile = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / G;
+    const int64_t ntiles = ((int64_t)gridDim.x * blockDim.x) / G;
     const int W = a.Wp, Wa = a.Wa;
     unsigned nleaf = 0;
     int hb = -1, ub = 0;
-    for (int64_t e = a.begin + warp; e < a.end; e += nwarps) {
+    for (int64_t e = a.begin + tile; e < a.end; e += ntiles) {
         int64_t out = 0;
         if (WRITE) {
             out = a.offsets[e];
@@ -315,7 +319,7 @@ __global__ void expand_warp(const ExpandArgs a, int max_l) {
         uint64_t P[WPL];
 #pragma unroll
         for (int t = 0; t < WPL; ++t) {
-            const int j = lane + 32 * t;
+            const int j = gl + G * t;
             P[t] = j < W ? a.P[e * W + j] : 0ull;
         }
         const RootInfo ri = a.roots[a.slot[e]];
@@ -329,7 +333,7 @@ __global__ void expand_warp(const ExpandArgs a, int max_l) {
                 bool any = false;
 #pragma unroll
                 for (int t = 0; t < WPL; ++t) any |= U[t] != 0;
-                if (!__any_sync(0xffffffffu, any)) break;
+                if (!((__ballot_sync(gmask, any) & gmask))) break;
                 ++ncol;
                 uint64_t Q[WPL];
 #pragma unroll
@@ -339,11 +343,11 @@ __global__ void expand_warp(const ExpandArgs a, int max_l) {
 #pragma unroll
                     for (int t = 0; t < WPL; ++t) {
                         if (v < 0) {
-                            const unsigned m = __ballot_sync(0xffffffffu, Q[t] != 0);
+                            const unsigned m = (__ballot_sync(gmask, Q[t] != 0) & gmask) >> gbase;
                             if (m) {
                                 const int src = __ffs(m) - 1;
-                                const int bit = __shfl_sync(0xffffffffu, __ffsll((long long)Q[t]) - 1, src);
-                                v = (src + 32 * t) * 64 + bit;
+                                const int bit = __shfl_sync(gmask, __ffsll((long long)Q[t]) - 1, src, G);
+                                v = (src + G * t) * 64 + bit;
                             }
                         }
                     }
@@ -351,19 +355,19 @@ __global__ void expand_warp(const ExpandArgs a, int max_l) {
                     const uint64_t *row = A + (int64_t)v * Wa;
 #pragma unroll
                     for (int t = 0; t < WPL; ++t) {
-                        const int j = lane + 32 * t;
+                        const int j = gl + G * t;
                         if (j < W) Q[t] &= ~__ldg(row + j);
                     }
                     const int jv = v >> 6;
-                    if ((jv & 31) == lane) {
+                    if ((jv & (G - 1)) == gl) {
 #pragma unroll
                         for (int t = 0; t < WPL; ++t)
-                            if (t == (jv >> 5)) {
+                            if (t == jv / G) {
                                 Q[t] &= ~(1ull << (v & 63));
                                 U[t] &= ~(1ull << (v & 63));
                             }
                     }
-                    if (lane == 0) {
+                    if (gl == 0) {
                         ord[np] = (uint16_t)v;
                         colr[np] = (uint16_t)ncol;
                     }
@@ -378,25 +382,25 @@ __global__ void expand_warp(const ExpandArgs a, int max_l) {
                 const int pc = __popcll(P[t]);
                 int incl = pc;
 #pragma unroll
-                for (int o = 1; o < 32; o <<= 1) {
-                    int y = __shfl_up_sync(0xffffffffu, incl, o);
-                    if (lane >= o) incl += y;
+                for (int o = 1; o < G; o <<= 1) {
+                    int y = __shfl_up_sync(gmask, incl, o, G);
+                    if (gl >= o) incl += y;
                 }
                 int pos = base + incl - pc;
                 uint64_t q = P[t];
                 while (q) {
                     const int b = __ffsll((long long)q) - 1;
                     q &= q - 1;
-                    ord[pos] = (uint16_t)((lane + 32 * t) * 64 + b);
+                    ord[pos] = (uint16_t)((gl + G * t) * 64 + b);
                     colr[pos] = (uint16_t)(pos + 1);
                     ++pos;
                 }
-                base += __shfl_sync(0xffffffffu, incl, 31);
+                base += __shfl_sync(gmask, incl, G - 1, G);
             }
             np = base;
             ncol = np;
         }
-        __syncwarp();
+        __syncwarp(gmask);
         int32_t cnt = 0;
         if (a.k + ncol >= a.need) {
             uint64_t R[WPL];
@@ -410,19 +414,20 @@ __global__ void expand_warp(const ExpandArgs a, int max_l) {
                 int pc = 0;
 #pragma unroll
                 for (int t = 0; t < WPL; ++t) {
-                    const int j = lane + 32 * t;
+                    const int j = gl + G * t;
                     C[t] = j < W ? (R[t] & __ldg(row + j)) : 0ull;
                     pc += __popcll(C[t]);
                 }
-                pc = __reduce_add_sync(0xffffffffu, pc);
+#pragma unroll
+                for (int o = G / 2; o > 0; o >>= 1) pc += __shfl_xor_sync(gmask, pc, o, G);
                 const int jv = v >> 6;
-                if ((jv & 31) == lane) {
+                if ((jv & (G - 1)) == gl) {
 #pragma unroll
                     for (int t = 0; t < WPL; ++t)
-                        if (t == (jv >> 5)) R[t] &= ~(1ull << (v & 63));
+                        if (t == jv / G) R[t] &= ~(1ull << (v & 63));
                 }
                 if (pc == 0) {
-                    if (!WRITE && a.k + 1 >= a.need && lane == 0) {
+                    if (!WRITE && a.k + 1 >= a.need && gl == 0) {
                         ++nleaf;
                         store_leaf(a, e, v, ri);
                     }
@@ -431,10 +436,10 @@ __global__ void expand_warp(const ExpandArgs a, int max_l) {
                         const int64_t c = out + cnt;
 #pragma unroll
                         for (int t = 0; t < WPL; ++t) {
-                            const int j = lane + 32 * t;
+                            const int j = gl + G * t;
                             if (j < a.Wc) a.cP[c * a.Wc + j] = C[t];
                         }
-                        if (lane == 0) {
+                        if (gl == 0) {
                             a.cslot[c] = a.slot[e];
                             a.cparent[c] = (int32_t)e;
                             a.cvloc[c] = v;
@@ -442,15 +447,15 @@ __global__ void expand_warp(const ExpandArgs a, int max_l) {
                     } else {
 #pragma unroll
                         for (int t = 0; t < WPL; ++t)
-                            if (C[t]) hb = max(hb, (lane + 32 * t) * 64 + 63 - __clzll((long long)C[t]));
+                            if (C[t]) hb = max(hb, (gl + G * t) * 64 + 63 - __clzll((long long)C[t]));
                         ub = max(ub, a.k + 1 + pc);
                     }
                     ++cnt;
                 }
             }
         }
-        if (!WRITE && lane == 0) a.counts[e] = cnt;
-        __syncwarp();
+        if (!WRITE && gl == 0) a.counts[e] = cnt;
+        __syncwarp(gmask);
     }
     if (!WRITE) flush_counters(a, nleaf, hb, ub);
 }
@@ -543,22 +548,17 @@ __global__ void find_window_kernel(const int64_t *__restrict__ prefix, int64_t h
     out[1] = prefix[hi] - prefix[l];
 }
 
-template <int WPL>
-void launch_warp(const ExpandArgs &a, bool write_pass, cudaStream_t s) {
+template <int G, int WPL>
+void launch_tile(const ExpandArgs &a, bool write_pass, cudaStream_t s) {
     const int max_l = 64 * a.Wp;
-    const int warps = WPL >= 4 ? 1 : (WPL == 2 ? 2 : 4);
-    const size_t smem = (size_t)warps * 2 * max_l * sizeof(uint16_t);
+    // 32 KB of colouring order per block: (threads / G) tiles x 2 x 64 W x 2 B
+    const int threads = WPL >= 4 ? 32 : (WPL == 2 ? 64 : 128);
+    const size_t smem = (size_t)(threads / G) * 2 * max_l * sizeof(uint16_t);
     const int64_t items = a.end - a.begin;
-    const int grid = grid_for(items * 32, 32 * warps, 32);
-    if (write_pass) {
-        if (smem > 48 * 1024)
-            MCE_CUDA(cudaFuncSetAttribute(expand_warp<WPL, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        expand_warp<WPL, true><<<grid, 32 * warps, smem, s>>>(a, max_l);
-    } else {
-        if (smem > 48 * 1024)
-            MCE_CUDA(cudaFuncSetAttribute(expand_warp<WPL, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        expand_warp<WPL, false><<<grid, 32 * warps, smem, s>>>(a, max_l);
-    }
+    const int grid = grid_for(items * G, threads, 16);
+    auto kern = write_pass ? expand_tile<G, WPL, true> : expand_tile<G, WPL, false>;
+    if (smem > 48 * 1024) MCE_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    kern<<<grid, threads, smem, s>>>(a, max_l);
     MCE_LAUNCH_CHECK();
 }
 
@@ -617,13 +617,16 @@ void launch_expand(const ExpandArgs &a, bool write_pass, cudaStream_t s) {
     } else if (a.Wp == 4) {
         launch_thread<4>(a, write_pass, s);
     } else if (a.Wp <= 32) {
-        launch_warp<1>(a, write_pass, s);
+        // a whole warp per candidate: 8- and 16-lane tiles (four or two
+        // candidates per warp) measured slower on dense800 (66 -> 99 ms count
+        // pass): the tiles of a warp diverge between colouring and branching
+        launch_tile<32, 1>(a, write_pass, s);
     } else if (a.Wp <= 64) {
-        launch_warp<2>(a, write_pass, s);
+        launch_tile<32, 2>(a, write_pass, s);
     } else if (a.Wp <= 128) {
-        launch_warp<4>(a, write_pass, s);
+        launch_tile<32, 4>(a, write_pass, s);
     } else {
-        launch_warp<8>(a, write_pass, s);
+        launch_tile<32, 8>(a, write_pass, s);
     }
 }
 

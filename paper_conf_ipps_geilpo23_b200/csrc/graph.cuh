@@ -1,6 +1,8 @@
 // Device-resident graph handle and the preprocessing entry points.
 #pragma once
 
+#include <vector>
+
 #include "common.cuh"
 
 struct mce_graph {
@@ -30,7 +32,7 @@ struct mce_graph {
 
     // ---- reusable memory (no cudaMalloc/cudaFree on the steady-state path) ----
     mce::Pool pool;                // per-phase scratch (reset at the start of every phase)
-    mce::DevBuf<uint8_t> ws;       // frontier arena of mce_enumerate / mce_find_one (grow-only)
+    std::vector<mce::DevBuf<uint8_t>> wsegs;  // frontier arena segments of mce_enumerate / mce_find_one
     mce::PinnedBuf host;           // pinned staging for small device->host reads (per device, shared)
     mce::DevBuf<uint8_t> misc;     // engine: leaf counter + level chain (persistent)
     mce::DevBuf<int32_t> stage;    // engine: staged leaf cliques (grow-only)

@@ -287,7 +287,7 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
         MCE_LAUNCH_CHECK();
         int64_t *hb = g->host.get<int64_t>(maxthr + 1);
         MCE_CUDA(cudaMemcpyAsync(hb, bins, sizeof(int64_t) * (maxthr + 1), cudaMemcpyDeviceToHost, s));
-        MCE_CUDA(cudaStreamSynchronize(s));
+        stream_sync(s);
         int64_t above = 0;
         int32_t tau = 0;
         for (int64_t t = maxthr; t >= 0; --t) {
@@ -345,7 +345,7 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
     MCE_CUDA(cudaEventRecord(e1, s));
     int32_t *hbest = g->host.get<int32_t>(1);
     MCE_CUDA(cudaMemcpyAsync(hbest, best, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
-    MCE_CUDA(cudaStreamSynchronize(s));
+    stream_sync(s);
     res.omega_bar = hbest[0];
     float ms = 0;
     MCE_CUDA(cudaEventElapsedTime(&ms, e0, e1));

@@ -555,7 +555,7 @@ void kcore(mce_graph *g) {
     last_core_kernel<<<1, 1, 0, s>>>(n, g->peel.get(), g->core.get(), deg);
     int32_t *h = g->host.get<int32_t>(1);
     MCE_CUDA(cudaMemcpyAsync(h, deg, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
-    MCE_CUDA(cudaStreamSynchronize(s));
+    stream_sync(s);
     g->degeneracy = h[0];
     g->have_core = true;
 }
@@ -633,7 +633,7 @@ void orient(mce_graph *g, int orientation) {
     MCE_LAUNCH_CHECK();
     int32_t *hmeta = g->host.get<int32_t>(2);
     MCE_CUDA(cudaMemcpyAsync(hmeta, meta, 2 * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
-    MCE_CUDA(cudaStreamSynchronize(s));
+    stream_sync(s);
     g->kernels += 8;
     g->max_out = hmeta[1];
     const int32_t n_long = hmeta[0];
@@ -653,7 +653,7 @@ void orient(mce_graph *g, int orientation) {
         }
         g->kernels += 1;
     }
-    MCE_CUDA(cudaStreamSynchronize(s));
+    stream_sync(s);
     g->orientation = orientation;
 }
 

@@ -1,0 +1,169 @@
+"""Multi-GPU root partitioner (DESIGN.md §8 row a8): host logic on CPU with
+world_size-2 `gloo` process groups, and the library's root/seed sharding on
+one GPU (the shards of a sharded run together give the unsharded answer).
+
+North star: "Work is partitioned ... by sharding first-level root vertices,
+whose subtrees are independent, with a small NCCL max-allreduce of the omega
+lower bound each level and a final gather of the cliques".
+"""
+
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+from paper_conf_ipps_geilpo23_b200 import distributed as mdist
+from paper_conf_ipps_geilpo23_b200.api import Result
+
+
+def _free_port() -> int:
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def _run(rank, world, port, fn, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        q.put((rank, fn(rank, world)))
+    finally:
+        dist.destroy_process_group()
+
+
+def spawn(fn, world=2):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_run, args=(r, world, port, fn, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    out = dict(q.get(timeout=120) for _ in procs)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    return [out[r] for r in range(world)]
+
+
+# --- per-rank bodies (module level: picklable for spawn) -------------------
+
+def _bound_sync_body(rank, world):
+    sync = mdist.make_bound_sync()
+    # step 1: rank 1 found a bigger clique, rank 0 still active
+    b1 = sync(5 if rank == 0 else 7, 1 if rank == 0 else 0)
+    # step 2: nobody active
+    b2 = sync(6, 0)
+    return b1, b2
+
+
+def _gather_body(rank, world):
+    # rank 0 holds two 3-cliques and one (stale) 2-clique-sized result on rank 1
+    if rank == 0:
+        r = Result(3, 2, np.array([[4, 5, 6], [0, 1, 2]], np.int32), False, [], {})
+    else:
+        r = Result(3, 1, np.array([[1, 2, 3]], np.int32), False, [], {})
+    g = mdist.gather_result(r)
+    return g.omega, g.count, g.cliques.tolist(), g.truncated
+
+
+def _gather_mixed_omega_body(rank, world):
+    # a rank whose subtrees only reach a smaller clique contributes nothing
+    if rank == 0:
+        r = Result(2, 5, np.array([[0, 1], [1, 2], [2, 3], [3, 4], [4, 0]], np.int32), False, [], {})
+    else:
+        r = Result(4, 1, np.array([[5, 6, 7, 8]], np.int32), True, [], {})
+    g = mdist.gather_result(r)
+    return g.omega, g.count, g.cliques.tolist(), g.truncated
+
+
+def _find_one_body(rank, world):
+    r = Result(3, 1, np.array([[9, 10, 11]], np.int32), False, [], {}) if rank == 1 else \
+        Result(2, 1, np.array([[0, 1]], np.int32), False, [], {})
+    g = mdist.gather_result(r, find_one=True)
+    return g.omega, g.count, g.cliques.tolist()
+
+
+def test_bound_sync_is_a_max_allreduce():
+    out = spawn(_bound_sync_body)
+    for b1, b2 in out:
+        assert b1 == (7, 1)  # global best, someone still active
+        assert b2 == (6, 0)
+
+
+def test_gather_adds_multiplicities_and_sorts():
+    out = spawn(_gather_body)
+    for omega, count, cliques, trunc in out:
+        assert omega == 3 and count == 3 and not trunc
+        assert cliques == [[0, 1, 2], [1, 2, 3], [4, 5, 6]]
+
+
+def test_gather_drops_smaller_local_results():
+    out = spawn(_gather_mixed_omega_body)
+    for omega, count, cliques, trunc in out:
+        assert omega == 4 and count == 1 and cliques == [[5, 6, 7, 8]] and trunc
+
+
+def test_find_one_gather_takes_a_holder_of_omega():
+    out = spawn(_find_one_body)
+    for omega, count, cliques in out:
+        assert omega == 3 and count == 1 and cliques == [[9, 10, 11]]
+
+
+def test_cyclic_deal_partitions_every_root():
+    for world in (1, 2, 3, 8):
+        for count in (0, 1, 7, 100):
+            seen = sorted(i for r in range(world) for i in mdist.owned(count, r, world))
+            assert seen == list(range(count))
+            assert all(mdist.shard_of(i, world) == r for r in range(world) for i in mdist.owned(count, r, world))
+
+
+# --- the library's sharding, on one GPU ------------------------------------
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("shards", [2, 3])
+@pytest.mark.parametrize("key", ["planted", "RMAT11", "T(30,6)", "ER400d"])
+def test_shards_union_is_the_full_answer(key, shards):
+    """Each shard enumerates its cyclic share of the roots (and heuristic seeds);
+    merged like gather_result, the shards give the oracle's answer."""
+    import oracle
+    from tests.test_gpu_parity import GRAPHS
+
+    import paper_conf_ipps_geilpo23_b200 as m
+
+    g = GRAPHS[key]()
+    om, cl = oracle.max_cliques(*g.numpy())
+    gg = m.Graph(g.rowptr, g.col)
+    parts = [gg.enumerate(shard_rank=r, shard_count=shards) for r in range(shards)]
+    gg.close()
+    omega = max(p.omega for p in parts)
+    count = sum(p.count for p in parts if p.omega == omega)
+    rows = np.concatenate([p.cliques for p in parts if p.omega == omega], 0)
+    rows = rows[np.lexsort(rows.T[::-1])]
+    assert omega == om and count == len(cl) and np.array_equal(rows, cl)
+
+
+@pytest.mark.gpu
+def test_bound_sync_callback_is_called_every_step():
+    import oracle
+    from tests.test_gpu_parity import GRAPHS
+
+    import paper_conf_ipps_geilpo23_b200 as m
+
+    g = GRAPHS["planted"]()
+    om, cl = oracle.max_cliques(*g.numpy())
+    calls = []
+
+    def sync(best, active):
+        calls.append((best, active))
+        return best, 0  # a single rank: the global state is the local one
+
+    gg = m.Graph(g.rowptr, g.col)
+    r = gg.enumerate(shard_rank=0, shard_count=1, bound_sync=sync)
+    gg.close()
+    assert r.omega == om and r.count == len(cl) and np.array_equal(r.cliques, cl)
+    assert len(calls) >= 2 and calls[-1][1] == 0
