@@ -228,6 +228,7 @@ def main():
         res = one_step(graph)
     times = []
     timings = []
+    py_ms = []
     start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(local) as clocks:
         for _ in range(args.steps):
@@ -236,7 +237,9 @@ def main():
                 dist.barrier()
             torch.cuda.synchronize()
             start.record(stream)
+            h0 = time.perf_counter()
             res = one_step(graph)
+            py_ms.append((time.perf_counter() - h0) * 1e3)
             end.record(stream)
             torch.cuda.synchronize()
             times.append(start.elapsed_time(end))
@@ -268,7 +271,11 @@ def main():
               "host_call_ms": statistics.mean(t["host_total_ms"] for t in timings),
               "host_preprocess_ms": statistics.mean(t["host_preprocess_ms"] for t in timings),
               "host_heuristic_ms": statistics.mean(t["host_heuristic_ms"] for t in timings),
-              "syncs_per_step": statistics.mean(t["syncs"] for t in timings)}
+              "host_setup_ms": statistics.mean(t["host_setup_ms"] for t in timings),
+              "host_enum_ms": statistics.mean(t["host_enum_ms"] for t in timings),
+              "host_readout_ms": statistics.mean(t["host_readout_ms"] for t in timings),
+              "syncs_per_step": statistics.mean(t["syncs"] for t in timings),
+              "python_step_ms": statistics.mean(py_ms)}
 
     # ---- end to end through the public API: pinned host CSR -> GPU -> cliques on the host
     e2e = None

@@ -162,7 +162,9 @@ mce_status mce_result_levels(const mce_result *r, int64_t *entries, int32_t cap,
  * [7] fused root-level kernel total, [8] its launches, [9] its algorithmic
  * bytes (16 + 20 L + 4 T per root: row bounds, V, and the out-rows of V),
  * [10] host wall time of the whole call, [11] of its preprocessing, [12] of
- * its heuristic, [13] host<->device synchronisations it made. */
+ * its heuristic, [13] host<->device synchronisations it made, [14] host
+ * time of the budget / workspace setup, [15] of the root classes + levels,
+ * [16] of the canonical read-out of the stored cliques (device sort + copy). */
 mce_status mce_result_timing(const mce_result *r, double *t, int32_t cap);
 void mce_result_free(mce_result *r);
 

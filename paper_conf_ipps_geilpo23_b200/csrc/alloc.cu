@@ -5,6 +5,7 @@
 // returning, and the internal frees (Pool::reset at the start of a phase, a
 // workspace regrow) happen after such a synchronisation, so a cached block is
 // never reused while in flight, whichever stream the next user runs on.
+#include <chrono>
 #include <map>
 #include <mutex>
 #include <unordered_map>
@@ -21,6 +22,8 @@ namespace {
 struct DeviceCache {
     std::multimap<size_t, void *> free_blocks;  // rounded size -> block
     size_t cached = 0;
+    size_t free_mem = 0;                        // last cudaMemGetInfo answer
+    std::chrono::steady_clock::time_point free_at;
     void *pinned = nullptr;
     size_t pinned_bytes = 0;
 };
@@ -100,6 +103,23 @@ void dev_empty_cache() {
     const int dev = current_device();
     std::lock_guard<std::mutex> lk(g_mu);
     release_all(g_cache[dev]);
+}
+
+size_t dev_free_memory() {
+    const int dev = current_device();
+    const auto now = std::chrono::steady_clock::now();
+    {
+        std::lock_guard<std::mutex> lk(g_mu);
+        DeviceCache &c = g_cache[dev];
+        if (c.free_mem && now - c.free_at < std::chrono::seconds(1)) return c.free_mem;
+    }
+    size_t f = 0, t = 0;
+    MCE_CUDA(cudaMemGetInfo(&f, &t));
+    std::lock_guard<std::mutex> lk(g_mu);
+    DeviceCache &c = g_cache[dev];
+    c.free_mem = f;
+    c.free_at = now;
+    return f;
 }
 
 void *host_pinned(size_t bytes) {

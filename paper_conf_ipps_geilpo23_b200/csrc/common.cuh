@@ -43,6 +43,7 @@ struct Error : std::runtime_error {
 void *dev_alloc(size_t bytes);           // throws MCE_ERR_NOMEM / MCE_ERR_CUDA
 void dev_free(void *p, size_t bytes);    // bytes = the size passed to dev_alloc
 size_t dev_cached_bytes();               // free bytes held by the cache on this device
+size_t dev_free_memory();                // cudaMemGetInfo free bytes, re-queried at most once a second
 void dev_empty_cache();
 void *host_pinned(size_t bytes);         // per-device pinned staging (grow-only, shared)
 

@@ -17,6 +17,7 @@
 
 #include "engine.cuh"
 #include "expand.cuh"
+#include "canon.cuh"
 #include "heuristic.cuh"
 
 namespace mce {
@@ -195,7 +196,8 @@ class Engine {
     int32_t *maxbit_ = nullptr;                 // g->misc[2]
     int64_t stage_rows_ = 0;
     int64_t stage_max_rows_ = 0;  // staging never exceeds a quarter of the budget (stored list truncated, count exact)
-    std::vector<int32_t> rows_;  // host copy of the stored cliques (width res_size_)
+    std::vector<int32_t> rows_;  // find-one: the clique held on the host (width res_size_)
+    int64_t stored_ = 0;         // enumerate: rows kept in g->store (device, width res_size_)
     int32_t res_size_ = 0;
     int64_t res_count_ = 0;
     bool truncated_ = false;
@@ -245,13 +247,13 @@ void Engine::handle_leaves(int32_t size, int64_t cnt, ExpandArgs &a) {
         return;
     }
     if (size > res_size_) {
-        rows_.clear();
+        stored_ = 0;
         res_size_ = size;
         res_count_ = 0;
         truncated_ = false;
     }
     if (size > best_) best_ = size;
-    const int64_t stored = (int64_t)rows_.size() / std::max(res_size_, 1);
+    const int64_t stored = stored_;
     // stored list capacity: max_cliques, and never more rows than a quarter of the budget holds
     const int64_t store_cap = o_.max_cliques > 0 ? std::min<int64_t>(o_.max_cliques, stage_max_rows_) : stage_max_rows_;
     const int64_t want = std::min<int64_t>(cnt, std::max<int64_t>(store_cap - stored, 0));
@@ -266,11 +268,19 @@ void Engine::handle_leaves(int32_t size, int64_t cnt, ExpandArgs &a) {
         stream_sync(s_);
     }
     const int64_t take = std::min<int64_t>(want, a.leaf_cap);
-    if (take > 0) {
-        size_t old = rows_.size();
-        rows_.resize(old + (size_t)take * size);
-        MCE_CUDA(cudaMemcpy(rows_.data() + old, g_->stage.get(), sizeof(int32_t) * take * size,
-                            cudaMemcpyDeviceToHost));
+    if (take > 0) {  // append to the device store (grown with copy; read out once at the end)
+        const size_t need = (size_t)(stored + take) * size;
+        if (g_->store.n < need) {
+            DevBuf<int32_t> bigger(std::max(need, g_->store.n * 2));
+            if (stored)
+                MCE_CUDA(cudaMemcpyAsync(bigger.get(), g_->store.get(), sizeof(int32_t) * stored * size,
+                                         cudaMemcpyDeviceToDevice, s_));
+            stream_sync(s_);  // the old block goes back to the cache only when unused
+            g_->store = std::move(bigger);
+        }
+        MCE_CUDA(cudaMemcpyAsync(g_->store.get() + (size_t)stored * size, g_->stage.get(),
+                                 sizeof(int32_t) * take * size, cudaMemcpyDeviceToDevice, s_));
+        stored_ += take;
     }
     if (take < cnt) truncated_ = true;
     res_count_ += cnt;
@@ -615,8 +625,8 @@ mce_result *Engine::run() {
 
     // frontier budget: the graph's workspace is reused across calls, so it
     // counts as free memory here
-    size_t free_b = 0, total_b = 0;
-    MCE_CUDA(cudaMemGetInfo(&free_b, &total_b));
+    const auto h2 = clk::now();
+    size_t free_b = dev_free_memory();  // (cudaMemGetInfo costs ~1 ms: cached for a second)
     size_t held = dev_cached_bytes();
     for (auto &sg : g_->wsegs) held += sg.n;
     free_b += held;
@@ -637,6 +647,8 @@ mce_result *Engine::run() {
     stage_rows_ = find_one_ ? 1 : 4096;
     g_->stage.ensure((size_t)stage_rows_ * std::max<int32_t>(g_->max_out + 2, 2));
 
+    res->h_setup_ms = ms_since(h2);
+    const auto h3 = clk::now();
     Timer tt(s_);
     tt.start();
     // roots worth expanding: 1 + |N+(r)| >= need, grouped by candidate-set width class
@@ -676,6 +688,7 @@ mce_result *Engine::run() {
         arena_.reset(mark);
     }
     tt.stop();
+    res->h_enum_ms = ms_since(h3);
     stream_sync(s_);
     res->t_enum_ms = tt.collect();
     clock_.collect(t_expand_ms_, t_count_ms_, t_root_ms_);
@@ -690,7 +703,25 @@ mce_result *Engine::run() {
     }
     res->omega = res_size_;
     res->count = res_count_;
-    res->rows = std::move(rows_);
+    if (find_one_) {
+        res->rows = std::move(rows_);
+    } else if (stored_ > 0 && res_size_ > 0) {
+        // canonical read-out on the device, one copy to the host (canon.cu)
+        const auto h4 = clk::now();
+        g_->pool.reset();
+        int32_t *out = g_->pool.take<int32_t>(stored_ * res_size_);
+        res->rows.resize((size_t)stored_ * res_size_);
+        if (canonicalize_device(g_->store.get(), stored_, res_size_, n, out, g_->pool, s_)) {
+            kernels_ += 3 + (res_size_ + 1) / 2 * 2;
+            res->canonical = true;
+        } else {
+            out = g_->store.get();  // rows too wide: the host sorts them (mce_result_cliques)
+        }
+        MCE_CUDA(cudaMemcpyAsync(res->rows.data(), out, sizeof(int32_t) * stored_ * res_size_,
+                                 cudaMemcpyDeviceToHost, s_));
+        stream_sync(s_);
+        res->h_readout_ms = ms_since(h4);
+    }
     res->stored = res_size_ > 0 ? (int64_t)res->rows.size() / res_size_ : 0;
     res->truncated = truncated_ ? 1 : 0;
     res->level_entries = level_entries_;

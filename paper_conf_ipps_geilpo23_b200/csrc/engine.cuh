@@ -18,6 +18,7 @@ struct mce_result {
     double t_root_ms = 0, root_bytes = 0;  // fused root-level kernel
     int64_t root_launches = 0;
     double h_total_ms = 0, h_pre_ms = 0, h_heur_ms = 0;  // host wall time of the call / its phases
+    double h_setup_ms = 0, h_enum_ms = 0, h_readout_ms = 0;
     int64_t syncs = 0;                                    // host<->device round trips
 };
 

@@ -35,7 +35,8 @@ struct mce_graph {
     std::vector<mce::DevBuf<uint8_t>> wsegs;  // frontier arena segments of mce_enumerate / mce_find_one
     mce::PinnedBuf host;           // pinned staging for small device->host reads (per device, shared)
     mce::DevBuf<uint8_t> misc;     // engine: leaf counter + level chain (persistent)
-    mce::DevBuf<int32_t> stage;    // engine: staged leaf cliques (grow-only)
+    mce::DevBuf<int32_t> stage;    // engine: staged leaf cliques of one launch (grow-only)
+    mce::DevBuf<int32_t> store;    // engine: stored maximum cliques of the run (grow-only)
 };
 
 namespace mce {

@@ -200,6 +200,7 @@ __global__ void __launch_bounds__(kPeelThreads)
             const unsigned long long slot = base + (lane >> 3);
             const int leader = lane & ~7;
             bool resolved = false, over = false;
+            int idle = 0;  // consecutive empty polls: back off, and only then look at the hot counters
             while (true) {
                 long long item = -1;
                 bool dead_slot = false;
@@ -208,7 +209,7 @@ __global__ void __launch_bounds__(kPeelThreads)
                         dead_slot = true;  // beyond the list: can never be filled
                     } else {
                         item = (long long)ld_relaxed((const unsigned long long *)(work + slot));
-                        if (item == -1) {
+                        if (item == -1 && idle >= 2) {
                             const unsigned long long dn = ld_relaxed(done);
                             const unsigned long long tl = ld_relaxed(tail);
                             dead_slot = dn == tl && slot >= tl;
@@ -247,7 +248,12 @@ __global__ void __launch_bounds__(kPeelThreads)
                     over = true;
                 }
                 if (__all_sync(0xffffffffu, resolved)) break;
-                if (!done_m) __nanosleep(64);
+                if (!done_m) {
+                    ++idle;
+                    __nanosleep(idle < 4 ? 32 : (idle < 16 ? 128 : 512));
+                } else {
+                    idle = 0;
+                }
             }
             if (__all_sync(0xffffffffu, over)) break;
         }
@@ -282,11 +288,11 @@ __global__ void degrees_kernel(int64_t n, const int64_t *__restrict__ rowptr, in
     }
 }
 
-// sort key of the CSR id space: core number (high word), degree (low word)
+// sort key of the CSR id space: core * (max_deg + 1) + degree
 __global__ void priority_keys_kernel(int64_t n, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ core,
-                                     uint64_t *keys, int32_t *vals) {
+                                     uint64_t span, uint64_t *keys, int32_t *vals) {
     for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
-        keys[v] = ((uint64_t)(uint32_t)core[v] << 32) | (uint64_t)(rowptr[v + 1] - rowptr[v]);
+        keys[v] = (uint64_t)(uint32_t)core[v] * span + (uint64_t)(rowptr[v + 1] - rowptr[v]);
         vals[v] = (int32_t)v;
     }
 }
@@ -360,8 +366,9 @@ __device__ void orient_fill_one(int64_t v, const int64_t *__restrict__ rowptr, c
 }
 
 // Warp w takes vertices [4w, 4w+4): 8-lane tiles when all four have degree
-// <= 64 (sparse graphs: a warp per vertex would leave most lanes idle),
-// otherwise one vertex after another on the whole warp.
+// <= 64 (a warp per vertex would leave most lanes idle), otherwise one vertex
+// after another on the whole warp.  (A lane per vertex was measured 4x
+// slower: its loads touch 32 separate rows, where a tile reads a row coalesced.)
 template <bool FILL>
 __global__ void __launch_bounds__(256) orient_kernel(int64_t n, const int64_t *__restrict__ rowptr,
                                                      const int32_t *__restrict__ col, const int32_t *__restrict__ rank,
@@ -600,10 +607,13 @@ void orient(mce_graph *g, int orientation) {
     if (orientation == 0) {
         uint64_t *keys = g->pool.take<uint64_t>(n), *keys_out = g->pool.take<uint64_t>(n);
         int32_t *vals = g->pool.take<int32_t>(n);
-        priority_keys_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(), g->core.get(), keys, vals);
+        const uint64_t span = (uint64_t)g->max_deg + 1;
+        priority_keys_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(), g->core.get(), span, keys, vals);
         MCE_LAUNCH_CHECK();
-        int end_bit = 32;
-        while (end_bit < 64 && (1ll << (end_bit - 32)) <= (int64_t)g->degeneracy) ++end_bit;
+        // only as many radix bits as the largest key needs (BA 1M: 15 bits, 2 passes)
+        const uint64_t kmax = ((uint64_t)g->degeneracy + 1) * span;
+        int end_bit = 1;
+        while (end_bit < 64 && (1ull << end_bit) < kmax) ++end_bit;
         size_t tmp_bytes = 0;
         MCE_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tmp_bytes, keys, keys_out, vals, g->vid.get(), (int)n, 0,
                                                  end_bit, s));
