@@ -90,6 +90,9 @@ typedef struct {
                                 kernel (adjacency build + first expansion in one warp, only
                                 surviving roots materialised); 1: the generic per-level path
                                 for every root (kept for A/B parity tests) */
+    int32_t no_fused_levels; /* 0 (default): consecutive levels of at most 1024 candidates (<= 256
+                                bits each) run inside one launch (expand_small); 1: every
+                                level takes the count -> scan -> write launches (A/B tests) */
 } mce_options;
 
 /* Fill `opt` with defaults: degeneracy orientation, multi-run degree heuristic

@@ -44,6 +44,7 @@ class Options(ctypes.Structure):
         ("bound_sync_user", ctypes.c_void_p),
         ("verbose", ctypes.c_int32),
         ("legacy_roots", ctypes.c_int32),
+        ("no_fused_levels", ctypes.c_int32),
     ]
 
 

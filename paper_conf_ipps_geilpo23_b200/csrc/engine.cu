@@ -174,6 +174,7 @@ class Engine {
    private:
     int32_t need() const { return find_one_ ? best_ + 1 : best_; }
     void process(int32_t k, const Level &L);
+    bool run_small(int32_t k, const Level &L);
     void do_class(int32_t cls, const int32_t *list, int64_t count);
     void do_class_w1(const int32_t *list, int64_t count);
     void handle_leaves(int32_t size, int64_t cnt, ExpandArgs &a);
@@ -286,7 +287,85 @@ void Engine::handle_leaves(int32_t size, int64_t cnt, ExpandArgs &a) {
     res_count_ += cnt;
 }
 
+// Small-frontier fused levels (expand_small): consecutive tiny levels in one
+// launch; the host then continues with whatever the kernel hands back.
+bool Engine::run_small(int32_t k, const Level &L) {
+    const Arena::Mark mark = arena_.mark();
+    const int64_t scratch_bytes = std::min<int64_t>((int64_t)(arena_.avail() / 2), 256ll << 20);
+    if (scratch_bytes < (16ll << 20)) return false;
+    uint8_t *scratch = arena_.alloc<uint8_t>(scratch_bytes);
+    SmallOut *dout = arena_.alloc<SmallOut>(1);
+    ExpandArgs a{};
+    a.P = L.P;
+    a.slot = L.slot;
+    a.parent = L.parent;
+    a.vloc = L.vloc;
+    a.begin = 0;
+    a.end = L.count;
+    a.k = k;
+    a.need = need();
+    a.bound = o_.bound;
+    a.Wp = L.W;
+    a.Wa = W_;
+    a.Wc = L.W;
+    a.roots = roots_;
+    a.adj = adj_;
+    a.ocol = g_->ocol.get();
+    a.order = g_->vid.get();
+    a.maxbit = maxbit_;
+    a.leaf_total = leaf_total_;
+    a.leaf_slot = leaf_slot_;
+    a.leaf_rows = g_->stage.get();
+    a.leaf_cap = stage_rows_;
+    a.chain = chain_dev_;
+    MCE_CUDA(cudaMemsetAsync(leaf_total_, 0, 2 * sizeof(unsigned long long), s_));
+    const int t = clock_.start(1);
+    launch_expand_small(a, scratch, scratch_bytes, dout, chain_dev_, s_);
+    clock_.stop(t);
+    ++kernels_;
+    SmallOut *h = g_->host.get<SmallOut>(1);
+    MCE_CUDA(cudaMemcpyAsync(h, dout, sizeof(SmallOut), cudaMemcpyDeviceToHost, s_));
+    stream_sync(s_);
+    if (h->levels == 0) {
+        arena_.reset(mark);
+        return false;
+    }
+    const SmallOut o = *h;  // the pinned staging is reused by the calls below
+    if ((int64_t)level_entries_.size() < k + o.levels) level_entries_.resize(k + o.levels, 0);
+    for (int64_t i = 0; i < o.levels; ++i) level_entries_[k + i] += o.level_n[i];
+    if (o_.verbose > 0)
+        fprintf(stderr, "[mce] fused levels k=%d..%lld entries=%lld -> children=%lld leaves=%lld status=%lld\n", k,
+                (long long)(k + o.levels - 1), (long long)L.count, (long long)o.children, (long long)o.leaves,
+                (long long)o.status);
+    if (o.leaves > 0) {  // leaves of size k_next from the last processed level
+        ExpandArgs la = a;
+        la.P = o.inP;
+        la.slot = o.inslot;
+        la.parent = o.inparent;
+        la.vloc = o.invloc;
+        la.end = o.inN;
+        la.k = (int32_t)o.k_next - 1;
+        la.Wp = la.Wc = (int32_t)o.inW;
+        la.counts = arena_.alloc<int32_t>(o.inN);  // for a count-pass replay if the staging must grow
+        handle_leaves((int32_t)o.k_next, o.leaves, la);
+    }
+    sync_bound(true);
+    if (o.status == 1 && o.children > 0) {
+        Level C;
+        C.count = o.children;
+        C.W = (int32_t)o.Wc;
+        C.P = o.P;
+        C.slot = o.slot;
+        C.parent = o.parent;
+        C.vloc = o.vloc;
+        process((int32_t)o.k_next, C);
+    }
+    arena_.reset(mark);
+    return true;
+}
+
 void Engine::process(int32_t k, const Level &L) {
+    if (!o_.no_fused_levels && L.count <= kSmallMax && L.W <= 4 && run_small(k, L)) return;
     if ((int64_t)level_entries_.size() <= k) level_entries_.resize(k + 1, 0);
     level_entries_[k] += L.count;
     if (k + 2 > chain_cap_) fail(MCE_ERR_INVALID, "clique depth above the supported maximum");
@@ -405,16 +484,17 @@ void Engine::process(int32_t k, const Level &L) {
 
 // W == 1 roots: the fused root level (roots.cu), then levels >= 2 as usual
 void Engine::do_class_w1(const int32_t *list, int64_t count) {
-    const int64_t mine = count > offset_ ? (count - offset_ + stride_ - 1) / stride_ : 0;
+    // the class list holds this shard's roots only (classify_roots deals them)
+    const int64_t mine = count;
     if (mine <= 0) return;
     W_ = 1;
-    const int32_t *base = list + offset_;
+    const int32_t *base = list;
     int32_t *len = arena_.alloc<int32_t>(mine);
     int64_t *prefix = arena_.alloc<int64_t>(mine + 1);
     int64_t *tmp = arena_.alloc<int64_t>(scan_tmp_items(mine));
     int64_t *win = arena_.alloc<int64_t>(2);
     unsigned long long *ctr = arena_.alloc<unsigned long long>(8);
-    launch_root_lengths(base, mine, stride_, g_->orp.get(), len, s_);
+    launch_root_lengths(base, mine, 1, g_->orp.get(), len, s_);
     exclusive_scan_i32(len, prefix, mine, tmp, s_);
     kernels_ += 4;
     // per candidate row: adjacency word + one level-2 entry (P, slot, parent, vloc)
@@ -433,9 +513,9 @@ void Engine::do_class_w1(const int32_t *list, int64_t count) {
         const int64_t lo = hw[0], rows = hw[1];
         const int64_t nw = hi - lo;
         RootArgs ra{};
-        ra.list = base + lo * stride_;
+        ra.list = base + lo;
         ra.count = nw;
-        ra.stride = stride_;
+        ra.stride = 1;
         ra.orp = g_->orp.get();
         ra.ocol = g_->ocol.get();
         ra.order = g_->vid.get();
@@ -516,18 +596,18 @@ void Engine::do_class(int32_t cls, const int32_t *list, int64_t count) {
         do_class_w1(list, count);
         return;
     }
-    // this shard's view: positions offset_, offset_+stride_, ...
-    const int64_t mine = count > offset_ ? (count - offset_ + stride_ - 1) / stride_ : 0;
+    // the class list holds this shard's roots only (classify_roots deals them)
+    const int64_t mine = count;
     if (mine <= 0) return;
     W_ = 1 << cls;
-    const int32_t *base = list + offset_;
+    const int32_t *base = list;
     // adjacency rows per root -> prefix; it stays on the device and windows
     // are cut there (one scalar read-back per window)
     int32_t *len = arena_.alloc<int32_t>(mine);
     int64_t *prefix = arena_.alloc<int64_t>(mine + 1);
     int64_t *tmp = arena_.alloc<int64_t>(scan_tmp_items(mine));
     int64_t *win = arena_.alloc<int64_t>(2);
-    launch_root_lengths(base, mine, stride_, g_->orp.get(), len, s_);
+    launch_root_lengths(base, mine, 1, g_->orp.get(), len, s_);
     exclusive_scan_i32(len, prefix, mine, tmp, s_);
     kernels_ += 4;
     const int64_t per_root = sizeof(RootInfo) + 8 * W_ + 12 + 64;
@@ -547,7 +627,7 @@ void Engine::do_class(int32_t cls, const int32_t *list, int64_t count) {
         const int64_t nw = hi - lo;
         RootInfo *roots = arena_.alloc<RootInfo>(nw);
         uint64_t *adj = arena_.alloc<uint64_t>(rows * W_);
-        launch_make_roots(base + lo * stride_, nw, stride_, W_, g_->orp.get(), prefix + lo, roots, s_);
+        launch_make_roots(base + lo, nw, 1, W_, g_->orp.get(), prefix + lo, roots, s_);
         launch_build_adj(roots, nw, W_, g_->orp.get(), g_->ocol.get(), adj, rows * W_, s_);
         kernels_ += 2;
         roots_ = roots;
@@ -660,7 +740,10 @@ mce_result *Engine::run() {
         int64_t *tmp = arena_.alloc<int64_t>(scan_tmp_items(n));
         int64_t *hist = arena_.alloc<int64_t>(kMaxClass + 1);
         MCE_CUDA(cudaMemsetAsync(hist, 0, sizeof(int64_t) * (kMaxClass + 1), s_));
-        launch_classify_roots(n, g_->orp.get(), std::max<int32_t>(need() - 1, 1), cls, hist, s_);
+        // roots are dealt to shards by CSR id (r % shard_count): independent of the
+        // lower bound, so ranks whose bounds differ still partition the roots exactly
+        launch_classify_roots(n, g_->orp.get(), std::max<int32_t>(need() - 1, 1), (int32_t)offset_,
+                              (int32_t)stride_, cls, hist, s_);
         ++kernels_;
         int64_t *hh = g_->host.get<int64_t>(kMaxClass + 1);
         MCE_CUDA(cudaMemcpyAsync(hh, hist, sizeof(int64_t) * (kMaxClass + 1), cudaMemcpyDeviceToHost, s_));

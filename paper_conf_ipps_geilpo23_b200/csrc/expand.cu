@@ -179,115 +179,270 @@ __device__ __forceinline__ void flush_counters(const ExpandArgs &a, unsigned lon
 // thread per candidate, W <= 4 words (|P| bits < 256): P, the running set R
 // and the child set C live in registers; the colouring order in local memory
 // ---------------------------------------------------------------------------
+// one candidate entry e (thread per candidate, W <= 4 words); returns its
+// number of surviving children (count pass) after writing them at `out`
+// (write pass).  Leaves, highest child bit and reachable depth accumulate
+// into the caller's counters.
+template <int W, bool WRITE>
+__device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, int64_t out, unsigned &nleaf,
+                                                int &hb, int &ub) {
+    uint64_t P[W];
+#pragma unroll
+    for (int w = 0; w < W; ++w) P[w] = a.P[e * W + w];
+    const RootInfo ri = a.roots[a.slot[e]];
+    const uint64_t *A = a.adj + ri.abase;
+    const int Wa = a.Wa;
+    uint8_t ord[64 * W];
+    uint8_t colr[64 * W];
+    int np = 0;
+    int ncol = 0;
+    if (a.bound == 1) {
+        uint64_t U[W];
+#pragma unroll
+        for (int w = 0; w < W; ++w) U[w] = P[w];
+        while (true) {
+            bool any = false;
+#pragma unroll
+            for (int w = 0; w < W; ++w) any |= U[w] != 0;
+            if (!any) break;
+            ++ncol;
+            uint64_t Q[W];
+#pragma unroll
+            for (int w = 0; w < W; ++w) Q[w] = U[w];
+#pragma unroll
+            for (int w = 0; w < W; ++w) {
+                while (Q[w]) {
+                    const int b = __ffsll((long long)Q[w]) - 1;
+                    const int v = w * 64 + b;
+                    const uint64_t *row = A + (int64_t)v * Wa;
+#pragma unroll
+                    for (int x = 0; x < W; ++x) Q[x] &= ~__ldg(row + x);
+                    Q[w] &= ~(1ull << b);
+                    U[w] &= ~(1ull << b);
+                    ord[np] = (uint8_t)v;
+                    colr[np] = (uint8_t)ncol;
+                    ++np;
+                }
+            }
+        }
+    } else {
+#pragma unroll
+        for (int w = 0; w < W; ++w) {
+            uint64_t q = P[w];
+            while (q) {
+                const int b = __ffsll((long long)q) - 1;
+                q &= q - 1;
+                ord[np] = (uint8_t)(w * 64 + b);
+                colr[np] = (uint8_t)(np + 1);
+                ++np;
+            }
+        }
+        ncol = np;
+    }
+    int32_t cnt = 0;
+    if (a.k + ncol >= a.need) {
+        uint64_t R[W];
+#pragma unroll
+        for (int w = 0; w < W; ++w) R[w] = P[w];
+        for (int i = np - 1; i >= 0; --i) {
+            if (a.k + colr[i] < a.need) break;
+            const int v = ord[i];
+            const uint64_t *row = A + (int64_t)v * Wa;
+            uint64_t C[W];
+            int pc = 0;
+#pragma unroll
+            for (int w = 0; w < W; ++w) {
+                C[w] = R[w] & __ldg(row + w);
+                pc += __popcll(C[w]);
+            }
+            R[v >> 6] &= ~(1ull << (v & 63));
+            if (pc == 0) {
+                if (!WRITE && a.k + 1 >= a.need) {
+                    ++nleaf;
+                    store_leaf(a, e, v, ri);
+                }
+            } else if (a.k + 1 + pc >= a.need) {
+                if (WRITE) {
+                    const int64_t c = out + cnt;
+#pragma unroll
+                    for (int w = 0; w < W; ++w)
+                        if (w < a.Wc) a.cP[c * a.Wc + w] = C[w];
+                    a.cslot[c] = a.slot[e];
+                    a.cparent[c] = (int32_t)e;
+                    a.cvloc[c] = v;
+                } else {
+                    hb = max(hb, top_bit<W>(C));
+                    ub = max(ub, a.k + 1 + pc);
+                }
+                ++cnt;
+            }
+        }
+    }
+    return cnt;
+}
+
 template <int W, bool WRITE>
 __global__ void __launch_bounds__(256) expand_thread(const ExpandArgs a) {
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     unsigned nleaf = 0;
     int hb = -1, ub = 0;
-    const int64_t e_end = a.begin + (a.end - a.begin + stride - 1) / stride * stride;  // warp-uniform trip count
-    for (int64_t e = a.begin + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < e_end; e += stride) {
-        if (e >= a.end) continue;
+    for (int64_t e = a.begin + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < a.end; e += stride) {
         int64_t out = 0;
         if (WRITE) {
             out = a.offsets[e];
             if (a.offsets[e + 1] == out) continue;
             out -= a.out_base;
         }
-        uint64_t P[W];
-#pragma unroll
-        for (int w = 0; w < W; ++w) P[w] = a.P[e * W + w];
-        const RootInfo ri = a.roots[a.slot[e]];
-        const uint64_t *A = a.adj + ri.abase;
-        const int Wa = a.Wa;
-        uint8_t ord[64 * W];
-        uint8_t colr[64 * W];
-        int np = 0;
-        int ncol = 0;
-        if (a.bound == 1) {
-            uint64_t U[W];
-#pragma unroll
-            for (int w = 0; w < W; ++w) U[w] = P[w];
-            while (true) {
-                bool any = false;
-#pragma unroll
-                for (int w = 0; w < W; ++w) any |= U[w] != 0;
-                if (!any) break;
-                ++ncol;
-                uint64_t Q[W];
-#pragma unroll
-                for (int w = 0; w < W; ++w) Q[w] = U[w];
-#pragma unroll
-                for (int w = 0; w < W; ++w) {
-                    while (Q[w]) {
-                        const int b = __ffsll((long long)Q[w]) - 1;
-                        const int v = w * 64 + b;
-                        const uint64_t *row = A + (int64_t)v * Wa;
-#pragma unroll
-                        for (int x = 0; x < W; ++x) Q[x] &= ~__ldg(row + x);
-                        Q[w] &= ~(1ull << b);
-                        U[w] &= ~(1ull << b);
-                        ord[np] = (uint8_t)v;
-                        colr[np] = (uint8_t)ncol;
-                        ++np;
-                    }
-                }
-            }
-        } else {
-#pragma unroll
-            for (int w = 0; w < W; ++w) {
-                uint64_t q = P[w];
-                while (q) {
-                    const int b = __ffsll((long long)q) - 1;
-                    q &= q - 1;
-                    ord[np] = (uint8_t)(w * 64 + b);
-                    colr[np] = (uint8_t)(np + 1);
-                    ++np;
-                }
-            }
-            ncol = np;
-        }
-        int32_t cnt = 0;
-        if (a.k + ncol >= a.need) {
-            uint64_t R[W];
-#pragma unroll
-            for (int w = 0; w < W; ++w) R[w] = P[w];
-            for (int i = np - 1; i >= 0; --i) {
-                if (a.k + colr[i] < a.need) break;
-                const int v = ord[i];
-                const uint64_t *row = A + (int64_t)v * Wa;
-                uint64_t C[W];
-                int pc = 0;
-#pragma unroll
-                for (int w = 0; w < W; ++w) {
-                    C[w] = R[w] & __ldg(row + w);
-                    pc += __popcll(C[w]);
-                }
-                R[v >> 6] &= ~(1ull << (v & 63));
-                if (pc == 0) {
-                    if (!WRITE && a.k + 1 >= a.need) {
-                        ++nleaf;
-                        store_leaf(a, e, v, ri);
-                    }
-                } else if (a.k + 1 + pc >= a.need) {
-                    if (WRITE) {
-                        const int64_t c = out + cnt;
-#pragma unroll
-                        for (int w = 0; w < W; ++w)
-                            if (w < a.Wc) a.cP[c * a.Wc + w] = C[w];
-                        a.cslot[c] = a.slot[e];
-                        a.cparent[c] = (int32_t)e;
-                        a.cvloc[c] = v;
-                    } else {
-                        hb = max(hb, top_bit<W>(C));
-                        ub = max(ub, a.k + 1 + pc);
-                    }
-                    ++cnt;
-                }
-            }
-        }
+        const int32_t cnt = expand_entry<W, WRITE>(a, e, out, nleaf, hb, ub);
         if (!WRITE) a.counts[e] = cnt;
     }
     if (!WRITE) flush_counters(a, nleaf, hb, ub);
+}
+
+// ---------------------------------------------------------------------------
+// small-frontier fused levels (see expand.cuh)
+// ---------------------------------------------------------------------------
+constexpr int kSmallThreads = 1024;
+
+template <bool WRITE>
+__device__ __forceinline__ int32_t expand_entry_w(int W, const ExpandArgs &a, int64_t e, int64_t out,
+                                                  unsigned &nleaf, int &hb, int &ub) {
+    if (W == 1) return expand_entry<1, WRITE>(a, e, out, nleaf, hb, ub);
+    if (W == 2) return expand_entry<2, WRITE>(a, e, out, nleaf, hb, ub);
+    return expand_entry<4, WRITE>(a, e, out, nleaf, hb, ub);
+}
+
+__global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a0, uint8_t *scratch,
+                                                              int64_t scratch_bytes, SmallOut *out,
+                                                              LevelLink *chain) {
+    __shared__ ExpandArgs A;
+    __shared__ int32_t offs[kSmallMax + 1];
+    __shared__ int32_t wsum[kSmallThreads / 32];
+    __shared__ unsigned s_leaf;
+    __shared__ int s_hb, s_ub;
+    __shared__ int64_t s_used;
+    const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
+    if (t == 0) {
+        A = a0;
+        s_used = 0;
+        out->levels = 0;
+        out->leaves = 0;
+        out->status = 2;
+        out->k_next = a0.k;
+        out->children = a0.end - a0.begin;
+        out->Wc = a0.Wp;
+        out->P = const_cast<uint64_t *>(a0.P);
+        out->slot = const_cast<int32_t *>(a0.slot);
+        out->parent = const_cast<int32_t *>(a0.parent);
+        out->vloc = const_cast<int32_t *>(a0.vloc);
+    }
+    __syncthreads();
+    for (int lev = 0; lev < kSmallMaxLevels; ++lev) {
+        const int64_t N = A.end - A.begin;
+        const int W = A.Wp;
+        // worst case of the children: every candidate bit a child
+        const int64_t worst = N * 64 * W * (8 * W + 12) + 4 * 256;
+        if (N > kSmallMax || W > 4 || s_used + worst > scratch_bytes) break;  // status 2: host takes level k
+        if (t == 0) {
+            s_leaf = 0;
+            s_hb = -1;
+            s_ub = 0;
+            chain[A.k] = LevelLink{A.parent, A.vloc};
+        }
+        __syncthreads();
+        // count pass, one candidate per thread
+        unsigned nleaf = 0;
+        int hb = -1, ub = 0;
+        int32_t cnt = 0;
+        if (t < N) cnt = expand_entry_w<false>(W, A, A.begin + t, 0, nleaf, hb, ub);
+        if (nleaf) atomicAdd(&s_leaf, nleaf);
+        if (hb >= 0) atomicMax(&s_hb, hb);
+        if (ub > 0) atomicMax(&s_ub, ub);
+        // block exclusive scan of the counts
+        int incl = cnt;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o) incl += y;
+        }
+        if (lane == 31) wsum[wid] = incl;
+        __syncthreads();
+        if (wid == 0) {
+            int w = wsum[lane];
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const int y = __shfl_up_sync(0xffffffffu, w, o);
+                if (lane >= o) w += y;
+            }
+            wsum[lane] = w;
+        }
+        __syncthreads();
+        const int excl = (wid ? wsum[wid - 1] : 0) + incl - cnt;
+        if (t < N) offs[t] = excl;
+        const int total = wsum[31];
+        if (t == 0) {
+            offs[N] = total;
+            out->level_n[lev] = N;
+            out->levels = lev + 1;
+            out->leaves = s_leaf;
+            out->inP = const_cast<uint64_t *>(A.P);
+            out->inslot = const_cast<int32_t *>(A.slot);
+            out->inparent = const_cast<int32_t *>(A.parent);
+            out->invloc = const_cast<int32_t *>(A.vloc);
+            out->inN = N;
+            out->inW = W;
+            out->k_next = A.k + 1;
+            out->children = total;
+            if (s_leaf) atomicAdd(A.leaf_total, (unsigned long long)s_leaf);
+        }
+        if (total == 0) {
+            if (t == 0) out->status = 0;
+            break;
+        }
+        __syncthreads();
+        // children arrays (narrowest stride holding the highest surviving bit)
+        if (t == 0) {
+            int Wc = 1;
+            while (Wc * 64 <= s_hb && Wc < W) Wc <<= 1;
+            uint8_t *p = scratch + s_used;
+            auto take = [&](int64_t bytes) {
+                uint8_t *q = p;
+                p += (bytes + 255) / 256 * 256;
+                return q;
+            };
+            A.cP = reinterpret_cast<uint64_t *>(take((int64_t)total * Wc * 8));
+            A.cslot = reinterpret_cast<int32_t *>(take((int64_t)total * 4));
+            A.cparent = reinterpret_cast<int32_t *>(take((int64_t)total * 4));
+            A.cvloc = reinterpret_cast<int32_t *>(take((int64_t)total * 4));
+            A.Wc = Wc;
+            A.out_base = 0;
+            s_used = p - scratch;
+        }
+        __syncthreads();
+        // write pass
+        if (t < N && cnt > 0) expand_entry_w<true>(W, A, A.begin + t, offs[t], nleaf, hb, ub);
+        __syncthreads();
+        const bool stop = s_leaf > 0 || total > kSmallMax;
+        if (t == 0) {
+            out->P = A.cP;
+            out->slot = A.cslot;
+            out->parent = A.cparent;
+            out->vloc = A.cvloc;
+            out->Wc = A.Wc;
+            out->status = 1;
+            // the children become the next level
+            A.P = A.cP;
+            A.slot = A.cslot;
+            A.parent = A.cparent;
+            A.vloc = A.cvloc;
+            A.begin = 0;
+            A.end = total;
+            A.Wp = A.Wc;
+            A.k = A.k + 1;
+        }
+        __syncthreads();
+        if (stop) break;
+    }
 }
 
 // ---------------------------------------------------------------------------
@@ -460,7 +615,8 @@ __global__ void expand_tile(const ExpandArgs a, int max_l) {
     if (!WRITE) flush_counters(a, nleaf, hb, ub);
 }
 
-__global__ void classify_roots_kernel(int64_t n, const int64_t *__restrict__ orp, int32_t min_len, int32_t *cls,
+__global__ void classify_roots_kernel(int64_t n, const int64_t *__restrict__ orp, int32_t min_len,
+                                      int32_t shard_rank, int32_t shard_count, int32_t *cls,
                                       unsigned long long *hist) {
     __shared__ unsigned int h[kMaxClass + 1];
     for (int i = threadIdx.x; i <= kMaxClass; i += blockDim.x) h[i] = 0;
@@ -468,7 +624,7 @@ __global__ void classify_roots_kernel(int64_t n, const int64_t *__restrict__ orp
     for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < n; r += (int64_t)gridDim.x * blockDim.x) {
         const int64_t L = orp[r + 1] - orp[r];
         int32_t c = -1;
-        if (L >= min_len && L > 0) {
+        if (L >= min_len && L > 0 && (shard_count <= 1 || r % shard_count == shard_rank)) {
             const int64_t words = (L + 63) / 64;
             c = 0;
             while ((1ll << c) < words) ++c;
@@ -630,9 +786,16 @@ void launch_expand(const ExpandArgs &a, bool write_pass, cudaStream_t s) {
     }
 }
 
-void launch_classify_roots(int64_t n, const int64_t *orp, int32_t min_len, int32_t *cls, int64_t *hist,
-                           cudaStream_t s) {
-    classify_roots_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, orp, min_len, cls, (unsigned long long *)hist);
+void launch_expand_small(const ExpandArgs &a, uint8_t *scratch, int64_t scratch_bytes, SmallOut *out,
+                         LevelLink *chain, cudaStream_t s) {
+    expand_small<<<1, kSmallThreads, 0, s>>>(a, scratch, scratch_bytes, out, chain);
+    MCE_LAUNCH_CHECK();
+}
+
+void launch_classify_roots(int64_t n, const int64_t *orp, int32_t min_len, int32_t shard_rank, int32_t shard_count,
+                           int32_t *cls, int64_t *hist, cudaStream_t s) {
+    classify_roots_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, orp, min_len, shard_rank, shard_count, cls,
+                                                           (unsigned long long *)hist);
     MCE_LAUNCH_CHECK();
 }
 void launch_find_window(const int64_t *prefix, int64_t hi, int64_t lo_min, int64_t room, int64_t row_bytes,

@@ -86,6 +86,32 @@ struct RootArgs {
 };
 void launch_root_expand_w1(const RootArgs &a, cudaStream_t s);
 
+// Small-frontier fused levels (expand.cu expand_small): one block runs
+// count -> scan -> write for consecutive levels while a level has at most
+// kSmallMax entries of at most 4 words, so chains of tiny levels (the planted
+// clique of er2000, the hub chain of R-MAT) cost one launch instead of ~7
+// launches and a host round trip each.  It stops after a level that recorded
+// leaves, produced more than kSmallMax children, or would not fit the scratch.
+constexpr int kSmallMax = 1024;
+constexpr int kSmallMaxLevels = 512;
+struct SmallOut {
+    int64_t status;    // 0: search below the input exhausted; 1: host continues with `children`;
+                       // 2: stopped before processing level k_next (host processes it)
+    int64_t levels;    // levels processed (|C| = k0 .. k0 + levels - 1)
+    int64_t k_next;    // |C| of the level the host continues with
+    int64_t children;  // its entries
+    int64_t Wc;        // its word stride
+    int64_t leaves;    // leaves (size k_next) recorded by the last processed level
+    uint64_t *P;       // the level the host continues with
+    int32_t *slot, *parent, *vloc;
+    uint64_t *inP;     // the last processed level (for a leaf replay)
+    int32_t *inslot, *inparent, *invloc;
+    int64_t inN, inW;
+    int64_t level_n[kSmallMaxLevels];  // entries of every processed level
+};
+void launch_expand_small(const ExpandArgs &a, uint8_t *scratch, int64_t scratch_bytes, SmallOut *out,
+                         LevelLink *chain, cudaStream_t s);
+
 // W classes: 0 -> 1 word, 1 -> 2, 2 -> 4, ... (W = 1 << class); L <= 64 W
 constexpr int kMaxClass = 9;  // W up to 256 words (L <= 16384)
 
@@ -94,8 +120,8 @@ void launch_build_adj(const RootInfo *roots, int64_t nroots, int W, const int64_
 void launch_init_level1(const RootInfo *roots, int64_t nroots, int W, uint64_t *P, int32_t *slot, int32_t *parent,
                         int32_t *vloc, cudaStream_t s);
 void launch_expand(const ExpandArgs &a, bool write_pass, cudaStream_t s);
-void launch_classify_roots(int64_t n, const int64_t *orp, int32_t min_len, int32_t *cls, int64_t *hist,
-                           cudaStream_t s);
+void launch_classify_roots(int64_t n, const int64_t *orp, int32_t min_len, int32_t shard_rank, int32_t shard_count,
+                           int32_t *cls, int64_t *hist, cudaStream_t s);
 void launch_find_window(const int64_t *prefix, int64_t hi, int64_t lo_min, int64_t room, int64_t row_bytes,
                         int64_t per_root, int64_t *out, cudaStream_t s);
 void launch_flag_eq(int64_t n, const int32_t *cls, int32_t c, int32_t *flag, cudaStream_t s);

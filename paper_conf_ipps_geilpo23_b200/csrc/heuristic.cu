@@ -38,6 +38,15 @@ __device__ __forceinline__ unsigned long long pick_key(const int32_t *__restrict
     return ((unsigned long long)(uint32_t)__ldg(thr + x) << 32) | (unsigned long long)(0x7fffffffu - (uint32_t)x);
 }
 
+// x ~ w?  Binary search in the shorter of the two sorted adjacency lists (the
+// picked vertex w is usually a hub, the candidate x rarely is).
+__device__ __forceinline__ bool adjacent(const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
+                                         int32_t x, int32_t w, int64_t wb, int64_t we) {
+    const int64_t xb = __ldg(rowptr + x), xe = __ldg(rowptr + x + 1);
+    if (xe - xb < we - wb) return contains_sorted(col, xb, xe, w);
+    return contains_sorted(col, wb, we, x);
+}
+
 // One greedy run for seed s by a tile of G lanes (G = 8 or 32) of the calling
 // warp.  Writes the clique (in order added) to `clique` when non-null.
 // Returns the clique size.
@@ -73,7 +82,7 @@ __device__ int32_t greedy_run(int32_t s, const int64_t *__restrict__ rowptr, con
         for (int64_t i0 = 0; i0 < len; i0 += G) {
             int64_t i = i0 + gl;
             int32_t x = i < len ? src[i] : -1;
-            bool keep = i < len && x != w && contains_sorted(col, wb, we, x);
+            bool keep = i < len && x != w && adjacent(rowptr, col, x, w, wb, we);
             const unsigned m = (__ballot_sync(gmask, keep) & gmask) >> gbase;
             if (keep) buf[out + __popc(m & ((1u << gl) - 1u))] = x;
             out += __popc(m);
@@ -182,7 +191,7 @@ __global__ void __launch_bounds__(kReplay) replay_kernel(const unsigned long lon
         for (int64_t i0 = 0; i0 < len; i0 += kReplay) {
             const int64_t i = i0 + threadIdx.x;
             const int32_t x = i < len ? src[i] : -1;
-            const bool keep = i < len && x != w && contains_sorted(col, wb, we, x);
+            const bool keep = i < len && x != w && adjacent(rowptr, col, x, w, wb, we);
             const unsigned m = __ballot_sync(0xffffffffu, keep);
             __syncthreads();  // wkey/wcnt reuse, and every read of this chunk precedes its writes
             if (lane == 0) wcnt[wid] = __popc(m);

@@ -5,8 +5,9 @@ whose subtrees are independent, with a small NCCL max-allreduce of the omega
 lower bound each level and a final gather of the cliques over NVLink."
 
  * every rank loads the whole graph and runs the same preprocessing;
- * heuristic runs and root vertices are dealt cyclically (index % world ==
-   rank) inside the library (mce_options.shard_rank / shard_count);
+ * heuristic seeds are dealt cyclically (seed position % world == rank) and
+   root vertices by CSR id (id % world == rank) inside the library
+   (mce_options.shard_rank / shard_count);
  * after every expansion step the library calls `bound_sync`, which
    max-allreduces (best clique size, still-active flag) across ranks, so a
    clique found on one GPU tightens the pruning bound on all of them and the
@@ -107,5 +108,5 @@ def shard_of(index: int, world: int) -> int:
 
 
 def owned(count: int, rank: int, world: int, offset: Optional[int] = None) -> range:
-    """Positions of a sorted root list owned by `rank` (mirrors the library's cyclic deal)."""
+    """Items 0..count-1 owned by `rank` under the cyclic deal the library uses for seeds and root ids."""
     return range(rank if offset is None else offset, count, world)

@@ -79,6 +79,15 @@ def test_enumerate_matches_oracle(key, legacy_roots):
     assert np.array_equal(r.cliques, cl)
 
 
+@pytest.mark.parametrize("key", ["er2000", "planted", "RMAT11", "RMAT13", "K130", "T(30,6)", "ER400d", "Paley17"])
+def test_unfused_levels_match(key):
+    """Every level through count -> scan -> write launches (no expand_small) gives the same answer."""
+    g = GRAPHS[key]()
+    om, cl = oracle_answer(key)
+    r = run_enum(g, fused_levels=False)
+    assert (r.omega, r.count) == (om, len(cl)) and np.array_equal(r.cliques, cl)
+
+
 @pytest.mark.parametrize("key", ["er2000", "planted", "RMAT11", "BA5k", "C9", "T(36,12)"])
 def test_no_heuristic_size2_leaves(key):
     """Heuristic 'none' with a lower bound of 2: size-2 leaves come out of the fused root kernel."""
