@@ -93,6 +93,11 @@ typedef struct {
     int32_t no_fused_levels; /* 0 (default): consecutive levels of at most 1024 candidates (<= 256
                                 bits each) run inside one launch (expand_small); 1: every
                                 level takes the count -> scan -> write launches (A/B tests) */
+    int32_t no_clique_shortcut; /* 0 (default, colouring bound only): a candidate (C, P) whose P is
+                                itself a clique with |C| + |P| equal to the size sought is
+                                recorded as the clique C + P instead of being expanded level by
+                                level (its only clique of that size; reading 10);
+                                1: Algorithm 2's expansion of every level (A/B tests) */
 } mce_options;
 
 /* Fill `opt` with defaults: degeneracy orientation, multi-run degree heuristic

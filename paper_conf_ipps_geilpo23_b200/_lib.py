@@ -45,6 +45,7 @@ class Options(ctypes.Structure):
         ("verbose", ctypes.c_int32),
         ("legacy_roots", ctypes.c_int32),
         ("no_fused_levels", ctypes.c_int32),
+        ("no_clique_shortcut", ctypes.c_int32),
     ]
 
 

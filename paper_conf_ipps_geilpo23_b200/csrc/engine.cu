@@ -177,7 +177,8 @@ class Engine {
     bool run_small(int32_t k, const Level &L);
     void do_class(int32_t cls, const int32_t *list, int64_t count);
     void do_class_w1(const int32_t *list, int64_t count);
-    void handle_leaves(int32_t size, int64_t cnt, ExpandArgs &a);
+    void handle_leaves(int32_t size, int64_t cnt, ExpandArgs &a, int kind = 0);
+    void leaf_args(ExpandArgs &a) const;
     void sync_bound(bool active);
     void launch_timed(const ExpandArgs &a, bool write);
 
@@ -194,8 +195,11 @@ class Engine {
     // leaves
     unsigned long long *leaf_total_ = nullptr;  // g->misc[0]
     unsigned long long *leaf_slot_ = nullptr;   // g->misc[1]
-    int32_t *maxbit_ = nullptr;                 // g->misc[2]
+    unsigned long long *clq_total_ = nullptr;   // g->misc[2] clique completions (reading 10)
+    unsigned long long *clq_slot_ = nullptr;    // g->misc[3]
+    int32_t *maxbit_ = nullptr;                 // g->misc[4]
     int64_t stage_rows_ = 0;
+    int64_t cstage_rows_ = 0;
     int64_t stage_max_rows_ = 0;  // staging never exceeds a quarter of the budget (stored list truncated, count exact)
     std::vector<int32_t> rows_;  // find-one: the clique held on the host (width res_size_)
     int64_t stored_ = 0;         // enumerate: rows kept in g->store (device, width res_size_)
@@ -236,15 +240,30 @@ void Engine::sync_bound(bool active) {
     if (gb > best_) best_ = gb;
 }
 
-void Engine::handle_leaves(int32_t size, int64_t cnt, ExpandArgs &a) {
+void Engine::leaf_args(ExpandArgs &a) const {
+    a.leaf_total = leaf_total_;
+    a.leaf_slot = leaf_slot_;
+    a.leaf_rows = g_->stage.get();
+    a.leaf_cap = stage_rows_;
+    a.shortcut = o_.no_clique_shortcut ? 0 : 1;
+    a.clq_total = clq_total_;
+    a.clq_slot = clq_slot_;
+    a.clq_rows = g_->cstage.get();
+    a.clq_cap = cstage_rows_;
+}
+
+// Record `cnt` cliques of `size` staged by a count pass: kind 0 = leaves
+// C + {v} (a.leaf_rows), kind 1 = clique completions C + P (a.clq_rows).
+void Engine::handle_leaves(int32_t size, int64_t cnt, ExpandArgs &a, int kind) {
     if (cnt <= 0) return;
+    DevBuf<int32_t> &stage = kind ? g_->cstage : g_->stage;
     if (find_one_) {
-        // all leaves of this launch have size k+1 > best: keep the first
+        // all cliques of this launch have size > best: keep the first
         best_ = size;
         res_size_ = size;
         res_count_ = 1;
         rows_.resize(size);
-        MCE_CUDA(cudaMemcpy(rows_.data(), g_->stage.get(), sizeof(int32_t) * size, cudaMemcpyDeviceToHost));
+        MCE_CUDA(cudaMemcpy(rows_.data(), stage.get(), sizeof(int32_t) * size, cudaMemcpyDeviceToHost));
         return;
     }
     if (size > res_size_) {
@@ -258,17 +277,18 @@ void Engine::handle_leaves(int32_t size, int64_t cnt, ExpandArgs &a) {
     // stored list capacity: max_cliques, and never more rows than a quarter of the budget holds
     const int64_t store_cap = o_.max_cliques > 0 ? std::min<int64_t>(o_.max_cliques, stage_max_rows_) : stage_max_rows_;
     const int64_t want = std::min<int64_t>(cnt, std::max<int64_t>(store_cap - stored, 0));
-    if (want > a.leaf_cap) {  // staging too small: grow and replay the count pass (idempotent)
-        stage_rows_ = want;
-        g_->stage.ensure((size_t)want * std::max<int32_t>(g_->max_out + 2, 2));
-        a.leaf_rows = g_->stage.get();
-        a.leaf_cap = want;
-        MCE_CUDA(cudaMemsetAsync(leaf_total_, 0, 2 * sizeof(unsigned long long), s_));
+    int64_t &cap = kind ? a.clq_cap : a.leaf_cap;
+    if (want > cap) {  // staging too small: grow and replay the count pass (idempotent)
+        (kind ? cstage_rows_ : stage_rows_) = want;
+        stage.ensure((size_t)want * std::max<int32_t>(g_->max_out + 2, 2));
+        (kind ? a.clq_rows : a.leaf_rows) = stage.get();
+        cap = want;
+        MCE_CUDA(cudaMemsetAsync(leaf_total_, 0, 4 * sizeof(unsigned long long), s_));
         launch_expand(a, false, s_);
         ++kernels_;
         stream_sync(s_);
     }
-    const int64_t take = std::min<int64_t>(want, a.leaf_cap);
+    const int64_t take = std::min<int64_t>(want, cap);
     if (take > 0) {  // append to the device store (grown with copy; read out once at the end)
         const size_t need = (size_t)(stored + take) * size;
         if (g_->store.n < need) {
@@ -279,7 +299,7 @@ void Engine::handle_leaves(int32_t size, int64_t cnt, ExpandArgs &a) {
             stream_sync(s_);  // the old block goes back to the cache only when unused
             g_->store = std::move(bigger);
         }
-        MCE_CUDA(cudaMemcpyAsync(g_->store.get() + (size_t)stored * size, g_->stage.get(),
+        MCE_CUDA(cudaMemcpyAsync(g_->store.get() + (size_t)stored * size, stage.get(),
                                  sizeof(int32_t) * take * size, cudaMemcpyDeviceToDevice, s_));
         stored_ += take;
     }
@@ -313,12 +333,9 @@ bool Engine::run_small(int32_t k, const Level &L) {
     a.ocol = g_->ocol.get();
     a.order = g_->vid.get();
     a.maxbit = maxbit_;
-    a.leaf_total = leaf_total_;
-    a.leaf_slot = leaf_slot_;
-    a.leaf_rows = g_->stage.get();
-    a.leaf_cap = stage_rows_;
+    leaf_args(a);
     a.chain = chain_dev_;
-    MCE_CUDA(cudaMemsetAsync(leaf_total_, 0, 2 * sizeof(unsigned long long), s_));
+    MCE_CUDA(cudaMemsetAsync(leaf_total_, 0, 4 * sizeof(unsigned long long), s_));
     const int t = clock_.start(1);
     launch_expand_small(a, scratch, scratch_bytes, dout, chain_dev_, s_);
     clock_.stop(t);
@@ -337,7 +354,7 @@ bool Engine::run_small(int32_t k, const Level &L) {
         fprintf(stderr, "[mce] fused levels k=%d..%lld entries=%lld -> children=%lld leaves=%lld status=%lld\n", k,
                 (long long)(k + o.levels - 1), (long long)L.count, (long long)o.children, (long long)o.leaves,
                 (long long)o.status);
-    if (o.leaves > 0) {  // leaves of size k_next from the last processed level
+    if (o.leaves > 0 || o.cliques > 0) {  // leaves of size k_next / completions of size need, last level
         ExpandArgs la = a;
         la.P = o.inP;
         la.slot = o.inslot;
@@ -347,7 +364,9 @@ bool Engine::run_small(int32_t k, const Level &L) {
         la.k = (int32_t)o.k_next - 1;
         la.Wp = la.Wc = (int32_t)o.inW;
         la.counts = arena_.alloc<int32_t>(o.inN);  // for a count-pass replay if the staging must grow
-        handle_leaves((int32_t)o.k_next, o.leaves, la);
+        handle_leaves((int32_t)o.k_next, o.leaves, la, 0);
+        if (o.cliques > 0 && (o.leaves == 0 || (!find_one_ && la.need == (int32_t)o.k_next)))
+            handle_leaves(la.need, o.cliques, la, 1);
     }
     sync_bound(true);
     if (o.status == 1 && o.children > 0) {
@@ -398,26 +417,24 @@ void Engine::process(int32_t k, const Level &L) {
     a.order = g_->vid.get();
     a.counts = counts;
     a.maxbit = maxbit_;
-    a.leaf_total = leaf_total_;
-    a.leaf_slot = leaf_slot_;
-    a.leaf_rows = g_->stage.get();
-    a.leaf_cap = stage_rows_;
+    leaf_args(a);
     a.chain = chain_dev_;
 
-    // misc[0..2] = leaf total, leaf slot, maxbit (-1)
-    MCE_CUDA(cudaMemsetAsync(leaf_total_, 0, 2 * sizeof(unsigned long long), s_));
+    // misc[0..4] = leaf total, leaf slot, completion total, completion slot, maxbit (-1)
+    MCE_CUDA(cudaMemsetAsync(leaf_total_, 0, 4 * sizeof(unsigned long long), s_));
     MCE_CUDA(cudaMemsetAsync(maxbit_, 0xff, 2 * sizeof(int32_t), s_));
     launch_timed(a, false);
     exclusive_scan_i32(counts, offs, N, tmp, s_);
     kernels_ += 3;
-    int64_t *h = g_->host.get<int64_t>(4);
+    int64_t *h = g_->host.get<int64_t>(6);
     MCE_CUDA(cudaMemcpyAsync(h, offs + N, sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
-    MCE_CUDA(cudaMemcpyAsync(h + 1, leaf_total_, 3 * sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
+    MCE_CUDA(cudaMemcpyAsync(h + 1, leaf_total_, 5 * sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
     stream_sync(s_);
     const int64_t total = h[0];
     const unsigned long long leaves = (unsigned long long)h[1];
-    const int32_t maxbit = (int32_t)(uint32_t)(uint64_t)h[3];
-    const int32_t maxub = (int32_t)(uint32_t)((uint64_t)h[3] >> 32);  // deepest reachable level
+    const int64_t completions = h[3];
+    const int32_t maxbit = (int32_t)(uint32_t)(uint64_t)h[5];
+    const int32_t maxub = (int32_t)(uint32_t)((uint64_t)h[5] >> 32);  // deepest reachable level
     // children's candidate sets only use bits <= maxbit: shrink their stride
     // (power of two, so the kernels stay specialised)
     int32_t Wc = 1;
@@ -426,7 +443,10 @@ void Engine::process(int32_t k, const Level &L) {
     if (o_.verbose > 0)
         fprintf(stderr, "[mce] level k=%d entries=%lld children=%lld leaves=%llu need=%d\n", k, (long long)N,
                 (long long)total, leaves, a.need);
-    if (leaves) handle_leaves(k + 1, (int64_t)leaves, a);
+    const int32_t need_counted = a.need;
+    if (leaves) handle_leaves(k + 1, (int64_t)leaves, a, 0);
+    if (completions > 0 && (leaves == 0 || (!find_one_ && need_counted == k + 1)))
+        handle_leaves(need_counted, completions, a, 1);
 
     const int64_t per_child = 8 * Wc + 12 + 12 + 16;
     // When the children do not fit they are produced in chunks.  Each chunk may
@@ -563,11 +583,10 @@ void Engine::do_class_w1(const int32_t *list, int64_t count) {
         if (leaves > 0) {
             ExpandArgs la{};
             la.k = 1;
+            leaf_args(la);
             la.leaf_rows = ra.leaf_rows;
             la.leaf_cap = ra.leaf_cap;
-            la.leaf_total = leaf_total_;
-            la.leaf_slot = leaf_slot_;
-            handle_leaves(2, leaves, la);
+            handle_leaves(2, leaves, la, 0);
         }
         const int64_t entries = (int64_t)hc[2];
         if (o_.verbose > 0)
@@ -721,11 +740,15 @@ mce_result *Engine::run() {
     g_->misc.ensure(256 + sizeof(LevelLink) * chain_cap_);
     leaf_total_ = reinterpret_cast<unsigned long long *>(g_->misc.get());
     leaf_slot_ = leaf_total_ + 1;
-    maxbit_ = reinterpret_cast<int32_t *>(leaf_total_ + 2);
+    clq_total_ = leaf_total_ + 2;
+    clq_slot_ = leaf_total_ + 3;
+    maxbit_ = reinterpret_cast<int32_t *>(leaf_total_ + 4);
     chain_dev_ = reinterpret_cast<LevelLink *>(g_->misc.get() + 256);
     stage_max_rows_ = std::max<int64_t>(1ll << 20, budget / 4 / (4ll * std::max<int32_t>(g_->max_out + 2, 2)));
     stage_rows_ = find_one_ ? 1 : 4096;
     g_->stage.ensure((size_t)stage_rows_ * std::max<int32_t>(g_->max_out + 2, 2));
+    cstage_rows_ = find_one_ ? 1 : 4096;
+    g_->cstage.ensure((size_t)cstage_rows_ * std::max<int32_t>(g_->max_out + 2, 2));
 
     res->h_setup_ms = ms_since(h2);
     const auto h3 = clk::now();

@@ -60,30 +60,53 @@ __global__ void build_adj_w1(const RootInfo *__restrict__ roots, int64_t nroots,
 
 // W >= 2: one block per root, warp per row.  Row i of the root-local
 // adjacency is N+(V[i]) ∩ V: the warp reads N+(V[i]) 32 elements at a time
-// (coalesced), every lane binary-searches its element in the staged V
-// (CSR ids order V but need not follow the orientation, so all of V),
-// and a hit at c sets bits (i, c) and (c, i).  The row stops at the first
-// chunk beyond V[L-1].  Bits go to a shared-memory bit matrix when it fits
-// (SMEM), else straight to the (zeroed) global matrix.
+// (coalesced) and every lane looks its element up in V (CSR ids order V but
+// need not follow the orientation, so all of V): a hit at c sets bits (i, c)
+// and (c, i).  The row stops at the first chunk beyond V[L-1].
+//   Lookup: when V's id span [V[0], V[L-1]] is at most kSpanBits, V is a bit
+// map over the span in shared memory with a rank per 32-bit word (position =
+// rank + popc of the lower bits): two shared loads instead of a log2(L)-step
+// binary search (the R-MAT hub core is a contiguous suffix of CSR-id space, so
+// the spans are short); otherwise binary search in the staged V.  Bits go to
+// a shared-memory bit matrix when it fits (SMEM), else straight to the
+// (zeroed) global matrix.
+constexpr int kSpanBits = 1 << 18;
+constexpr int kSpanWords = kSpanBits / 32;
 template <bool SMEM>
 __global__ void build_adj_block(const RootInfo *__restrict__ roots, int64_t nroots, int W,
                                 const int64_t *__restrict__ orp, const int32_t *__restrict__ ocol,
-                                uint64_t *__restrict__ adj) {
+                                uint64_t *__restrict__ adj, int Lmax, int use_map) {
     extern __shared__ int32_t dsm[];
     const int lane = threadIdx.x & 31;
     const int wib = threadIdx.x >> 5, nwb = blockDim.x >> 5;
+    int32_t *sV = dsm;
+    uint32_t *sA = reinterpret_cast<uint32_t *>(dsm + ((Lmax + 3) & ~3));
+    uint32_t *sMap = sA + (SMEM ? (size_t)Lmax * W * 2 : 0);
+    uint16_t *sRank = reinterpret_cast<uint16_t *>(sMap + (use_map ? kSpanWords : 0));
     for (int64_t j = blockIdx.x; j < nroots; j += gridDim.x) {
         const RootInfo ri = roots[j];
         const int L = ri.L;
-        int32_t *sV = dsm;
-        uint32_t *sA = reinterpret_cast<uint32_t *>(dsm + ((L + 3) & ~3));
         uint32_t *gA = reinterpret_cast<uint32_t *>(adj + ri.abase);
         uint32_t *A = SMEM ? sA : gA;
         for (int i = threadIdx.x; i < L; i += blockDim.x) sV[i] = __ldg(ocol + ri.vbase + i);
         if (SMEM)
             for (int64_t w = threadIdx.x; w < (int64_t)L * W * 2; w += blockDim.x) sA[w] = 0u;
         __syncthreads();
-        const int32_t vmax = sV[L - 1];
+        const int32_t vmin = sV[0], vmax = sV[L - 1];
+        const bool map = use_map && (int64_t)vmax - vmin < kSpanBits;
+        if (map) {
+            const int nw = ((vmax - vmin) >> 5) + 1;
+            for (int w = threadIdx.x; w < nw; w += blockDim.x) sMap[w] = 0u;
+            __syncthreads();
+            for (int p = threadIdx.x; p < L; p += blockDim.x) {
+                const int off = sV[p] - vmin, w = off >> 5;
+                atomicOr(sMap + w, 1u << (off & 31));
+                // words after the previous member's word up to this one start with rank p
+                const int wprev = p ? ((sV[p - 1] - vmin) >> 5) : -1;
+                for (int x = wprev + 1; x <= w; ++x) sRank[x] = (uint16_t)p;
+            }
+            __syncthreads();
+        }
         for (int i = wib; i < L; i += nwb) {
             const int32_t a = sV[i];
             const int64_t pb = __ldg(orp + a), pe = __ldg(orp + a + 1);
@@ -91,8 +114,15 @@ __global__ void build_adj_block(const RootInfo *__restrict__ roots, int64_t nroo
                 const int64_t p = p0 + lane;
                 const int32_t u = p < pe ? __ldg(ocol + p) : INT32_MAX;
                 if (__shfl_sync(0xffffffffu, u, 0) > vmax) break;
-                if (u <= vmax) {
-                    int lo = 0, hi = L;  // CSR-id order need not follow the orientation
+                int c = -1;
+                if (map) {
+                    if (u >= vmin && u <= vmax) {
+                        const int off = u - vmin, w = off >> 5;
+                        const uint32_t bits = sMap[w], bit = 1u << (off & 31);
+                        if (bits & bit) c = sRank[w] + __popc(bits & (bit - 1u));
+                    }
+                } else if (u <= vmax) {
+                    int lo = 0, hi = L;
                     while (lo < hi) {
                         const int mid = (lo + hi) >> 1;
                         if (sV[mid] < u)
@@ -100,19 +130,20 @@ __global__ void build_adj_block(const RootInfo *__restrict__ roots, int64_t nroo
                         else
                             hi = mid;
                     }
-                    if (lo < L && sV[lo] == u) {  // local indices L-1-position (expand.cuh)
-                        const int li = L - 1 - i, lc = L - 1 - lo;
-                        atomicOr(A + (int64_t)li * 2 * W + (lc >> 5), 1u << (lc & 31));
-                        atomicOr(A + (int64_t)lc * 2 * W + (li >> 5), 1u << (li & 31));
-                    }
+                    if (lo < L && sV[lo] == u) c = lo;
+                }
+                if (c >= 0) {  // local indices L-1-position (expand.cuh)
+                    const int li = L - 1 - i, lc = L - 1 - c;
+                    atomicOr(A + (int64_t)li * 2 * W + (lc >> 5), 1u << (lc & 31));
+                    atomicOr(A + (int64_t)lc * 2 * W + (li >> 5), 1u << (li & 31));
                 }
             }
         }
         __syncthreads();
         if (SMEM) {
             for (int64_t w = threadIdx.x; w < (int64_t)L * W * 2; w += blockDim.x) gA[w] = sA[w];
-            __syncthreads();
         }
+        __syncthreads();
     }
 }
 
@@ -151,6 +182,55 @@ __device__ void store_leaf(const ExpandArgs &a, int64_t e, int32_t v, const Root
     row[0] = a.order[ri.r];
 }
 
+// Store one clique completion C + P of size a.need (count pass): the caller
+// checked that P is a clique and k + |P| == need.  G lanes of a tile hold the
+// words of P (lane gl: words gl, gl + G, ...; WPL per lane); returns with the
+// row written by the whole tile.
+template <int G, int WPL>
+__device__ void store_clique_leaf(const ExpandArgs &a, int64_t e, const uint64_t (&P)[WPL], const RootInfo &ri,
+                                  unsigned gmask) {
+    const int gl = (threadIdx.x & 31) & (G - 1);
+    unsigned long long idx = 0;
+    if (gl == 0) {
+        idx = ~0ull;
+        if (*(volatile unsigned long long *)a.clq_slot < (unsigned long long)a.clq_cap) {
+            idx = atomicAdd(a.clq_slot, 1ull);
+            if ((int64_t)idx >= a.clq_cap) idx = ~0ull;
+        }
+    }
+    if (G > 1) idx = __shfl_sync(gmask, idx, 0, G);
+    if (idx == ~0ull) return;
+    int32_t *row = a.clq_rows + (int64_t)idx * a.need;
+    const int32_t *V = a.ocol + ri.vbase;
+    if (gl == 0) {
+        int64_t cur = e;
+        for (int32_t lev = a.k; lev >= 2; --lev) {
+            row[lev - 1] = a.order[V[ri.L - 1 - a.chain[lev].vloc[cur]]];
+            cur = a.chain[lev].parent[cur];
+        }
+        row[0] = a.order[ri.r];
+    }
+    int pc = 0;
+#pragma unroll
+    for (int t = 0; t < WPL; ++t) pc += __popcll(P[t]);
+    int incl = pc;
+#pragma unroll
+    for (int o = 1; o < G; o <<= 1) {
+        const int y = __shfl_up_sync(gmask, incl, o, G);
+        if (gl >= o) incl += y;
+    }
+    int pos = a.k + incl - pc;
+#pragma unroll
+    for (int t = 0; t < WPL; ++t) {
+        uint64_t q = P[t];
+        while (q) {
+            const int b = __ffsll((long long)q) - 1;
+            q &= q - 1;
+            row[pos++] = a.order[V[ri.L - 1 - ((gl + G * t) * 64 + b)]];
+        }
+    }
+}
+
 // highest set bit of a W-word set (-1 if empty)
 template <int W>
 __device__ __forceinline__ int top_bit(const uint64_t (&C)[W]) {
@@ -164,12 +244,15 @@ __device__ __forceinline__ int top_bit(const uint64_t (&C)[W]) {
 // end-of-kernel reductions of the count pass: leaves (sum) and the highest
 // candidate bit of any surviving child (max) -> the children's word stride
 // ... and the deepest level any descendant can reach (max of k + 1 + |P'|)
-__device__ __forceinline__ void flush_counters(const ExpandArgs &a, unsigned long long nleaf, int hb, int ub) {
+__device__ __forceinline__ void flush_counters(const ExpandArgs &a, unsigned long long nleaf, unsigned long long nclq,
+                                               int hb, int ub) {
     nleaf = __reduce_add_sync(0xffffffffu, (unsigned)nleaf);
+    nclq = __reduce_add_sync(0xffffffffu, (unsigned)nclq);
     hb = __reduce_max_sync(0xffffffffu, hb + 1) - 1;
     ub = __reduce_max_sync(0xffffffffu, ub);
     if ((threadIdx.x & 31) == 0) {
         if (nleaf) atomicAdd(a.leaf_total, nleaf);
+        if (nclq) atomicAdd(a.clq_total, nclq);
         if (hb >= 0) atomicMax(a.maxbit, hb);
         if (ub > 0) atomicMax(a.maxbit + 1, ub);
     }
@@ -185,7 +268,7 @@ __device__ __forceinline__ void flush_counters(const ExpandArgs &a, unsigned lon
 // into the caller's counters.
 template <int W, bool WRITE>
 __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, int64_t out, unsigned &nleaf,
-                                                int &hb, int &ub) {
+                                                unsigned &nclq, int &hb, int &ub) {
     uint64_t P[W];
 #pragma unroll
     for (int w = 0; w < W; ++w) P[w] = a.P[e * W + w];
@@ -193,7 +276,7 @@ __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, 
     const uint64_t *A = a.adj + ri.abase;
     const int Wa = a.Wa;
     uint8_t ord[64 * W];
-    uint8_t colr[64 * W];
+    uint8_t colr[64 * W];  // colour - 1 (a full 4-word set has 256 colours)
     int np = 0;
     int ncol = 0;
     if (a.bound == 1) {
@@ -220,7 +303,7 @@ __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, 
                     Q[w] &= ~(1ull << b);
                     U[w] &= ~(1ull << b);
                     ord[np] = (uint8_t)v;
-                    colr[np] = (uint8_t)ncol;
+                    colr[np] = (uint8_t)(ncol - 1);
                     ++np;
                 }
             }
@@ -233,11 +316,19 @@ __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, 
                 const int b = __ffsll((long long)q) - 1;
                 q &= q - 1;
                 ord[np] = (uint8_t)(w * 64 + b);
-                colr[np] = (uint8_t)(np + 1);
+                colr[np] = (uint8_t)np;
                 ++np;
             }
         }
         ncol = np;
+    }
+    // P is a clique iff every colour class is a single vertex (reading 10)
+    if (a.shortcut && a.bound == 1 && np >= 2 && ncol == np && a.k + np == a.need) {
+        if (!WRITE) {
+            ++nclq;
+            store_clique_leaf<1, W>(a, e, P, ri, 0xffffffffu);
+        }
+        return 0;
     }
     int32_t cnt = 0;
     if (a.k + ncol >= a.need) {
@@ -245,7 +336,7 @@ __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, 
 #pragma unroll
         for (int w = 0; w < W; ++w) R[w] = P[w];
         for (int i = np - 1; i >= 0; --i) {
-            if (a.k + colr[i] < a.need) break;
+            if (a.k + 1 + colr[i] < a.need) break;
             const int v = ord[i];
             const uint64_t *row = A + (int64_t)v * Wa;
             uint64_t C[W];
@@ -284,7 +375,7 @@ __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, 
 template <int W, bool WRITE>
 __global__ void __launch_bounds__(256) expand_thread(const ExpandArgs a) {
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    unsigned nleaf = 0;
+    unsigned nleaf = 0, nclq = 0;
     int hb = -1, ub = 0;
     for (int64_t e = a.begin + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < a.end; e += stride) {
         int64_t out = 0;
@@ -293,10 +384,10 @@ __global__ void __launch_bounds__(256) expand_thread(const ExpandArgs a) {
             if (a.offsets[e + 1] == out) continue;
             out -= a.out_base;
         }
-        const int32_t cnt = expand_entry<W, WRITE>(a, e, out, nleaf, hb, ub);
+        const int32_t cnt = expand_entry<W, WRITE>(a, e, out, nleaf, nclq, hb, ub);
         if (!WRITE) a.counts[e] = cnt;
     }
-    if (!WRITE) flush_counters(a, nleaf, hb, ub);
+    if (!WRITE) flush_counters(a, nleaf, nclq, hb, ub);
 }
 
 // ---------------------------------------------------------------------------
@@ -306,10 +397,10 @@ constexpr int kSmallThreads = 1024;
 
 template <bool WRITE>
 __device__ __forceinline__ int32_t expand_entry_w(int W, const ExpandArgs &a, int64_t e, int64_t out,
-                                                  unsigned &nleaf, int &hb, int &ub) {
-    if (W == 1) return expand_entry<1, WRITE>(a, e, out, nleaf, hb, ub);
-    if (W == 2) return expand_entry<2, WRITE>(a, e, out, nleaf, hb, ub);
-    return expand_entry<4, WRITE>(a, e, out, nleaf, hb, ub);
+                                                  unsigned &nleaf, unsigned &nclq, int &hb, int &ub) {
+    if (W == 1) return expand_entry<1, WRITE>(a, e, out, nleaf, nclq, hb, ub);
+    if (W == 2) return expand_entry<2, WRITE>(a, e, out, nleaf, nclq, hb, ub);
+    return expand_entry<4, WRITE>(a, e, out, nleaf, nclq, hb, ub);
 }
 
 __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a0, uint8_t *scratch,
@@ -318,7 +409,7 @@ __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a
     __shared__ ExpandArgs A;
     __shared__ int32_t offs[kSmallMax + 1];
     __shared__ int32_t wsum[kSmallThreads / 32];
-    __shared__ unsigned s_leaf;
+    __shared__ unsigned s_leaf, s_clq;
     __shared__ int s_hb, s_ub;
     __shared__ int64_t s_used;
     const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
@@ -327,6 +418,7 @@ __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a
         s_used = 0;
         out->levels = 0;
         out->leaves = 0;
+        out->cliques = 0;
         out->status = 2;
         out->k_next = a0.k;
         out->children = a0.end - a0.begin;
@@ -345,17 +437,19 @@ __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a
         if (N > kSmallMax || W > 4 || s_used + worst > scratch_bytes) break;  // status 2: host takes level k
         if (t == 0) {
             s_leaf = 0;
+            s_clq = 0;
             s_hb = -1;
             s_ub = 0;
             chain[A.k] = LevelLink{A.parent, A.vloc};
         }
         __syncthreads();
         // count pass, one candidate per thread
-        unsigned nleaf = 0;
+        unsigned nleaf = 0, nclq = 0;
         int hb = -1, ub = 0;
         int32_t cnt = 0;
-        if (t < N) cnt = expand_entry_w<false>(W, A, A.begin + t, 0, nleaf, hb, ub);
+        if (t < N) cnt = expand_entry_w<false>(W, A, A.begin + t, 0, nleaf, nclq, hb, ub);
         if (nleaf) atomicAdd(&s_leaf, nleaf);
+        if (nclq) atomicAdd(&s_clq, nclq);
         if (hb >= 0) atomicMax(&s_hb, hb);
         if (ub > 0) atomicMax(&s_ub, ub);
         // block exclusive scan of the counts
@@ -385,6 +479,7 @@ __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a
             out->level_n[lev] = N;
             out->levels = lev + 1;
             out->leaves = s_leaf;
+            out->cliques = s_clq;
             out->inP = const_cast<uint64_t *>(A.P);
             out->inslot = const_cast<int32_t *>(A.slot);
             out->inparent = const_cast<int32_t *>(A.parent);
@@ -394,6 +489,7 @@ __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a
             out->k_next = A.k + 1;
             out->children = total;
             if (s_leaf) atomicAdd(A.leaf_total, (unsigned long long)s_leaf);
+            if (s_clq) atomicAdd(A.clq_total, (unsigned long long)s_clq);
         }
         if (total == 0) {
             if (t == 0) out->status = 0;
@@ -420,9 +516,9 @@ __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a
         }
         __syncthreads();
         // write pass
-        if (t < N && cnt > 0) expand_entry_w<true>(W, A, A.begin + t, offs[t], nleaf, hb, ub);
+        if (t < N && cnt > 0) expand_entry_w<true>(W, A, A.begin + t, offs[t], nleaf, nclq, hb, ub);
         __syncthreads();
-        const bool stop = s_leaf > 0 || total > kSmallMax;
+        const bool stop = s_leaf > 0 || s_clq > 0 || total > kSmallMax;
         if (t == 0) {
             out->P = A.cP;
             out->slot = A.cslot;
@@ -462,7 +558,7 @@ __global__ void expand_tile(const ExpandArgs a, int max_l) {
     const int64_t tile = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / G;
     const int64_t ntiles = ((int64_t)gridDim.x * blockDim.x) / G;
     const int W = a.Wp, Wa = a.Wa;
-    unsigned nleaf = 0;
+    unsigned nleaf = 0, nclq = 0;
     int hb = -1, ub = 0;
     for (int64_t e = a.begin + tile; e < a.end; e += ntiles) {
         int64_t out = 0;
@@ -556,6 +652,15 @@ __global__ void expand_tile(const ExpandArgs a, int max_l) {
             ncol = np;
         }
         __syncwarp(gmask);
+        if (a.shortcut && a.bound == 1 && np >= 2 && ncol == np && a.k + np == a.need) {
+            if (!WRITE) {
+                if (gl == 0) ++nclq;
+                store_clique_leaf<G, WPL>(a, e, P, ri, gmask);
+                if (gl == 0) a.counts[e] = 0;
+            }
+            __syncwarp(gmask);
+            continue;
+        }
         int32_t cnt = 0;
         if (a.k + ncol >= a.need) {
             uint64_t R[WPL];
@@ -612,7 +717,7 @@ __global__ void expand_tile(const ExpandArgs a, int max_l) {
         if (!WRITE && gl == 0) a.counts[e] = cnt;
         __syncwarp(gmask);
     }
-    if (!WRITE) flush_counters(a, nleaf, hb, ub);
+    if (!WRITE) flush_counters(a, nleaf, nclq, hb, ub);
 }
 
 __global__ void classify_roots_kernel(int64_t n, const int64_t *__restrict__ orp, int32_t min_len,
@@ -726,21 +831,32 @@ void launch_build_adj(const RootInfo *roots, int64_t nroots, int W, const int64_
     if (W == 1) {
         build_adj_w1<<<grid_for(nroots * 32, 256, 16), 256, 0, s>>>(roots, nroots, orp, ocol, adj);
     } else {
-        // shared-memory bit matrix up to W = 16 (L <= 1024: 128 KB + V)
+        // shared-memory bit matrix up to W = 16 (L <= 1024: 128 KB), the
+        // staged V, and the span bit map + word ranks (48 KB)
         const int64_t Lmax = 64ll * W;
-        const size_t smem = sizeof(int32_t) * (size_t)Lmax + (size_t)Lmax * W * 8;
+        const size_t map_bytes = (size_t)kSpanWords * 4 + (size_t)kSpanWords * 2;
+        const size_t base = sizeof(int32_t) * (size_t)((Lmax + 3) & ~3ll);
         if (W <= 16) {
+            const size_t smem = base + (size_t)Lmax * W * 8 + map_bytes;
             static size_t attr_set = 0;
-            if (smem > 48 * 1024 && attr_set < smem) {
+            if (attr_set < smem) {
                 MCE_CUDA(cudaFuncSetAttribute(build_adj_block<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                               (int)smem));
                 attr_set = smem;
             }
-            build_adj_block<true><<<grid_for(nroots, 1, 8), 512, smem, s>>>(roots, nroots, W, orp, ocol, adj);
+            build_adj_block<true><<<grid_for(nroots, 1, 8), 1024, smem, s>>>(roots, nroots, W, orp, ocol, adj,
+                                                                              (int)Lmax, 1);
         } else {
+            const size_t smem = base + map_bytes;
+            static size_t attr_set = 0;
+            if (attr_set < smem) {
+                MCE_CUDA(cudaFuncSetAttribute(build_adj_block<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                              (int)smem));
+                attr_set = smem;
+            }
             MCE_CUDA(cudaMemsetAsync(adj, 0, sizeof(uint64_t) * (size_t)adj_words, s));
-            build_adj_block<false><<<grid_for(nroots, 1, 8), 512, sizeof(int32_t) * Lmax, s>>>(roots, nroots, W, orp,
-                                                                                                ocol, adj);
+            build_adj_block<false><<<grid_for(nroots, 1, 8), 1024, smem, s>>>(roots, nroots, W, orp, ocol, adj,
+                                                                               (int)Lmax, 1);
         }
     }
     MCE_LAUNCH_CHECK();

@@ -63,6 +63,15 @@ struct ExpandArgs {
     int32_t *leaf_rows;
     int64_t leaf_cap;  // rows
     const LevelLink *chain;  // chain[1..k]
+    // clique completions (count pass, reading 10): an entry whose
+    // candidate set P is itself a clique with k + |P| == need has exactly one
+    // clique of interest below it, C + P; it is recorded (size need) instead of
+    // expanded.  shortcut = 0 expands every level as Algorithm 2 does.
+    int32_t shortcut;
+    unsigned long long *clq_total;
+    unsigned long long *clq_slot;
+    int32_t *clq_rows;
+    int64_t clq_cap;  // rows of `need` vertices
 };
 
 // Fused root level for W == 1 roots (roots.cu): one warp per root builds the
@@ -102,6 +111,7 @@ struct SmallOut {
     int64_t children;  // its entries
     int64_t Wc;        // its word stride
     int64_t leaves;    // leaves (size k_next) recorded by the last processed level
+    int64_t cliques;   // clique completions (size need) recorded by the last processed level
     uint64_t *P;       // the level the host continues with
     int32_t *slot, *parent, *vloc;
     uint64_t *inP;     // the last processed level (for a leaf replay)

@@ -36,6 +36,7 @@ struct mce_graph {
     mce::PinnedBuf host;           // pinned staging for small device->host reads (per device, shared)
     mce::DevBuf<uint8_t> misc;     // engine: leaf counter + level chain (persistent)
     mce::DevBuf<int32_t> stage;    // engine: staged leaf cliques of one launch (grow-only)
+    mce::DevBuf<int32_t> cstage;   // engine: staged clique completions of one launch (grow-only)
     mce::DevBuf<int32_t> store;    // engine: stored maximum cliques of the run (grow-only)
 };
 

@@ -47,12 +47,24 @@ __device__ __forceinline__ bool adjacent(const int64_t *__restrict__ rowptr, con
     return contains_sorted(col, wb, we, x);
 }
 
+// Early abort (exact).  A run's final size is at most |C| + |P| at any
+// point, and at most t(s) + 1 from the start, t(s) = min(deg(s), core(s)) (a
+// clique through s has at most core(s) + 1 vertices).  Unless every run size
+// is wanted, a run stops as soon as that cap falls STRICTLY below the best
+// size found so far: it can no longer reach the best, so neither the best
+// size nor the winning seed (the first in seed order among runs reaching it)
+// changes.  The size it stores is then < the final best, never equal.
+__device__ __forceinline__ int32_t ld_best(const int32_t *best) {
+    int32_t v;
+    asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(best) : "memory");
+    return v;
+}
+
 // One greedy run for seed s by a tile of G lanes (G = 8 or 32) of the calling
-// warp.  Writes the clique (in order added) to `clique` when non-null.
-// Returns the clique size.
+// warp.  Returns the clique size (a partial size < the best when aborted).
 template <int G>
 __device__ int32_t greedy_run(int32_t s, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
-                              const int32_t *__restrict__ thr, int32_t *__restrict__ scratch, int32_t *clique) {
+                              const int32_t *__restrict__ thr, int32_t *__restrict__ scratch, const int32_t *best) {
     const int lane = threadIdx.x & 31;
     const int gl = lane & (G - 1);
     const int gbase = lane & ~(G - 1);
@@ -62,8 +74,13 @@ __device__ int32_t greedy_run(int32_t s, const int64_t *__restrict__ rowptr, con
     const int32_t *src = col + base;  // first round reads the CSR row directly
     int32_t *buf = scratch + base;    // later rounds work in place in the seed's segment
     int32_t csize = 1;
-    if (clique && gl == 0) clique[0] = s;
     while (len > 0) {
+        if (best) {
+            int32_t b = 0;
+            if (gl == 0) b = ld_best(best);
+            b = __shfl_sync(gmask, b, 0, G);
+            if (csize + len < b) break;
+        }
         unsigned long long key = 0;
         for (int64_t i = gl; i < len; i += G) {
             unsigned long long k2 = pick_key(thr, src[i]);
@@ -75,7 +92,6 @@ __device__ int32_t greedy_run(int32_t s, const int64_t *__restrict__ rowptr, con
             key = y > key ? y : key;
         }
         const int32_t w = (int32_t)(0x7fffffffu - (uint32_t)(key & 0xffffffffull));
-        if (clique && gl == 0) clique[csize] = w;
         ++csize;
         const int64_t wb = rowptr[w], we = rowptr[w + 1];
         int64_t out = 0;
@@ -94,48 +110,211 @@ __device__ int32_t greedy_run(int32_t s, const int64_t *__restrict__ rowptr, con
     return csize;
 }
 
-// Warp w takes seeds [4w, 4w+4): when all four have degree <= 64 they run in
-// parallel on 8-lane tiles (low-degree seeds leave most of a warp idle),
-// otherwise one after another on the whole warp.  The best size is reduced
-// per block before one atomicMax per block.
+// One greedy run for seed s by the whole block (NT threads): block-wide argmax
+// and an order-preserving in-place compaction.  Hub seeds (degree > kBigSeed)
+// run this way so a long run is not serialised on one warp; the replay of the
+// winning run uses it too, writing the clique (in order added).
+constexpr int kBlockRun = 512;
+constexpr int64_t kBigSeed = 1024;
+template <int NT>
+__device__ int32_t block_run(int32_t s, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
+                             const int32_t *__restrict__ thr, int32_t *__restrict__ scratch, int32_t *clique,
+                             const int32_t *best) {
+    __shared__ unsigned long long wkey[NT / 32];
+    __shared__ int32_t wcnt[NT / 32];
+    __shared__ int32_t sbest;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int64_t base = rowptr[s];
+    int64_t len = rowptr[s + 1] - base;
+    const int32_t *src = col + base;
+    int32_t *buf = scratch + base;
+    int32_t csize = 1;
+    if (clique && threadIdx.x == 0) clique[0] = s;
+    while (len > 0) {
+        if (best) {
+            if (threadIdx.x == 0) sbest = ld_best(best);
+            __syncthreads();
+            const int32_t b = sbest;
+            __syncthreads();
+            if (csize + len < b) break;
+        }
+        unsigned long long key = 0;
+        for (int64_t i = threadIdx.x; i < len; i += NT) {
+            const unsigned long long k2 = pick_key(thr, src[i]);
+            key = k2 > key ? k2 : key;
+        }
+        key = warp_max_u64(key);
+        if (lane == 0) wkey[wid] = key;
+        __syncthreads();
+        if (wid == 0) {
+            key = warp_max_u64(lane < NT / 32 ? wkey[lane] : 0ull);
+            if (lane == 0) wkey[0] = key;
+        }
+        __syncthreads();
+        key = wkey[0];
+        const int32_t w = (int32_t)(0x7fffffffu - (uint32_t)(key & 0xffffffffull));
+        if (clique && threadIdx.x == 0) clique[csize] = w;
+        ++csize;
+        const int64_t wb = rowptr[w], we = rowptr[w + 1];
+        int64_t out = 0;
+        for (int64_t i0 = 0; i0 < len; i0 += NT) {
+            const int64_t i = i0 + threadIdx.x;
+            const int32_t x = i < len ? src[i] : -1;
+            const bool keep = i < len && x != w && adjacent(rowptr, col, x, w, wb, we);
+            const unsigned m = __ballot_sync(0xffffffffu, keep);
+            __syncthreads();  // wkey/wcnt reuse, and every read of this chunk precedes its writes
+            if (lane == 0) wcnt[wid] = __popc(m);
+            __syncthreads();
+            int32_t before = 0, total = 0;
+#pragma unroll
+            for (int j = 0; j < NT / 32; ++j) {
+                const int32_t c = wcnt[j];
+                before += j < wid ? c : 0;
+                total += c;
+            }
+            if (keep) buf[out + before + __popc(m & lanemask_lt())] = x;
+            out += total;
+        }
+        __syncthreads();
+        src = buf;
+        len = out;
+    }
+    return csize;
+}
+
+// cap t(s) + 1 on the size of any run from seed s (see ld_best)
+__device__ __forceinline__ int64_t seed_cap(int32_t s, const int64_t *__restrict__ rowptr,
+                                            const int32_t *__restrict__ core) {
+    int64_t c = rowptr[s + 1] - rowptr[s];
+    if (core) c = min(c, (int64_t)__ldg(core + s));
+    return c + 1;
+}
+
+// Hub seeds (degree > kBigSeed): one block per run, launched before the rest
+// so the long runs start first and their sizes prune the short ones.
+__global__ void __launch_bounds__(kBlockRun) greedy_big_kernel(int64_t nbig, const int32_t *__restrict__ big,
+                                                               const int64_t *__restrict__ rowptr,
+                                                               const int32_t *__restrict__ col,
+                                                               const int32_t *__restrict__ thr,
+                                                               const int32_t *__restrict__ core,
+                                                               int32_t *__restrict__ scratch,
+                                                               int32_t *__restrict__ run_size, int32_t *best_size,
+                                                               int abort_runs) {
+    for (int64_t i = blockIdx.x; i < nbig; i += gridDim.x) {
+        const int32_t s = big[i];
+        int32_t c = 1;
+        if (!abort_runs || seed_cap(s, rowptr, core) >= ld_best(best_size))
+            c = block_run<kBlockRun>(s, rowptr, col, thr, scratch, nullptr, abort_runs ? best_size : nullptr);
+        if (threadIdx.x == 0) {
+            run_size[s] = c;
+            atomicMax(best_size, c);
+        }
+        __syncthreads();
+    }
+}
+
+// One greedy run for a seed of degree <= kThreadSeed by ONE thread: the
+// candidates and their pick keys stay in registers, alive ones marked in a
+// bit mask (no compaction, so no local memory); same picks as greedy_run.
+constexpr int kThreadSeed = 16;
+__device__ int32_t greedy_thread(int32_t s, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
+                                 const int32_t *__restrict__ thr, const int32_t *best) {
+    const int64_t base = rowptr[s];
+    const int len0 = (int)(rowptr[s + 1] - base);
+    int32_t P[kThreadSeed];
+    unsigned long long key[kThreadSeed];
+    uint32_t alive = 0;
+#pragma unroll
+    for (int i = 0; i < kThreadSeed; ++i) {
+        P[i] = i < len0 ? __ldg(col + base + i) : 0;
+        key[i] = i < len0 ? pick_key(thr, P[i]) : 0ull;
+        if (i < len0) alive |= 1u << i;
+    }
+    int32_t csize = 1;
+    while (alive) {
+        if (best && csize + __popc(alive) < ld_best(best)) break;
+        unsigned long long km = 0;
+#pragma unroll
+        for (int i = 0; i < kThreadSeed; ++i)
+            if (((alive >> i) & 1u) && key[i] > km) km = key[i];
+        const int32_t w = (int32_t)(0x7fffffffu - (uint32_t)(km & 0xffffffffull));
+        ++csize;
+        const int64_t wb = rowptr[w], we = rowptr[w + 1];
+#pragma unroll
+        for (int i = 0; i < kThreadSeed; ++i)
+            if ((alive >> i) & 1u)
+                if (P[i] == w || !adjacent(rowptr, col, P[i], w, wb, we)) alive &= ~(1u << i);
+    }
+    return csize;
+}
+
+// The other seeds (degree <= kBigSeed), thread per seed: degree <= kThreadSeed
+// runs on the seed's own thread, longer ones are queued in shared memory and
+// run by whole warps (greedy_run<32>) once the block's threads are done.  The
+// best size is published with one atomicMax per warp and group, so later
+// runs abort against it.
 __global__ void __launch_bounds__(256) greedy_kernel(int64_t nseeds, const int32_t *__restrict__ seeds,
                                                      const int64_t *__restrict__ rowptr,
                                                      const int32_t *__restrict__ col, const int32_t *__restrict__ thr,
+                                                     const int32_t *__restrict__ core,
                                                      int32_t *__restrict__ scratch, int32_t *__restrict__ run_size,
-                                                     int32_t *best_size) {
-    __shared__ int32_t block_best;
-    if (threadIdx.x == 0) block_best = 0;
+                                                     int32_t *best_size, int abort_runs) {
+    __shared__ int32_t queue[256];
+    __shared__ int qn;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int32_t *best = abort_runs ? best_size : nullptr;
+    if (threadIdx.x == 0) qn = 0;
     __syncthreads();
-    const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    const int lane = threadIdx.x & 31;
-    int32_t mybest = 0;
-    for (int64_t i0 = warp * 4; i0 < nseeds; i0 += nwarps * 4) {
-        const int64_t my = i0 + (lane >> 3);
-        const int32_t s_mine = my < nseeds ? seeds[my] : -1;
-        const int64_t d_mine = s_mine >= 0 ? rowptr[s_mine + 1] - rowptr[s_mine] : 0;
-        const bool small = __all_sync(0xffffffffu, d_mine <= 64);
-        if (small) {
-            if (s_mine >= 0) {
-                const int32_t c = greedy_run<8>(s_mine, rowptr, col, thr, scratch, nullptr);
-                if ((lane & 7) == 0) run_size[s_mine] = c;
-                mybest = max(mybest, c);
-            }
-        } else {
-            for (int t = 0; t < 4; ++t) {
-                const int32_t s = __shfl_sync(0xffffffffu, s_mine, 8 * t);
-                if (s < 0) break;
-                const int32_t c = greedy_run<32>(s, rowptr, col, thr, scratch, nullptr);
-                if (lane == 0) run_size[s] = c;
-                mybest = max(mybest, c);
-            }
+    int32_t published = 0;
+    for (int64_t b0 = (int64_t)blockIdx.x * blockDim.x; b0 < nseeds; b0 += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t i = b0 + threadIdx.x;
+        int32_t sd = i < nseeds ? seeds[i] : -1;
+        int64_t d = sd >= 0 ? rowptr[sd + 1] - rowptr[sd] : 0;
+        if (d > kBigSeed) sd = -1;  // run by greedy_big_kernel
+        if (sd >= 0 && best && seed_cap(sd, rowptr, core) < ld_best(best_size)) {
+            run_size[sd] = 1;  // cannot reach the best: not run
+            sd = -1;
         }
-        __syncwarp();
+        if (sd >= 0 && d > kThreadSeed) {
+            queue[atomicAdd(&qn, 1)] = sd;
+            sd = -1;
+        }
+        int32_t mybest = 0;
+        if (sd >= 0) {
+            mybest = greedy_thread(sd, rowptr, col, thr, best);
+            run_size[sd] = mybest;
+        }
+        __syncthreads();
+        const int nq = qn;
+        for (int q = wid; q < nq; q += blockDim.x >> 5) {
+            const int32_t sq = queue[q];
+            const int32_t c = greedy_run<32>(sq, rowptr, col, thr, scratch, best);
+            if (lane == 0) run_size[sq] = c;
+            mybest = max(mybest, c);
+        }
+        mybest = __reduce_max_sync(0xffffffffu, mybest);
+        if (lane == 0 && mybest > published) {
+            atomicMax(best_size, mybest);
+            published = mybest;
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) qn = 0;
+        __syncthreads();
     }
-    mybest = __reduce_max_sync(0xffffffffu, mybest);
-    if (lane == 0 && mybest) atomicMax(&block_best, mybest);
-    __syncthreads();
-    if (threadIdx.x == 0 && block_best) atomicMax(best_size, block_best);
+}
+
+__global__ void big_flags_kernel(int64_t nseeds, const int32_t *__restrict__ seeds,
+                                 const int64_t *__restrict__ rowptr, int32_t *flag) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nseeds; i += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t s = seeds[i];
+        flag[i] = rowptr[s + 1] - rowptr[s] > kBigSeed;
+    }
+}
+
+__global__ void gather_flagged_kernel(int64_t n, const int32_t *__restrict__ in, const int32_t *__restrict__ flag,
+                                      const int64_t *__restrict__ pos, int32_t *out) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        if (flag[i]) out[pos[i]] = in[i];
 }
 
 // among seeds whose run reached best, the first in seed order (threshold desc, id asc)
@@ -148,67 +327,15 @@ __global__ void best_seed_kernel(int64_t nseeds, const int32_t *__restrict__ see
     }
 }
 
-// Replay of the winning run to recover its clique: the same greedy steps as
-// greedy_run, by one block of kReplay threads (block-wide argmax and an
-// order-preserving in-place compaction), since a single run on a hub seed is
-// long and nothing else is running.
+// Replay of the winning run to recover its clique (one block, nothing else running)
 constexpr int kReplay = 1024;
 __global__ void __launch_bounds__(kReplay) replay_kernel(const unsigned long long *best_key,
                                                          const int64_t *__restrict__ rowptr,
                                                          const int32_t *__restrict__ col,
                                                          const int32_t *__restrict__ thr,
                                                          int32_t *__restrict__ scratch, int32_t *clique) {
-    __shared__ unsigned long long wkey[kReplay / 32];
-    __shared__ int32_t wcnt[kReplay / 32];
-    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     const int32_t s = (int32_t)(0x7fffffffu - (uint32_t)(*best_key & 0xffffffffull));
-    const int64_t base = rowptr[s];
-    int64_t len = rowptr[s + 1] - base;
-    const int32_t *src = col + base;
-    int32_t *buf = scratch + base;
-    int32_t csize = 1;
-    if (threadIdx.x == 0) clique[0] = s;
-    while (len > 0) {
-        unsigned long long key = 0;
-        for (int64_t i = threadIdx.x; i < len; i += kReplay) {
-            const unsigned long long k2 = pick_key(thr, src[i]);
-            key = k2 > key ? k2 : key;
-        }
-        key = warp_max_u64(key);
-        if (lane == 0) wkey[wid] = key;
-        __syncthreads();
-        if (wid == 0) {
-            key = warp_max_u64(wkey[lane]);
-            if (lane == 0) wkey[0] = key;
-        }
-        __syncthreads();
-        key = wkey[0];
-        const int32_t w = (int32_t)(0x7fffffffu - (uint32_t)(key & 0xffffffffull));
-        if (threadIdx.x == 0) clique[csize] = w;
-        ++csize;
-        const int64_t wb = rowptr[w], we = rowptr[w + 1];
-        int64_t out = 0;
-        for (int64_t i0 = 0; i0 < len; i0 += kReplay) {
-            const int64_t i = i0 + threadIdx.x;
-            const int32_t x = i < len ? src[i] : -1;
-            const bool keep = i < len && x != w && adjacent(rowptr, col, x, w, wb, we);
-            const unsigned m = __ballot_sync(0xffffffffu, keep);
-            __syncthreads();  // wkey/wcnt reuse, and every read of this chunk precedes its writes
-            if (lane == 0) wcnt[wid] = __popc(m);
-            __syncthreads();
-            int32_t before = 0, total = 0;
-            for (int j = 0; j < kReplay / 32; ++j) {
-                const int32_t c = wcnt[j];
-                before += j < wid ? c : 0;
-                total += c;
-            }
-            if (keep) buf[out + before + __popc(m & lanemask_lt())] = x;
-            out += total;
-        }
-        __syncthreads();
-        src = buf;
-        len = out;
-    }
+    block_run<kReplay>(s, rowptr, col, thr, scratch, clique, nullptr);
 }
 
 __global__ void degree_thr_kernel(int64_t n, const int64_t *__restrict__ rowptr, int32_t *thr) {
@@ -333,7 +460,7 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
         seed_ptr = sh;
         nseeds = mine;
     }
-    // ---- the runs
+    // ---- the runs: hub seeds first (block per run), then the rest
     int32_t *scratch = pool.take<int32_t>(std::max<int64_t>(g->nnz, 1));
     int32_t *run_size = pool.take<int32_t>(n), *best = pool.take<int32_t>(1);
     unsigned long long *best_key = pool.take<unsigned long long>(1);
@@ -341,9 +468,33 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
     MCE_CUDA(cudaMemsetAsync(run_size, 0, sizeof(int32_t) * n, s));
     MCE_CUDA(cudaMemsetAsync(best, 0, sizeof(int32_t), s));
     MCE_CUDA(cudaMemsetAsync(best_key, 0, sizeof(unsigned long long), s));
+    const int32_t *core = g->have_core ? g->core.get() : nullptr;
+    const int abort_runs = want_runs ? 0 : 1;
     if (nseeds > 0) {
-        greedy_kernel<<<grid_for(nseeds * 8, 256), 256, 0, s>>>(nseeds, seed_ptr, g->rowptr.get(), g->col.get(),
-                                                                  thr, scratch, run_size, best);
+        if (g->max_deg > kBigSeed) {
+            int32_t *flag = pool.take<int32_t>(nseeds);
+            int64_t *pos = pool.take<int64_t>(nseeds + 1), *tmp = pool.take<int64_t>(scan_tmp_items(nseeds));
+            int32_t *big = pool.take<int32_t>(nseeds);
+            big_flags_kernel<<<grid_for(nseeds, 256), 256, 0, s>>>(nseeds, seed_ptr, g->rowptr.get(), flag);
+            MCE_LAUNCH_CHECK();
+            exclusive_scan_i32(flag, pos, nseeds, tmp, s);
+            gather_flagged_kernel<<<grid_for(nseeds, 256), 256, 0, s>>>(nseeds, seed_ptr, flag, pos, big);
+            MCE_LAUNCH_CHECK();
+            int64_t *hnb = g->host.get<int64_t>(1);
+            MCE_CUDA(cudaMemcpyAsync(hnb, pos + nseeds, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+            stream_sync(s);
+            const int64_t nbig = hnb[0];
+            kernels += 5;
+            if (nbig > 0) {
+                const int blocks = (int)std::min<int64_t>(nbig, (int64_t)num_sms() * 4);
+                greedy_big_kernel<<<blocks, kBlockRun, 0, s>>>(nbig, big, g->rowptr.get(), g->col.get(), thr, core,
+                                                               scratch, run_size, best, abort_runs);
+                MCE_LAUNCH_CHECK();
+                ++kernels;
+            }
+        }
+        greedy_kernel<<<grid_for(nseeds, 256), 256, 0, s>>>(nseeds, seed_ptr, g->rowptr.get(), g->col.get(),
+                                                                  thr, core, scratch, run_size, best, abort_runs);
         MCE_LAUNCH_CHECK();
         best_seed_kernel<<<grid_for(nseeds, 256), 256, 0, s>>>(nseeds, seed_ptr, thr, run_size, best, best_key);
         MCE_LAUNCH_CHECK();

@@ -224,32 +224,202 @@ __device__ void root_step(const RootArgs &a, int32_t r, RootSmem<G * RPL> &sm, u
     __syncwarp(gmask);
 }
 
-// Warp w takes roots [4w, 4w+4): four 8-lane tiles when all four have
-// |N+(r)| <= 8 (the sparse case: BA m=4 roots have 4), else one root after
-// another on the whole warp (|N+(r)| <= 64).
-__global__ void __launch_bounds__(kRootWarps * 32) root_expand_w1(const RootArgs a) {
-    __shared__ RootSmem<64> sm_all[kRootWarps];
+// 8x8 bit-matrix transpose (row i = byte i, column j = bit j)
+__device__ __forceinline__ uint64_t transpose8(uint64_t x) {
+    uint64_t t;
+    t = (x ^ (x >> 7)) & 0x00AA00AA00AA00AAull;
+    x = x ^ t ^ (t << 7);
+    t = (x ^ (x >> 14)) & 0x0000CCCC0000CCCCull;
+    x = x ^ t ^ (t << 14);
+    t = (x ^ (x >> 28)) & 0x00000000F0F0F0F0ull;
+    x = x ^ t ^ (t << 28);
+    return x;
+}
+
+// warp exclusive prefix sum of x (all 32 lanes)
+__device__ __forceinline__ unsigned long long warp_excl(unsigned long long x, unsigned long long &total) {
     const int lane = threadIdx.x & 31;
-    RootSmem<64> &sm = sm_all[threadIdx.x >> 5];
-    RootSmem<8> *tiles = reinterpret_cast<RootSmem<8> *>(&sm);  // 4 x RootSmem<8> fit in one RootSmem<64>
-    static_assert(4 * sizeof(RootSmem<8>) <= sizeof(RootSmem<64>), "tile scratch");
-    const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    unsigned long long bytes = 0;  // algorithmic bytes read, tile leaders
-    for (int64_t i0 = warp * 4; i0 < a.count; i0 += nwarps * 4) {
-        const int64_t i = i0 + (lane >> 3);
-        const int32_t r = i < a.count ? __ldg(a.list + i * a.stride) : -1;
-        const int L = r >= 0 ? (int)(__ldg(a.orp + r + 1) - __ldg(a.orp + r)) : 0;
-        if (__all_sync(0xffffffffu, L <= 8)) {
-            if (r >= 0) root_step<8, 1>(a, r, tiles[lane >> 3], bytes);
-        } else {
-            for (int t = 0; t < 4; ++t) {
-                const int32_t rt = __shfl_sync(0xffffffffu, r, 8 * t);
-                if (rt < 0) break;
-                root_step<32, 2>(a, rt, sm, bytes);
+    unsigned long long inc = x;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const unsigned long long y = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= o) inc += y;
+    }
+    total = __shfl_sync(0xffffffffu, inc, 31);
+    return inc - x;
+}
+
+// The whole first expansion step of a root with L = |N+(r)| <= 8 by ONE
+// thread (the sparse case: BA m = 4 roots have L = 4).  Same steps as
+// root_step, in registers: the L x L bit matrix is one uint64 (row li = byte
+// li), built by testing every element of each out-row N+(V[p]) against the
+// L staged ids (or, for a long out-row, binary-searching the L ids in it) and
+// closed under symmetry with an 8x8 transpose; the colouring order, colours
+// and children are packed nibbles / bytes.  Called by all 32 lanes of a warp
+// (r < 0: no root) so survivors are materialised with warp-aggregated atomics.
+__device__ void root_thread(const RootArgs &a, int32_t r, unsigned long long &bytes) {
+    int L = 0;
+    int64_t vb = 0;
+    uint64_t adj = 0;
+    unsigned long long T = 0;
+    if (r >= 0) {
+        vb = __ldg(a.orp + r);
+        L = (int)(__ldg(a.orp + r + 1) - vb);
+        int32_t V[8];
+#pragma unroll
+        for (int p = 0; p < 8; ++p) V[p] = p < L ? __ldg(a.ocol + vb + p) : -1;
+        int64_t s0[8], s1[8];
+#pragma unroll
+        for (int p = 0; p < 8; ++p) {
+            s0[p] = s1[p] = 0;
+            if (p < L) {
+                s0[p] = __ldg(a.orp + V[p]);
+                s1[p] = __ldg(a.orp + V[p] + 1);
             }
         }
-        __syncwarp();
+#pragma unroll
+        for (int p = 0; p < 8; ++p) {
+            if (p >= L) break;
+            const int64_t d = s1[p] - s0[p];
+            T += (unsigned long long)d;
+            unsigned m = 0;  // positions c with V[c] in N+(V[p])
+            if (d <= 16) {
+                for (int64_t q = s0[p]; q < s1[p]; ++q) {
+                    const int32_t u = __ldg(a.ocol + q);
+#pragma unroll
+                    for (int c = 0; c < 8; ++c) m |= (unsigned)(V[c] == u) << c;
+                }
+            } else {
+#pragma unroll
+                for (int c = 0; c < 8; ++c)
+                    if (c < L && c != p && contains_sorted(a.ocol, s0[p], s1[p], V[c])) m |= 1u << c;
+            }
+            // local index = L-1-position (expand.cuh): reverse rows and columns
+            const unsigned lm = (__brev(m) >> (32 - L)) & 0xffu;
+            adj |= (uint64_t)lm << (8 * (L - 1 - p));
+        }
+        adj |= transpose8(adj);
+        bytes += 16ull + 20ull * (unsigned long long)L + 4ull * T;
+    }
+    auto row = [&](int v) -> uint64_t { return (adj >> (8 * v)) & 0xffull; };
+    // bound + children (|C| = 1)
+    const uint64_t P = (1ull << L) - 1;
+    uint32_t ord = 0, colr = 0;  // nibble j: j-th vertex in colouring order, its colour
+    int np = 0, ncol = 0;
+    if (a.bound == 1) {
+        uint64_t U = P;
+        while (U) {
+            ++ncol;
+            uint64_t Q = U;
+            while (Q) {
+                const int v = __ffsll((long long)Q) - 1;
+                Q &= ~row(v);
+                Q &= ~(1ull << v);
+                U &= ~(1ull << v);
+                ord |= (uint32_t)v << (4 * np);
+                colr |= (uint32_t)ncol << (4 * np);
+                ++np;
+            }
+        }
+    } else {
+        for (int j = 0; j < L; ++j) {
+            ord |= (uint32_t)j << (4 * j);
+            colr |= (uint32_t)(j + 1) << (4 * j);
+        }
+        np = ncol = L;
+    }
+    int cnt = 0;
+    uint64_t chP = 0;   // byte j: candidate set of child j
+    uint32_t chv = 0;   // nibble j: its local vertex
+    if (r >= 0 && 1 + ncol >= a.need) {
+        uint64_t R = P;
+        for (int j = np - 1; j >= 0; --j) {
+            if (1 + (int)((colr >> (4 * j)) & 0xf) < a.need) break;
+            const int v = (ord >> (4 * j)) & 0xf;
+            const uint64_t C = R & row(v);
+            R &= ~(1ull << v);
+            const int pc = __popcll(C);
+            if (pc == 0) {
+                if (2 >= a.need) {  // {r, v} is a leaf clique of interest
+                    const unsigned long long idx = atomicAdd(a.ctr + 3, 1ull);
+                    if ((int64_t)idx < a.leaf_cap) {
+                        a.leaf_rows[idx * 2] = __ldg(a.order + r);
+                        a.leaf_rows[idx * 2 + 1] = __ldg(a.order + __ldg(a.ocol + vb + (L - 1 - v)));
+                    }
+                }
+            } else if (2 + pc >= a.need) {
+                chP |= C << (8 * cnt);
+                chv |= (uint32_t)v << (4 * cnt);
+                ++cnt;
+            }
+        }
+    }
+    // materialise surviving roots: warp-aggregated slots for the three arrays
+    const bool surv = cnt > 0;
+    if (__any_sync(0xffffffffu, surv)) {
+        unsigned long long ts, tl, tc;
+        const unsigned long long os = warp_excl(surv ? 1ull : 0ull, ts);
+        const unsigned long long ol = warp_excl(surv ? (unsigned long long)L : 0ull, tl);
+        const unsigned long long oc = warp_excl((unsigned long long)cnt, tc);
+        unsigned long long bs = 0, bl = 0, bc = 0;
+        if ((threadIdx.x & 31) == 0) {
+            bs = atomicAdd(a.ctr + 0, ts);
+            bl = atomicAdd(a.ctr + 1, tl);
+            bc = atomicAdd(a.ctr + 2, tc);
+        }
+        bs = __shfl_sync(0xffffffffu, bs, 0) + os;
+        bl = __shfl_sync(0xffffffffu, bl, 0) + ol;
+        bc = __shfl_sync(0xffffffffu, bc, 0) + oc;
+        if (surv) {
+            RootInfo ri;
+            ri.r = r;
+            ri.L = L;
+            ri.vbase = vb;
+            ri.abase = (int64_t)bl;
+            a.roots[bs] = ri;
+            for (int i = 0; i < L; ++i) a.adj[bl + i] = row(i);
+            for (int j = 0; j < cnt; ++j) {
+                a.cP[bc + j] = (chP >> (8 * j)) & 0xffull;
+                a.cslot[bc + j] = (int32_t)bs;
+                a.cparent[bc + j] = -1;
+                a.cvloc[bc + j] = (int32_t)((chv >> (4 * j)) & 0xf);
+            }
+        }
+    }
+}
+
+// Thread per root: roots with |N+(r)| <= 8 run root_thread on their own lane;
+// longer ones (<= 64) are queued in shared memory and taken by whole warps
+// (root_step<32, 2>) once the block's threads are done.
+constexpr int kThreadRootMax = 8;
+__global__ void __launch_bounds__(kRootWarps * 32) root_expand_w1(const RootArgs a) {
+    __shared__ RootSmem<64> sm_all[kRootWarps];
+    __shared__ int32_t queue[kRootWarps * 32];
+    __shared__ int qn;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    RootSmem<64> &sm = sm_all[wid];
+    if (threadIdx.x == 0) qn = 0;
+    __syncthreads();
+    unsigned long long bytes = 0;  // algorithmic bytes read
+    for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < a.count; base += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t i = base + threadIdx.x;
+        int32_t r = i < a.count ? __ldg(a.list + i * a.stride) : -1;
+        const int L = r >= 0 ? (int)(__ldg(a.orp + r + 1) - __ldg(a.orp + r)) : 0;
+        if (r >= 0 && L > kThreadRootMax) {
+            queue[atomicAdd(&qn, 1)] = r;
+            r = -1;
+        }
+        root_thread(a, r, bytes);
+        __syncthreads();
+        const int nq = qn;
+        for (int q = wid; q < nq; q += kRootWarps) {
+            unsigned long long wb = 0;
+            root_step<32, 2>(a, queue[q], sm, wb);
+            if (lane == 0) bytes += wb;
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) qn = 0;
+        __syncthreads();
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) bytes += __shfl_xor_sync(0xffffffffu, bytes, o);
@@ -260,7 +430,7 @@ __global__ void __launch_bounds__(kRootWarps * 32) root_expand_w1(const RootArgs
 
 void launch_root_expand_w1(const RootArgs &a, cudaStream_t s) {
     if (a.count <= 0) return;
-    root_expand_w1<<<grid_for(a.count * 8, kRootWarps * 32, 8), kRootWarps * 32, 0, s>>>(a);
+    root_expand_w1<<<grid_for(a.count, kRootWarps * 32, 8), kRootWarps * 32, 0, s>>>(a);
     MCE_LAUNCH_CHECK();
 }
 

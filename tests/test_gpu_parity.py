@@ -39,6 +39,7 @@ GRAPHS = {
     "K64": lambda: G.complete_graph(64),
     "K65": lambda: G.complete_graph(65),
     "K130": lambda: G.complete_graph(130),
+    "K257": lambda: G.complete_graph(257),  # a full 4-word candidate set: 256 colours
     "C5": lambda: G.cycle_graph(5),
     "C9": lambda: G.cycle_graph(9),
     "T(12,4)": lambda: G.turan_graph(12, 4),
@@ -52,6 +53,7 @@ GRAPHS = {
     "ER400d": lambda: G.erdos_renyi(400, 0.35, seed=7),
     "RMAT11": lambda: G.rmat(11, 8, 0.57, 0.19, 0.19, seed=3),
     "RMAT13": lambda: G.rmat(13, 8, 0.45, 0.2, 0.2, seed=2),
+    "RMAT15": lambda: G.rmat(15, 16, 0.57, 0.19, 0.19, seed=5),  # 121 hubs of degree > 1024
     "BA5k": lambda: G.barabasi_albert(5000, 4, seed=2),
     "planted": lambda: G.plant_cliques(G.erdos_renyi(3000, 0.004, seed=9), 3, 9, seed=9),
     "er2000": lambda: G.make_config("er2000"),
@@ -257,3 +259,63 @@ def test_config_dense800_find_one():
     r = gg.find_one(window=32)
     assert r.omega == 15  # tests/golden/dense800.json (oracle, scripts/make_golden.py)
     assert oracle.is_clique(*g.numpy(), r.cliques[0])
+
+
+def cocktail_join(j, t, seed):
+    """Cocktail-party graph CP(j) (K_2j minus a perfect matching) joined with K_t,
+    vertex ids permuted: omega = j + t with 2^j maximum cliques (one vertex of
+    every non-adjacent pair), the structure of the R-MAT hub core."""
+    n = 2 * j + t
+    u, v = np.triu_indices(n, 1)
+    keep = ~((u < 2 * j) & (v < 2 * j) & (u // 2 == v // 2))
+    perm = np.random.default_rng(seed).permutation(n)
+    return G.from_edges(n, torch.from_numpy(perm[u[keep]].astype(np.int64)),
+                        torch.from_numpy(perm[v[keep]].astype(np.int64)))
+
+
+@pytest.mark.parametrize("shortcut", [True, False])
+@pytest.mark.parametrize("j,t", [(13, 5), (12, 300), (6, 60), (3, 1)])
+def test_clique_completions_closed_form(j, t, shortcut):
+    """Completions (P a clique, reading 10) on the thread (W <= 4) and
+    tile (W >= 8) kernels: 2^13 > the 4096-row staging forces growth + replay."""
+    g = cocktail_join(j, t, seed=j * 1000 + t)
+    om, cl = oracle.max_cliques(*g.numpy())
+    assert om == j + t and len(cl) == 2 ** j  # closed form pins the oracle here too
+    for fused in (True, False):
+        r = run_enum(g, clique_shortcut=shortcut, fused_levels=fused)
+        assert (r.omega, r.count) == (om, len(cl)) and np.array_equal(r.cliques, cl)
+    r = run_enum(g, clique_shortcut=shortcut, budget_bytes=4 << 20)
+    assert (r.omega, r.count) == (om, len(cl)) and np.array_equal(r.cliques, cl)
+    m = mce()
+    f = m.Graph(g.rowptr, g.col).find_one(window=4)
+    assert f.omega == om and oracle.is_clique(*g.numpy(), f.cliques[0])
+
+
+@pytest.mark.parametrize("key", ["er2000", "planted", "RMAT11", "RMAT13", "K65", "K130", "K257", "T(36,12)", "ER400d",
+                                 "Paley17", "BA5k"])
+def test_clique_shortcut_off_matches(key):
+    """Algorithm 2's level-by-level expansion (no completions) gives the same answer."""
+    g = GRAPHS[key]()
+    om, cl = oracle_answer(key)
+    r = run_enum(g, clique_shortcut=False)
+    assert (r.omega, r.count) == (om, len(cl)) and np.array_equal(r.cliques, cl)
+    r = run_enum(g, clique_shortcut=False, fused_levels=False, heuristic="none")
+    assert (r.omega, r.count) == (om, len(cl)) and np.array_equal(r.cliques, cl)
+
+
+@pytest.mark.parametrize("key", ["RMAT15", "RMAT13", "BA5k", "planted"])
+def test_heuristic_hub_runs(key):
+    """Runs on hub seeds (degree > 1024: block per run) and the exact early abort:
+    the bound and the winning clique equal the oracle's; with every run size
+    requested nothing is aborted."""
+    g = GRAPHS[key]()
+    rp, col = g.numpy()
+    m = mce()
+    gg = m.Graph(g.rowptr, g.col)
+    w_o, runs_o, best_o = oracle.greedy(rp, col, np.diff(rp), g.n)
+    r = gg.enumerate()  # aborting heuristic inside the pipeline
+    w, clique, runs = gg.heuristic("multi_degree", g.n)
+    assert w == w_o and clique == best_o.tolist()
+    order = np.lexsort((np.arange(g.n), -np.diff(rp).astype(np.int64)))
+    assert np.array_equal(runs[order], runs_o)
+    assert r.omega == oracle_answer(key)[0]
