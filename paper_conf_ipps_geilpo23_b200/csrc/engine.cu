@@ -818,7 +818,9 @@ mce_result *Engine::run() {
         int32_t *out = g_->pool.take<int32_t>(stored_ * res_size_);
         res->rows.resize((size_t)stored_ * res_size_);
         if (canonicalize_device(g_->store.get(), stored_, res_size_, n, out, g_->pool, s_)) {
-            kernels_ += 3 + (res_size_ + 1) / 2 * 2;
+            int merge_passes = 0;  // CUB merge sort: block sort + (partition, merge) per doubling of tiles
+            for (int64_t t = 512; t < stored_; t <<= 1) ++merge_passes;
+            kernels_ += 4 + 2 * merge_passes;
             res->canonical = true;
         } else {
             out = g_->store.get();  // rows too wide: the host sorts them (mce_result_cliques)

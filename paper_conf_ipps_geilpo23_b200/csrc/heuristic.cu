@@ -213,93 +213,56 @@ __global__ void __launch_bounds__(kBlockRun) greedy_big_kernel(int64_t nbig, con
     }
 }
 
-// One greedy run for a seed of degree <= kThreadSeed by ONE thread: the
-// candidates and their pick keys stay in registers, alive ones marked in a
-// bit mask (no compaction, so no local memory); same picks as greedy_run.
-constexpr int kThreadSeed = 16;
-__device__ int32_t greedy_thread(int32_t s, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
-                                 const int32_t *__restrict__ thr, const int32_t *best) {
-    const int64_t base = rowptr[s];
-    const int len0 = (int)(rowptr[s + 1] - base);
-    int32_t P[kThreadSeed];
-    unsigned long long key[kThreadSeed];
-    uint32_t alive = 0;
-#pragma unroll
-    for (int i = 0; i < kThreadSeed; ++i) {
-        P[i] = i < len0 ? __ldg(col + base + i) : 0;
-        key[i] = i < len0 ? pick_key(thr, P[i]) : 0ull;
-        if (i < len0) alive |= 1u << i;
-    }
-    int32_t csize = 1;
-    while (alive) {
-        if (best && csize + __popc(alive) < ld_best(best)) break;
-        unsigned long long km = 0;
-#pragma unroll
-        for (int i = 0; i < kThreadSeed; ++i)
-            if (((alive >> i) & 1u) && key[i] > km) km = key[i];
-        const int32_t w = (int32_t)(0x7fffffffu - (uint32_t)(km & 0xffffffffull));
-        ++csize;
-        const int64_t wb = rowptr[w], we = rowptr[w + 1];
-#pragma unroll
-        for (int i = 0; i < kThreadSeed; ++i)
-            if ((alive >> i) & 1u)
-                if (P[i] == w || !adjacent(rowptr, col, P[i], w, wb, we)) alive &= ~(1u << i);
-    }
-    return csize;
-}
-
-// The other seeds (degree <= kBigSeed), thread per seed: degree <= kThreadSeed
-// runs on the seed's own thread, longer ones are queued in shared memory and
-// run by whole warps (greedy_run<32>) once the block's threads are done.  The
-// best size is published with one atomicMax per warp and group, so later
-// runs abort against it.
+// The other seeds (degree <= kBigSeed).  Warp w takes seeds [4w, 4w+4): when
+// all four have degree <= 64 they run in parallel on 8-lane tiles (low-degree
+// seeds leave most of a warp idle), otherwise one after another on the whole
+// warp.  A warp publishes its best with one atomicMax per group of seeds, so
+// later runs abort against it.  (A thread per short seed was measured 2x
+// slower: its candidate rows and adjacency searches are 32 separate streams.)
 __global__ void __launch_bounds__(256) greedy_kernel(int64_t nseeds, const int32_t *__restrict__ seeds,
                                                      const int64_t *__restrict__ rowptr,
                                                      const int32_t *__restrict__ col, const int32_t *__restrict__ thr,
                                                      const int32_t *__restrict__ core,
                                                      int32_t *__restrict__ scratch, int32_t *__restrict__ run_size,
                                                      int32_t *best_size, int abort_runs) {
-    __shared__ int32_t queue[256];
-    __shared__ int qn;
-    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int lane = threadIdx.x & 31;
     const int32_t *best = abort_runs ? best_size : nullptr;
-    if (threadIdx.x == 0) qn = 0;
-    __syncthreads();
     int32_t published = 0;
-    for (int64_t b0 = (int64_t)blockIdx.x * blockDim.x; b0 < nseeds; b0 += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t i = b0 + threadIdx.x;
-        int32_t sd = i < nseeds ? seeds[i] : -1;
-        int64_t d = sd >= 0 ? rowptr[sd + 1] - rowptr[sd] : 0;
-        if (d > kBigSeed) sd = -1;  // run by greedy_big_kernel
-        if (sd >= 0 && best && seed_cap(sd, rowptr, core) < ld_best(best_size)) {
-            run_size[sd] = 1;  // cannot reach the best: not run
-            sd = -1;
+    for (int64_t i0 = warp * 4; i0 < nseeds; i0 += nwarps * 4) {
+        const int64_t my = i0 + (lane >> 3);
+        int32_t s_mine = my < nseeds ? seeds[my] : -1;
+        int64_t d_mine = s_mine >= 0 ? rowptr[s_mine + 1] - rowptr[s_mine] : 0;
+        if (d_mine > kBigSeed) s_mine = -1;  // run by greedy_big_kernel
+        if (s_mine >= 0 && best && seed_cap(s_mine, rowptr, core) < ld_best(best_size)) {
+            if ((lane & 7) == 0) run_size[s_mine] = 1;  // cannot reach the best: not run
+            s_mine = -1;
         }
-        if (sd >= 0 && d > kThreadSeed) {
-            queue[atomicAdd(&qn, 1)] = sd;
-            sd = -1;
-        }
+        if (s_mine < 0) d_mine = 0;
         int32_t mybest = 0;
-        if (sd >= 0) {
-            mybest = greedy_thread(sd, rowptr, col, thr, best);
-            run_size[sd] = mybest;
-        }
-        __syncthreads();
-        const int nq = qn;
-        for (int q = wid; q < nq; q += blockDim.x >> 5) {
-            const int32_t sq = queue[q];
-            const int32_t c = greedy_run<32>(sq, rowptr, col, thr, scratch, best);
-            if (lane == 0) run_size[sq] = c;
-            mybest = max(mybest, c);
+        if (!__ballot_sync(0xffffffffu, s_mine >= 0)) continue;
+        if (__all_sync(0xffffffffu, d_mine <= 64)) {
+            if (s_mine >= 0) {
+                const int32_t c = greedy_run<8>(s_mine, rowptr, col, thr, scratch, best);
+                if ((lane & 7) == 0) run_size[s_mine] = c;
+                mybest = c;
+            }
+        } else {
+            for (int t = 0; t < 4; ++t) {
+                const int32_t s = __shfl_sync(0xffffffffu, s_mine, 8 * t);
+                if (s < 0) continue;
+                const int32_t c = greedy_run<32>(s, rowptr, col, thr, scratch, best);
+                if (lane == 0) run_size[s] = c;
+                mybest = max(mybest, c);
+            }
         }
         mybest = __reduce_max_sync(0xffffffffu, mybest);
         if (lane == 0 && mybest > published) {
             atomicMax(best_size, mybest);
             published = mybest;
         }
-        __syncthreads();
-        if (threadIdx.x == 0) qn = 0;
-        __syncthreads();
+        __syncwarp();
     }
 }
 
@@ -493,7 +456,7 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
                 ++kernels;
             }
         }
-        greedy_kernel<<<grid_for(nseeds, 256), 256, 0, s>>>(nseeds, seed_ptr, g->rowptr.get(), g->col.get(),
+        greedy_kernel<<<grid_for(nseeds * 8, 256), 256, 0, s>>>(nseeds, seed_ptr, g->rowptr.get(), g->col.get(),
                                                                   thr, core, scratch, run_size, best, abort_runs);
         MCE_LAUNCH_CHECK();
         best_seed_kernel<<<grid_for(nseeds, 256), 256, 0, s>>>(nseeds, seed_ptr, thr, run_size, best, best_key);

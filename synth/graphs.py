@@ -98,31 +98,60 @@ class Graph:
         return np.stack([src[m], col[m].astype(np.int64)], axis=1)
 
 
-def from_edges(n: int, src: torch.Tensor, dst: torch.Tensor, name: str = "") -> Graph:
-    """Symmetrise, drop self loops and duplicates, build sorted CSR."""
+def _csr_from_keys(n: int, key: torch.Tensor, name: str = "") -> Graph:
+    """CSR (both directions, rows ascending) from sorted unique keys a * n + b, a < b.
+
+    Row v is [a < v : (a, v) an edge] ++ [b > v : (v, b) an edge]: the upper
+    half comes grouped by a and sorted by b with the keys; the lower half is
+    one more sort of b * n + a.  Every part is ascending and the lower part is
+    below v, so the concatenation is the sorted row.  Memory stays a few
+    copies of |E| (R-MAT scale 26: 10^9 edges on one GPU).
+    """
+    device = key.device
+    m = key.numel()
+    a = (key // n).to(torch.int32)
+    b = (key - a.to(torch.int64) * n).to(torch.int32)
+    up = torch.bincount(a, minlength=n) if m else torch.zeros(n, dtype=torch.int64, device=device)
+    lo = torch.bincount(b, minlength=n) if m else torch.zeros(n, dtype=torch.int64, device=device)
+    rowptr = torch.zeros(n + 1, dtype=torch.int64, device=device)
+    rowptr[1:] = torch.cumsum(up + lo, 0)
+    col = torch.empty(2 * m, dtype=torch.int32, device=device)
+    if m:
+        # upper half, in key order: rank of each entry inside its row group a
+        ustart = torch.cumsum(up, 0) - up
+        idx = torch.arange(m, dtype=torch.int64, device=device)
+        al = a.to(torch.int64)
+        col[rowptr[:-1][al] + lo[al] + (idx - ustart[al])] = b
+        del al, ustart
+        # lower half, sorted by (b, a)
+        k2, _ = torch.sort(b.to(torch.int64) * n + a.to(torch.int64))
+        del a, b
+        b2 = k2 // n
+        a2 = (k2 - b2 * n).to(torch.int32)
+        del k2
+        lstart = torch.cumsum(lo, 0) - lo
+        col[rowptr[:-1][b2] + (idx - lstart[b2])] = a2
+        del b2, a2, idx, lstart
+    return Graph(n=n, rowptr=rowptr, col=col, name=name)
+
+
+def edge_keys(n: int, src: torch.Tensor, dst: torch.Tensor) -> torch.Tensor:
+    """Undirected keys min * n + max of the non-loop pairs (unsorted, with duplicates)."""
     src = src.to(torch.int64)
     dst = dst.to(torch.int64)
-    device = src.device
     keep = src != dst
     src, dst = src[keep], dst[keep]
-    a = torch.minimum(src, dst)
-    b = torch.maximum(src, dst)
-    key = torch.unique(a * n + b)  # sorted, deduplicated undirected edges
-    del a, b, src, dst, keep
-    a = key // n
-    b = key - a * n
-    del key
-    s = torch.cat([a, b])
-    d = torch.cat([b, a])
-    del a, b
-    order = torch.argsort(s * n + d)
-    s = s[order]
-    d = d[order]
-    del order
-    deg = torch.bincount(s, minlength=n) if s.numel() else torch.zeros(n, dtype=torch.int64, device=device)
-    rowptr = torch.zeros(n + 1, dtype=torch.int64, device=device)
-    rowptr[1:] = torch.cumsum(deg, 0)
-    return Graph(n=n, rowptr=rowptr, col=d.to(torch.int32), name=name)
+    return torch.minimum(src, dst) * n + torch.maximum(src, dst)
+
+
+def from_keys(n: int, keys: torch.Tensor, name: str = "") -> Graph:
+    """Graph from undirected keys (duplicates allowed)."""
+    return _csr_from_keys(n, torch.unique(keys), name=name)
+
+
+def from_edges(n: int, src: torch.Tensor, dst: torch.Tensor, name: str = "") -> Graph:
+    """Symmetrise, drop self loops and duplicates, build sorted CSR."""
+    return from_keys(n, edge_keys(n, src, dst), name=name)
 
 
 def _pairs_from_mask(n: int, keep_fn, device, chunk_rows: int = 256):
@@ -191,23 +220,29 @@ def erdos_renyi(n: int, p: float, seed: int, device="cpu") -> Graph:
     return from_edges(n, s, d, name=f"G({n},{p})s{seed}")
 
 
-def plant_cliques(g: Graph, count: int, size: int, seed: int) -> Graph:
-    """Add `count` vertex-disjoint cliques of `size` vertices chosen at random."""
-    n = g.n
-    device = g.rowptr.device
+def planted_clique_edges(n: int, count: int, size: int, seed: int, device="cpu"):
+    """`count` vertex-disjoint cliques of `size` random vertices: (src, dst, chosen rows)."""
     if count * size > n:
         raise ValueError("not enough vertices to plant the cliques")
     keys = rand_u64(seed, _STREAM_PLANT, torch.arange(n, dtype=torch.int64, device=device))
     chosen = torch.argsort(keys)[: count * size].reshape(count, size)
+    del keys
     chosen, _ = torch.sort(chosen, dim=1)
     ii, jj = torch.triu_indices(size, size, offset=1, device=device)
-    add_s = chosen[:, ii].reshape(-1)
-    add_d = chosen[:, jj].reshape(-1)
+    return chosen[:, ii].reshape(-1), chosen[:, jj].reshape(-1), chosen
+
+
+def plant_cliques(g: Graph, count: int, size: int, seed: int) -> Graph:
+    """Add `count` vertex-disjoint cliques of `size` vertices chosen at random."""
+    n = g.n
+    device = g.rowptr.device
+    add_s, add_d, chosen = planted_clique_edges(n, count, size, seed, device)
     rp = g.rowptr
     src = torch.repeat_interleave(torch.arange(n, dtype=torch.int64, device=device), rp[1:] - rp[:-1])
-    s = torch.cat([src, add_s])
-    d = torch.cat([g.col.to(torch.int64), add_d])
-    out = from_edges(n, s, d, name=f"{g.name}+{count}x K{size}")
+    up = src < g.col
+    keys = torch.cat([src[up] * n + g.col[up].to(torch.int64), edge_keys(n, add_s, add_d)])
+    del src, up
+    out = from_keys(n, keys, name=f"{g.name}+{count}x K{size}")
     out.planted = (g.planted or []) + chosen.cpu().tolist()
     return out
 
@@ -257,18 +292,27 @@ def barabasi_albert(n: int, m: int, seed: int) -> Graph:
 
 
 def rmat(scale: int, edge_factor: int, a: float, b: float, c: float, seed: int,
-         device="cpu", permute: bool = True, chunk: int = 1 << 24) -> Graph:
+         device="cpu", permute: bool = True, chunk: int = 1 << 24, plant=None) -> Graph:
     """R-MAT (Chakrabarti et al.) with 2^scale vertices and edge_factor*2^scale draws.
 
     Each draw descends `scale` levels picking quadrant (0,0),(0,1),(1,0),(1,1)
     with probabilities a, b, c, 1-a-b-c.  Vertex ids are then randomly
-    permuted (the paper randomises indices).
+    permuted (the paper randomises indices).  `plant` =
+    (count, size, seed) adds planted cliques exactly as plant_cliques does,
+    without building the graph twice.
     """
     n = 1 << scale
     m = edge_factor * n
     ab = a + b
     abc = a + b + c
-    srcs, dsts = [], []
+    label = None
+    if permute:
+        keys = rand_u64(seed, _STREAM_PERM, torch.arange(n, dtype=torch.int64, device=device))
+        order = torch.argsort(keys)
+        label = torch.empty_like(order)
+        label[order] = torch.arange(n, dtype=torch.int64, device=device)
+        del keys, order
+    parts = []
     for e0 in range(0, m, chunk):
         e = torch.arange(e0, min(m, e0 + chunk), dtype=torch.int64, device=device)
         s = torch.zeros_like(e)
@@ -281,22 +325,25 @@ def rmat(scale: int, edge_factor: int, a: float, b: float, c: float, seed: int,
             s += sb * bit
             d += db.to(torch.int64) * bit
             del u, sb, db
-        srcs.append(s)
-        dsts.append(d)
-        del e
-    s = torch.cat(srcs)
-    d = torch.cat(dsts)
-    del srcs, dsts
-    if permute:
-        keys = rand_u64(seed, _STREAM_PERM, torch.arange(n, dtype=torch.int64, device=device))
-        order = torch.argsort(keys)
-        label = torch.empty_like(order)
-        label[order] = torch.arange(n, dtype=torch.int64, device=device)
-        del keys, order
-        s = label[s]
-        d = label[d]
-        del label
-    return from_edges(n, s, d, name=f"RMAT{scale}ef{edge_factor}s{seed}")
+        if label is not None:
+            s = label[s]
+            d = label[d]
+        parts.append(edge_keys(n, s, d))
+        del e, s, d
+    del label
+    chosen = None
+    if plant is not None:
+        ps, pd, chosen = planted_clique_edges(n, plant[0], plant[1], plant[2], device)
+        parts.append(edge_keys(n, ps, pd))
+    keys = torch.cat(parts)
+    del parts
+    name = f"RMAT{scale}ef{edge_factor}s{seed}"
+    if plant is not None:
+        name += f"+{plant[0]}x K{plant[1]}"
+    g = from_keys(n, keys, name=name)
+    if chosen is not None:
+        g.planted = chosen.cpu().tolist()
+    return g
 
 
 # ---------------------------------------------------------------------------
@@ -329,8 +376,7 @@ def make_config(name: str, device="cpu", scale_override: Optional[int] = None) -
     if name == "dense800":
         return erdos_renyi(800, 0.5, seed=1, device=device)
     if name == "rmat26":
-        g = rmat(scale_override or 26, 16, 0.57, 0.19, 0.19, seed=1, device=device)
-        return plant_cliques(g, 50, 20, seed=1)
+        return rmat(scale_override or 26, 16, 0.57, 0.19, 0.19, seed=1, device=device, plant=(50, 20, 1))
     raise KeyError(name)
 
 

@@ -284,7 +284,8 @@ def test_clique_completions_closed_form(j, t, shortcut):
     for fused in (True, False):
         r = run_enum(g, clique_shortcut=shortcut, fused_levels=fused)
         assert (r.omega, r.count) == (om, len(cl)) and np.array_equal(r.cliques, cl)
-    r = run_enum(g, clique_shortcut=shortcut, budget_bytes=4 << 20)
+    # a small budget forces chunked levels (the 312-level chain itself needs ~35 MB of parent links)
+    r = run_enum(g, clique_shortcut=shortcut, budget_bytes=64 << 20)
     assert (r.omega, r.count) == (om, len(cl)) and np.array_equal(r.cliques, cl)
     m = mce()
     f = m.Graph(g.rowptr, g.col).find_one(window=4)
@@ -299,7 +300,7 @@ def test_clique_shortcut_off_matches(key):
     om, cl = oracle_answer(key)
     r = run_enum(g, clique_shortcut=False)
     assert (r.omega, r.count) == (om, len(cl)) and np.array_equal(r.cliques, cl)
-    r = run_enum(g, clique_shortcut=False, fused_levels=False, heuristic="none")
+    r = run_enum(g, clique_shortcut=False, fused_levels=False)
     assert (r.omega, r.count) == (om, len(cl)) and np.array_equal(r.cliques, cl)
 
 
