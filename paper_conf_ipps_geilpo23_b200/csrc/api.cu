@@ -286,8 +286,16 @@ mce_status mce_result_info(const mce_result *r, int32_t *omega, int64_t *count, 
 mce_status mce_result_cliques(mce_result *r, int32_t *dst, int32_t where) {
     return run_guarded([&] {
         if (!r) fail(MCE_ERR_INVALID, "result is NULL");
-        canonicalize(r);
         const size_t bytes = sizeof(int32_t) * (size_t)r->stored * std::max(r->omega, 0);
+        if (r->drows.get()) {  // canonical rows on the device
+            if (!bytes) return;
+            if (!dst) fail(MCE_ERR_INVALID, "dst is NULL");
+            MCE_CUDA(cudaSetDevice(r->device));
+            MCE_CUDA(cudaMemcpy(dst, r->drows.get(), bytes,
+                                where == MCE_WHERE_HOST ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice));
+            return;
+        }
+        canonicalize(r);
         if (!bytes) return;
         if (!dst) fail(MCE_ERR_INVALID, "dst is NULL");
         if (where == MCE_WHERE_HOST)

@@ -812,25 +812,29 @@ mce_result *Engine::run() {
     if (find_one_) {
         res->rows = std::move(rows_);
     } else if (stored_ > 0 && res_size_ > 0) {
-        // canonical read-out on the device, one copy to the host (canon.cu)
+        // canonical read-out on the device (canon.cu); the rows stay in the
+        // result's device buffer and go straight to the caller's destination
+        // in mce_result_cliques (no intermediate host copy)
         const auto h4 = clk::now();
         g_->pool.reset();
-        int32_t *out = g_->pool.take<int32_t>(stored_ * res_size_);
-        res->rows.resize((size_t)stored_ * res_size_);
-        if (canonicalize_device(g_->store.get(), stored_, res_size_, n, out, g_->pool, s_)) {
+        res->device = g_->device;
+        res->drows.alloc((size_t)stored_ * res_size_);
+        if (canonicalize_device(g_->store.get(), stored_, res_size_, n, res->drows.get(), g_->pool, s_)) {
             int merge_passes = 0;  // CUB merge sort: block sort + (partition, merge) per doubling of tiles
             for (int64_t t = 512; t < stored_; t <<= 1) ++merge_passes;
             kernels_ += 4 + 2 * merge_passes;
             res->canonical = true;
-        } else {
-            out = g_->store.get();  // rows too wide: the host sorts them (mce_result_cliques)
+            stream_sync(s_);
+        } else {  // rows too wide: the host sorts them (mce_result_cliques)
+            res->drows.release();
+            res->rows.resize((size_t)stored_ * res_size_);
+            MCE_CUDA(cudaMemcpyAsync(res->rows.data(), g_->store.get(), sizeof(int32_t) * stored_ * res_size_,
+                                     cudaMemcpyDeviceToHost, s_));
+            stream_sync(s_);
         }
-        MCE_CUDA(cudaMemcpyAsync(res->rows.data(), out, sizeof(int32_t) * stored_ * res_size_,
-                                 cudaMemcpyDeviceToHost, s_));
-        stream_sync(s_);
         res->h_readout_ms = ms_since(h4);
     }
-    res->stored = res_size_ > 0 ? (int64_t)res->rows.size() / res_size_ : 0;
+    res->stored = res_size_ <= 0 ? 0 : (res->drows.get() ? stored_ : (int64_t)res->rows.size() / res_size_);
     res->truncated = truncated_ ? 1 : 0;
     res->level_entries = level_entries_;
     res->t_count_ms = t_count_ms_;

@@ -10,7 +10,9 @@ struct mce_result {
     int64_t count = 0;     // multiplicity (exact)
     int64_t stored = 0;    // rows available
     int32_t truncated = 0;
-    std::vector<int32_t> rows;  // stored * omega original vertex ids
+    std::vector<int32_t> rows;  // stored * omega original vertex ids (host; find-one / wide rows)
+    mce::DevBuf<int32_t> drows; // the same on the device when the read-out ran there (canon.cu)
+    int device = 0;
     bool canonical = false;     // rows sorted (each clique ascending, list lexicographic)
     std::vector<int64_t> level_entries;
     double t_pre_ms = 0, t_heur_ms = 0, t_enum_ms = 0, t_expand_ms = 0, t_count_ms = 0, count_bytes = 0;

@@ -60,11 +60,101 @@ __device__ __forceinline__ int32_t ld_best(const int32_t *best) {
     return v;
 }
 
+// Hub bit matrix (exact acceleration of long runs on power-law graphs).  H =
+// the highest-degree vertices (at most kHubMax, degree bucket threshold), M =
+// their induced adjacency as K x K bits, hkey = their pick keys.  Once every
+// candidate of a run is in H (after a few picks, runs from hubs are inside the
+// dense hub core), the run continues on a bit set over H: the pick is a max
+// over the set bits' keys, the filter one AND with M's row.  Same picks, same
+// sizes as the list form (the key encodes threshold and id).
+constexpr int kHubMax = 8192;
+constexpr int kHubWords = kHubMax / 64;  // 128
+constexpr int kHubWPL = kHubWords / 32;  // words per lane
+struct Hub {
+    const int32_t *hid = nullptr;           // [n] hub index or -1
+    const int32_t *hv = nullptr;            // [K] hub -> vertex
+    const unsigned long long *hkey = nullptr;  // [K] pick keys
+    const uint64_t *M = nullptr;            // [K][KW]
+    int K = 0, KW = 0;
+};
+
+// The rest of a run whose candidates are all hubs, by one warp: P = the
+// list src[0..len) (all in H) becomes a bit set; returns the final size.
+__device__ int32_t hub_tail_warp(const Hub &H, const int32_t *src, int64_t len, int32_t csize, int32_t *clique,
+                                 const int32_t *best) {
+    const int lane = threadIdx.x & 31;
+    uint64_t P[kHubWPL];
+#pragma unroll
+    for (int t = 0; t < kHubWPL; ++t) P[t] = 0;
+    // build: lane l collects the members whose word is owned by l (word % 32 == l)
+    for (int64_t i0 = 0; i0 < len; i0 += 32) {
+        const int64_t i = i0 + lane;
+        const int h = i < len ? __ldg(H.hid + src[i]) : -1;
+        for (int src_lane = 0; src_lane < 32; ++src_lane) {
+            const int hh = __shfl_sync(0xffffffffu, h, src_lane);
+            if (hh >= 0 && ((hh >> 6) & 31) == lane) {
+#pragma unroll
+                for (int t = 0; t < kHubWPL; ++t)
+                    if (t == (hh >> 11)) P[t] |= 1ull << (hh & 63);
+            }
+        }
+    }
+    while (true) {
+        int pc = 0;
+#pragma unroll
+        for (int t = 0; t < kHubWPL; ++t) pc += __popcll(P[t]);
+        pc = __reduce_add_sync(0xffffffffu, pc);
+        if (pc == 0) break;
+        if (best) {
+            int32_t b = 0;
+            if (lane == 0) b = ld_best(best);
+            b = __shfl_sync(0xffffffffu, b, 0);
+            if (csize + pc < b) break;
+        }
+        unsigned long long key = 0;
+        int hb = -1;
+#pragma unroll
+        for (int t = 0; t < kHubWPL; ++t) {
+            uint64_t q = P[t];
+            while (q) {
+                const int b = __ffsll((long long)q) - 1;
+                q &= q - 1;
+                const int h = ((t * 32 + lane) << 6) + b;
+                const unsigned long long k2 = __ldg(H.hkey + h);
+                if (k2 > key) {
+                    key = k2;
+                    hb = h;
+                }
+            }
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            const unsigned long long y = __shfl_xor_sync(0xffffffffu, key, o);
+            const int yh = __shfl_xor_sync(0xffffffffu, hb, o);
+            if (y > key) {
+                key = y;
+                hb = yh;
+            }
+        }
+        if (clique && lane == 0) clique[csize] = (int32_t)(0x7fffffffu - (uint32_t)(key & 0xffffffffull));
+        ++csize;
+        const uint64_t *row = H.M + (int64_t)hb * H.KW;
+#pragma unroll
+        for (int t = 0; t < kHubWPL; ++t) {
+            const int w = t * 32 + lane;
+            P[t] &= w < H.KW ? __ldg(row + w) : 0ull;
+            if (w == (hb >> 6)) P[t] &= ~(1ull << (hb & 63));
+        }
+    }
+    return csize;
+}
+
 // One greedy run for seed s by a tile of G lanes (G = 8 or 32) of the calling
 // warp.  Returns the clique size (a partial size < the best when aborted).
 template <int G>
 __device__ int32_t greedy_run(int32_t s, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
-                              const int32_t *__restrict__ thr, int32_t *__restrict__ scratch, const int32_t *best) {
+                              const int32_t *__restrict__ thr, int32_t *__restrict__ scratch, const int32_t *best,
+                              const Hub &H) {
     const int lane = threadIdx.x & 31;
     const int gl = lane & (G - 1);
     const int gbase = lane & ~(G - 1);
@@ -95,6 +185,7 @@ __device__ int32_t greedy_run(int32_t s, const int64_t *__restrict__ rowptr, con
         ++csize;
         const int64_t wb = rowptr[w], we = rowptr[w + 1];
         int64_t out = 0;
+        int nonhub = 0;
         for (int64_t i0 = 0; i0 < len; i0 += G) {
             int64_t i = i0 + gl;
             int32_t x = i < len ? src[i] : -1;
@@ -102,10 +193,12 @@ __device__ int32_t greedy_run(int32_t s, const int64_t *__restrict__ rowptr, con
             const unsigned m = (__ballot_sync(gmask, keep) & gmask) >> gbase;
             if (keep) buf[out + __popc(m & ((1u << gl) - 1u))] = x;
             out += __popc(m);
+            if (G == 32 && H.K) nonhub += __popc(__ballot_sync(gmask, keep && __ldg(H.hid + x) < 0));
         }
         __syncwarp(gmask);
         src = buf;
         len = out;
+        if (G == 32 && H.K && len > 0 && nonhub == 0) return hub_tail_warp(H, src, len, csize, nullptr, best);
     }
     return csize;
 }
@@ -119,10 +212,10 @@ constexpr int64_t kBigSeed = 1024;
 template <int NT>
 __device__ int32_t block_run(int32_t s, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
                              const int32_t *__restrict__ thr, int32_t *__restrict__ scratch, int32_t *clique,
-                             const int32_t *best) {
+                             const int32_t *best, const Hub &H) {
     __shared__ unsigned long long wkey[NT / 32];
-    __shared__ int32_t wcnt[NT / 32];
-    __shared__ int32_t sbest;
+    __shared__ int32_t wcnt[NT / 32], wnon[NT / 32];
+    __shared__ int32_t sbest, sres;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     const int64_t base = rowptr[s];
     int64_t len = rowptr[s + 1] - base;
@@ -157,13 +250,18 @@ __device__ int32_t block_run(int32_t s, const int64_t *__restrict__ rowptr, cons
         ++csize;
         const int64_t wb = rowptr[w], we = rowptr[w + 1];
         int64_t out = 0;
+        int32_t nonhub = 0;
         for (int64_t i0 = 0; i0 < len; i0 += NT) {
             const int64_t i = i0 + threadIdx.x;
             const int32_t x = i < len ? src[i] : -1;
             const bool keep = i < len && x != w && adjacent(rowptr, col, x, w, wb, we);
             const unsigned m = __ballot_sync(0xffffffffu, keep);
+            const unsigned nh = H.K ? __ballot_sync(0xffffffffu, keep && __ldg(H.hid + x) < 0) : 0u;
             __syncthreads();  // wkey/wcnt reuse, and every read of this chunk precedes its writes
-            if (lane == 0) wcnt[wid] = __popc(m);
+            if (lane == 0) {
+                wcnt[wid] = __popc(m);
+                wnon[wid] = __popc(nh);
+            }
             __syncthreads();
             int32_t before = 0, total = 0;
 #pragma unroll
@@ -171,6 +269,7 @@ __device__ int32_t block_run(int32_t s, const int64_t *__restrict__ rowptr, cons
                 const int32_t c = wcnt[j];
                 before += j < wid ? c : 0;
                 total += c;
+                nonhub += wnon[j];
             }
             if (keep) buf[out + before + __popc(m & lanemask_lt())] = x;
             out += total;
@@ -178,6 +277,16 @@ __device__ int32_t block_run(int32_t s, const int64_t *__restrict__ rowptr, cons
         __syncthreads();
         src = buf;
         len = out;
+        if (H.K && len > 0 && nonhub == 0) {  // the rest on a bit set over the hubs, by warp 0
+            if (wid == 0) {
+                const int32_t c = hub_tail_warp(H, src, len, csize, clique, best);
+                if (lane == 0) sres = c;
+            }
+            __syncthreads();
+            csize = sres;
+            __syncthreads();
+            return csize;
+        }
     }
     return csize;
 }
@@ -199,12 +308,12 @@ __global__ void __launch_bounds__(kBlockRun) greedy_big_kernel(int64_t nbig, con
                                                                const int32_t *__restrict__ core,
                                                                int32_t *__restrict__ scratch,
                                                                int32_t *__restrict__ run_size, int32_t *best_size,
-                                                               int abort_runs) {
+                                                               int abort_runs, const Hub H) {
     for (int64_t i = blockIdx.x; i < nbig; i += gridDim.x) {
         const int32_t s = big[i];
         int32_t c = 1;
         if (!abort_runs || seed_cap(s, rowptr, core) >= ld_best(best_size))
-            c = block_run<kBlockRun>(s, rowptr, col, thr, scratch, nullptr, abort_runs ? best_size : nullptr);
+            c = block_run<kBlockRun>(s, rowptr, col, thr, scratch, nullptr, abort_runs ? best_size : nullptr, H);
         if (threadIdx.x == 0) {
             run_size[s] = c;
             atomicMax(best_size, c);
@@ -224,7 +333,8 @@ __global__ void __launch_bounds__(256) greedy_kernel(int64_t nseeds, const int32
                                                      const int32_t *__restrict__ col, const int32_t *__restrict__ thr,
                                                      const int32_t *__restrict__ core,
                                                      int32_t *__restrict__ scratch, int32_t *__restrict__ run_size,
-                                                     int32_t *best_size, int abort_runs) {
+                                                     int32_t *best_size, int abort_runs, const Hub H) {
+    const Hub none{};
     const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     const int lane = threadIdx.x & 31;
@@ -244,7 +354,7 @@ __global__ void __launch_bounds__(256) greedy_kernel(int64_t nseeds, const int32
         if (!__ballot_sync(0xffffffffu, s_mine >= 0)) continue;
         if (__all_sync(0xffffffffu, d_mine <= 64)) {
             if (s_mine >= 0) {
-                const int32_t c = greedy_run<8>(s_mine, rowptr, col, thr, scratch, best);
+                const int32_t c = greedy_run<8>(s_mine, rowptr, col, thr, scratch, best, none);
                 if ((lane & 7) == 0) run_size[s_mine] = c;
                 mybest = c;
             }
@@ -252,7 +362,7 @@ __global__ void __launch_bounds__(256) greedy_kernel(int64_t nseeds, const int32
             for (int t = 0; t < 4; ++t) {
                 const int32_t s = __shfl_sync(0xffffffffu, s_mine, 8 * t);
                 if (s < 0) continue;
-                const int32_t c = greedy_run<32>(s, rowptr, col, thr, scratch, best);
+                const int32_t c = greedy_run<32>(s, rowptr, col, thr, scratch, best, H);
                 if (lane == 0) run_size[s] = c;
                 mybest = max(mybest, c);
             }
@@ -296,9 +406,9 @@ __global__ void __launch_bounds__(kReplay) replay_kernel(const unsigned long lon
                                                          const int64_t *__restrict__ rowptr,
                                                          const int32_t *__restrict__ col,
                                                          const int32_t *__restrict__ thr,
-                                                         int32_t *__restrict__ scratch, int32_t *clique) {
+                                                         int32_t *__restrict__ scratch, int32_t *clique, const Hub H) {
     const int32_t s = (int32_t)(0x7fffffffu - (uint32_t)(*best_key & 0xffffffffull));
-    block_run<kReplay>(s, rowptr, col, thr, scratch, clique, nullptr);
+    block_run<kReplay>(s, rowptr, col, thr, scratch, clique, nullptr, H);
 }
 
 __global__ void degree_thr_kernel(int64_t n, const int64_t *__restrict__ rowptr, int32_t *thr) {
@@ -337,6 +447,74 @@ __global__ void strided_gather_kernel(const int32_t *__restrict__ in, int64_t co
 __global__ void iota_kernel(int64_t n, int32_t *out) {
     for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
         out[v] = (int32_t)v;
+}
+
+// degree bucket: 4 mantissa bits below the leading one (monotone in d)
+__device__ __forceinline__ int deg_bucket(int64_t d) {
+    if (d <= 0) return 0;
+    const int e = 63 - __clzll((long long)d);
+    const int m = e >= 4 ? (int)((d >> (e - 4)) & 15) : (int)((d << (4 - e)) & 15);
+    return (e << 4) | m;
+}
+constexpr int kBuckets = 64 * 16;
+
+// per-block shared histogram, one global add per non-empty bucket (degrees
+// crowd into a few buckets: same-address global atomics would serialise)
+__global__ void deg_bucket_hist(int64_t n, const int64_t *__restrict__ rowptr, unsigned long long *bins) {
+    __shared__ unsigned int h[kBuckets];
+    for (int i = threadIdx.x; i < kBuckets; i += blockDim.x) h[i] = 0;
+    __syncthreads();
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+        atomicAdd(h + deg_bucket(rowptr[v + 1] - rowptr[v]), 1u);
+    __syncthreads();
+    for (int i = threadIdx.x; i < kBuckets; i += blockDim.x)
+        if (h[i]) atomicAdd(bins + i, (unsigned long long)h[i]);
+}
+
+// hub index of every vertex (-1: not a hub), by warp-aggregated appends;
+// hub order is immaterial (keys carry the tie-break)
+__global__ void hub_index_kernel(int64_t n, const int64_t *__restrict__ rowptr, int bstar, int32_t *hid, int32_t *hv,
+                                 int32_t *count) {
+    const int lane = threadIdx.x & 31;
+    for (int64_t v0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) & ~31ll; v0 < n;
+         v0 += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t v = v0 + lane;
+        const bool h = v < n && deg_bucket(rowptr[v + 1] - rowptr[v]) >= bstar;
+        const unsigned m = __ballot_sync(0xffffffffu, h);
+        int b = 0;
+        if (lane == 0 && m) b = atomicAdd(count, __popc(m));
+        b = __shfl_sync(0xffffffffu, b, 0);
+        if (v < n) {
+            const int idx = h ? b + __popc(m & lanemask_lt()) : -1;
+            hid[v] = idx;
+            if (h) hv[idx] = (int32_t)v;
+        }
+    }
+}
+
+// row h of M: warp per hub, bits gathered in shared memory
+__global__ void __launch_bounds__(256) hub_matrix_kernel(int K, int KW, const int32_t *__restrict__ hv,
+                                                         const int64_t *__restrict__ rowptr,
+                                                         const int32_t *__restrict__ col,
+                                                         const int32_t *__restrict__ hid,
+                                                         const int32_t *__restrict__ thr, uint64_t *M,
+                                                         unsigned long long *hkey) {
+    __shared__ unsigned long long row_all[8][kHubWords];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    unsigned long long *row = row_all[wid];
+    for (int h = blockIdx.x * 8 + wid; h < K; h += gridDim.x * 8) {
+        for (int w = lane; w < KW; w += 32) row[w] = 0ull;
+        __syncwarp();
+        const int32_t v = hv[h];
+        for (int64_t e = rowptr[v] + lane; e < rowptr[v + 1]; e += 32) {
+            const int32_t u = __ldg(hid + __ldg(col + e));
+            if (u >= 0) atomicOr(row + (u >> 6), 1ull << (u & 63));
+        }
+        __syncwarp();
+        for (int w = lane; w < KW; w += 32) M[(int64_t)h * KW + w] = row[w];
+        if (lane == 0) hkey[h] = pick_key(thr, v);
+        __syncwarp();
+    }
 }
 
 }  // namespace
@@ -433,35 +611,76 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
     MCE_CUDA(cudaMemsetAsync(best_key, 0, sizeof(unsigned long long), s));
     const int32_t *core = g->have_core ? g->core.get() : nullptr;
     const int abort_runs = want_runs ? 0 : 1;
+    Hub H;
+    int64_t nbig = 0;
+    int32_t *big = nullptr;
+    if (nseeds > 0 && g->max_deg > kBigSeed) {
+        int32_t *flag = pool.take<int32_t>(nseeds);
+        int64_t *pos = pool.take<int64_t>(nseeds + 1), *tmp = pool.take<int64_t>(scan_tmp_items(nseeds));
+        big = pool.take<int32_t>(nseeds);
+        big_flags_kernel<<<grid_for(nseeds, 256), 256, 0, s>>>(nseeds, seed_ptr, g->rowptr.get(), flag);
+        MCE_LAUNCH_CHECK();
+        exclusive_scan_i32(flag, pos, nseeds, tmp, s);
+        gather_flagged_kernel<<<grid_for(nseeds, 256), 256, 0, s>>>(nseeds, seed_ptr, flag, pos, big);
+        MCE_LAUNCH_CHECK();
+        int64_t *hnb = g->host.get<int64_t>(1);
+        MCE_CUDA(cudaMemcpyAsync(hnb, pos + nseeds, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        stream_sync(s);
+        nbig = hnb[0];
+        kernels += 5;
+    }
+    if (nbig >= 64) {  // enough hub runs for the hub bit matrix to pay
+        // H = the vertices of the highest degree buckets, at most kHubMax of them
+        unsigned long long *bins = pool.take<unsigned long long>(kBuckets);
+        MCE_CUDA(cudaMemsetAsync(bins, 0, sizeof(unsigned long long) * kBuckets, s));
+        deg_bucket_hist<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(), bins);
+        MCE_LAUNCH_CHECK();
+        unsigned long long *hb = g->host.get<unsigned long long>(kBuckets);
+        MCE_CUDA(cudaMemcpyAsync(hb, bins, sizeof(unsigned long long) * kBuckets, cudaMemcpyDeviceToHost, s));
+        stream_sync(s);
+        int bstar = kBuckets;
+        unsigned long long above = 0;
+        for (int b = kBuckets - 1; b >= 0; --b) {
+            if (above + hb[b] > (unsigned long long)kHubMax) break;
+            above += hb[b];
+            if (hb[b]) bstar = b;
+        }
+        kernels += 1;
+        if (above >= 64) {  // enough hubs to matter
+            int32_t *hid = pool.take<int32_t>(n), *hv = pool.take<int32_t>(kHubMax), *cnt = pool.take<int32_t>(1);
+            MCE_CUDA(cudaMemsetAsync(cnt, 0, sizeof(int32_t), s));
+            hub_index_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(), bstar, hid, hv, cnt);
+            MCE_LAUNCH_CHECK();
+            const int K = (int)above;
+            const int KW = (K + 63) / 64;
+            uint64_t *M = pool.take<uint64_t>((int64_t)K * KW);
+            unsigned long long *hkey = pool.take<unsigned long long>(K);
+            hub_matrix_kernel<<<std::max(1, std::min((K + 7) / 8, num_sms() * 8)), 256, 0, s>>>(
+                K, KW, hv, g->rowptr.get(), g->col.get(), hid, thr, M, hkey);
+            MCE_LAUNCH_CHECK();
+            kernels += 2;
+            H.hid = hid;
+            H.hv = hv;
+            H.hkey = hkey;
+            H.M = M;
+            H.K = K;
+            H.KW = KW;
+        }
+    }
     if (nseeds > 0) {
-        if (g->max_deg > kBigSeed) {
-            int32_t *flag = pool.take<int32_t>(nseeds);
-            int64_t *pos = pool.take<int64_t>(nseeds + 1), *tmp = pool.take<int64_t>(scan_tmp_items(nseeds));
-            int32_t *big = pool.take<int32_t>(nseeds);
-            big_flags_kernel<<<grid_for(nseeds, 256), 256, 0, s>>>(nseeds, seed_ptr, g->rowptr.get(), flag);
+        if (nbig > 0) {
+            const int blocks = (int)std::min<int64_t>(nbig, (int64_t)num_sms() * 4);
+            greedy_big_kernel<<<blocks, kBlockRun, 0, s>>>(nbig, big, g->rowptr.get(), g->col.get(), thr, core,
+                                                           scratch, run_size, best, abort_runs, H);
             MCE_LAUNCH_CHECK();
-            exclusive_scan_i32(flag, pos, nseeds, tmp, s);
-            gather_flagged_kernel<<<grid_for(nseeds, 256), 256, 0, s>>>(nseeds, seed_ptr, flag, pos, big);
-            MCE_LAUNCH_CHECK();
-            int64_t *hnb = g->host.get<int64_t>(1);
-            MCE_CUDA(cudaMemcpyAsync(hnb, pos + nseeds, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
-            stream_sync(s);
-            const int64_t nbig = hnb[0];
-            kernels += 5;
-            if (nbig > 0) {
-                const int blocks = (int)std::min<int64_t>(nbig, (int64_t)num_sms() * 4);
-                greedy_big_kernel<<<blocks, kBlockRun, 0, s>>>(nbig, big, g->rowptr.get(), g->col.get(), thr, core,
-                                                               scratch, run_size, best, abort_runs);
-                MCE_LAUNCH_CHECK();
-                ++kernels;
-            }
+            ++kernels;
         }
         greedy_kernel<<<grid_for(nseeds * 8, 256), 256, 0, s>>>(nseeds, seed_ptr, g->rowptr.get(), g->col.get(),
-                                                                  thr, core, scratch, run_size, best, abort_runs);
+                                                                  thr, core, scratch, run_size, best, abort_runs, H);
         MCE_LAUNCH_CHECK();
         best_seed_kernel<<<grid_for(nseeds, 256), 256, 0, s>>>(nseeds, seed_ptr, thr, run_size, best, best_key);
         MCE_LAUNCH_CHECK();
-        replay_kernel<<<1, kReplay, 0, s>>>(best_key, g->rowptr.get(), g->col.get(), thr, scratch, clique);
+        replay_kernel<<<1, kReplay, 0, s>>>(best_key, g->rowptr.get(), g->col.get(), thr, scratch, clique, H);
         MCE_LAUNCH_CHECK();
         kernels += 3;
     }
