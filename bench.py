@@ -145,6 +145,19 @@ def cpu_baseline(graph_np, edges, budget_s=25.0):
             "seconds": dt, "omega": om, "count": len(cl)}
 
 
+def ncu_traffic(config: str, kname: str):
+    """DRAM bytes per launch (dram__bytes_read.sum + dram__bytes_write.sum) of this config's dominant
+    kernel from the committed `ncu --set full` capture (profiles/ncu_traffic.json), or None."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
+            rec = json.load(f).get(config)
+    except (OSError, ValueError):
+        return None
+    if not rec or rec.get("kernel", "") not in kname:
+        return None
+    return rec.get("bytes_per_launch")
+
+
 def build_graph(config: str, device: str):
     from synth import graphs as G
 
@@ -261,9 +274,10 @@ def main():
         kname = "root_expand_w1 (fused root level: adjacency build + first expansion)"
         k_ms, k_bytes, launches = root_ms, tm["root_kernel_bytes"], max(tm["root_launches"], 1)
     else:
-        kname = "expand_count (mce::expand_thread/expand_warp count pass)"
+        kname = "expand (fused count + write pass of levels >= 2: mce::expand_thread / expand_tile)"
         k_ms, k_bytes, launches = cnt_ms, tm["count_kernel_bytes"], max(tm["count_launches"], 1)
     achieved = (k_bytes / launches) / ((k_ms / launches) / 1e3) / 1e9 if k_ms > 0 else 0.0
+    traffic = ncu_traffic(args.config, kname)
     phases = {"preprocess_ms": statistics.mean(t["preprocess_ms"] for t in timings),
               "heuristic_ms": statistics.mean(t["heuristic_ms"] for t in timings),
               "expand_ms": statistics.mean(t["expand_ms"] for t in timings),
@@ -330,7 +344,7 @@ def main():
                        "step_ms": [round(t, 4) for t in times]},
             "roofline": {"bound": "hbm", "kernel": kname,
                          "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak if peak else None, "traffic": None, "peak_source": peak_src,
+                         "frac": achieved / peak if peak else None, "traffic": traffic, "peak_source": peak_src,
                          "bytes_per_launch": k_bytes / launches, "launches_per_step": launches,
                          "kernel_ms_per_step": k_ms},
             "cpu_baseline": cpu,

@@ -98,6 +98,9 @@ typedef struct {
                                 recorded as the clique C + P instead of being expanded level by
                                 level (its only clique of that size; reading 10);
                                 1: Algorithm 2's expansion of every level (A/B tests) */
+    int32_t no_fused_expand; /* 0 (default): a level's count pass also writes the children (slots
+                                reserved per warp, colouring computed once) whenever they fit half
+                                of the free budget; 1: count -> scan -> write passes (A/B tests) */
 } mce_options;
 
 /* Fill `opt` with defaults: degeneracy orientation, multi-run degree heuristic

@@ -46,6 +46,7 @@ class Options(ctypes.Structure):
         ("legacy_roots", ctypes.c_int32),
         ("no_fused_levels", ctypes.c_int32),
         ("no_clique_shortcut", ctypes.c_int32),
+        ("no_fused_expand", ctypes.c_int32),
     ]
 
 

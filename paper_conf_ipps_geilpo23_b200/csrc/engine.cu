@@ -57,8 +57,9 @@ struct Arena {
         off = m.off;
         before = m.before;
     }
+    // at != nullptr: receives the mark just before the allocation (after a segment switch)
     template <typename T>
-    T *alloc(int64_t count) {
+    T *alloc(int64_t count, Mark *at = nullptr) {
         const size_t bytes = ((size_t)std::max<int64_t>(count, 1) * sizeof(T) + kAlign - 1) / kAlign * kAlign;
         if (off + bytes > (*segs)[cur].n) {  // next segment (the rest of this one is skipped)
             const size_t nb = before + (*segs)[cur].n;
@@ -76,6 +77,7 @@ struct Arena {
             fail(MCE_ERR_BUDGET, "frontier budget exhausted (need " + std::to_string(bytes) + " more bytes, " +
                                      std::to_string(avail()) + " available)");
         T *p = reinterpret_cast<T *>((*segs)[cur].p + off);
+        if (at) *at = Mark{cur, off, before};
         off += bytes;
         return p;
     }
@@ -83,7 +85,8 @@ struct Arena {
 
 struct Level {
     int64_t count = 0;
-    int32_t W = 1;  // words per candidate set (stride of P)
+    int32_t W = 1;   // words per candidate set (kernel width)
+    int32_t Ps = 0;  // P stride in words (0: = W; a fused pass writes the parent's width)
     uint64_t *P = nullptr;
     int32_t *slot = nullptr;
     int32_t *parent = nullptr;
@@ -198,6 +201,7 @@ class Engine {
     unsigned long long *clq_total_ = nullptr;   // g->misc[2] clique completions (reading 10)
     unsigned long long *clq_slot_ = nullptr;    // g->misc[3]
     int32_t *maxbit_ = nullptr;                 // g->misc[4]
+    unsigned long long *out_count_ = nullptr;   // g->misc[5] fused-pass children
     int64_t stage_rows_ = 0;
     int64_t cstage_rows_ = 0;
     int64_t stage_max_rows_ = 0;  // staging never exceeds a quarter of the budget (stored list truncated, count exact)
@@ -326,6 +330,7 @@ bool Engine::run_small(int32_t k, const Level &L) {
     a.need = need();
     a.bound = o_.bound;
     a.Wp = L.W;
+    a.Ps = L.Ps > 0 ? L.Ps : L.W;
     a.Wa = W_;
     a.Wc = L.W;
     a.roots = roots_;
@@ -363,6 +368,7 @@ bool Engine::run_small(int32_t k, const Level &L) {
         la.end = o.inN;
         la.k = (int32_t)o.k_next - 1;
         la.Wp = la.Wc = (int32_t)o.inW;
+        la.Ps = (int32_t)o.inPs;
         la.counts = arena_.alloc<int32_t>(o.inN);  // for a count-pass replay if the staging must grow
         handle_leaves((int32_t)o.k_next, o.leaves, la, 0);
         if (o.cliques > 0 && (o.leaves == 0 || (!find_one_ && la.need == (int32_t)o.k_next)))
@@ -373,6 +379,7 @@ bool Engine::run_small(int32_t k, const Level &L) {
         Level C;
         C.count = o.children;
         C.W = (int32_t)o.Wc;
+        C.Ps = (int32_t)o.Wc;
         C.P = o.P;
         C.slot = o.slot;
         C.parent = o.parent;
@@ -409,6 +416,7 @@ void Engine::process(int32_t k, const Level &L) {
     a.need = need();
     a.bound = o_.bound;
     a.Wp = L.W;
+    a.Ps = L.Ps > 0 ? L.Ps : L.W;
     a.Wa = W_;
     a.Wc = L.W;
     a.roots = roots_;
@@ -420,17 +428,50 @@ void Engine::process(int32_t k, const Level &L) {
     leaf_args(a);
     a.chain = chain_dev_;
 
-    // misc[0..4] = leaf total, leaf slot, completion total, completion slot, maxbit (-1)
+    // Fused count + write: the children are written by the count pass into
+    // arrays sized for half of the free budget; if they fit they are compacted
+    // and the next level starts without a scan or a write pass.
+    const int64_t per_child = 8 * L.W + 12;
+    Arena::Mark fmark = arena_.mark();
+    bool fused = false;
+    int64_t fcap = 0;
+    uint64_t *fP = nullptr;
+    int32_t *fslot = nullptr, *fparent = nullptr, *fvloc = nullptr;
+    if (!o_.no_fused_expand) {
+        // capacity: half of the free budget, at most 16 children per entry (+1M);
+        // a level that branches wider overflows into scan + chunked writes
+        fcap = std::min<int64_t>((int64_t)(arena_.avail() / 2) / (per_child + 64), 16 * N + (1 << 20));
+        if (fcap >= 1024) {
+            fP = arena_.alloc<uint64_t>(fcap * L.W, &fmark);
+            fslot = arena_.alloc<int32_t>(fcap);
+            fparent = arena_.alloc<int32_t>(fcap);
+            fvloc = arena_.alloc<int32_t>(fcap);
+            fused = true;
+            a.fused = 1;
+            a.out_count = out_count_;
+            a.out_cap = fcap;
+            a.cP = fP;
+            a.cslot = fslot;
+            a.cparent = fparent;
+            a.cvloc = fvloc;
+        }
+    }
+
+    // misc[0..4] = leaf total, leaf slot, completion total, completion slot, maxbit (-1); misc[5] = fused children
     MCE_CUDA(cudaMemsetAsync(leaf_total_, 0, 4 * sizeof(unsigned long long), s_));
     MCE_CUDA(cudaMemsetAsync(maxbit_, 0xff, 2 * sizeof(int32_t), s_));
+    if (fused) MCE_CUDA(cudaMemsetAsync(out_count_, 0, sizeof(unsigned long long), s_));
     launch_timed(a, false);
-    exclusive_scan_i32(counts, offs, N, tmp, s_);
-    kernels_ += 3;
-    int64_t *h = g_->host.get<int64_t>(6);
-    MCE_CUDA(cudaMemcpyAsync(h, offs + N, sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
-    MCE_CUDA(cudaMemcpyAsync(h + 1, leaf_total_, 5 * sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
+    kernels_ += 1;
+    if (!fused) {
+        exclusive_scan_i32(counts, offs, N, tmp, s_);
+        kernels_ += 2;
+    }
+    int64_t *h = g_->host.get<int64_t>(8);
+    if (!fused) MCE_CUDA(cudaMemcpyAsync(h, offs + N, sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
+    MCE_CUDA(cudaMemcpyAsync(h + 1, leaf_total_, 6 * sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
     stream_sync(s_);
-    const int64_t total = h[0];
+    const int64_t total = fused ? h[6] : h[0];
     const unsigned long long leaves = (unsigned long long)h[1];
     const int64_t completions = h[3];
     const int32_t maxbit = (int32_t)(uint32_t)(uint64_t)h[5];
@@ -441,14 +482,52 @@ void Engine::process(int32_t k, const Level &L) {
     while (Wc * 64 <= maxbit && Wc < L.W) Wc <<= 1;
     a.Wc = Wc;
     if (o_.verbose > 0)
-        fprintf(stderr, "[mce] level k=%d entries=%lld children=%lld leaves=%llu need=%d\n", k, (long long)N,
-                (long long)total, leaves, a.need);
+        fprintf(stderr, "[mce] level k=%d entries=%lld children=%lld leaves=%llu need=%d%s\n", k, (long long)N,
+                (long long)total, leaves, a.need, fused ? (total <= fcap ? " fused" : " fused-overflow") : "");
     const int32_t need_counted = a.need;
+    a.fused = 0;  // a count-pass replay (staging growth) must not write children again
     if (leaves) handle_leaves(k + 1, (int64_t)leaves, a, 0);
     if (completions > 0 && (leaves == 0 || (!find_one_ && need_counted == k + 1)))
         handle_leaves(need_counted, completions, a, 1);
 
-    const int64_t per_child = 8 * Wc + 12 + 12 + 16;
+    if (fused && total <= fcap) {
+        count_bytes_ += (double)total * (8.0 * L.W + 12.0);  // the children the fused pass wrote
+        Level C;
+        C.count = total;
+        C.W = Wc;
+        C.Ps = L.W;
+        if (total > 0) {
+            // compact: slot/parent/vloc go to a temporary behind the fcap-sized
+            // arrays, then to tight arrays right behind P (P stays in place);
+            // the tight arrays end before the temporary starts (total <= fcap)
+            int32_t *tmp3 = arena_.alloc<int32_t>(3 * total);
+            MCE_CUDA(cudaMemcpyAsync(tmp3, fslot, sizeof(int32_t) * total, cudaMemcpyDeviceToDevice, s_));
+            MCE_CUDA(cudaMemcpyAsync(tmp3 + total, fparent, sizeof(int32_t) * total, cudaMemcpyDeviceToDevice, s_));
+            MCE_CUDA(cudaMemcpyAsync(tmp3 + 2 * total, fvloc, sizeof(int32_t) * total, cudaMemcpyDeviceToDevice,
+                                     s_));
+            arena_.reset(fmark);
+            C.P = arena_.alloc<uint64_t>(total * L.W);  // == fP
+            C.slot = arena_.alloc<int32_t>(total);
+            C.parent = arena_.alloc<int32_t>(total);
+            C.vloc = arena_.alloc<int32_t>(total);
+            MCE_CUDA(cudaMemcpyAsync(C.slot, tmp3, sizeof(int32_t) * total, cudaMemcpyDeviceToDevice, s_));
+            MCE_CUDA(cudaMemcpyAsync(C.parent, tmp3 + total, sizeof(int32_t) * total, cudaMemcpyDeviceToDevice, s_));
+            MCE_CUDA(cudaMemcpyAsync(C.vloc, tmp3 + 2 * total, sizeof(int32_t) * total, cudaMemcpyDeviceToDevice,
+                                     s_));
+            if (C.P != fP) fail(MCE_ERR_INVALID, "internal: fused level moved");
+        }
+        sync_bound(true);
+        if (total > 0) process(k + 1, C);
+        arena_.reset(mark);
+        return;
+    }
+    if (fused) {  // overflow: the children did not fit; scan the counts and write in chunks
+        arena_.reset(fmark);
+        exclusive_scan_i32(counts, offs, N, tmp, s_);
+        kernels_ += 2;
+    }
+
+    const int64_t per_child2 = 8 * Wc + 12 + 12 + 16;
     // When the children do not fit they are produced in chunks.  Each chunk may
     // take 1/(levels still reachable below it + 1) of the free arena, so a
     // frontier that keeps growing for many levels (R-MAT: 2x per level over the
@@ -456,8 +535,8 @@ void Engine::process(int32_t k, const Level &L) {
     const int64_t depth_left = std::max<int64_t>(1, (int64_t)maxub - (k + 1));
     int64_t a0 = 0;
     while (total > 0 && a0 < N) {
-        const int64_t share = total * per_child <= (int64_t)(arena_.avail() / 2) ? 2 : depth_left + 1;
-        const int64_t cap = (int64_t)(arena_.avail() / share) / per_child;
+        const int64_t share = total * per_child2 <= (int64_t)(arena_.avail() / 2) ? 2 : depth_left + 1;
+        const int64_t cap = (int64_t)(arena_.avail() / share) / per_child2;
         int64_t b, cnt, base;
         if (a0 == 0 && total <= cap) {
             b = N;
@@ -743,6 +822,7 @@ mce_result *Engine::run() {
     clq_total_ = leaf_total_ + 2;
     clq_slot_ = leaf_total_ + 3;
     maxbit_ = reinterpret_cast<int32_t *>(leaf_total_ + 4);
+    out_count_ = leaf_total_ + 5;
     chain_dev_ = reinterpret_cast<LevelLink *>(g_->misc.get() + 256);
     stage_max_rows_ = std::max<int64_t>(1ll << 20, budget / 4 / (4ll * std::max<int32_t>(g_->max_out + 2, 2)));
     stage_rows_ = find_one_ ? 1 : 4096;

@@ -266,13 +266,36 @@ __device__ __forceinline__ void flush_counters(const ExpandArgs &a, unsigned lon
 // number of surviving children (count pass) after writing them at `out`
 // (write pass).  Leaves, highest child bit and reachable depth accumulate
 // into the caller's counters.
+// warp exclusive prefix sum of x over all 32 lanes (total in `total`)
+__device__ __forceinline__ unsigned long long warp_excl_u64(unsigned long long x, unsigned long long &total) {
+    const int lane = threadIdx.x & 31;
+    unsigned long long inc = x;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const unsigned long long y = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= o) inc += y;
+    }
+    total = __shfl_sync(0xffffffffu, inc, 31);
+    return inc - x;
+}
+
+// one candidate entry e (thread per candidate, W <= 4 words); returns its
+// number of surviving children (count pass) after writing them at `out`
+// (write pass).  Leaves, highest child bit and reachable depth accumulate
+// into the caller's counters.  FUSED (count pass, called by all 32 lanes of
+// the warp; `active` = lane has an entry): the children are also written, at
+// slots reserved for the whole warp with one atomicAdd, by replaying the
+// cheap branching loop after the colouring (which the separate write pass
+// would recompute).
 template <int W, bool WRITE>
 __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, int64_t out, unsigned &nleaf,
-                                                unsigned &nclq, int &hb, int &ub) {
+                                                unsigned &nclq, int &hb, int &ub, bool active = true,
+                                                bool fused = false) {
     uint64_t P[W];
 #pragma unroll
-    for (int w = 0; w < W; ++w) P[w] = a.P[e * W + w];
-    const RootInfo ri = a.roots[a.slot[e]];
+    for (int w = 0; w < W; ++w) P[w] = active ? a.P[e * a.Ps + w] : 0ull;
+    RootInfo ri{};
+    if (active) ri = a.roots[a.slot[e]];
     const uint64_t *A = a.adj + ri.abase;
     const int Wa = a.Wa;
     uint8_t ord[64 * W];
@@ -323,15 +346,20 @@ __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, 
         ncol = np;
     }
     // P is a clique iff every colour class is a single vertex (reading 10)
+    bool done = false;
     if (a.shortcut && a.bound == 1 && np >= 2 && ncol == np && a.k + np == a.need) {
         if (!WRITE) {
             ++nclq;
             store_clique_leaf<1, W>(a, e, P, ri, 0xffffffffu);
         }
-        return 0;
+        done = true;
+        if (!fused) return 0;
     }
-    int32_t cnt = 0;
-    if (a.k + ncol >= a.need) {
+    // the branching loop (Algorithm 2 lines 3-9 with the colouring order):
+    // MODE 0 count (+ leaves), 1 write at `at` with word stride `ws`
+    auto branch = [&](int mode, int64_t at, int ws) -> int32_t {
+        int32_t cnt = 0;
+        if (done || a.k + ncol < a.need) return 0;
         uint64_t R[W];
 #pragma unroll
         for (int w = 0; w < W; ++w) R[w] = P[w];
@@ -348,16 +376,16 @@ __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, 
             }
             R[v >> 6] &= ~(1ull << (v & 63));
             if (pc == 0) {
-                if (!WRITE && a.k + 1 >= a.need) {
+                if (mode == 0 && a.k + 1 >= a.need) {
                     ++nleaf;
                     store_leaf(a, e, v, ri);
                 }
             } else if (a.k + 1 + pc >= a.need) {
-                if (WRITE) {
-                    const int64_t c = out + cnt;
+                if (mode == 1) {
+                    const int64_t c = at + cnt;
 #pragma unroll
                     for (int w = 0; w < W; ++w)
-                        if (w < a.Wc) a.cP[c * a.Wc + w] = C[w];
+                        if (w < ws) a.cP[c * ws + w] = C[w];
                     a.cslot[c] = a.slot[e];
                     a.cparent[c] = (int32_t)e;
                     a.cvloc[c] = v;
@@ -368,6 +396,17 @@ __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, 
                 ++cnt;
             }
         }
+        return cnt;
+    };
+    if (WRITE) return branch(1, out, a.Wc);
+    const int32_t cnt = branch(0, 0, 0);
+    if (fused) {
+        unsigned long long total;
+        const unsigned long long excl = warp_excl_u64((unsigned long long)cnt, total);
+        unsigned long long base = 0;
+        if ((threadIdx.x & 31) == 0 && total) base = atomicAdd(a.out_count, total);
+        base = __shfl_sync(0xffffffffu, base, 0) + excl;
+        if (cnt > 0 && (int64_t)(base + cnt) <= a.out_cap) branch(1, (int64_t)base, W);
     }
     return cnt;
 }
@@ -377,6 +416,17 @@ __global__ void __launch_bounds__(256) expand_thread(const ExpandArgs a) {
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     unsigned nleaf = 0, nclq = 0;
     int hb = -1, ub = 0;
+    if (!WRITE && a.fused) {  // warp-uniform loop: the whole warp reserves its children's slots at once
+        for (int64_t e0 = a.begin + (int64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31); e0 < a.end;
+             e0 += stride) {
+            const int64_t e = e0 + (threadIdx.x & 31);
+            const bool active = e < a.end;
+            const int32_t cnt = expand_entry<W, false>(a, e, 0, nleaf, nclq, hb, ub, active, true);
+            if (active) a.counts[e] = cnt;
+        }
+        flush_counters(a, nleaf, nclq, hb, ub);
+        return;
+    }
     for (int64_t e = a.begin + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < a.end; e += stride) {
         int64_t out = 0;
         if (WRITE) {
@@ -486,6 +536,7 @@ __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a
             out->invloc = const_cast<int32_t *>(A.vloc);
             out->inN = N;
             out->inW = W;
+            out->inPs = A.Ps;
             out->k_next = A.k + 1;
             out->children = total;
             if (s_leaf) atomicAdd(A.leaf_total, (unsigned long long)s_leaf);
@@ -534,6 +585,7 @@ __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a
             A.begin = 0;
             A.end = total;
             A.Wp = A.Wc;
+            A.Ps = A.Wc;
             A.k = A.k + 1;
         }
         __syncthreads();
@@ -571,7 +623,7 @@ __global__ void expand_tile(const ExpandArgs a, int max_l) {
 #pragma unroll
         for (int t = 0; t < WPL; ++t) {
             const int j = gl + G * t;
-            P[t] = j < W ? a.P[e * W + j] : 0ull;
+            P[t] = j < W ? a.P[e * a.Ps + j] : 0ull;
         }
         const RootInfo ri = a.roots[a.slot[e]];
         const uint64_t *A = a.adj + ri.abase;
@@ -715,6 +767,52 @@ __global__ void expand_tile(const ExpandArgs a, int max_l) {
             }
         }
         if (!WRITE && gl == 0) a.counts[e] = cnt;
+        if (!WRITE && a.fused && cnt > 0) {  // fused: reserve and replay the branching, writing
+            unsigned long long base = 0;
+            if (gl == 0) base = atomicAdd(a.out_count, (unsigned long long)cnt);
+            base = __shfl_sync(gmask, base, 0, G);
+            if ((int64_t)(base + cnt) <= a.out_cap) {
+                uint64_t R[WPL];
+#pragma unroll
+                for (int t = 0; t < WPL; ++t) R[t] = P[t];
+                int32_t c2 = 0;
+                for (int i = np - 1; i >= 0; --i) {
+                    if (a.k + colr[i] < a.need) break;
+                    const int v = ord[i];
+                    const uint64_t *row = A + (int64_t)v * Wa;
+                    uint64_t C[WPL];
+                    int pc = 0;
+#pragma unroll
+                    for (int t = 0; t < WPL; ++t) {
+                        const int j = gl + G * t;
+                        C[t] = j < W ? (R[t] & __ldg(row + j)) : 0ull;
+                        pc += __popcll(C[t]);
+                    }
+#pragma unroll
+                    for (int o = G / 2; o > 0; o >>= 1) pc += __shfl_xor_sync(gmask, pc, o, G);
+                    const int jv = v >> 6;
+                    if ((jv & (G - 1)) == gl) {
+#pragma unroll
+                        for (int t = 0; t < WPL; ++t)
+                            if (t == jv / G) R[t] &= ~(1ull << (v & 63));
+                    }
+                    if (pc > 0 && a.k + 1 + pc >= a.need) {
+                        const int64_t c = (int64_t)base + c2;
+#pragma unroll
+                        for (int t = 0; t < WPL; ++t) {
+                            const int j = gl + G * t;
+                            if (j < W) a.cP[c * W + j] = C[t];
+                        }
+                        if (gl == 0) {
+                            a.cslot[c] = a.slot[e];
+                            a.cparent[c] = (int32_t)e;
+                            a.cvloc[c] = v;
+                        }
+                        ++c2;
+                    }
+                }
+            }
+        }
         __syncwarp(gmask);
     }
     if (!WRITE) flush_counters(a, nleaf, nclq, hb, ub);

@@ -38,7 +38,8 @@ struct ExpandArgs {
     int32_t k;           // |C|
     int32_t need;        // smallest clique size still of interest
     int32_t bound;       // 0: |C|+|P|, 1: colouring
-    int32_t Wp;          // words per candidate set of this level (its P stride; 1, 2, 4, 8, ...)
+    int32_t Wp;          // words per candidate set of this level (kernel width; 1, 2, 4, 8, ...)
+    int32_t Ps;          // P stride of this level in words (>= Wp: a fused pass writes the parent's width)
     int32_t Wa;          // words per adjacency row of the root window (>= Wp)
     int32_t Wc;          // write pass: words per child candidate set (<= Wp, from *maxbit)
     const RootInfo *roots;
@@ -72,6 +73,12 @@ struct ExpandArgs {
     unsigned long long *clq_slot;
     int32_t *clq_rows;
     int64_t clq_cap;  // rows of `need` vertices
+    // fused count + write (count pass only): children are appended at
+    // cP/cslot/... + atomicAdd(out_count) with stride Wp while they fit out_cap;
+    // counts[] is written as usual so an overflowing level falls back to scan + write
+    int32_t fused;
+    unsigned long long *out_count;
+    int64_t out_cap;
 };
 
 // Fused root level for W == 1 roots (roots.cu): one warp per root builds the
@@ -116,7 +123,7 @@ struct SmallOut {
     int32_t *slot, *parent, *vloc;
     uint64_t *inP;     // the last processed level (for a leaf replay)
     int32_t *inslot, *inparent, *invloc;
-    int64_t inN, inW;
+    int64_t inN, inW, inPs;
     int64_t level_n[kSmallMaxLevels];  // entries of every processed level
 };
 void launch_expand_small(const ExpandArgs &a, uint8_t *scratch, int64_t scratch_bytes, SmallOut *out,

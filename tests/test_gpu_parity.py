@@ -320,3 +320,25 @@ def test_heuristic_hub_runs(key):
     order = np.lexsort((np.arange(g.n), -np.diff(rp).astype(np.int64)))
     assert np.array_equal(runs[order], runs_o)
     assert r.omega == oracle_answer(key)[0]
+
+
+@pytest.mark.parametrize("key", ["er2000", "planted", "RMAT11", "RMAT13", "K130", "K257", "T(30,6)", "ER400d",
+                                 "Paley17", "BA5k"])
+def test_fused_expand_off_matches(key):
+    """The separate count -> scan -> write passes (no fused count + write) give the same answer."""
+    g = GRAPHS[key]()
+    om, cl = oracle_answer(key)
+    for fused_levels in (True, False):
+        r = run_enum(g, fused_expand=False, fused_levels=fused_levels)
+        assert (r.omega, r.count) == (om, len(cl)) and np.array_equal(r.cliques, cl)
+
+
+@pytest.mark.parametrize("key", ["ER400d", "RMAT13", "T(36,12)"])
+def test_fused_expand_overflow(key):
+    """A budget too small for a level's children makes the fused pass overflow
+    (falls back to scan + chunked writes); find-one under the same budget."""
+    g = GRAPHS[key]()
+    om, cl = oracle_answer(key)
+    for budget in (2 << 20, 6 << 20, 32 << 20):
+        r = run_enum(g, budget_bytes=budget, heuristic="none", fused_levels=False)
+        assert r.omega == om and np.array_equal(r.cliques, cl)
