@@ -441,6 +441,11 @@ void Engine::process(int32_t k, const Level &L) {
         // capacity: half of the free budget, at most 16 children per entry (+1M);
         // a level that branches wider overflows into scan + chunked writes
         fcap = std::min<int64_t>((int64_t)(arena_.avail() / 2) / (per_child + 64), 16 * N + (1 << 20));
+        // a power of two: budget jitter between calls then asks for the same
+        // sizes, so the arena's kept segments are reused (no re-allocation)
+        int64_t p2 = 1;
+        while (p2 * 2 <= fcap) p2 <<= 1;
+        fcap = p2;
         if (fcap >= 1024) {
             fP = arena_.alloc<uint64_t>(fcap * L.W, &fmark);
             fslot = arena_.alloc<int32_t>(fcap);
@@ -825,10 +830,13 @@ mce_result *Engine::run() {
     out_count_ = leaf_total_ + 5;
     chain_dev_ = reinterpret_cast<LevelLink *>(g_->misc.get() + 256);
     stage_max_rows_ = std::max<int64_t>(1ll << 20, budget / 4 / (4ll * std::max<int32_t>(g_->max_out + 2, 2)));
-    stage_rows_ = find_one_ ? 1 : 4096;
-    g_->stage.ensure((size_t)stage_rows_ * std::max<int32_t>(g_->max_out + 2, 2));
-    cstage_rows_ = find_one_ ? 1 : 4096;
-    g_->cstage.ensure((size_t)cstage_rows_ * std::max<int32_t>(g_->max_out + 2, 2));
+    // staging rows: whatever the buffers kept from earlier calls hold (a count
+    // pass is replayed when the staging is too small, so reuse avoids replays)
+    const int64_t row_w = std::max<int32_t>(g_->max_out + 2, 2);
+    stage_rows_ = find_one_ ? 1 : std::max<int64_t>(4096, (int64_t)g_->stage.n / row_w);
+    g_->stage.ensure((size_t)stage_rows_ * row_w);
+    cstage_rows_ = find_one_ ? 1 : std::max<int64_t>(4096, (int64_t)g_->cstage.n / row_w);
+    g_->cstage.ensure((size_t)cstage_rows_ * row_w);
 
     res->h_setup_ms = ms_since(h2);
     const auto h3 = clk::now();

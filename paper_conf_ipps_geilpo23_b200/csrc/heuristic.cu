@@ -15,6 +15,8 @@
 // in place with __ballot_sync/__popc, so every run stays in one warp's
 // registers + one contiguous scratch segment and no host round trip is needed
 // per iteration.
+#include <cub/device/device_radix_sort.cuh>
+
 #include <algorithm>
 #include <vector>
 
@@ -149,6 +151,21 @@ __device__ int32_t hub_tail_warp(const Hub &H, const int32_t *src, int64_t len, 
     return csize;
 }
 
+// x ~ w with the hub bit matrix when both are hubs (hw = hid[w] or -1);
+// also reports whether x is a hub
+__device__ __forceinline__ bool adjacent_h(const Hub &H, int hw, const int64_t *__restrict__ rowptr,
+                                           const int32_t *__restrict__ col, int32_t x, int32_t w, int64_t wb,
+                                           int64_t we, bool &x_hub) {
+    if (H.K) {
+        const int hx = __ldg(H.hid + x);
+        x_hub = hx >= 0;
+        if (x_hub && hw >= 0) return (__ldg(H.M + (int64_t)hw * H.KW + (hx >> 6)) >> (hx & 63)) & 1ull;
+    } else {
+        x_hub = false;
+    }
+    return adjacent(rowptr, col, x, w, wb, we);
+}
+
 // One greedy run for seed s by a tile of G lanes (G = 8 or 32) of the calling
 // warp.  Returns the clique size (a partial size < the best when aborted).
 template <int G>
@@ -184,16 +201,18 @@ __device__ int32_t greedy_run(int32_t s, const int64_t *__restrict__ rowptr, con
         const int32_t w = (int32_t)(0x7fffffffu - (uint32_t)(key & 0xffffffffull));
         ++csize;
         const int64_t wb = rowptr[w], we = rowptr[w + 1];
+        const int hw = H.K ? __ldg(H.hid + w) : -1;
         int64_t out = 0;
         int nonhub = 0;
         for (int64_t i0 = 0; i0 < len; i0 += G) {
             int64_t i = i0 + gl;
             int32_t x = i < len ? src[i] : -1;
-            bool keep = i < len && x != w && adjacent(rowptr, col, x, w, wb, we);
+            bool xh = true;
+            bool keep = i < len && x != w && adjacent_h(H, hw, rowptr, col, x, w, wb, we, xh);
             const unsigned m = (__ballot_sync(gmask, keep) & gmask) >> gbase;
             if (keep) buf[out + __popc(m & ((1u << gl) - 1u))] = x;
             out += __popc(m);
-            if (G == 32 && H.K) nonhub += __popc(__ballot_sync(gmask, keep && __ldg(H.hid + x) < 0));
+            if (G == 32 && H.K) nonhub += __popc(__ballot_sync(gmask, keep && !xh));
         }
         __syncwarp(gmask);
         src = buf;
@@ -249,14 +268,16 @@ __device__ int32_t block_run(int32_t s, const int64_t *__restrict__ rowptr, cons
         if (clique && threadIdx.x == 0) clique[csize] = w;
         ++csize;
         const int64_t wb = rowptr[w], we = rowptr[w + 1];
+        const int hw = H.K ? __ldg(H.hid + w) : -1;
         int64_t out = 0;
         int32_t nonhub = 0;
         for (int64_t i0 = 0; i0 < len; i0 += NT) {
             const int64_t i = i0 + threadIdx.x;
             const int32_t x = i < len ? src[i] : -1;
-            const bool keep = i < len && x != w && adjacent(rowptr, col, x, w, wb, we);
+            bool xh = true;
+            const bool keep = i < len && x != w && adjacent_h(H, hw, rowptr, col, x, w, wb, we, xh);
             const unsigned m = __ballot_sync(0xffffffffu, keep);
-            const unsigned nh = H.K ? __ballot_sync(0xffffffffu, keep && __ldg(H.hid + x) < 0) : 0u;
+            const unsigned nh = H.K ? __ballot_sync(0xffffffffu, keep && !xh) : 0u;
             __syncthreads();  // wkey/wcnt reuse, and every read of this chunk precedes its writes
             if (lane == 0) {
                 wcnt[wid] = __popc(m);
@@ -382,6 +403,12 @@ __global__ void big_flags_kernel(int64_t nseeds, const int32_t *__restrict__ see
         const int32_t s = seeds[i];
         flag[i] = rowptr[s + 1] - rowptr[s] > kBigSeed;
     }
+}
+
+__global__ void seed_degree_kernel(int64_t nbig, const int32_t *__restrict__ big, const int64_t *__restrict__ rowptr,
+                                   int32_t *deg) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nbig; i += (int64_t)gridDim.x * blockDim.x)
+        deg[i] = (int32_t)(rowptr[big[i] + 1] - rowptr[big[i]]);
 }
 
 __global__ void gather_flagged_kernel(int64_t n, const int32_t *__restrict__ in, const int32_t *__restrict__ flag,
@@ -669,11 +696,29 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
     }
     if (nseeds > 0) {
         if (nbig > 0) {
-            const int blocks = (int)std::min<int64_t>(nbig, (int64_t)num_sms() * 4);
-            greedy_big_kernel<<<blocks, kBlockRun, 0, s>>>(nbig, big, g->rowptr.get(), g->col.get(), thr, core,
-                                                           scratch, run_size, best, abort_runs, H);
+            // hub runs by descending degree, the first SM-count of them alone: the
+            // longest runs publish their sizes before the rest start, which then abort
+            // earlier (the order of runs never changes a result: ties go by key)
+            int32_t *dk = pool.take<int32_t>(nbig), *dk2 = pool.take<int32_t>(nbig);
+            int32_t *big2 = pool.take<int32_t>(nbig);
+            seed_degree_kernel<<<grid_for(nbig, 256), 256, 0, s>>>(nbig, big, g->rowptr.get(), dk);
             MCE_LAUNCH_CHECK();
-            ++kernels;
+            size_t tb = 0;
+            MCE_CUDA(cub::DeviceRadixSort::SortPairsDescending(nullptr, tb, dk, dk2, big, big2, (int)nbig, 0, 32, s));
+            void *tmpb = pool.take<uint8_t>((int64_t)tb);
+            MCE_CUDA(cub::DeviceRadixSort::SortPairsDescending(tmpb, tb, dk, dk2, big, big2, (int)nbig, 0, 32, s));
+            const int64_t first = std::min<int64_t>(nbig, num_sms());
+            greedy_big_kernel<<<(int)first, kBlockRun, 0, s>>>(first, big2, g->rowptr.get(), g->col.get(), thr, core,
+                                                               scratch, run_size, best, abort_runs, H);
+            MCE_LAUNCH_CHECK();
+            if (nbig > first) {
+                const int blocks = (int)std::min<int64_t>(nbig - first, (int64_t)num_sms() * 4);
+                greedy_big_kernel<<<blocks, kBlockRun, 0, s>>>(nbig - first, big2 + first, g->rowptr.get(),
+                                                               g->col.get(), thr, core, scratch, run_size, best,
+                                                               abort_runs, H);
+                MCE_LAUNCH_CHECK();
+            }
+            kernels += 5;
         }
         greedy_kernel<<<grid_for(nseeds * 8, 256), 256, 0, s>>>(nseeds, seed_ptr, g->rowptr.get(), g->col.get(),
                                                                   thr, core, scratch, run_size, best, abort_runs, H);

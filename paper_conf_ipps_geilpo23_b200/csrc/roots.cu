@@ -392,7 +392,7 @@ __device__ void root_thread(const RootArgs &a, int32_t r, unsigned long long &by
 // longer ones (<= 64) are queued in shared memory and taken by whole warps
 // (root_step<32, 2>) once the block's threads are done.
 constexpr int kThreadRootMax = 8;
-__global__ void __launch_bounds__(kRootWarps * 32) root_expand_w1(const RootArgs a) {
+__global__ void __launch_bounds__(kRootWarps * 32, 4) root_expand_w1(const RootArgs a) {
     __shared__ RootSmem<64> sm_all[kRootWarps];
     __shared__ int32_t queue[kRootWarps * 32];
     __shared__ int qn;
