@@ -101,6 +101,9 @@ typedef struct {
     int32_t no_fused_expand; /* 0 (default): a level's count pass also writes the children (slots
                                 reserved per warp, colouring computed once) whenever they fit half
                                 of the free budget; 1: count -> scan -> write passes (A/B tests) */
+    int32_t no_overlap;      /* 0 (default): the degree heuristics run on a second stream and host
+                                thread while the k-core / orientation preprocessing runs (they
+                                share no data); 1: one after the other */
 } mce_options;
 
 /* Fill `opt` with defaults: degeneracy orientation, multi-run degree heuristic

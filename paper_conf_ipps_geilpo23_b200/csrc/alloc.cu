@@ -24,8 +24,8 @@ struct DeviceCache {
     size_t cached = 0;
     size_t free_mem = 0;                        // last cudaMemGetInfo answer
     std::chrono::steady_clock::time_point free_at;
-    void *pinned = nullptr;
-    size_t pinned_bytes = 0;
+    void *pinned[2] = {nullptr, nullptr};  // slot 0: the calling thread, slot 1: the overlapped heuristic
+    size_t pinned_bytes[2] = {0, 0};
 };
 
 std::mutex g_mu;
@@ -122,17 +122,17 @@ size_t dev_free_memory() {
     return f;
 }
 
-void *host_pinned(size_t bytes) {
+void *host_pinned(size_t bytes, int slot) {
     const int dev = current_device();
     std::lock_guard<std::mutex> lk(g_mu);
     DeviceCache &c = g_cache[dev];
-    if (c.pinned_bytes < bytes) {
-        if (c.pinned) cudaFreeHost(c.pinned);
-        c.pinned = nullptr;
-        c.pinned_bytes = std::max<size_t>(bytes, 1 << 16);
-        MCE_CUDA(cudaMallocHost(&c.pinned, c.pinned_bytes));
+    if (c.pinned_bytes[slot] < bytes) {
+        if (c.pinned[slot]) cudaFreeHost(c.pinned[slot]);
+        c.pinned[slot] = nullptr;
+        c.pinned_bytes[slot] = std::max<size_t>(bytes, 1 << 16);
+        MCE_CUDA(cudaMallocHost(&c.pinned[slot], c.pinned_bytes[slot]));
     }
-    return c.pinned;
+    return c.pinned[slot];
 }
 
 }  // namespace mce

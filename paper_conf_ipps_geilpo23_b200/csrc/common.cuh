@@ -45,7 +45,7 @@ void dev_free(void *p, size_t bytes);    // bytes = the size passed to dev_alloc
 size_t dev_cached_bytes();               // free bytes held by the cache on this device
 size_t dev_free_memory();                // cudaMemGetInfo free bytes, re-queried at most once a second
 void dev_empty_cache();
-void *host_pinned(size_t bytes);         // per-device pinned staging (grow-only, shared)
+void *host_pinned(size_t bytes, int slot = 0);  // per-device pinned staging (grow-only; slot per thread role)
 
 // ---------------------------------------------------------------------------
 // owning device buffer
@@ -85,9 +85,10 @@ struct DevBuf {
 // pinned host staging (small scalar read-backs without pageable copies);
 // the memory is the device's shared staging block (host_pinned)
 struct PinnedBuf {
+    int slot = 0;
     template <typename T>
     T *get(size_t count) {
-        return reinterpret_cast<T *>(host_pinned(count * sizeof(T)));
+        return reinterpret_cast<T *>(host_pinned(count * sizeof(T), slot));
     }
 };
 

@@ -10,6 +10,8 @@
 //           Windowing"), so the frontier never exceeds the budget.
 #include <algorithm>
 #include <chrono>
+#include <exception>
+#include <thread>
 #include <cstdio>
 #include <cstring>
 #include <numeric>
@@ -783,17 +785,57 @@ mce_result *Engine::run() {
         sync_bound(false);
         return res;
     }
-    preprocess(g_, o_.orientation);
-    res->t_pre_ms = g_->t_pre_ms;
-    res->h_pre_ms = ms_since(h0);
-    const auto h1 = clk::now();
-    kernels_ += g_->kernels;
-
     int heur = o_.heuristic;
     if (find_one_ && heur == 0) heur = 1;  // find-one needs an incumbent clique
-    HeuristicResult hr = run_heuristic(g_, heur, o_.heuristic_runs, (int32_t)offset_, (int32_t)stride_, false);
-    res->t_heur_ms = hr.ms;
-    res->h_heur_ms = ms_since(h1);
+    HeuristicResult hr;
+    const bool need_pre = !(g_->have_core && g_->orientation == o_.orientation);
+    if (!o_.no_overlap && need_pre && (heur == MCE_HEUR_SINGLE_DEGREE || heur == MCE_HEUR_MULTI_DEGREE)) {
+        // the degree heuristics read only the CSR: run them on a second stream
+        // and host thread while the k-core peel and the orientation run here
+        if (!g_->hstream) MCE_CUDA(cudaStreamCreateWithFlags(&g_->hstream, cudaStreamNonBlocking));
+        cudaEvent_t ready;
+        MCE_CUDA(cudaEventCreateWithFlags(&ready, cudaEventDisableTiming));
+        MCE_CUDA(cudaEventRecord(ready, s_));  // the CSR is on the device
+        std::exception_ptr err;
+        double h_heur = 0.0;
+        const int dev = g_->device;
+        std::thread th([&] {
+            try {
+                const auto t0 = clk::now();
+                MCE_CUDA(cudaSetDevice(dev));
+                MCE_CUDA(cudaStreamWaitEvent(g_->hstream, ready, 0));
+                hr = run_heuristic(g_, heur, o_.heuristic_runs, (int32_t)offset_, (int32_t)stride_, false, true);
+                h_heur = ms_since(t0);
+            } catch (...) {
+                err = std::current_exception();
+            }
+        });
+        try {
+            preprocess(g_, o_.orientation);
+        } catch (...) {
+            th.join();
+            cudaEventDestroy(ready);
+            throw;
+        }
+        th.join();
+        cudaEventDestroy(ready);
+        if (err) std::rethrow_exception(err);
+        res->t_pre_ms = g_->t_pre_ms;
+        res->h_pre_ms = ms_since(h0);
+        res->t_heur_ms = hr.ms;
+        res->h_heur_ms = h_heur;
+        res->overlapped = 1;
+        kernels_ += g_->kernels;
+    } else {
+        preprocess(g_, o_.orientation);
+        res->t_pre_ms = g_->t_pre_ms;
+        res->h_pre_ms = ms_since(h0);
+        const auto h1 = clk::now();
+        kernels_ += g_->kernels;
+        hr = run_heuristic(g_, heur, o_.heuristic_runs, (int32_t)offset_, (int32_t)stride_, false);
+        res->t_heur_ms = hr.ms;
+        res->h_heur_ms = ms_since(h1);
+    }
     kernels_ += hr.kernels;
     best_ = std::max<int32_t>(hr.omega_bar, 2);
     if (find_one_) {

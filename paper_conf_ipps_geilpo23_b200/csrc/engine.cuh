@@ -22,6 +22,7 @@ struct mce_result {
     double h_total_ms = 0, h_pre_ms = 0, h_heur_ms = 0;  // host wall time of the call / its phases
     double h_setup_ms = 0, h_enum_ms = 0, h_readout_ms = 0;
     int64_t syncs = 0;                                    // host<->device round trips
+    int32_t overlapped = 0;                               // heuristic ran concurrently with preprocessing
 };
 
 namespace mce {

@@ -34,6 +34,14 @@ struct mce_graph {
     mce::Pool pool;                // per-phase scratch (reset at the start of every phase)
     std::vector<mce::DevBuf<uint8_t>> wsegs;  // frontier arena segments of mce_enumerate / mce_find_one
     mce::PinnedBuf host;           // pinned staging for small device->host reads (per device, shared)
+    // the heuristic overlapped with preprocessing (engine.cu) runs on its own
+    // thread, stream, scratch pool and pinned slot
+    mce::Pool hpool;
+    mce::PinnedBuf hhost{1};
+    cudaStream_t hstream = nullptr;
+    ~mce_graph() {
+        if (hstream) cudaStreamDestroy(hstream);
+    }
     mce::DevBuf<uint8_t> misc;     // engine: leaf counter + level chain (persistent)
     mce::DevBuf<int32_t> stage;    // engine: staged leaf cliques of one launch (grow-only)
     mce::DevBuf<int32_t> cstage;   // engine: staged clique completions of one launch (grow-only)

@@ -22,6 +22,7 @@
 
 #include "graph.cuh"
 #include "heuristic.cuh"
+#include "mce.h"
 
 namespace mce {
 
@@ -547,23 +548,27 @@ __global__ void __launch_bounds__(256) hub_matrix_kernel(int K, int KW, const in
 }  // namespace
 
 HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_rank, int32_t shard_count,
-                              bool want_runs) {
+                              bool want_runs, bool concurrent) {
     HeuristicResult res;
     const int64_t n = g->n;
-    cudaStream_t s = g->stream;
+    cudaStream_t s = concurrent ? g->hstream : g->stream;
+    PinnedBuf &host = concurrent ? g->hhost : g->host;
     if (n == 0 || kind == 0) return res;
     bool use_core = (kind == 2 || kind == 4);
     bool single = (kind == 1 || kind == 2);
     if (single) h = 1;
     if (h <= 0 || h > n) h = n;
-    if (use_core) kcore(g);
+    if (use_core) {
+        if (concurrent) fail(MCE_ERR_INVALID, "internal: core-number heuristics cannot overlap preprocessing");
+        kcore(g);
+    }
     cudaEvent_t e0, e1;
     MCE_CUDA(cudaEventCreate(&e0));
     MCE_CUDA(cudaEventCreate(&e1));
     MCE_CUDA(cudaEventRecord(e0, s));
     int64_t kernels = 0;
 
-    Pool &pool = g->pool;
+    Pool &pool = concurrent ? g->hpool : g->pool;
     pool.reset();
     const int32_t *thr;
     if (use_core) {
@@ -589,7 +594,7 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
         MCE_CUDA(cudaMemsetAsync(bins, 0, sizeof(int64_t) * (maxthr + 1), s));
         thr_hist_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, thr, bins);
         MCE_LAUNCH_CHECK();
-        int64_t *hb = g->host.get<int64_t>(maxthr + 1);
+        int64_t *hb = host.get<int64_t>(maxthr + 1);
         MCE_CUDA(cudaMemcpyAsync(hb, bins, sizeof(int64_t) * (maxthr + 1), cudaMemcpyDeviceToHost, s));
         stream_sync(s);
         int64_t above = 0;
@@ -636,7 +641,7 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
     MCE_CUDA(cudaMemsetAsync(run_size, 0, sizeof(int32_t) * n, s));
     MCE_CUDA(cudaMemsetAsync(best, 0, sizeof(int32_t), s));
     MCE_CUDA(cudaMemsetAsync(best_key, 0, sizeof(unsigned long long), s));
-    const int32_t *core = g->have_core ? g->core.get() : nullptr;
+    const int32_t *core = (!concurrent && g->have_core) ? g->core.get() : nullptr;
     const int abort_runs = want_runs ? 0 : 1;
     Hub H;
     int64_t nbig = 0;
@@ -650,7 +655,7 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
         exclusive_scan_i32(flag, pos, nseeds, tmp, s);
         gather_flagged_kernel<<<grid_for(nseeds, 256), 256, 0, s>>>(nseeds, seed_ptr, flag, pos, big);
         MCE_LAUNCH_CHECK();
-        int64_t *hnb = g->host.get<int64_t>(1);
+        int64_t *hnb = host.get<int64_t>(1);
         MCE_CUDA(cudaMemcpyAsync(hnb, pos + nseeds, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
         stream_sync(s);
         nbig = hnb[0];
@@ -662,7 +667,7 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
         MCE_CUDA(cudaMemsetAsync(bins, 0, sizeof(unsigned long long) * kBuckets, s));
         deg_bucket_hist<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(), bins);
         MCE_LAUNCH_CHECK();
-        unsigned long long *hb = g->host.get<unsigned long long>(kBuckets);
+        unsigned long long *hb = host.get<unsigned long long>(kBuckets);
         MCE_CUDA(cudaMemcpyAsync(hb, bins, sizeof(unsigned long long) * kBuckets, cudaMemcpyDeviceToHost, s));
         stream_sync(s);
         int bstar = kBuckets;
@@ -730,7 +735,7 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
         kernels += 3;
     }
     MCE_CUDA(cudaEventRecord(e1, s));
-    int32_t *hbest = g->host.get<int32_t>(1);
+    int32_t *hbest = host.get<int32_t>(1);
     MCE_CUDA(cudaMemcpyAsync(hbest, best, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
     stream_sync(s);
     res.omega_bar = hbest[0];
@@ -742,11 +747,14 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
     cudaEventDestroy(e1);
     if (res.omega_bar > 0) {
         res.clique.resize(res.omega_bar);
-        MCE_CUDA(cudaMemcpy(res.clique.data(), clique, sizeof(int32_t) * res.omega_bar, cudaMemcpyDeviceToHost));
+        MCE_CUDA(cudaMemcpyAsync(res.clique.data(), clique, sizeof(int32_t) * res.omega_bar, cudaMemcpyDeviceToHost,
+                                 s));
+        stream_sync(s);
     }
     if (want_runs) {
         res.run_size.resize(n);
-        MCE_CUDA(cudaMemcpy(res.run_size.data(), run_size, sizeof(int32_t) * n, cudaMemcpyDeviceToHost));
+        MCE_CUDA(cudaMemcpyAsync(res.run_size.data(), run_size, sizeof(int32_t) * n, cudaMemcpyDeviceToHost, s));
+        stream_sync(s);
     }
     return res;
 }

@@ -12,6 +12,8 @@ struct HeuristicResult {
     int64_t kernels = 0;
 };
 // kind: MCE_HEUR_*; h <= 0 means |V|; runs sharded cyclically when shard_count > 1
+// concurrent: run on g->hstream / g->hpool / g->hhost without core numbers
+// (overlapped with preprocessing by the engine; degree kinds only)
 HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_rank, int32_t shard_count,
-                              bool want_runs);
+                              bool want_runs, bool concurrent = false);
 }  // namespace mce

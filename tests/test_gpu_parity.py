@@ -342,3 +342,16 @@ def test_fused_expand_overflow(key):
     for budget in (2 << 20, 6 << 20, 32 << 20):
         r = run_enum(g, budget_bytes=budget, heuristic="none", fused_levels=False)
         assert r.omega == om and np.array_equal(r.cliques, cl)
+
+
+@pytest.mark.parametrize("key", ["er2000", "planted", "RMAT15", "BA5k", "ER400d"])
+def test_overlap_off_matches(key):
+    """Heuristic after preprocessing (no second stream / thread) gives the same answer."""
+    g = GRAPHS[key]()
+    om, cl = oracle_answer(key)
+    for heuristic in ("multi_degree", "single_degree"):
+        r = run_enum(g, overlap=False, heuristic=heuristic)
+        assert (r.omega, r.count) == (om, len(cl)) and np.array_equal(r.cliques, cl)
+        m = mce()
+        f = m.Graph(g.rowptr, g.col).find_one(window=8)
+        assert f.omega == om and oracle.is_clique(*g.numpy(), f.cliques[0])
