@@ -45,6 +45,9 @@ def parse():
                         "(~10^8 maximum cliques of size ~223 there), unbounded otherwise")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--shard-depth", type=int, default=-1,
+                   help="N > 1: <= 1 deals roots, d >= 2 replicates levels < d and deals the level-d candidates "
+                        "by hash (mce_options.shard_depth); -1: 3 for rmat26 (work under a few hub roots), else 0")
     return p.parse_args()
 
 
@@ -219,6 +222,7 @@ def main():
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     mode = args.mode or ("find_one" if args.config == "dense800" else "enumerate")
+    shard_depth = args.shard_depth if args.shard_depth >= 0 else (3 if args.config == "rmat26" else 0)
     max_cl = args.max_cliques if args.max_cliques >= 0 else (1 << 16 if args.config.startswith("rmat") else 0)
 
     g = build_graph(args.config, f"cuda:{local}")
@@ -231,7 +235,7 @@ def main():
         gr.clear_cache()
         if world > 1:
             if mode == "enumerate":
-                return mdist.enumerate_distributed(gr, max_cliques=max_cl)
+                return mdist.enumerate_distributed(gr, max_cliques=max_cl, shard_depth=shard_depth)
             return mdist.find_one_distributed(gr, window=args.window)
         if mode == "enumerate":
             return gr.enumerate(max_cliques=max_cl)
@@ -302,7 +306,7 @@ def main():
             torch.cuda.synchronize()
             t0 = time.perf_counter()
             gh = mce.Graph(rp_h, col_h, device=local)
-            r2 = mdist.enumerate_distributed(gh, max_cliques=max_cl) if (world > 1 and mode == "enumerate") else (
+            r2 = mdist.enumerate_distributed(gh, max_cliques=max_cl, shard_depth=shard_depth) if (world > 1 and mode == "enumerate") else (
                 mdist.find_one_distributed(gh, window=args.window) if world > 1 else
                 (gh.enumerate(max_cliques=max_cl) if mode == "enumerate" else gh.find_one(window=args.window)))
             dt = time.perf_counter() - t0
@@ -339,7 +343,8 @@ def main():
             "config": {"workload": args.config, "baseline_config_index": CONFIG_INDEX[args.config],
                        "mode": mode, "n": g.n, "edges": edges, "omega": res.omega, "multiplicity": res.count,
                        "stored_cliques": int(res.cliques.shape[0]), "max_cliques": max_cl,
-                       "parallelism": f"root-shard x{world}", "l2": "flushed (256 MiB write) before every step",
+                       "parallelism": (f"root-shard x{world}" if shard_depth < 2 else
+                                       f"level-{shard_depth} candidate shard x{world}"), "l2": "flushed (256 MiB write) before every step",
                        "phases_ms": phases, "levels": res.levels,
                        "step_ms": [round(t, 4) for t in times]},
             "roofline": {"bound": "hbm", "kernel": kname,

@@ -101,6 +101,11 @@ typedef struct {
     int32_t no_fused_expand; /* 0 (default): a level's count pass also writes the children (slots
                                 reserved per warp, colouring computed once) whenever they fit half
                                 of the free budget; 1: count -> scan -> write passes (A/B tests) */
+    int32_t shard_depth;     /* with shard_count > 1: <= 1 (default): roots are dealt to shards by CSR
+                                id; d >= 2: every shard expands all roots through level d - 1 and
+                                keeps the level-d candidates (d-cliques) whose vertex-path hash
+                                % shard_count == shard_rank (balances work that sits under a few
+                                hub roots); cliques found above level d are reported by shard 0 */
     int32_t no_overlap;      /* 0 (default): the degree heuristics run on a second stream and host
                                 thread while the k-core / orientation preprocessing runs (they
                                 share no data); 1: one after the other */

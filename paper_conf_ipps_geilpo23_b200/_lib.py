@@ -47,6 +47,7 @@ class Options(ctypes.Structure):
         ("no_fused_levels", ctypes.c_int32),
         ("no_clique_shortcut", ctypes.c_int32),
         ("no_fused_expand", ctypes.c_int32),
+        ("shard_depth", ctypes.c_int32),
         ("no_overlap", ctypes.c_int32),
     ]
 

@@ -120,6 +120,7 @@ void mce_default_options(mce_options *o) {
     o->no_clique_shortcut = 0;
     o->no_fused_expand = 0;
     o->no_overlap = 0;
+    o->shard_depth = 0;
 }
 
 mce_status mce_load_csr(int32_t device, int64_t n, const int64_t *row_ptr, const int32_t *col_idx, int32_t where,

@@ -196,6 +196,8 @@ class Engine {
     int32_t best_ = 0;
     int32_t W_ = 1;   // words per adjacency row of the current root window
     int64_t stride_ = 1, offset_ = 0;
+    bool entry_shard_ = false;  // shard_depth >= 2: levels < depth replicated, level-depth entries dealt by hash
+    bool split_ = false;        // inside a subtree whose level-depth entries were dealt
 
     // leaves
     unsigned long long *leaf_total_ = nullptr;  // g->misc[0]
@@ -262,6 +264,10 @@ void Engine::leaf_args(ExpandArgs &a) const {
 // C + {v} (a.leaf_rows), kind 1 = clique completions C + P (a.clq_rows).
 void Engine::handle_leaves(int32_t size, int64_t cnt, ExpandArgs &a, int kind) {
     if (cnt <= 0) return;
+    if (entry_shard_ && !split_ && offset_ != 0) {  // found above the split depth by every shard: shard 0 reports
+        if (size > best_) best_ = size;
+        return;
+    }
     DevBuf<int32_t> &stage = kind ? g_->cstage : g_->stage;
     if (find_one_) {
         // all cliques of this launch have size > best: keep the first
@@ -393,7 +399,41 @@ bool Engine::run_small(int32_t k, const Level &L) {
 }
 
 void Engine::process(int32_t k, const Level &L) {
-    if (!o_.no_fused_levels && L.count <= kSmallMax && L.W <= 4 && run_small(k, L)) return;
+    if (entry_shard_ && !split_ && k >= o_.shard_depth) {  // deal this level's entries by path hash
+        if (k + 2 > chain_cap_) fail(MCE_ERR_INVALID, "clique depth above the supported maximum");
+        LevelLink link{L.parent, L.vloc};
+        MCE_CUDA(cudaMemcpyAsync(chain_dev_ + k, &link, sizeof(link), cudaMemcpyHostToDevice, s_));
+        const Arena::Mark mark = arena_.mark();
+        const int64_t N = L.count;
+        const int32_t Ps = L.Ps > 0 ? L.Ps : L.W;
+        int32_t *flag = arena_.alloc<int32_t>(N);
+        int64_t *pos = arena_.alloc<int64_t>(N + 1);
+        int64_t *tmp = arena_.alloc<int64_t>(scan_tmp_items(N));
+        launch_shard_flags(roots_, L.slot, chain_dev_, N, k, (int32_t)offset_, (int32_t)stride_, flag, s_);
+        exclusive_scan_i32(flag, pos, N, tmp, s_);
+        int64_t *h = g_->host.get<int64_t>(1);
+        MCE_CUDA(cudaMemcpyAsync(h, pos + N, sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
+        stream_sync(s_);
+        kernels_ += 4;
+        const int64_t mine = h[0];
+        Level F;
+        F.count = mine;
+        F.W = L.W;
+        F.P = arena_.alloc<uint64_t>(mine * L.W);
+        F.slot = arena_.alloc<int32_t>(mine);
+        F.parent = arena_.alloc<int32_t>(mine);
+        F.vloc = arena_.alloc<int32_t>(mine);
+        launch_gather_level(N, flag, pos, L.W, Ps, L.P, L.slot, L.parent, L.vloc, F.P, F.slot, F.parent, F.vloc,
+                            s_);
+        ++kernels_;
+        split_ = true;
+        if (mine > 0) process(k, F);
+        split_ = false;
+        arena_.reset(mark);
+        return;
+    }
+    const bool pre_split = entry_shard_ && !split_;  // fused tiny levels would run past the split depth
+    if (!pre_split && !o_.no_fused_levels && L.count <= kSmallMax && L.W <= 4 && run_small(k, L)) return;
     if ((int64_t)level_entries_.size() <= k) level_entries_.resize(k + 1, 0);
     level_entries_[k] += L.count;
     if (k + 2 > chain_cap_) fail(MCE_ERR_INVALID, "clique depth above the supported maximum");
@@ -762,6 +802,7 @@ mce_result *Engine::run() {
     const int64_t n = g_->n;
     stride_ = o_.shard_count > 1 ? o_.shard_count : 1;
     offset_ = o_.shard_count > 1 ? o_.shard_rank : 0;
+    entry_shard_ = stride_ > 1 && o_.shard_depth >= 2;
     if (n == 0) {  // the empty clique is the only clique of the null graph
         res->omega = 0;
         res->count = 1;
@@ -895,8 +936,8 @@ mce_result *Engine::run() {
         MCE_CUDA(cudaMemsetAsync(hist, 0, sizeof(int64_t) * (kMaxClass + 1), s_));
         // roots are dealt to shards by CSR id (r % shard_count): independent of the
         // lower bound, so ranks whose bounds differ still partition the roots exactly
-        launch_classify_roots(n, g_->orp.get(), std::max<int32_t>(need() - 1, 1), (int32_t)offset_,
-                              (int32_t)stride_, cls, hist, s_);
+        launch_classify_roots(n, g_->orp.get(), std::max<int32_t>(need() - 1, 1), entry_shard_ ? 0 : (int32_t)offset_,
+                              entry_shard_ ? 1 : (int32_t)stride_, cls, hist, s_);
         ++kernels_;
         int64_t *hh = g_->host.get<int64_t>(kMaxClass + 1);
         MCE_CUDA(cudaMemcpyAsync(hh, hist, sizeof(int64_t) * (kMaxClass + 1), cudaMemcpyDeviceToHost, s_));

@@ -818,6 +818,41 @@ __global__ void expand_tile(const ExpandArgs a, int max_l) {
     if (!WRITE) flush_counters(a, nleaf, nclq, hb, ub);
 }
 
+__device__ __forceinline__ uint64_t mix64(uint64_t z) {
+    z += 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
+__global__ void shard_flags_kernel(const RootInfo *__restrict__ roots, const int32_t *__restrict__ slot,
+                                   const LevelLink *__restrict__ chain, int64_t n, int32_t k, int32_t rank,
+                                   int32_t count, int32_t *flag) {
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x) {
+        uint64_t h = mix64((uint64_t)(uint32_t)roots[slot[e]].r);
+        int64_t cur = e;
+        for (int32_t lev = k; lev >= 2; --lev) {
+            h = mix64(h ^ (uint64_t)(uint32_t)chain[lev].vloc[cur]);
+            cur = chain[lev].parent[cur];
+        }
+        flag[e] = (int32_t)(h % (uint64_t)count) == rank;
+    }
+}
+
+__global__ void gather_level_kernel(int64_t n, const int32_t *__restrict__ flag, const int64_t *__restrict__ pos,
+                                    int W, int Ps, const uint64_t *__restrict__ P, const int32_t *__restrict__ slot,
+                                    const int32_t *__restrict__ parent, const int32_t *__restrict__ vloc,
+                                    uint64_t *oP, int32_t *oslot, int32_t *oparent, int32_t *ovloc) {
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x) {
+        if (!flag[e]) continue;
+        const int64_t o = pos[e];
+        for (int w = 0; w < W; ++w) oP[o * W + w] = P[e * Ps + w];
+        oslot[o] = slot[e];
+        oparent[o] = parent[e];
+        ovloc[o] = vloc[e];
+    }
+}
+
 __global__ void classify_roots_kernel(int64_t n, const int64_t *__restrict__ orp, int32_t min_len,
                                       int32_t shard_rank, int32_t shard_count, int32_t *cls,
                                       unsigned long long *hist) {
@@ -1006,6 +1041,20 @@ void launch_expand_small(const ExpandArgs &a, uint8_t *scratch, int64_t scratch_
     MCE_LAUNCH_CHECK();
 }
 
+void launch_shard_flags(const RootInfo *roots, const int32_t *slot, const LevelLink *chain, int64_t n, int32_t k,
+                        int32_t rank, int32_t count, int32_t *flag, cudaStream_t s) {
+    if (n <= 0) return;
+    shard_flags_kernel<<<grid_for(n, 256), 256, 0, s>>>(roots, slot, chain, n, k, rank, count, flag);
+    MCE_LAUNCH_CHECK();
+}
+void launch_gather_level(int64_t n, const int32_t *flag, const int64_t *pos, int W, int Ps, const uint64_t *P,
+                         const int32_t *slot, const int32_t *parent, const int32_t *vloc, uint64_t *oP,
+                         int32_t *oslot, int32_t *oparent, int32_t *ovloc, cudaStream_t s) {
+    if (n <= 0) return;
+    gather_level_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, flag, pos, W, Ps, P, slot, parent, vloc, oP, oslot,
+                                                          oparent, ovloc);
+    MCE_LAUNCH_CHECK();
+}
 void launch_classify_roots(int64_t n, const int64_t *orp, int32_t min_len, int32_t shard_rank, int32_t shard_count,
                            int32_t *cls, int64_t *hist, cudaStream_t s) {
     classify_roots_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, orp, min_len, shard_rank, shard_count, cls,

@@ -147,6 +147,15 @@ void launch_make_roots(const int32_t *list, int64_t count, int64_t stride, int W
                        const int64_t *row_prefix, RootInfo *roots, cudaStream_t s);
 void launch_root_lengths(const int32_t *list, int64_t count, int64_t stride, const int64_t *orp, int32_t *len,
                          cudaStream_t s);
+// depth-d entry sharding (mce_options.shard_depth): flag[e] = 1 when the hash
+// of entry e's vertex path (root CSR id, then the local vertices of levels
+// 2..k) modulo `count` is `rank`; chain[2..k] must be set
+void launch_shard_flags(const RootInfo *roots, const int32_t *slot, const LevelLink *chain, int64_t n, int32_t k,
+                        int32_t rank, int32_t count, int32_t *flag, cudaStream_t s);
+// out = the flagged entries of a level (P re-strided from Ps to W words)
+void launch_gather_level(int64_t n, const int32_t *flag, const int64_t *pos, int W, int Ps, const uint64_t *P,
+                         const int32_t *slot, const int32_t *parent, const int32_t *vloc, uint64_t *oP,
+                         int32_t *oslot, int32_t *oparent, int32_t *ovloc, cudaStream_t s);
 void launch_find_chunk_end(const int64_t *offsets, int64_t a, int64_t n, int64_t cap, int64_t *out,
                            cudaStream_t s);
 

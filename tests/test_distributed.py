@@ -125,11 +125,14 @@ def test_cyclic_deal_partitions_every_root():
 # --- the library's sharding, on one GPU ------------------------------------
 
 @pytest.mark.gpu
+@pytest.mark.parametrize("depth", [0, 2, 3, 5])
 @pytest.mark.parametrize("shards", [2, 3])
-@pytest.mark.parametrize("key", ["planted", "RMAT11", "T(30,6)", "ER400d"])
-def test_shards_union_is_the_full_answer(key, shards):
-    """Each shard enumerates its cyclic share of the roots (and heuristic seeds);
-    merged like gather_result, the shards give the oracle's answer."""
+@pytest.mark.parametrize("key", ["planted", "RMAT11", "T(30,6)", "ER400d", "er2000"])
+def test_shards_union_is_the_full_answer(key, shards, depth):
+    """Each shard enumerates its cyclic share of the roots (depth 0) or, with
+    shard_depth d >= 2, every root down to level d - 1 and its hash share of
+    the level-d candidates (heuristic seeds dealt either way); merged like
+    gather_result, the shards give the oracle's answer."""
     import oracle
     from tests.test_gpu_parity import GRAPHS
 
@@ -138,7 +141,7 @@ def test_shards_union_is_the_full_answer(key, shards):
     g = GRAPHS[key]()
     om, cl = oracle.max_cliques(*g.numpy())
     gg = m.Graph(g.rowptr, g.col)
-    parts = [gg.enumerate(shard_rank=r, shard_count=shards) for r in range(shards)]
+    parts = [gg.enumerate(shard_rank=r, shard_count=shards, shard_depth=depth) for r in range(shards)]
     gg.close()
     omega = max(p.omega for p in parts)
     count = sum(p.count for p in parts if p.omega == omega)
