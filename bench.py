@@ -39,7 +39,9 @@ def parse():
     p.add_argument("--config", default="ba1m", choices=list(CONFIG_INDEX))
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
     p.add_argument("--mode", default=None, choices=[None, "enumerate", "find_one"])
-    p.add_argument("--window", type=int, default=0)
+    p.add_argument("--window", type=int, default=-1,
+                   help="find-one roots per window (PAPER.md IV-E); -1: 64 for dense800 (the best of the "
+                        "window sweep, profiles/r01_window_sweep_dense800_*.json), else 0 = all roots")
     p.add_argument("--max-cliques", type=int, default=-1,
                    help="stored-clique capacity (multiplicity stays exact); -1: 2^16 for the R-MAT configs "
                         "(~10^8 maximum cliques of size ~223 there), unbounded otherwise")
@@ -223,6 +225,8 @@ def main():
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     mode = args.mode or ("find_one" if args.config == "dense800" else "enumerate")
     shard_depth = args.shard_depth if args.shard_depth >= 0 else (3 if args.config == "rmat26" else 0)
+    if args.window < 0:
+        args.window = 64 if args.config == "dense800" else 0
     max_cl = args.max_cliques if args.max_cliques >= 0 else (1 << 16 if args.config.startswith("rmat") else 0)
 
     g = build_graph(args.config, f"cuda:{local}")
@@ -341,7 +345,7 @@ def main():
             "dtype": "int32",
             "data": "synthetic",
             "config": {"workload": args.config, "baseline_config_index": CONFIG_INDEX[args.config],
-                       "mode": mode, "n": g.n, "edges": edges, "omega": res.omega, "multiplicity": res.count,
+                       "mode": mode, "window": args.window if mode == "find_one" else None, "n": g.n, "edges": edges, "omega": res.omega, "multiplicity": res.count,
                        "stored_cliques": int(res.cliques.shape[0]), "max_cliques": max_cl,
                        "parallelism": (f"root-shard x{world}" if shard_depth < 2 else
                                        f"level-{shard_depth} candidate shard x{world}"), "l2": "flushed (256 MiB write) before every step",

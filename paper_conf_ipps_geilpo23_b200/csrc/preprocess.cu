@@ -330,50 +330,35 @@ struct Tile {
     __device__ unsigned lt() const { return (1u << gl) - 1u; }
 };
 
-// out-degree of vertex v's rank (tile of G lanes over v's neighbours)
+// count + stage: the up-neighbours of v (as CSR ids) are written compacted at
+// the start of v's own undirected row in `stage` (rowptr-indexed), their
+// number at odeg[pid[v]]; orient_copy moves them to the oriented CSR once the
+// out-degrees are scanned (one gather pass over rank/pid instead of two)
 template <int G>
-__device__ void out_degree_one(int64_t v, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
-                               const int32_t *__restrict__ rank, const int32_t *__restrict__ pid, int32_t *odeg) {
+__device__ void stage_one(int64_t v, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
+                          const int32_t *__restrict__ rank, const int32_t *__restrict__ pid, int32_t *odeg,
+                          int32_t *stage) {
     Tile<G> t;
     const int32_t r = rank[v];
-    int32_t cnt = 0;
     const int64_t eb = rowptr[v], ee = rowptr[v + 1];
-    for (int64_t e0 = eb; e0 < ee; e0 += G) {
-        const int64_t e = e0 + t.gl;
-        cnt += __popc(t.ballot(e < ee && rank[col[e]] > r));
-    }
-    if (t.gl == 0) odeg[pid[v]] = cnt;
-}
-
-// oriented row of v (in CSR order of the source; sorted afterwards)
-template <int G>
-__device__ void orient_fill_one(int64_t v, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
-                                const int32_t *__restrict__ rank, const int32_t *__restrict__ pid,
-                                const int64_t *__restrict__ orp, int32_t *ocol) {
-    Tile<G> t;
-    const int32_t r = rank[v];
-    int64_t out = orp[pid[v]];
-    const int64_t eb = rowptr[v], ee = rowptr[v + 1];
+    int64_t out = eb;
     for (int64_t e0 = eb; e0 < ee; e0 += G) {
         const int64_t e = e0 + t.gl;
         const int32_t u = e < ee ? col[e] : 0;
-        const int32_t ru = e < ee ? rank[u] : -1;
-        const bool up = ru > r;
+        const bool up = e < ee && rank[u] > r;
         const unsigned m = t.ballot(up);
-        if (up) ocol[out + __popc(m & t.lt())] = pid[u];
+        if (up) stage[out + __popc(m & t.lt())] = pid[u];
         out += __popc(m);
     }
+    if (t.gl == 0) odeg[pid[v]] = (int32_t)(out - eb);
 }
 
-// Warp w takes vertices [4w, 4w+4): 8-lane tiles when all four have degree
-// <= 64 (a warp per vertex would leave most lanes idle), otherwise one vertex
-// after another on the whole warp.  (A lane per vertex was measured 4x
-// slower: its loads touch 32 separate rows, where a tile reads a row coalesced.)
-template <bool FILL>
-__global__ void __launch_bounds__(256) orient_kernel(int64_t n, const int64_t *__restrict__ rowptr,
-                                                     const int32_t *__restrict__ col, const int32_t *__restrict__ rank,
-                                                     const int32_t *__restrict__ pid, int32_t *odeg,
-                                                     const int64_t *__restrict__ orp, int32_t *ocol) {
+// Warp w takes vertices [4w, 4w+4): 8-lane tiles when all four have degree <= 64, else a warp each
+__global__ void __launch_bounds__(256) orient_stage_kernel(int64_t n, const int64_t *__restrict__ rowptr,
+                                                           const int32_t *__restrict__ col,
+                                                           const int32_t *__restrict__ rank,
+                                                           const int32_t *__restrict__ pid, int32_t *odeg,
+                                                           int32_t *stage) {
     const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     const int lane = threadIdx.x & 31;
@@ -381,18 +366,38 @@ __global__ void __launch_bounds__(256) orient_kernel(int64_t n, const int64_t *_
         const int64_t v = v0 + (lane >> 3);
         const int64_t d = v < n ? rowptr[v + 1] - rowptr[v] : 0;
         if (__all_sync(0xffffffffu, d <= 64)) {
-            if (v < n) {
-                if (FILL)
-                    orient_fill_one<8>(v, rowptr, col, rank, pid, orp, ocol);
-                else
-                    out_degree_one<8>(v, rowptr, col, rank, pid, odeg);
-            }
+            if (v < n) stage_one<8>(v, rowptr, col, rank, pid, odeg, stage);
         } else {
-            for (int t = 0; t < 4 && v0 + t < n; ++t) {
-                if (FILL)
-                    orient_fill_one<32>(v0 + t, rowptr, col, rank, pid, orp, ocol);
-                else
-                    out_degree_one<32>(v0 + t, rowptr, col, rank, pid, odeg);
+            for (int t = 0; t < 4 && v0 + t < n; ++t) stage_one<32>(v0 + t, rowptr, col, rank, pid, odeg, stage);
+        }
+        __syncwarp();
+    }
+}
+
+// oriented row of CSR id i = the staged prefix of vertex vid[i]'s row (8-lane
+// tile per row, 4 rows per warp; a warp per row when a row exceeds 64)
+__global__ void __launch_bounds__(256) orient_copy_kernel(int64_t n, const int64_t *__restrict__ rowptr,
+                                                          const int32_t *__restrict__ vid,
+                                                          const int64_t *__restrict__ orp,
+                                                          const int32_t *__restrict__ stage, int32_t *ocol) {
+    const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    for (int64_t i0 = warp * 4; i0 < n; i0 += nwarps * 4) {
+        const int64_t i = i0 + (lane >> 3);
+        int64_t ob = 0, len = 0, sb = 0;
+        if (i < n) {
+            ob = orp[i];
+            len = orp[i + 1] - ob;
+            sb = rowptr[vid[i]];
+        }
+        if (__all_sync(0xffffffffu, len <= 64)) {
+            for (int64_t j = lane & 7; j < len; j += 8) ocol[ob + j] = stage[sb + j];
+        } else {
+            for (int t = 0; t < 4; ++t) {
+                const int64_t bo = __shfl_sync(0xffffffffu, ob, 8 * t), bl = __shfl_sync(0xffffffffu, len, 8 * t);
+                const int64_t bs = __shfl_sync(0xffffffffu, sb, 8 * t);
+                for (int64_t j = lane; j < bl; j += 32) ocol[bo + j] = stage[bs + j];
             }
         }
         __syncwarp();
@@ -628,12 +633,13 @@ void orient(mce_graph *g, int orientation) {
         MCE_CUDA(cudaMemcpyAsync(g->pid.get(), g->rank.get(), sizeof(int32_t) * n, cudaMemcpyDeviceToDevice, s));
     }
     int32_t *odeg = g->pool.take<int32_t>(n);
-    orient_kernel<false><<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), g->rank.get(),
-                                                               g->pid.get(), odeg, nullptr, nullptr);
+    int32_t *stage = g->pool.take<int32_t>(std::max<int64_t>(g->nnz, 1));
+    orient_stage_kernel<<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), g->rank.get(),
+                                                              g->pid.get(), odeg, stage);
     MCE_LAUNCH_CHECK();
     exclusive_scan_i32(odeg, g->orp.get(), n, g->pool.take<int64_t>(scan_tmp_items(n)), s);
-    orient_kernel<true><<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), g->rank.get(),
-                                                              g->pid.get(), nullptr, g->orp.get(), g->ocol.get());
+    orient_copy_kernel<<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->vid.get(), g->orp.get(), stage,
+                                                             g->ocol.get());
     MCE_LAUNCH_CHECK();
     sort_rows_warp<<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->orp.get(), g->ocol.get());
     MCE_LAUNCH_CHECK();
