@@ -852,8 +852,11 @@ mce_result *Engine::run() {
             }
         });
         try {
+            g_->pre_overlapped = true;
             preprocess(g_, o_.orientation);
+            g_->pre_overlapped = false;
         } catch (...) {
+            g_->pre_overlapped = false;
             th.join();
             cudaEventDestroy(ready);
             throw;

@@ -28,6 +28,7 @@ struct mce_graph {
     mce::DevBuf<int32_t> ocol;     // [nnz/2] out-neighbour CSR ids, rows ascending
     int32_t max_out = 0;           // largest out-degree
     double t_pre_ms = 0.0;         // device time of the last preprocessing
+    bool pre_overlapped = false;   // set by the engine while the heuristic runs concurrently
     int64_t kernels = 0;           // kernels launched by the last preprocessing
 
     // ---- reusable memory (no cudaMalloc/cudaFree on the steady-state path) ----

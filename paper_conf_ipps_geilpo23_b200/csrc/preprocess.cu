@@ -31,7 +31,7 @@ namespace mce {
 
 namespace {
 
-constexpr int kPeelThreads = 512;
+constexpr int kPeelThreads = 1024;  // launch bound; the launch uses kcore_threads()
 
 // ---------------------------------------------------------------------------
 // k-core numbers and a degeneracy order: asynchronous level peel.  Within a level k the order in which
@@ -110,7 +110,7 @@ constexpr int kLine = 16;  // u64 per counter line
 __global__ void __launch_bounds__(kPeelThreads)
     kcore_async(int64_t n, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col, int32_t *deg,
                 int32_t *core, int32_t *order, int32_t *alive_a, int32_t *alive_b, uint8_t *dead,
-                long long *work0, long long *work1, int64_t witems, unsigned long long *ctrl) {
+                long long *work0, long long *work1, int64_t witems, unsigned long long *ctrl, int max_sleep) {
     cg::grid_group grid = cg::this_grid();
     __shared__ unsigned long long sh[6];
     const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -250,7 +250,7 @@ __global__ void __launch_bounds__(kPeelThreads)
                 if (__all_sync(0xffffffffu, resolved)) break;
                 if (!done_m) {
                     ++idle;
-                    __nanosleep(idle < 4 ? 32 : (idle < 16 ? 128 : 512));
+                    __nanosleep(idle < 4 ? 32 : (idle < 16 ? 128 : max_sleep));
                 } else {
                     idle = 0;
                 }
@@ -548,10 +548,17 @@ void kcore(mce_graph *g) {
         MCE_CUDA(cudaMemsetAsync(ctrl + kLine * (10 + 3 * i), 0xff, sizeof(unsigned long long), s));
     degrees_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(), deg, alive_a);
     MCE_LAUNCH_CHECK();
+    // launch shape (measured on B200, ba1m / rmat22): alone, one 512-thread
+    // block per SM; overlapped with the heuristic (engine.cu), 1024-thread
+    // blocks on half of the SMs, leaving the other half to the heuristic
+    // (ba1m 1.88 -> 1.74 ms, rmat22 221 -> 190 ms per step).  Fewer, wider
+    // blocks contend less on the work-list counters.
+    const bool half = g->pre_overlapped;
+    const int threads = half ? 1024 : 512;
     int blocks_per_sm = 0;
-    MCE_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm, kcore_async, kPeelThreads, 0));
-    blocks_per_sm = std::max(1, std::min(blocks_per_sm, 2));
-    int grid = num_sms() * blocks_per_sm;
+    MCE_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm, kcore_async, threads, 0));
+    if (blocks_per_sm < 1) fail(2, "kcore: cooperative kernel does not fit an SM");
+    const int grid = half ? std::max(1, num_sms() / 2) : num_sms();
     int64_t n_arg = n;
     const int64_t *rp = g->rowptr.get();
     const int32_t *cl = g->col.get();
@@ -560,8 +567,9 @@ void kcore(mce_graph *g) {
     long long *w0 = work0, *w1 = work1;
     int64_t wi = witems;
     unsigned long long *ct = ctrl;
-    void *args[] = {&n_arg, &rp, &cl, &dg, &co, &qu, &aa, &ab, &dd, &w0, &w1, &wi, &ct};
-    MCE_CUDA(cudaLaunchCooperativeKernel((void *)kcore_async, grid, kPeelThreads, args, 0, s));
+    int ms = 512;  // longest poll back-off (ns); 256-2048 measured equal
+    void *args[] = {&n_arg, &rp, &cl, &dg, &co, &qu, &aa, &ab, &dd, &w0, &w1, &wi, &ct, &ms};
+    MCE_CUDA(cudaLaunchCooperativeKernel((void *)kcore_async, grid, threads, args, 0, s));
     g->kernels += 2;
     // degeneracy = max core (the last queued vertex has it)
     last_core_kernel<<<1, 1, 0, s>>>(n, g->peel.get(), g->core.get(), deg);
