@@ -184,6 +184,11 @@ class Engine {
     void do_class_w1(const int32_t *list, int64_t count);
     void handle_leaves(int32_t size, int64_t cnt, ExpandArgs &a, int kind = 0);
     void leaf_args(ExpandArgs &a) const;
+    void materialize_pairs(ExpandArgs &a);
+    void reset_leaf_counters() {
+        MCE_CUDA(cudaMemsetAsync(leaf_total_, 0, 4 * sizeof(unsigned long long), s_));
+        MCE_CUDA(cudaMemsetAsync(pair_n_, 0, sizeof(unsigned long long), s_));
+    }
     void sync_bound(bool active);
     void launch_timed(const ExpandArgs &a, bool write);
 
@@ -206,6 +211,8 @@ class Engine {
     unsigned long long *clq_slot_ = nullptr;    // g->misc[3]
     int32_t *maxbit_ = nullptr;                 // g->misc[4]
     unsigned long long *out_count_ = nullptr;   // g->misc[5] fused-pass children
+    unsigned long long *pair_n_ = nullptr;      // g->misc[6] pair-completion descriptors
+    int64_t pair_cap_ = 0;
     int64_t stage_rows_ = 0;
     int64_t cstage_rows_ = 0;
     int64_t stage_max_rows_ = 0;  // staging never exceeds a quarter of the budget (stored list truncated, count exact)
@@ -258,6 +265,34 @@ void Engine::leaf_args(ExpandArgs &a) const {
     a.clq_slot = clq_slot_;
     a.clq_rows = g_->cstage.get();
     a.clq_cap = cstage_rows_;
+    a.pair_n = pair_n_;
+    a.pair_desc = g_->pdesc.get();
+    a.pair_cap = pair_cap_;
+}
+
+// Pair completions (reading 13): the count pass reserved their staging rows
+// and left descriptors; write the rows (growing the descriptor list and
+// replaying the count pass once if it overflowed)
+void Engine::materialize_pairs(ExpandArgs &a) {
+    for (int attempt = 0; attempt < 2; ++attempt) {
+        unsigned long long *hp = g_->host.get<unsigned long long>(1);
+        MCE_CUDA(cudaMemcpyAsync(hp, pair_n_, sizeof(unsigned long long), cudaMemcpyDeviceToHost, s_));
+        stream_sync(s_);
+        const int64_t np = (int64_t)hp[0];
+        if (np > a.pair_cap && attempt == 0) {
+            pair_cap_ = np;
+            g_->pdesc.ensure((size_t)pair_cap_ * 3);
+            a.pair_desc = g_->pdesc.get();
+            a.pair_cap = pair_cap_;
+            reset_leaf_counters();
+            launch_expand(a, false, s_);
+            ++kernels_;
+            continue;
+        }
+        launch_materialize_pairs(a, std::min<int64_t>(np, a.pair_cap), s_);
+        ++kernels_;
+        return;
+    }
 }
 
 // Record `cnt` cliques of `size` staged by a count pass: kind 0 = leaves
@@ -269,13 +304,15 @@ void Engine::handle_leaves(int32_t size, int64_t cnt, ExpandArgs &a, int kind) {
         return;
     }
     DevBuf<int32_t> &stage = kind ? g_->cstage : g_->stage;
+    if (kind == 1) materialize_pairs(a);
     if (find_one_) {
         // all cliques of this launch have size > best: keep the first
         best_ = size;
         res_size_ = size;
         res_count_ = 1;
         rows_.resize(size);
-        MCE_CUDA(cudaMemcpy(rows_.data(), stage.get(), sizeof(int32_t) * size, cudaMemcpyDeviceToHost));
+        MCE_CUDA(cudaMemcpyAsync(rows_.data(), stage.get(), sizeof(int32_t) * size, cudaMemcpyDeviceToHost, s_));
+        stream_sync(s_);
         return;
     }
     if (size > res_size_) {
@@ -295,9 +332,10 @@ void Engine::handle_leaves(int32_t size, int64_t cnt, ExpandArgs &a, int kind) {
         stage.ensure((size_t)want * std::max<int32_t>(g_->max_out + 2, 2));
         (kind ? a.clq_rows : a.leaf_rows) = stage.get();
         cap = want;
-        MCE_CUDA(cudaMemsetAsync(leaf_total_, 0, 4 * sizeof(unsigned long long), s_));
+        reset_leaf_counters();
         launch_expand(a, false, s_);
         ++kernels_;
+        if (kind == 1) materialize_pairs(a);
         stream_sync(s_);
     }
     const int64_t take = std::min<int64_t>(want, cap);
@@ -348,7 +386,7 @@ bool Engine::run_small(int32_t k, const Level &L) {
     a.maxbit = maxbit_;
     leaf_args(a);
     a.chain = chain_dev_;
-    MCE_CUDA(cudaMemsetAsync(leaf_total_, 0, 4 * sizeof(unsigned long long), s_));
+    reset_leaf_counters();
     const int t = clock_.start(1);
     launch_expand_small(a, scratch, scratch_bytes, dout, chain_dev_, s_);
     clock_.stop(t);
@@ -505,7 +543,7 @@ void Engine::process(int32_t k, const Level &L) {
     }
 
     // misc[0..4] = leaf total, leaf slot, completion total, completion slot, maxbit (-1); misc[5] = fused children
-    MCE_CUDA(cudaMemsetAsync(leaf_total_, 0, 4 * sizeof(unsigned long long), s_));
+    reset_leaf_counters();
     MCE_CUDA(cudaMemsetAsync(maxbit_, 0xff, 2 * sizeof(int32_t), s_));
     if (fused) MCE_CUDA(cudaMemsetAsync(out_count_, 0, sizeof(unsigned long long), s_));
     launch_timed(a, false);
@@ -914,6 +952,9 @@ mce_result *Engine::run() {
     clq_slot_ = leaf_total_ + 3;
     maxbit_ = reinterpret_cast<int32_t *>(leaf_total_ + 4);
     out_count_ = leaf_total_ + 5;
+    pair_n_ = leaf_total_ + 6;
+    pair_cap_ = std::max<int64_t>(4096, (int64_t)g_->pdesc.n / 3);
+    g_->pdesc.ensure((size_t)pair_cap_ * 3);
     chain_dev_ = reinterpret_cast<LevelLink *>(g_->misc.get() + 256);
     stage_max_rows_ = std::max<int64_t>(1ll << 20, budget / 4 / (4ll * std::max<int32_t>(g_->max_out + 2, 2)));
     // staging rows: whatever the buffers kept from earlier calls hold (a count

@@ -247,7 +247,8 @@ __device__ __forceinline__ int top_bit(const uint64_t (&C)[W]) {
 __device__ __forceinline__ void flush_counters(const ExpandArgs &a, unsigned long long nleaf, unsigned long long nclq,
                                                int hb, int ub) {
     nleaf = __reduce_add_sync(0xffffffffu, (unsigned)nleaf);
-    nclq = __reduce_add_sync(0xffffffffu, (unsigned)nclq);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) nclq += __shfl_xor_sync(0xffffffffu, nclq, o);
     hb = __reduce_max_sync(0xffffffffu, hb + 1) - 1;
     ub = __reduce_max_sync(0xffffffffu, ub);
     if ((threadIdx.x & 31) == 0) {
@@ -266,6 +267,82 @@ __device__ __forceinline__ void flush_counters(const ExpandArgs &a, unsigned lon
 // number of surviving children (count pass) after writing them at `out`
 // (write pass).  Leaves, highest child bit and reachable depth accumulate
 // into the caller's counters.
+// Pair completions (thread path, reading 13): P's complement is a
+// matching (every vertex of P misses at most one other), so the cliques of
+// size need below (C, P) are C + one vertex of each of the m non-adjacent
+// pairs + every other vertex of P: 2^m of them.  The count pass reserves
+// their staging rows and records a descriptor; materialize_pairs (a block
+// per descriptor) writes the rows: combination c takes the higher vertex of
+// pair j when bit j of c is set.
+__device__ void reserve_pair_completions(const ExpandArgs &a, int64_t e, int m) {
+    if (*(volatile unsigned long long *)a.clq_slot >= (unsigned long long)a.clq_cap) return;
+    const unsigned long long base = atomicAdd(a.clq_slot, 1ull << m);
+    if ((int64_t)base >= a.clq_cap) return;
+    const unsigned long long d = atomicAdd(a.pair_n, 1ull);
+    if ((int64_t)d >= a.pair_cap) return;  // the host sees the overflow and replays with more room
+    a.pair_desc[3 * d] = e;
+    a.pair_desc[3 * d + 1] = (int64_t)base;
+    a.pair_desc[3 * d + 2] = m;
+}
+
+constexpr int kMatThreads = 256;
+__global__ void __launch_bounds__(kMatThreads) materialize_pairs_kernel(const ExpandArgs a, int64_t n) {
+    __shared__ int32_t tmpl[4096];  // C + unpaired vertices (need - m <= 4096 checked by the host)
+    __shared__ int32_t plo[40], phi[40];
+    __shared__ int s_np2, s_len;
+    for (int64_t d = blockIdx.x; d < n; d += gridDim.x) {
+        const int64_t e = a.pair_desc[3 * d];
+        const int64_t base = a.pair_desc[3 * d + 1];
+        const int m = (int)a.pair_desc[3 * d + 2];
+        if (threadIdx.x == 0) {
+            const RootInfo ri = a.roots[a.slot[e]];
+            const int32_t *V = a.ocol + ri.vbase;
+            const uint64_t *A = a.adj + ri.abase;
+            int64_t cur = e;
+            for (int32_t lev = a.k; lev >= 2; --lev) {
+                tmpl[lev - 1] = a.order[V[ri.L - 1 - a.chain[lev].vloc[cur]]];
+                cur = a.chain[lev].parent[cur];
+            }
+            tmpl[0] = a.order[ri.r];
+            int pos = a.k, np2 = 0;
+            for (int w = 0; w < a.Wp; ++w) {
+                uint64_t q = a.P[e * a.Ps + w];
+                while (q) {
+                    const int b = __ffsll((long long)q) - 1;
+                    q &= q - 1;
+                    const int v = w * 64 + b;
+                    const uint64_t *row = A + (int64_t)v * a.Wa;
+                    int u = -1;
+                    for (int x = 0; x < a.Wp; ++x) {
+                        uint64_t nb = a.P[e * a.Ps + x] & ~row[x];
+                        if (x == w) nb &= ~(1ull << b);
+                        if (nb) u = x * 64 + __ffsll((long long)nb) - 1;
+                    }
+                    if (u < 0) {
+                        tmpl[pos++] = a.order[V[ri.L - 1 - v]];
+                    } else if (v < u && np2 < 40) {
+                        plo[np2] = a.order[V[ri.L - 1 - v]];
+                        phi[np2] = a.order[V[ri.L - 1 - u]];
+                        ++np2;
+                    }
+                }
+            }
+            s_np2 = np2;
+            s_len = pos;
+        }
+        __syncthreads();
+        const int np2 = s_np2, len = s_len;
+        const int64_t last = min((int64_t)(base + (1ll << m)), (int64_t)a.clq_cap);
+        for (int64_t r = base + threadIdx.x; r < last; r += blockDim.x) {
+            const unsigned long long c = (unsigned long long)(r - base);
+            int32_t *row = a.clq_rows + r * a.need;
+            for (int i = 0; i < len; ++i) row[i] = tmpl[i];
+            for (int j = 0; j < np2; ++j) row[len + j] = ((c >> j) & 1ull) ? phi[j] : plo[j];
+        }
+        __syncthreads();
+    }
+}
+
 // warp exclusive prefix sum of x over all 32 lanes (total in `total`)
 __device__ __forceinline__ unsigned long long warp_excl_u64(unsigned long long x, unsigned long long &total) {
     const int lane = threadIdx.x & 31;
@@ -289,7 +366,7 @@ __device__ __forceinline__ unsigned long long warp_excl_u64(unsigned long long x
 // would recompute).
 template <int W, bool WRITE>
 __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, int64_t out, unsigned &nleaf,
-                                                unsigned &nclq, int &hb, int &ub, bool active = true,
+                                                unsigned long long &nclq, int &hb, int &ub, bool active = true,
                                                 bool fused = false) {
     uint64_t P[W];
 #pragma unroll
@@ -355,6 +432,33 @@ __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, 
         done = true;
         if (!fused) return 0;
     }
+    // P's complement a matching with |C| + #colours == need: 2^m completions
+    // (the greedy colouring then makes every colour class a pair or a single
+    // vertex, so #colours = |P| - m)
+    if (!done && a.shortcut && a.bound == 1 && ncol < np && np - ncol <= 40 && a.k + ncol == a.need &&
+        a.need <= 4096) {
+        bool matching = true;
+        for (int i = 0; i < np && matching; ++i) {
+            const int v = ord[i];
+            const uint64_t *row = A + (int64_t)v * Wa;
+            int miss = 0;
+#pragma unroll
+            for (int x = 0; x < W; ++x) {
+                uint64_t nb = P[x] & ~__ldg(row + x);
+                if (x == (v >> 6)) nb &= ~(1ull << (v & 63));
+                miss += __popcll(nb);
+            }
+            matching = miss <= 1;
+        }
+        if (matching) {
+            if (!WRITE) {
+                nclq += 1ull << (np - ncol);
+                reserve_pair_completions(a, e, np - ncol);
+            }
+            done = true;
+            if (!fused) return 0;
+        }
+    }
     // the branching loop (Algorithm 2 lines 3-9 with the colouring order):
     // MODE 0 count (+ leaves), 1 write at `at` with word stride `ws`
     auto branch = [&](int mode, int64_t at, int ws) -> int32_t {
@@ -414,7 +518,8 @@ __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, 
 template <int W, bool WRITE>
 __global__ void __launch_bounds__(256) expand_thread(const ExpandArgs a) {
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    unsigned nleaf = 0, nclq = 0;
+    unsigned nleaf = 0;
+    unsigned long long nclq = 0;
     int hb = -1, ub = 0;
     if (!WRITE && a.fused) {  // warp-uniform loop: the whole warp reserves its children's slots at once
         for (int64_t e0 = a.begin + (int64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31); e0 < a.end;
@@ -447,7 +552,7 @@ constexpr int kSmallThreads = 1024;
 
 template <bool WRITE>
 __device__ __forceinline__ int32_t expand_entry_w(int W, const ExpandArgs &a, int64_t e, int64_t out,
-                                                  unsigned &nleaf, unsigned &nclq, int &hb, int &ub) {
+                                                  unsigned &nleaf, unsigned long long &nclq, int &hb, int &ub) {
     if (W == 1) return expand_entry<1, WRITE>(a, e, out, nleaf, nclq, hb, ub);
     if (W == 2) return expand_entry<2, WRITE>(a, e, out, nleaf, nclq, hb, ub);
     return expand_entry<4, WRITE>(a, e, out, nleaf, nclq, hb, ub);
@@ -459,7 +564,8 @@ __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a
     __shared__ ExpandArgs A;
     __shared__ int32_t offs[kSmallMax + 1];
     __shared__ int32_t wsum[kSmallThreads / 32];
-    __shared__ unsigned s_leaf, s_clq;
+    __shared__ unsigned s_leaf;
+    __shared__ unsigned long long s_clq;
     __shared__ int s_hb, s_ub;
     __shared__ int64_t s_used;
     const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
@@ -494,7 +600,8 @@ __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a
         }
         __syncthreads();
         // count pass, one candidate per thread
-        unsigned nleaf = 0, nclq = 0;
+        unsigned nleaf = 0;
+        unsigned long long nclq = 0;
         int hb = -1, ub = 0;
         int32_t cnt = 0;
         if (t < N) cnt = expand_entry_w<false>(W, A, A.begin + t, 0, nleaf, nclq, hb, ub);
@@ -610,7 +717,8 @@ __global__ void expand_tile(const ExpandArgs a, int max_l) {
     const int64_t tile = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / G;
     const int64_t ntiles = ((int64_t)gridDim.x * blockDim.x) / G;
     const int W = a.Wp, Wa = a.Wa;
-    unsigned nleaf = 0, nclq = 0;
+    unsigned nleaf = 0;
+    unsigned long long nclq = 0;
     int hb = -1, ub = 0;
     for (int64_t e = a.begin + tile; e < a.end; e += ntiles) {
         int64_t out = 0;
@@ -1033,6 +1141,12 @@ void launch_expand(const ExpandArgs &a, bool write_pass, cudaStream_t s) {
     } else {
         launch_tile<32, 8>(a, write_pass, s);
     }
+}
+
+void launch_materialize_pairs(const ExpandArgs &a, int64_t n, cudaStream_t s) {
+    if (n <= 0) return;
+    materialize_pairs_kernel<<<(int)std::min<int64_t>(n, (int64_t)num_sms() * 8), kMatThreads, 0, s>>>(a, n);
+    MCE_LAUNCH_CHECK();
 }
 
 void launch_expand_small(const ExpandArgs &a, uint8_t *scratch, int64_t scratch_bytes, SmallOut *out,

@@ -73,6 +73,11 @@ struct ExpandArgs {
     unsigned long long *clq_slot;
     int32_t *clq_rows;
     int64_t clq_cap;  // rows of `need` vertices
+    // pair completions (reading 13): the count pass reserves their rows and
+    // records (entry, first row, m) here; materialize_pairs writes the rows
+    unsigned long long *pair_n;  // descriptors recorded
+    int64_t *pair_desc;          // 3 x int64 each
+    int64_t pair_cap;
     // fused count + write (count pass only): children are appended at
     // cP/cslot/... + atomicAdd(out_count) with stride Wp while they fit out_cap;
     // counts[] is written as usual so an overflowing level falls back to scan + write
@@ -126,6 +131,9 @@ struct SmallOut {
     int64_t inN, inW, inPs;
     int64_t level_n[kSmallMaxLevels];  // entries of every processed level
 };
+// write the rows of the pair completions recorded by the last count pass over
+// the level described by `a` (its P / slot / chain); n = descriptors recorded
+void launch_materialize_pairs(const ExpandArgs &a, int64_t n, cudaStream_t s);
 void launch_expand_small(const ExpandArgs &a, uint8_t *scratch, int64_t scratch_bytes, SmallOut *out,
                          LevelLink *chain, cudaStream_t s);
 

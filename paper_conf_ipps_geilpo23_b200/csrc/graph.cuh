@@ -46,6 +46,7 @@ struct mce_graph {
     mce::DevBuf<uint8_t> misc;     // engine: leaf counter + level chain (persistent)
     mce::DevBuf<int32_t> stage;    // engine: staged leaf cliques of one launch (grow-only)
     mce::DevBuf<int32_t> cstage;   // engine: staged clique completions of one launch (grow-only)
+    mce::DevBuf<int64_t> pdesc;    // engine: pair-completion descriptors of one launch (grow-only)
     mce::DevBuf<int32_t> store;    // engine: stored maximum cliques of the run (grow-only)
 };
 
