@@ -149,7 +149,7 @@ class Graph:
             st = ctypes.c_int64()
             tr = ctypes.c_int32()
             check(L.mce_result_info(handle, ctypes.byref(om), ctypes.byref(cnt), ctypes.byref(st), ctypes.byref(tr)))
-            cl = np.zeros((st.value, max(om.value, 0)), np.int32)
+            cl = np.empty((st.value, max(om.value, 0)), np.int32)
             check(L.mce_result_cliques(handle, cl.ctypes.data_as(ctypes.c_void_p) if cl.size else None,
                                        _lib.WHERE_HOST))
             nl = ctypes.c_int32()

@@ -2,6 +2,9 @@
 // status codes, graph upload and result read-out; all compute is in the
 // kernels of preprocess.cu, heuristic.cu, expand.cu.
 #include <algorithm>
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <numeric>
 #include <string>
@@ -135,9 +138,17 @@ mce_status mce_load_csr(int32_t device, int64_t n, const int64_t *row_ptr, const
         MCE_CUDA(cudaGetDeviceCount(&ndev));
         if (device < 0 || device >= ndev) fail(MCE_ERR_INVALID, "bad device index");
         MCE_CUDA(cudaSetDevice(device));
-        cudaDeviceProp prop;
-        MCE_CUDA(cudaGetDeviceProperties(&prop, device));
-        if (prop.major < 10) fail(MCE_ERR_CUDA, "libmce_b200 needs an sm_100 (Blackwell) device");
+        int major = 0;  // (cudaGetDeviceProperties costs milliseconds: one attribute instead)
+        MCE_CUDA(cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, device));
+        if (major < 10) fail(MCE_ERR_CUDA, "libmce_b200 needs an sm_100 (Blackwell) device");
+        const bool trace = getenv("MCE_TRACE_LOAD") != nullptr;
+        using lclk = std::chrono::steady_clock;
+        const auto t0 = lclk::now();
+        auto lap = [&](const char *what) {
+            if (trace)
+                fprintf(stderr, "[mce] load %s %.3f ms\n", what,
+                        std::chrono::duration<double, std::milli>(lclk::now() - t0).count());
+        };
         auto g = new mce_graph();
         try {
             g->device = device;
@@ -152,11 +163,14 @@ mce_status mce_load_csr(int32_t device, int64_t n, const int64_t *row_ptr, const
             if (nnz < 0 || (nnz & 1)) fail(MCE_ERR_INVALID, "row_ptr[n] must be 2|E| (even, >= 0)");
             if (nnz > 0 && !col_idx) fail(MCE_ERR_INVALID, "col_idx is NULL");
             g->nnz = nnz;
+            lap("start");
             g->rowptr.alloc(n + 1);
             g->col.alloc(std::max<int64_t>(nnz, 1));
+            lap("alloc");
             MCE_CUDA(cudaMemcpyAsync(g->rowptr.get(), row_ptr, sizeof(int64_t) * (n + 1), kind, g->stream));
             if (nnz)
                 MCE_CUDA(cudaMemcpyAsync(g->col.get(), col_idx, sizeof(int32_t) * nnz, kind, g->stream));
+            lap("copies issued");
             if (n > 0) {
                 g->pool.reset();
                 unsigned long long *md = g->pool.take<unsigned long long>(1);
@@ -166,6 +180,7 @@ mce_status mce_load_csr(int32_t device, int64_t n, const int64_t *row_ptr, const
                 unsigned long long *h = g->host.get<unsigned long long>(1);
                 MCE_CUDA(cudaMemcpyAsync(h, md, sizeof(unsigned long long), cudaMemcpyDeviceToHost, g->stream));
                 stream_sync(g->stream);
+                lap("copied + max degree");
                 g->max_deg = (int64_t)h[0];
                 if (validate) {
                     int32_t *bad = g->pool.take<int32_t>(1);
