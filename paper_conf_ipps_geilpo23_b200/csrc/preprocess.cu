@@ -193,6 +193,7 @@ __global__ void __launch_bounds__(kPeelThreads)
         // unwritten slot may be waiting for an item that a sibling tile's item
         // appends.  The tiles' edge loops run in warp lock-step so appends and
         // done counts are aggregated over the whole warp (one atomic each).
+        unsigned long long pending = 0;  // lane 0: items processed, not yet added to `done`
         while (true) {
             unsigned long long base = 0;
             if (lane == 0) base = atomicAdd(head, 4ull);
@@ -209,7 +210,7 @@ __global__ void __launch_bounds__(kPeelThreads)
                         dead_slot = true;  // beyond the list: can never be filled
                     } else {
                         item = (long long)ld_relaxed((const unsigned long long *)(work + slot));
-                        if (item == -1 && idle >= 2) {
+                        if (item == -1 && idle >= 4) {
                             const unsigned long long dn = ld_relaxed(done);
                             const unsigned long long tl = ld_relaxed(tail);
                             dead_slot = dn == tl && slot >= tl;
@@ -238,10 +239,7 @@ __global__ void __launch_bounds__(kPeelThreads)
                     async_append<32>(fell, u, rowptr, core, order, dead, work, otail, tail, k);
                 }
                 const unsigned done_m = __ballot_sync(0xffffffffu, work_now && (lane & 7) == 0);
-                if (lane == 0 && done_m) {
-                    __threadfence();  // this warp's appends before its done count
-                    atomicAdd(done, (unsigned long long)__popc(done_m));
-                }
+                if (lane == 0) pending += (unsigned long long)__popc(done_m);
                 if (work_now) resolved = true;
                 if (!resolved && dead_slot) {
                     resolved = true;
@@ -249,6 +247,13 @@ __global__ void __launch_bounds__(kPeelThreads)
                 }
                 if (__all_sync(0xffffffffu, resolved)) break;
                 if (!done_m) {
+                    // about to wait: publish the processed count first (a warp with work
+                    // batches it; termination needs every warp idle, hence flushed)
+                    if (lane == 0 && pending) {
+                        __threadfence();  // this warp's appends before its done count
+                        atomicAdd(done, pending);
+                        pending = 0;
+                    }
                     ++idle;
                     __nanosleep(idle < 4 ? 32 : (idle < 16 ? 128 : max_sleep));
                 } else {
@@ -256,6 +261,10 @@ __global__ void __launch_bounds__(kPeelThreads)
                 }
             }
             if (__all_sync(0xffffffffu, over)) break;
+        }
+        if (lane == 0 && pending) {  // (cannot happen: `over` needs an idle, flushed warp)
+            __threadfence();
+            atomicAdd(done, pending);
         }
         grid.sync();
         // ---- clear this level's work list (the next level fills the other one)
