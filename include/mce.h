@@ -154,7 +154,11 @@ mce_status mce_heuristic(mce_graph *g, int32_t kind, int64_t h, int32_t *omega_b
                          int32_t *clique_len_out, int32_t *run_size_out);
 
 /* Enumerate every maximum clique (PAPER.md IV-D, Algorithm 2, breadth-first).
- * On success *out holds omega, the multiplicity and the cliques. */
+ * On success *out holds omega, the multiplicity and the cliques.  Work is
+ * ordered on `stream` (mce_load_csr); the overlapped heuristic uses a second,
+ * library-owned stream that waits on `stream` and is joined before return.
+ * Errors: MCE_ERR_BUDGET when one candidate's children exceed the frontier
+ * budget, MCE_ERR_CUDA / MCE_ERR_NOMEM from the runtime; *out is NULL then. */
 mce_status mce_enumerate(mce_graph *g, const mce_options *opt, mce_result **out);
 
 /* Find one maximum clique with the windowed search (PAPER.md IV-E): roots are
@@ -168,14 +172,18 @@ mce_status mce_find_one(mce_graph *g, int64_t window, const mce_options *opt, mc
 mce_status mce_result_info(const mce_result *r, int32_t *omega, int64_t *count, int64_t *stored,
                            int32_t *truncated);
 /* Copy the stored cliques, each sorted ascending, the list in lexicographic
- * order, as int32[stored * omega] into dst (host or device per `where`). */
+ * order, as int32[stored * omega] into dst (host or device per `where`).
+ * The canonical rows stay in device memory owned by the result until this
+ * call copies them (one device-to-host or device-to-device copy). */
 mce_status mce_result_cliques(mce_result *r, int32_t *dst, int32_t where);
 /* Per-level statistics of the last run: entries[k] = candidates (C, P) with
  * |C| = k+1 that were expanded, for k < levels (host int64 array of capacity
  * `cap`).  *levels_out = number of levels recorded. */
 mce_status mce_result_levels(const mce_result *r, int64_t *entries, int32_t cap, int32_t *levels_out);
 /* Kernel timing of the last run, milliseconds measured with CUDA events on
- * the run's stream: [0] preprocess, [1] heuristic, [2] expansion total,
+ * the run's stream: [0] preprocess, [1] heuristic ([0] and [1] overlap when
+ * the degree heuristic runs on the library's second stream, mce_options.no_overlap),
+ * [2] expansion total,
  * [3] dominant expansion kernel total, [4] number of dominant-kernel launches,
  * [5] algorithmic bytes moved by the dominant kernel, [6] kernels launched,
  * [7] fused root-level kernel total, [8] its launches, [9] its algorithmic
