@@ -8,6 +8,7 @@
 #include <cstring>
 #include <numeric>
 #include <string>
+#include <thread>
 #include <vector>
 
 #include "engine.cuh"
@@ -309,8 +310,52 @@ mce_status mce_result_cliques(mce_result *r, int32_t *dst, int32_t where) {
             if (!bytes) return;
             if (!dst) fail(MCE_ERR_INVALID, "dst is NULL");
             MCE_CUDA(cudaSetDevice(r->device));
-            MCE_CUDA(cudaMemcpy(dst, r->drows.get(), bytes,
-                                where == MCE_WHERE_HOST ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice));
+            if (where != MCE_WHERE_HOST) {
+                MCE_CUDA(cudaMemcpy(dst, r->drows.get(), bytes, cudaMemcpyDeviceToDevice));
+                return;
+            }
+            if (bytes < (8u << 20)) {
+                MCE_CUDA(cudaMemcpy(dst, r->drows.get(), bytes, cudaMemcpyDeviceToHost));
+                return;
+            }
+            // large: through the cached pinned staging at full link speed, in
+            // chunks, the host copies of a chunk spread over threads and
+            // overlapped with the next chunk's transfer
+            constexpr size_t kChunkBytes = 32u << 20;
+            char *stage = static_cast<char *>(mce::host_pinned(2 * kChunkBytes));
+            cudaStream_t st;
+            MCE_CUDA(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking));
+            cudaEvent_t ev[2];
+            MCE_CUDA(cudaEventCreateWithFlags(&ev[0], cudaEventDisableTiming));
+            MCE_CUDA(cudaEventCreateWithFlags(&ev[1], cudaEventDisableTiming));
+            const char *src = reinterpret_cast<const char *>(r->drows.get());
+            char *out = reinterpret_cast<char *>(dst);
+            const size_t nchunks = (bytes + kChunkBytes - 1) / kChunkBytes;
+            auto issue = [&](size_t c) {
+                const size_t off = c * kChunkBytes, len = std::min(kChunkBytes, bytes - off);
+                MCE_CUDA(cudaMemcpyAsync(stage + (c & 1) * kChunkBytes, src + off, len, cudaMemcpyDeviceToHost, st));
+                MCE_CUDA(cudaEventRecord(ev[c & 1], st));
+            };
+            issue(0);
+            for (size_t c = 0; c < nchunks; ++c) {
+                if (c + 1 < nchunks) issue(c + 1);
+                MCE_CUDA(cudaEventSynchronize(ev[c & 1]));
+                const size_t off = c * kChunkBytes, len = std::min(kChunkBytes, bytes - off);
+                const char *from = stage + (c & 1) * kChunkBytes;
+                const int nt = 8;
+                std::vector<std::thread> th;
+                const size_t part = (len + nt - 1) / nt;
+                for (int t = 0; t < nt; ++t) {
+                    const size_t b = t * part;
+                    if (b >= len) break;
+                    th.emplace_back([=] { std::memcpy(out + off + b, from + b, std::min(part, len - b)); });
+                }
+                for (auto &x : th) x.join();
+
+            }
+            cudaEventDestroy(ev[0]);
+            cudaEventDestroy(ev[1]);
+            cudaStreamDestroy(st);
             return;
         }
         canonicalize(r);
