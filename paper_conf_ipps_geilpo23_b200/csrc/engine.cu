@@ -425,7 +425,7 @@ bool Engine::run_small(int32_t k, const Level &L) {
         Level C;
         C.count = o.children;
         C.W = (int32_t)o.Wc;
-        C.Ps = (int32_t)o.Wc;
+        C.Ps = (int32_t)o.Ps;
         C.P = o.P;
         C.slot = o.slot;
         C.parent = o.parent;

@@ -552,23 +552,23 @@ constexpr int kSmallThreads = 1024;
 
 template <bool WRITE>
 __device__ __forceinline__ int32_t expand_entry_w(int W, const ExpandArgs &a, int64_t e, int64_t out,
-                                                  unsigned &nleaf, unsigned long long &nclq, int &hb, int &ub) {
-    if (W == 1) return expand_entry<1, WRITE>(a, e, out, nleaf, nclq, hb, ub);
-    if (W == 2) return expand_entry<2, WRITE>(a, e, out, nleaf, nclq, hb, ub);
-    return expand_entry<4, WRITE>(a, e, out, nleaf, nclq, hb, ub);
+                                                  unsigned &nleaf, unsigned long long &nclq, int &hb, int &ub,
+                                                  bool active = true, bool fused = false) {
+    if (W == 1) return expand_entry<1, WRITE>(a, e, out, nleaf, nclq, hb, ub, active, fused);
+    if (W == 2) return expand_entry<2, WRITE>(a, e, out, nleaf, nclq, hb, ub, active, fused);
+    return expand_entry<4, WRITE>(a, e, out, nleaf, nclq, hb, ub, active, fused);
 }
 
 __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a0, uint8_t *scratch,
                                                               int64_t scratch_bytes, SmallOut *out,
                                                               LevelLink *chain) {
     __shared__ ExpandArgs A;
-    __shared__ int32_t offs[kSmallMax + 1];
-    __shared__ int32_t wsum[kSmallThreads / 32];
     __shared__ unsigned s_leaf;
-    __shared__ unsigned long long s_clq;
+    __shared__ unsigned long long s_clq, s_cnt;
+    __shared__ int64_t s_end;
     __shared__ int s_hb, s_ub;
     __shared__ int64_t s_used;
-    const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
+    const int t = threadIdx.x;
     if (t == 0) {
         A = a0;
         s_used = 0;
@@ -579,6 +579,7 @@ __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a
         out->k_next = a0.k;
         out->children = a0.end - a0.begin;
         out->Wc = a0.Wp;
+        out->Ps = a0.Ps;
         out->P = const_cast<uint64_t *>(a0.P);
         out->slot = const_cast<int32_t *>(a0.slot);
         out->parent = const_cast<int32_t *>(a0.parent);
@@ -599,40 +600,40 @@ __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a
             chain[A.k] = LevelLink{A.parent, A.vloc};
         }
         __syncthreads();
-        // count pass, one candidate per thread
+        // fused count + write, one candidate per thread: the children go to
+        // worst-case arrays (every candidate bit a child) at slots reserved
+        // per warp, then are compacted behind P
+        if (t == 0) {
+            const int64_t cap = N * 64 * W;
+            uint8_t *p = scratch + s_used;
+            auto take = [&](int64_t bytes) {
+                uint8_t *q = p;
+                p += (bytes + 255) / 256 * 256;
+                return q;
+            };
+            A.cP = reinterpret_cast<uint64_t *>(take(cap * W * 8));
+            A.cslot = reinterpret_cast<int32_t *>(take(cap * 4));
+            A.cparent = reinterpret_cast<int32_t *>(take(cap * 4));
+            A.cvloc = reinterpret_cast<int32_t *>(take(cap * 4));
+            A.out_cap = cap;
+            A.out_count = &s_cnt;
+            A.fused = 1;
+            s_cnt = 0;
+            s_end = p - scratch;
+        }
+        __syncthreads();
         unsigned nleaf = 0;
         unsigned long long nclq = 0;
         int hb = -1, ub = 0;
-        int32_t cnt = 0;
-        if (t < N) cnt = expand_entry_w<false>(W, A, A.begin + t, 0, nleaf, nclq, hb, ub);
+        const int32_t cnt = expand_entry_w<false>(W, A, A.begin + t, 0, nleaf, nclq, hb, ub, t < N, true);
+        (void)cnt;
         if (nleaf) atomicAdd(&s_leaf, nleaf);
         if (nclq) atomicAdd(&s_clq, nclq);
         if (hb >= 0) atomicMax(&s_hb, hb);
         if (ub > 0) atomicMax(&s_ub, ub);
-        // block exclusive scan of the counts
-        int incl = cnt;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const int y = __shfl_up_sync(0xffffffffu, incl, o);
-            if (lane >= o) incl += y;
-        }
-        if (lane == 31) wsum[wid] = incl;
         __syncthreads();
-        if (wid == 0) {
-            int w = wsum[lane];
-#pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const int y = __shfl_up_sync(0xffffffffu, w, o);
-                if (lane >= o) w += y;
-            }
-            wsum[lane] = w;
-        }
-        __syncthreads();
-        const int excl = (wid ? wsum[wid - 1] : 0) + incl - cnt;
-        if (t < N) offs[t] = excl;
-        const int total = wsum[31];
+        const int64_t total = (int64_t)s_cnt;
         if (t == 0) {
-            offs[N] = total;
             out->level_n[lev] = N;
             out->levels = lev + 1;
             out->leaves = s_leaf;
@@ -653,28 +654,35 @@ __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a
             if (t == 0) out->status = 0;
             break;
         }
-        __syncthreads();
-        // children arrays (narrowest stride holding the highest surviving bit)
+        // compaction: slot / parent / vloc right behind the used part of P
+        // (the new ranges end before the old ones start when total <= cap / 2)
+        const int64_t cap = N * 64 * W;
+        if (total <= cap / 2) {
+            uint8_t *base = reinterpret_cast<uint8_t *>(A.cP);
+            auto at = [&](int64_t off) { return base + (off + 255) / 256 * 256; };
+            int32_t *ns = reinterpret_cast<int32_t *>(at(total * W * 8));
+            int32_t *np_ = reinterpret_cast<int32_t *>(at(reinterpret_cast<uint8_t *>(ns) - base + total * 4));
+            int32_t *nv = reinterpret_cast<int32_t *>(at(reinterpret_cast<uint8_t *>(np_) - base + total * 4));
+            for (int64_t i = t; i < total; i += blockDim.x) ns[i] = A.cslot[i];
+            __syncthreads();
+            for (int64_t i = t; i < total; i += blockDim.x) np_[i] = A.cparent[i];
+            __syncthreads();
+            for (int64_t i = t; i < total; i += blockDim.x) nv[i] = A.cvloc[i];
+            __syncthreads();
+            if (t == 0) {
+                A.cslot = ns;
+                A.cparent = np_;
+                A.cvloc = nv;
+                s_used = (reinterpret_cast<uint8_t *>(nv) - scratch) + (total * 4 + 255) / 256 * 256;
+            }
+        } else if (t == 0) {
+            s_used = s_end;
+        }
         if (t == 0) {
             int Wc = 1;
             while (Wc * 64 <= s_hb && Wc < W) Wc <<= 1;
-            uint8_t *p = scratch + s_used;
-            auto take = [&](int64_t bytes) {
-                uint8_t *q = p;
-                p += (bytes + 255) / 256 * 256;
-                return q;
-            };
-            A.cP = reinterpret_cast<uint64_t *>(take((int64_t)total * Wc * 8));
-            A.cslot = reinterpret_cast<int32_t *>(take((int64_t)total * 4));
-            A.cparent = reinterpret_cast<int32_t *>(take((int64_t)total * 4));
-            A.cvloc = reinterpret_cast<int32_t *>(take((int64_t)total * 4));
             A.Wc = Wc;
-            A.out_base = 0;
-            s_used = p - scratch;
         }
-        __syncthreads();
-        // write pass
-        if (t < N && cnt > 0) expand_entry_w<true>(W, A, A.begin + t, offs[t], nleaf, nclq, hb, ub);
         __syncthreads();
         const bool stop = s_leaf > 0 || s_clq > 0 || total > kSmallMax;
         if (t == 0) {
@@ -683,6 +691,7 @@ __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a
             out->parent = A.cparent;
             out->vloc = A.cvloc;
             out->Wc = A.Wc;
+            out->Ps = A.Wp;
             out->status = 1;
             // the children become the next level
             A.P = A.cP;
@@ -691,8 +700,8 @@ __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a
             A.vloc = A.cvloc;
             A.begin = 0;
             A.end = total;
+            A.Ps = A.Wp;  // written with the parent's width
             A.Wp = A.Wc;
-            A.Ps = A.Wc;
             A.k = A.k + 1;
         }
         __syncthreads();

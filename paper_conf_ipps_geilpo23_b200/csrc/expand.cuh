@@ -121,7 +121,8 @@ struct SmallOut {
     int64_t levels;    // levels processed (|C| = k0 .. k0 + levels - 1)
     int64_t k_next;    // |C| of the level the host continues with
     int64_t children;  // its entries
-    int64_t Wc;        // its word stride
+    int64_t Wc;        // its word width
+    int64_t Ps;        // its P stride in words (>= Wc)
     int64_t leaves;    // leaves (size k_next) recorded by the last processed level
     int64_t cliques;   // clique completions (size need) recorded by the last processed level
     uint64_t *P;       // the level the host continues with
