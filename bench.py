@@ -220,9 +220,17 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # test hooks for the multi-process path on a one-GPU box: every rank on
+    # cuda:0, gloo instead of NCCL (the driver's N-GPU runs use neither)
+    if os.environ.get("MCE_BENCH_SAME_DEVICE") == "1":
+        local = 0
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if os.environ.get("MCE_BENCH_BACKEND") == "gloo":
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    rdev = "cpu" if (world > 1 and dist.get_backend() == "gloo") else f"cuda:{local}"
     mode = args.mode or ("find_one" if args.config == "dense800" else "enumerate")
     shard_depth = args.shard_depth if args.shard_depth >= 0 else (3 if args.config == "rmat26" else 0)
     if args.window < 0:
@@ -267,7 +275,7 @@ def main():
             timings.append(res.timing)
     t_ms = sum(times) / len(times)  # exactly K timed steps
     if world > 1:
-        tt = torch.tensor([t_ms], dtype=torch.float64, device=f"cuda:{local}")
+        tt = torch.tensor([t_ms], dtype=torch.float64, device=rdev)
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         t_ms = float(tt.item())
     value = edges / (t_ms / 1e3)
@@ -321,7 +329,7 @@ def main():
             d2h = int(r2.cliques.nbytes) + 32
         et = statistics.mean(e2e_times)
         if world > 1:
-            tt = torch.tensor([et], dtype=torch.float64, device=f"cuda:{local}")
+            tt = torch.tensor([et], dtype=torch.float64, device=rdev)
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
             et = float(tt.item())
         e2e = {"value": edges / et, "unit": "edges/s", "h2d_bytes_per_step": int(rp_h.nbytes + col_h.nbytes),

@@ -144,6 +144,17 @@ mce_status mce_graph_clear_cache(mce_graph *g);
 mce_status mce_preprocess(mce_graph *g, int32_t orientation, int32_t *core_out, int32_t *order_out,
                           int32_t where, int32_t *degeneracy_out);
 
+/* Replace the orientation order with `order` (int32[n], a permutation of the
+ * vertices: vertex of rank i; host or device per `where`) and rebuild the
+ * oriented CSR from it; core numbers are computed if missing.  Multi-GPU:
+ * the k-core peel order is not deterministic across processes and root /
+ * candidate sharding needs every rank to orient edges the same way, so
+ * rank 0's order is broadcast and set on the others (distributed.py).  For
+ * MCE_ORIENT_DEGENERACY the order must be a degeneracy order (each vertex
+ * has at most core(v) later neighbours) -- e.g. another rank's
+ * mce_preprocess output; MCE_ERR_INVALID for a NULL order. */
+mce_status mce_set_order(mce_graph *g, int32_t orientation, const int32_t *order, int32_t where);
+
 /* Greedy heuristic (PAPER.md IV-A, Algorithm 1).  kind = MCE_HEUR_*; h = runs
  * (<=0: |V|; single-run kinds ignore h and use 1).  *omega_bar_out = size of the
  * best clique found; clique_out (host, capacity >= max degree + 1, may be NULL)

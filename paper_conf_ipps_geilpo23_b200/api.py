@@ -130,6 +130,19 @@ class Graph:
                                    order.ctypes.data_as(ctypes.c_void_p), _lib.WHERE_HOST, ctypes.byref(d)))
         return core[: self.n], order[: self.n], int(d.value)
 
+    def order_into(self, out, orientation: str = "degeneracy"):
+        """Preprocess (cached) and copy the orientation order into `out` (int32[n]
+        torch tensor on this graph's device, or a host array)."""
+        ptr, where, _keep = _ptr_and_where(out, np.int32)
+        d = ctypes.c_int32()
+        check(lib().mce_preprocess(self._h, ORIENT[orientation], None, ptr, where, ctypes.byref(d)))
+        return out
+
+    def set_order(self, order, orientation: str = "degeneracy"):
+        """mce_set_order: orient the edges along `order` (vertex of rank i)."""
+        ptr, where, _keep = _ptr_and_where(order, np.int32)
+        check(lib().mce_set_order(self._h, ORIENT[orientation], ptr, where))
+
     def heuristic(self, kind: str = "multi_degree", h: int = 0):
         """(omega_bar, clique in order added, run size per seed vertex (0 = not a seed))."""
         w = ctypes.c_int32()

@@ -216,6 +216,17 @@ mce_status mce_graph_clear_cache(mce_graph *g) {
     });
 }
 
+mce_status mce_set_order(mce_graph *g, int32_t orientation, const int32_t *order, int32_t where) {
+    return run_guarded([&] {
+        if (!g) fail(MCE_ERR_INVALID, "graph is NULL");
+        if (orientation != MCE_ORIENT_DEGENERACY && orientation != MCE_ORIENT_DEGREE)
+            fail(MCE_ERR_INVALID, "bad orientation");
+        if (!order && g->n) fail(MCE_ERR_INVALID, "order is NULL");
+        MCE_CUDA(cudaSetDevice(g->device));
+        orient_from(g, orientation, order, where == MCE_WHERE_DEVICE);
+    });
+}
+
 mce_status mce_preprocess(mce_graph *g, int32_t orientation, int32_t *core_out, int32_t *order_out, int32_t where,
                           int32_t *degeneracy_out) {
     return run_guarded([&] {

@@ -29,6 +29,7 @@ struct mce_graph {
     int32_t max_out = 0;           // largest out-degree
     double t_pre_ms = 0.0;         // device time of the last preprocessing
     bool pre_overlapped = false;   // set by the engine while the heuristic runs concurrently
+    bool order_given = false;      // g->order was set by mce_set_order: orient() keeps it
     int64_t kernels = 0;           // kernels launched by the last preprocessing
 
     // ---- reusable memory (no cudaMalloc/cudaFree on the steady-state path) ----
@@ -57,4 +58,6 @@ void kcore(mce_graph *g);
 void orient(mce_graph *g, int orientation);
 // both, cached on the handle
 void preprocess(mce_graph *g, int orientation);
+// orientation from a given order (mce_set_order)
+void orient_from(mce_graph *g, int orientation, const int32_t *order, bool on_device);
 }  // namespace mce

@@ -606,7 +606,8 @@ void orient(mce_graph *g, int orientation) {
         g->max_out = 0;
         return;
     }
-    if (orientation == 0) {  // degeneracy: the peel queue
+    if (g->order_given) {  // mce_set_order: g->order already holds the order
+    } else if (orientation == 0) {  // degeneracy: the peel queue
         MCE_CUDA(cudaMemcpyAsync(g->order.get(), g->peel.get(), sizeof(int32_t) * n, cudaMemcpyDeviceToDevice, s));
     } else {  // degree order
         int64_t nb = g->max_deg + 1;
@@ -688,6 +689,20 @@ void orient(mce_graph *g, int orientation) {
     }
     stream_sync(s);
     g->orientation = orientation;
+}
+
+void orient_from(mce_graph *g, int orientation, const int32_t *order, bool on_device) {
+    kcore(g);  // core numbers (deterministic) for the CSR-id space and the heuristics
+    const int64_t n = g->n;
+    g->order.ensure(std::max<int64_t>(n, 1));
+    if (n)
+        MCE_CUDA(cudaMemcpyAsync(g->order.get(), order, sizeof(int32_t) * n,
+                                 on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, g->stream));
+    g->order_given = true;
+    g->orientation = -1;
+    orient(g, orientation);
+    g->order_given = false;
+    stream_sync(g->stream);
 }
 
 void preprocess(mce_graph *g, int orientation) {

@@ -4,7 +4,9 @@ North star: "Work is partitioned ... by sharding first-level root vertices,
 whose subtrees are independent, with a small NCCL max-allreduce of the omega
 lower bound each level and a final gather of the cliques over NVLink."
 
- * every rank loads the whole graph and runs the same preprocessing;
+ * every rank loads the whole graph and runs the same preprocessing, then
+   takes rank 0's orientation order (agree_orientation: the peel order is not
+   deterministic across processes, and clique ownership depends on it);
  * heuristic seeds are dealt cyclically (seed position % world == rank) and
    root vertices by CSR id (id % world == rank) inside the library
    (mce_options.shard_rank / shard_count);
@@ -18,6 +20,7 @@ lower bound each level and a final gather of the cliques over NVLink."
 
 from __future__ import annotations
 
+import os
 from typing import Optional
 
 import numpy as np
@@ -51,6 +54,9 @@ def gather_result(res: Result, group=None, find_one: bool = False) -> Result:
     dev = _device(group)
     world = dist.get_world_size(group)
     rank = dist.get_rank(group)
+    if os.environ.get("MCE_DEBUG_GATHER"):
+        print(f"[gather] rank {rank}/{world}: local omega {res.omega} count {res.count} "
+              f"stored {res.cliques.shape[0]}", flush=True)
     t = torch.tensor([res.omega], dtype=torch.int64, device=dev)
     dist.all_reduce(t, op=dist.ReduceOp.MAX, group=group)
     omega = int(t.item())
@@ -87,9 +93,30 @@ def gather_result(res: Result, group=None, find_one: bool = False) -> Result:
     return Result(omega, total, allrows, bool(trunc), res.levels, res.timing)
 
 
+def agree_orientation(graph: Graph, group=None, orientation: str = "degeneracy"):
+    """Make every rank orient the edges like rank 0.  The asynchronous k-core
+    peel is not deterministic across processes, and the root of a clique (its
+    lowest-rank vertex) -- hence the rank that owns it -- depends on the
+    order: rank 0's order is broadcast and set on the others."""
+    if dist.get_world_size(group) == 1 or graph.n == 0:
+        return
+    dev = _device(group)
+    if dev.type == "cuda":
+        order = torch.empty(graph.n, dtype=torch.int32, device=torch.device("cuda", graph.device))
+    else:
+        order = torch.empty(graph.n, dtype=torch.int32)
+    src = dist.get_global_rank(group, 0) if group is not None else 0
+    if dist.get_rank(group) == 0:
+        graph.order_into(order, orientation)
+    dist.broadcast(order, src=src, group=group)
+    if dist.get_rank(group) != 0:
+        graph.set_order(order, orientation)
+
+
 def enumerate_distributed(graph: Graph, group=None, **opts) -> Result:
     rank = dist.get_rank(group)
     world = dist.get_world_size(group)
+    agree_orientation(graph, group, opts.get("orientation", "degeneracy"))
     res = graph.enumerate(shard_rank=rank, shard_count=world, bound_sync=make_bound_sync(group), **opts)
     return gather_result(res, group)
 
@@ -97,6 +124,7 @@ def enumerate_distributed(graph: Graph, group=None, **opts) -> Result:
 def find_one_distributed(graph: Graph, window: int = 0, group=None, **opts) -> Result:
     rank = dist.get_rank(group)
     world = dist.get_world_size(group)
+    agree_orientation(graph, group, opts.get("orientation", "degeneracy"))
     res = graph.find_one(window=window, shard_rank=rank, shard_count=world, bound_sync=make_bound_sync(group),
                          **opts)
     return gather_result(res, group, find_one=True)

@@ -170,3 +170,36 @@ def test_bound_sync_callback_is_called_every_step():
     gg.close()
     assert r.omega == om and r.count == len(cl) and np.array_equal(r.cliques, cl)
     assert len(calls) >= 2 and calls[-1][1] == 0
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("depth", [0, 3])
+@pytest.mark.parametrize("key", ["RMAT13", "planted", "ER400d", "T(30,6)"])
+def test_shards_on_separate_handles_agree_after_set_order(key, depth):
+    """Each "rank" has its own graph handle (its own, possibly different, k-core
+    peel order); after mce_set_order with handle 0's order the shards still
+    partition the maximum cliques exactly (agree_orientation)."""
+    import torch
+
+    import oracle
+    from tests.test_gpu_parity import GRAPHS
+
+    import paper_conf_ipps_geilpo23_b200 as m
+
+    g = GRAPHS[key]()
+    om, cl = oracle.max_cliques(*g.numpy())
+    shards = 2
+    hs = [m.Graph(g.rowptr, g.col) for _ in range(shards)]
+    order = hs[0].order_into(torch.empty(g.n, dtype=torch.int32, device="cuda"))
+    for h in hs[1:]:
+        h.set_order(order)
+    o2 = hs[1].order_into(torch.empty(g.n, dtype=torch.int32, device="cuda"))
+    assert torch.equal(order, o2)
+    parts = [h.enumerate(shard_rank=r, shard_count=shards, shard_depth=depth) for r, h in enumerate(hs)]
+    for h in hs:
+        h.close()
+    omega = max(p.omega for p in parts)
+    count = sum(p.count for p in parts if p.omega == omega)
+    rows = np.concatenate([p.cliques for p in parts if p.omega == omega], 0)
+    rows = rows[np.lexsort(rows.T[::-1])]
+    assert omega == om and count == len(cl) and np.array_equal(rows, cl)
