@@ -27,7 +27,9 @@ struct mce_graph {
     mce::DevBuf<int64_t> orp;      // [n+1] oriented CSR (edges to higher rank), indexed by CSR id
     mce::DevBuf<int32_t> ocol;     // [nnz/2] out-neighbour CSR ids, rows ascending
     int32_t max_out = 0;           // largest out-degree
-    double t_pre_ms = 0.0;         // device time of the last preprocessing
+    double t_pre_ms = 0.0;         // device time of the last preprocessing (see preprocess_ms)
+    cudaEvent_t pre_ev[2] = {nullptr, nullptr};
+    bool pre_pending = false;
     bool pre_overlapped = false;   // set by the engine while the heuristic runs concurrently
     bool order_given = false;      // g->order was set by mce_set_order: orient() keeps it
     int64_t kernels = 0;           // kernels launched by the last preprocessing
@@ -43,6 +45,8 @@ struct mce_graph {
     cudaStream_t hstream = nullptr;
     ~mce_graph() {
         if (hstream) cudaStreamDestroy(hstream);
+        if (pre_ev[0]) cudaEventDestroy(pre_ev[0]);
+        if (pre_ev[1]) cudaEventDestroy(pre_ev[1]);
     }
     mce::DevBuf<uint8_t> misc;     // engine: leaf counter + level chain (persistent)
     mce::DevBuf<int32_t> stage;    // engine: staged leaf cliques of one launch (grow-only)
@@ -58,6 +62,8 @@ void kcore(mce_graph *g);
 void orient(mce_graph *g, int orientation);
 // both, cached on the handle
 void preprocess(mce_graph *g, int orientation);
+// device time of the last preprocessing (waits for it if still pending)
+double preprocess_ms(mce_graph *g);
 // orientation from a given order (mce_set_order)
 void orient_from(mce_graph *g, int orientation, const int32_t *order, bool on_device);
 }  // namespace mce

@@ -687,8 +687,7 @@ void orient(mce_graph *g, int orientation) {
         }
         g->kernels += 1;
     }
-    stream_sync(s);
-    g->orientation = orientation;
+    g->orientation = orientation;  // (stream-ordered: no sync needed before the consumers)
 }
 
 void orient_from(mce_graph *g, int orientation, const int32_t *order, bool on_device) {
@@ -707,20 +706,28 @@ void orient_from(mce_graph *g, int orientation, const int32_t *order, bool on_de
 
 void preprocess(mce_graph *g, int orientation) {
     if (g->have_core && g->orientation == orientation) return;
-    cudaEvent_t e0, e1;
-    MCE_CUDA(cudaEventCreate(&e0));
-    MCE_CUDA(cudaEventCreate(&e1));
-    MCE_CUDA(cudaEventRecord(e0, g->stream));
+    if (!g->pre_ev[0]) {
+        MCE_CUDA(cudaEventCreate(&g->pre_ev[0]));
+        MCE_CUDA(cudaEventCreate(&g->pre_ev[1]));
+    }
+    MCE_CUDA(cudaEventRecord(g->pre_ev[0], g->stream));
     g->kernels = 0;
     kcore(g);
     orient(g, orientation);
-    MCE_CUDA(cudaEventRecord(e1, g->stream));
-    MCE_CUDA(cudaEventSynchronize(e1));
-    float ms = 0;
-    MCE_CUDA(cudaEventElapsedTime(&ms, e0, e1));
-    g->t_pre_ms = ms;
-    cudaEventDestroy(e0);
-    cudaEventDestroy(e1);
+    // no host sync here: the device time is read after the caller's next one
+    MCE_CUDA(cudaEventRecord(g->pre_ev[1], g->stream));
+    g->pre_pending = true;
+}
+
+double preprocess_ms(mce_graph *g) {
+    if (g->pre_pending) {
+        MCE_CUDA(cudaEventSynchronize(g->pre_ev[1]));
+        float ms = 0;
+        MCE_CUDA(cudaEventElapsedTime(&ms, g->pre_ev[0], g->pre_ev[1]));
+        g->t_pre_ms = ms;
+        g->pre_pending = false;
+    }
+    return g->t_pre_ms;
 }
 
 }  // namespace mce
