@@ -284,7 +284,16 @@ __device__ void root_thread(const RootArgs &a, int32_t r, unsigned long long &by
             T += (unsigned long long)d;
             unsigned m = 0;  // positions c with V[c] in N+(V[p])
             if (d <= 16) {
-                for (int64_t q = s0[p]; q < s1[p]; ++q) {
+                // the first four elements as independent loads (sparse out-rows are
+                // that short), so a row costs one load latency, not d of them
+                const int32_t u0 = d > 0 ? __ldg(a.ocol + s0[p]) : -2;
+                const int32_t u1 = d > 1 ? __ldg(a.ocol + s0[p] + 1) : -2;
+                const int32_t u2 = d > 2 ? __ldg(a.ocol + s0[p] + 2) : -2;
+                const int32_t u3 = d > 3 ? __ldg(a.ocol + s0[p] + 3) : -2;
+#pragma unroll
+                for (int c = 0; c < 8; ++c)
+                    m |= (unsigned)((V[c] == u0) | (V[c] == u1) | (V[c] == u2) | (V[c] == u3)) << c;
+                for (int64_t q = s0[p] + 4; q < s1[p]; ++q) {
                     const int32_t u = __ldg(a.ocol + q);
 #pragma unroll
                     for (int c = 0; c < 8; ++c) m |= (unsigned)(V[c] == u) << c;
