@@ -598,7 +598,7 @@ void orient(mce_graph *g, int orientation) {
     g->vid.ensure(std::max<int64_t>(n, 1));
     g->pid.ensure(std::max<int64_t>(n, 1));
     g->orp.ensure(n + 1);
-    g->ocol.ensure(std::max<int64_t>(g->nnz / 2, 1));
+    g->ocol.ensure(std::max<int64_t>(g->nnz / 2, 1) + 4);  // + 4: int4 over-reads of the root level (roots.cu load4)
     g->pool.reset();
     if (n == 0) {
         MCE_CUDA(cudaMemsetAsync(g->orp.get(), 0, sizeof(int64_t), s));

@@ -257,28 +257,75 @@ __device__ __forceinline__ unsigned long long warp_excl(unsigned long long x, un
 // closed under symmetry with an 8x8 transpose; the colouring order, colours
 // and children are packed nibbles / bytes.  Called by all 32 lanes of a warp
 // (r < 0: no root) so survivors are materialised with warp-aggregated atomics.
-__device__ void root_thread(const RootArgs &a, int32_t r, unsigned long long &bytes) {
-    int L = 0;
-    int64_t vb = 0;
+// Thread-per-root loads are scattered (every lane its own line), so the L1
+// wavefronts they cost, not bytes, bound the root level (ncu: LSU data-pipe
+// wavefronts 77% of peak).  These helpers fetch what one lane needs with
+// aligned 16-byte loads: a row's bounds orp[v], orp[v+1] in one load when v is
+// even, up to four consecutive ids in one or two.
+__device__ __forceinline__ void row_bounds(const int64_t *__restrict__ orp, int32_t v, int64_t &b, int64_t &e) {
+    const longlong2 x = __ldg(reinterpret_cast<const longlong2 *>(orp + (v & ~1)));
+    if (v & 1) {
+        b = x.y;
+        e = __ldg(orp + v + 1);
+    } else {
+        b = x.x;
+        e = x.y;
+    }
+}
+
+// u[k] = col[s + k] for k < d (d <= 4), else fill.  The int4 loads may read up
+// to three ids past the end of `col` (the oriented CSR is allocated with that
+// padding, preprocess.cu).
+__device__ __forceinline__ void load4(const int32_t *__restrict__ col, int64_t s, int d, int32_t fill,
+                                      int32_t (&u)[4]) {
+    const int64_t al = s & ~3ll;
+    const int o = (int)(s - al);
+    int4 w0 = make_int4(fill, fill, fill, fill), w1 = w0;
+    if (d > 0) w0 = __ldg(reinterpret_cast<const int4 *>(col + al));
+    if (o + d > 4) w1 = __ldg(reinterpret_cast<const int4 *>(col + al + 4));
+    const int32_t x[8] = {w0.x, w0.y, w0.z, w0.w, w1.x, w1.y, w1.z, w1.w};
+    int32_t y[6];
+#pragma unroll
+    for (int i = 0; i < 6; ++i) y[i] = (o & 2) ? x[i + 2] : x[i];
+#pragma unroll
+    for (int k = 0; k < 4; ++k) u[k] = k < d ? ((o & 1) ? y[k + 1] : y[k]) : fill;
+}
+
+template <int LM>
+__device__ void root_thread(const RootArgs &a, int32_t r, int64_t vb, int L, unsigned long long &bytes) {
     uint64_t adj = 0;
     unsigned long long T = 0;
+    if (r < 0) {
+        vb = 0;
+        L = 0;
+    }
     if (r >= 0) {
-        vb = __ldg(a.orp + r);
-        L = (int)(__ldg(a.orp + r + 1) - vb);
-        int32_t V[8];
+        int32_t V[LM];
+        if constexpr (LM == 4) {
+            load4(a.ocol, vb, L, -1, V);
+        } else {
 #pragma unroll
-        for (int p = 0; p < 8; ++p) V[p] = p < L ? __ldg(a.ocol + vb + p) : -1;
-        int64_t s0[8], s1[8];
+            for (int p = 0; p < LM; ++p) V[p] = p < L ? __ldg(a.ocol + vb + p) : -1;
+        }
+        int64_t s0[LM], s1[LM];
 #pragma unroll
-        for (int p = 0; p < 8; ++p) {
+        for (int p = 0; p < LM; ++p) {
             s0[p] = s1[p] = 0;
-            if (p < L) {
-                s0[p] = __ldg(a.orp + V[p]);
-                s1[p] = __ldg(a.orp + V[p] + 1);
+            if (p < L) row_bounds(a.orp, V[p], s0[p], s1[p]);
+        }
+        // LM == 4 (sparse roots): the first four elements of every out-row,
+        // all issued before any is used, so the adjacency costs one load
+        // latency, not one per row
+        int32_t u[LM == 4 ? 4 : 1][4];
+        if constexpr (LM == 4) {
+#pragma unroll
+            for (int p = 0; p < 4; ++p) {
+                const int64_t d = s1[p] - s0[p];
+                load4(a.ocol, s0[p], (p < L && d <= 16) ? (int)min(d, (int64_t)4) : 0, -2, u[p]);
             }
         }
 #pragma unroll
-        for (int p = 0; p < 8; ++p) {
+        for (int p = 0; p < LM; ++p) {
             if (p >= L) break;
             const int64_t d = s1[p] - s0[p];
             T += (unsigned long long)d;
@@ -286,21 +333,29 @@ __device__ void root_thread(const RootArgs &a, int32_t r, unsigned long long &by
             if (d <= 16) {
                 // the first four elements as independent loads (sparse out-rows are
                 // that short), so a row costs one load latency, not d of them
-                const int32_t u0 = d > 0 ? __ldg(a.ocol + s0[p]) : -2;
-                const int32_t u1 = d > 1 ? __ldg(a.ocol + s0[p] + 1) : -2;
-                const int32_t u2 = d > 2 ? __ldg(a.ocol + s0[p] + 2) : -2;
-                const int32_t u3 = d > 3 ? __ldg(a.ocol + s0[p] + 3) : -2;
+                int32_t u0, u1, u2, u3;
+                if constexpr (LM == 4) {
+                    u0 = u[p][0];
+                    u1 = u[p][1];
+                    u2 = u[p][2];
+                    u3 = u[p][3];
+                } else {
+                    u0 = d > 0 ? __ldg(a.ocol + s0[p]) : -2;
+                    u1 = d > 1 ? __ldg(a.ocol + s0[p] + 1) : -2;
+                    u2 = d > 2 ? __ldg(a.ocol + s0[p] + 2) : -2;
+                    u3 = d > 3 ? __ldg(a.ocol + s0[p] + 3) : -2;
+                }
 #pragma unroll
-                for (int c = 0; c < 8; ++c)
+                for (int c = 0; c < LM; ++c)
                     m |= (unsigned)((V[c] == u0) | (V[c] == u1) | (V[c] == u2) | (V[c] == u3)) << c;
                 for (int64_t q = s0[p] + 4; q < s1[p]; ++q) {
                     const int32_t u = __ldg(a.ocol + q);
 #pragma unroll
-                    for (int c = 0; c < 8; ++c) m |= (unsigned)(V[c] == u) << c;
+                    for (int c = 0; c < LM; ++c) m |= (unsigned)(V[c] == u) << c;
                 }
             } else {
 #pragma unroll
-                for (int c = 0; c < 8; ++c)
+                for (int c = 0; c < LM; ++c)
                     if (c < L && c != p && contains_sorted(a.ocol, s0[p], s1[p], V[c])) m |= 1u << c;
             }
             // local index = L-1-position (expand.cuh): reverse rows and columns
@@ -413,12 +468,17 @@ __global__ void __launch_bounds__(kRootWarps * 32, 4) root_expand_w1(const RootA
     for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < a.count; base += (int64_t)gridDim.x * blockDim.x) {
         const int64_t i = base + threadIdx.x;
         int32_t r = i < a.count ? __ldg(a.list + i * a.stride) : -1;
-        const int L = r >= 0 ? (int)(__ldg(a.orp + r + 1) - __ldg(a.orp + r)) : 0;
+        int64_t vb = 0, ve = 0;
+        if (r >= 0) row_bounds(a.orp, r, vb, ve);
+        const int L = (int)(ve - vb);
         if (r >= 0 && L > kThreadRootMax) {
             queue[atomicAdd(&qn, 1)] = r;
             r = -1;
         }
-        root_thread(a, r, bytes);
+        if (__all_sync(0xffffffffu, r < 0 || L <= 4))
+            root_thread<4>(a, r, vb, L, bytes);
+        else
+            root_thread<kThreadRootMax>(a, r, vb, L, bytes);
         __syncthreads();
         const int nq = qn;
         for (int q = wid; q < nq; q += kRootWarps) {
