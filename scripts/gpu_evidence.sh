@@ -19,3 +19,4 @@ timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --lo
   python bench.py --config rmat22 --steps 1 --warmup 1 --no-cpu-baseline --no-e2e > gpurun_out/${TAG}_launches_rmat22.log 2>&1; echo launches rmat rc=$?
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:root_expand -c 1 -o gpurun_out/${TAG}_full_root_ba1m \
   python bench.py --config ba1m --steps 1 --warmup 1 --no-cpu-baseline --no-e2e > gpurun_out/${TAG}_full_root.log 2>&1; echo full root rc=$?
+timeout 1500 python bench.py --config rmat26 --steps 1 --warmup 3 --no-cpu-baseline --no-e2e > gpurun_out/${TAG}_bench_rmat26.log 2>&1; echo bench rmat26 rc=$?
