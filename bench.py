@@ -287,7 +287,7 @@ def main():
     cnt_ms = statistics.mean(t["count_kernel_ms"] for t in timings)
     root_ms = statistics.mean(t["root_kernel_ms"] for t in timings)
     if root_ms >= cnt_ms and tm["root_launches"] > 0:
-        kname = "root_expand_w1 (fused root level: adjacency build + first expansion)"
+        kname = "root_expand_l4 / root_expand_w1 (fused root level: adjacency build + first expansion)"
         k_ms, k_bytes, launches = root_ms, tm["root_kernel_bytes"], max(tm["root_launches"], 1)
     else:
         kname = "expand (fused count + write pass of levels >= 2: mce::expand_thread / expand_tile)"

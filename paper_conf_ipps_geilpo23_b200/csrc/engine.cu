@@ -718,7 +718,7 @@ void Engine::do_class_w1(const int32_t *list, int64_t count) {
         for (int attempt = 0; attempt < 2; ++attempt) {
             MCE_CUDA(cudaMemsetAsync(ctr, 0, 8 * sizeof(unsigned long long), s_));
             const int t = clock_.start(2);
-            launch_root_expand_w1(ra, s_);
+            launch_root_expand_w1(ra, g_->max_out, s_);
             clock_.stop(t);
             ++kernels_;
             ++root_launches_;

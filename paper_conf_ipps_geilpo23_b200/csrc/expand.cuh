@@ -105,7 +105,8 @@ struct RootArgs {
     int32_t *leaf_rows;  // size-2 leaves (only when need <= 2)
     int64_t leaf_cap;
 };
-void launch_root_expand_w1(const RootArgs &a, cudaStream_t s);
+// max_len: an upper bound on |N+(r)| over the launch's roots (<= 4 selects the sparse kernel)
+void launch_root_expand_w1(const RootArgs &a, int max_len, cudaStream_t s);
 
 // Small-frontier fused levels (expand.cu expand_small): one block runs
 // count -> scan -> write for consecutive levels while a level has at most

@@ -495,10 +495,38 @@ __global__ void __launch_bounds__(kRootWarps * 32, 4) root_expand_w1(const RootA
     if (lane == 0 && bytes) atomicAdd(a.ctr + 4, bytes);
 }
 
+// Every root of the launch has L <= 4 (the host knows the largest out-degree
+// of the orientation: sparse graphs such as BA m = 4 have degeneracy 4): only
+// the register-resident thread path, no queue, no barriers, and a register
+// budget cut for more resident roots (ROOT_SPARSE_BLOCKS blocks per SM).
+#ifndef ROOT_SPARSE_BLOCKS
+#define ROOT_SPARSE_BLOCKS 4  // measured: 4 / 5 / 6 blocks per SM = 52 / 69 / 93 us on ba1m (5, 6 spill)
+#endif
+__global__ void __launch_bounds__(kRootWarps * 32, ROOT_SPARSE_BLOCKS) root_expand_l4(const RootArgs a) {
+    unsigned long long bytes = 0;  // algorithmic bytes read
+    for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < a.count; base += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t i = base + threadIdx.x;
+        const int32_t r = i < a.count ? __ldg(a.list + i * a.stride) : -1;
+        int64_t vb = 0, ve = 0;
+        if (r >= 0) row_bounds(a.orp, r, vb, ve);
+        root_thread<4>(a, r, vb, (int)(ve - vb), bytes);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) bytes += __shfl_xor_sync(0xffffffffu, bytes, o);
+    if ((threadIdx.x & 31) == 0 && bytes) atomicAdd(a.ctr + 4, bytes);
+}
+
 }  // namespace
 
-void launch_root_expand_w1(const RootArgs &a, cudaStream_t s) {
+void launch_root_expand_w1(const RootArgs &a, int max_len, cudaStream_t s) {
     if (a.count <= 0) return;
+#if !ROOT_NO_SPARSE
+    if (max_len <= 4) {
+        root_expand_l4<<<grid_for(a.count, kRootWarps * 32, 8), kRootWarps * 32, 0, s>>>(a);
+        MCE_LAUNCH_CHECK();
+        return;
+    }
+#endif
     root_expand_w1<<<grid_for(a.count, kRootWarps * 32, 8), kRootWarps * 32, 0, s>>>(a);
     MCE_LAUNCH_CHECK();
 }

@@ -55,6 +55,10 @@ GRAPHS = {
     "RMAT13": lambda: G.rmat(13, 8, 0.45, 0.2, 0.2, seed=2),
     "RMAT15": lambda: G.rmat(15, 16, 0.57, 0.19, 0.19, seed=5),  # 121 hubs of degree > 1024
     "BA5k": lambda: G.barabasi_albert(5000, 4, seed=2),
+    # degeneracy <= 3: every root has |N+(r)| <= 4, the sparse root kernel (root_expand_l4)
+    "BA3k_m1": lambda: G.barabasi_albert(3000, 1, seed=11),  # a tree: omega 2, every edge maximum
+    "BA3k_m2": lambda: G.barabasi_albert(3000, 2, seed=11),
+    "BA3k_m3": lambda: G.barabasi_albert(3000, 3, seed=11),
     "planted": lambda: G.plant_cliques(G.erdos_renyi(3000, 0.004, seed=9), 3, 9, seed=9),
     "er2000": lambda: G.make_config("er2000"),
 }
@@ -90,7 +94,7 @@ def test_unfused_levels_match(key):
     assert (r.omega, r.count) == (om, len(cl)) and np.array_equal(r.cliques, cl)
 
 
-@pytest.mark.parametrize("key", ["er2000", "planted", "RMAT11", "BA5k", "C9", "T(36,12)"])
+@pytest.mark.parametrize("key", ["er2000", "planted", "RMAT11", "BA5k", "BA3k_m1", "BA3k_m2", "C9", "T(36,12)"])
 def test_no_heuristic_size2_leaves(key):
     """Heuristic 'none' with a lower bound of 2: size-2 leaves come out of the fused root kernel."""
     g = GRAPHS[key]()
