@@ -236,13 +236,14 @@ __device__ __forceinline__ uint64_t transpose8(uint64_t x) {
     return x;
 }
 
-// warp exclusive prefix sum of x (all 32 lanes)
-__device__ __forceinline__ unsigned long long warp_excl(unsigned long long x, unsigned long long &total) {
+// warp exclusive prefix sum of x (all 32 lanes; per-lane values and the warp
+// total fit 32 bits: at most 32 roots x 64 rows or children)
+__device__ __forceinline__ unsigned warp_excl(unsigned x, unsigned &total) {
     const int lane = threadIdx.x & 31;
-    unsigned long long inc = x;
+    unsigned inc = x;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
-        const unsigned long long y = __shfl_up_sync(0xffffffffu, inc, o);
+        const unsigned y = __shfl_up_sync(0xffffffffu, inc, o);
         if (lane >= o) inc += y;
     }
     total = __shfl_sync(0xffffffffu, inc, 31);
@@ -291,7 +292,9 @@ __device__ __forceinline__ void load4(const int32_t *__restrict__ col, int64_t s
     for (int k = 0; k < 4; ++k) u[k] = k < d ? ((o & 1) ? y[k + 1] : y[k]) : fill;
 }
 
-template <int LM>
+// kShort: every out-row of the launch has <= 4 ids (the orientation's largest
+// out-degree is <= 4), so the tail and binary-search paths are compiled out
+template <int LM, bool kShort = false>
 __device__ void root_thread(const RootArgs &a, int32_t r, int64_t vb, int L, unsigned long long &bytes) {
     uint64_t adj = 0;
     unsigned long long T = 0;
@@ -321,7 +324,7 @@ __device__ void root_thread(const RootArgs &a, int32_t r, int64_t vb, int L, uns
 #pragma unroll
             for (int p = 0; p < 4; ++p) {
                 const int64_t d = s1[p] - s0[p];
-                load4(a.ocol, s0[p], (p < L && d <= 16) ? (int)min(d, (int64_t)4) : 0, -2, u[p]);
+                load4(a.ocol, s0[p], (p < L && (kShort || d <= 16)) ? (int)min(d, (int64_t)4) : 0, -2, u[p]);
             }
         }
 #pragma unroll
@@ -330,7 +333,7 @@ __device__ void root_thread(const RootArgs &a, int32_t r, int64_t vb, int L, uns
             const int64_t d = s1[p] - s0[p];
             T += (unsigned long long)d;
             unsigned m = 0;  // positions c with V[c] in N+(V[p])
-            if (d <= 16) {
+            if (kShort || d <= 16) {
                 // the first four elements as independent loads (sparse out-rows are
                 // that short), so a row costs one load latency, not d of them
                 int32_t u0, u1, u2, u3;
@@ -348,10 +351,12 @@ __device__ void root_thread(const RootArgs &a, int32_t r, int64_t vb, int L, uns
 #pragma unroll
                 for (int c = 0; c < LM; ++c)
                     m |= (unsigned)((V[c] == u0) | (V[c] == u1) | (V[c] == u2) | (V[c] == u3)) << c;
-                for (int64_t q = s0[p] + 4; q < s1[p]; ++q) {
-                    const int32_t u = __ldg(a.ocol + q);
+                if constexpr (!kShort) {
+                    for (int64_t q = s0[p] + 4; q < s1[p]; ++q) {
+                        const int32_t u = __ldg(a.ocol + q);
 #pragma unroll
-                    for (int c = 0; c < LM; ++c) m |= (unsigned)(V[c] == u) << c;
+                        for (int c = 0; c < LM; ++c) m |= (unsigned)(V[c] == u) << c;
+                    }
                 }
             } else {
 #pragma unroll
@@ -421,15 +426,15 @@ __device__ void root_thread(const RootArgs &a, int32_t r, int64_t vb, int L, uns
     // materialise surviving roots: warp-aggregated slots for the three arrays
     const bool surv = cnt > 0;
     if (__any_sync(0xffffffffu, surv)) {
-        unsigned long long ts, tl, tc;
-        const unsigned long long os = warp_excl(surv ? 1ull : 0ull, ts);
-        const unsigned long long ol = warp_excl(surv ? (unsigned long long)L : 0ull, tl);
-        const unsigned long long oc = warp_excl((unsigned long long)cnt, tc);
+        unsigned ts, tl, tc;
+        const unsigned os = warp_excl(surv ? 1u : 0u, ts);
+        const unsigned ol = warp_excl(surv ? (unsigned)L : 0u, tl);
+        const unsigned oc = warp_excl((unsigned)cnt, tc);
         unsigned long long bs = 0, bl = 0, bc = 0;
         if ((threadIdx.x & 31) == 0) {
-            bs = atomicAdd(a.ctr + 0, ts);
-            bl = atomicAdd(a.ctr + 1, tl);
-            bc = atomicAdd(a.ctr + 2, tc);
+            bs = atomicAdd(a.ctr + 0, (unsigned long long)ts);
+            bl = atomicAdd(a.ctr + 1, (unsigned long long)tl);
+            bc = atomicAdd(a.ctr + 2, (unsigned long long)tc);
         }
         bs = __shfl_sync(0xffffffffu, bs, 0) + os;
         bl = __shfl_sync(0xffffffffu, bl, 0) + ol;
@@ -509,7 +514,7 @@ __global__ void __launch_bounds__(kRootWarps * 32, ROOT_SPARSE_BLOCKS) root_expa
         const int32_t r = i < a.count ? __ldg(a.list + i * a.stride) : -1;
         int64_t vb = 0, ve = 0;
         if (r >= 0) row_bounds(a.orp, r, vb, ve);
-        root_thread<4>(a, r, vb, (int)(ve - vb), bytes);
+        root_thread<4, true>(a, r, vb, (int)(ve - vb), bytes);
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) bytes += __shfl_xor_sync(0xffffffffu, bytes, o);
