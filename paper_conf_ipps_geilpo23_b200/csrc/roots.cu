@@ -504,14 +504,41 @@ __global__ void __launch_bounds__(kRootWarps * 32, 4) root_expand_w1(const RootA
 // of the orientation: sparse graphs such as BA m = 4 have degeneracy 4): only
 // the register-resident thread path, no queue, no barriers, and a register
 // budget cut for more resident roots (ROOT_SPARSE_BLOCKS blocks per SM).
+#ifndef ROOT_L4_PREFETCH
+#define ROOT_L4_PREFETCH 1  // measured: 0 / 1 = 50.3 / 49.8 us on ba1m
+#endif
 #ifndef ROOT_SPARSE_BLOCKS
 #define ROOT_SPARSE_BLOCKS 4  // measured: 4 / 5 / 6 blocks per SM = 52 / 69 / 93 us on ba1m (5, 6 spill)
 #endif
 __global__ void __launch_bounds__(kRootWarps * 32, ROOT_SPARSE_BLOCKS) root_expand_l4(const RootArgs a) {
     unsigned long long bytes = 0;  // algorithmic bytes read
+#if ROOT_L4_PREFETCH
+    // the next root id is loaded one iteration ahead (one latency off the
+    // chain); with ROOT_L4_PREFETCH 2 its row bounds too
+    const int64_t step = (int64_t)gridDim.x * blockDim.x;
+    int64_t in = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    int32_t rn = in < a.count ? __ldg(a.list + in * a.stride) : -1;
+#if ROOT_L4_PREFETCH == 2
+    int64_t vbn = 0, ven = 0;
+    if (rn >= 0) row_bounds(a.orp, rn, vbn, ven);
+#endif
+    for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < a.count; base += step) {
+        const int32_t r = rn;
+        in += step;
+        rn = in < a.count ? __ldg(a.list + in * a.stride) : -1;
+#if ROOT_L4_PREFETCH == 2
+        {
+            root_thread<4, true>(a, r, vbn, (int)(ven - vbn), bytes);
+            vbn = ven = 0;
+            if (rn >= 0) row_bounds(a.orp, rn, vbn, ven);
+            continue;
+        }
+#endif
+#else
     for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < a.count; base += (int64_t)gridDim.x * blockDim.x) {
         const int64_t i = base + threadIdx.x;
         const int32_t r = i < a.count ? __ldg(a.list + i * a.stride) : -1;
+#endif
         int64_t vb = 0, ve = 0;
         if (r >= 0) row_bounds(a.orp, r, vb, ve);
         root_thread<4, true>(a, r, vb, (int)(ve - vb), bytes);
