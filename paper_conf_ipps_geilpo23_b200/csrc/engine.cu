@@ -718,7 +718,8 @@ void Engine::do_class_w1(const int32_t *list, int64_t count) {
         for (int attempt = 0; attempt < 2; ++attempt) {
             MCE_CUDA(cudaMemsetAsync(ctr, 0, 8 * sizeof(unsigned long long), s_));
             const int t = clock_.start(2);
-            launch_root_expand_w1(ra, g_->max_out, s_);
+            // the sparse kernel takes 32-bit offsets into the oriented CSR
+            launch_root_expand_w1(ra, g_->nnz / 2 < INT32_MAX ? g_->max_out : 64, s_);
             clock_.stop(t);
             ++kernels_;
             ++root_launches_;

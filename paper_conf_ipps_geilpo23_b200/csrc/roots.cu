@@ -22,6 +22,7 @@
 //
 // On sparse graphs almost every root is pruned in step 3, so the level-1
 // frontier and the adjacency of pruned roots never touch HBM.
+#include <type_traits>
 #include "expand.cuh"
 
 namespace mce {
@@ -297,7 +298,7 @@ __device__ __forceinline__ void load4(const int32_t *__restrict__ col, int64_t s
 template <int LM, bool kShort = false>
 __device__ void root_thread(const RootArgs &a, int32_t r, int64_t vb, int L, unsigned long long &bytes) {
     uint64_t adj = 0;
-    unsigned long long T = 0;
+    typename std::conditional<kShort, unsigned, unsigned long long>::type T = 0;
     if (r < 0) {
         vb = 0;
         L = 0;
@@ -310,11 +311,18 @@ __device__ void root_thread(const RootArgs &a, int32_t r, int64_t vb, int L, uns
 #pragma unroll
             for (int p = 0; p < LM; ++p) V[p] = p < L ? __ldg(a.ocol + vb + p) : -1;
         }
-        int64_t s0[LM], s1[LM];
+        // kShort launches also guarantee |E+| < 2^31 (engine.cu): 32-bit offsets
+        using Off = typename std::conditional<kShort, int32_t, int64_t>::type;
+        Off s0[LM], s1[LM];
 #pragma unroll
         for (int p = 0; p < LM; ++p) {
             s0[p] = s1[p] = 0;
-            if (p < L) row_bounds(a.orp, V[p], s0[p], s1[p]);
+            if (p < L) {
+                int64_t b, e;
+                row_bounds(a.orp, V[p], b, e);
+                s0[p] = (Off)b;
+                s1[p] = (Off)e;
+            }
         }
         // LM == 4 (sparse roots): the first four elements of every out-row,
         // all issued before any is used, so the adjacency costs one load
@@ -323,15 +331,15 @@ __device__ void root_thread(const RootArgs &a, int32_t r, int64_t vb, int L, uns
         if constexpr (LM == 4) {
 #pragma unroll
             for (int p = 0; p < 4; ++p) {
-                const int64_t d = s1[p] - s0[p];
-                load4(a.ocol, s0[p], (p < L && (kShort || d <= 16)) ? (int)min(d, (int64_t)4) : 0, -2, u[p]);
+                const Off d = s1[p] - s0[p];
+                load4(a.ocol, s0[p], (p < L && (kShort || d <= 16)) ? (int)min(d, (Off)4) : 0, -2, u[p]);
             }
         }
 #pragma unroll
         for (int p = 0; p < LM; ++p) {
             if (p >= L) break;
             const int64_t d = s1[p] - s0[p];
-            T += (unsigned long long)d;
+            T += d;
             unsigned m = 0;  // positions c with V[c] in N+(V[p])
             if (kShort || d <= 16) {
                 // the first four elements as independent loads (sparse out-rows are
