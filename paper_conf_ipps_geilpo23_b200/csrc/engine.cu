@@ -673,28 +673,42 @@ void Engine::do_class_w1(const int32_t *list, int64_t count) {
     if (mine <= 0) return;
     W_ = 1;
     const int32_t *base = list;
-    int32_t *len = arena_.alloc<int32_t>(mine);
-    int64_t *prefix = arena_.alloc<int64_t>(mine + 1);
-    int64_t *tmp = arena_.alloc<int64_t>(scan_tmp_items(mine));
-    int64_t *win = arena_.alloc<int64_t>(2);
     unsigned long long *ctr = arena_.alloc<unsigned long long>(8);
-    launch_root_lengths(base, mine, 1, g_->orp.get(), len, s_);
-    exclusive_scan_i32(len, prefix, mine, tmp, s_);
-    kernels_ += 4;
     // per candidate row: adjacency word + one level-2 entry (P, slot, parent, vloc)
     const int64_t row_bytes = 8 + 8 + 12;
     const int64_t per_root = sizeof(RootInfo) + 64;
+    // Sparse orientation (every |N+(r)| <= 4, no window requested): when
+    // max_out rows per root fit, the whole class is one window sized by that
+    // bound, with no row-count pass, scan or read-back
+    const bool one_window = o_.window <= 0 && g_->max_out <= 4 &&
+                            (int64_t)(arena_.avail() / 3) >= mine * (per_root + row_bytes * std::max(g_->max_out, 1));
+    int64_t *prefix = nullptr, *win = nullptr;
+    if (!one_window) {
+        int32_t *len = arena_.alloc<int32_t>(mine);
+        prefix = arena_.alloc<int64_t>(mine + 1);
+        int64_t *tmp = arena_.alloc<int64_t>(scan_tmp_items(mine));
+        win = arena_.alloc<int64_t>(2);
+        launch_root_lengths(base, mine, 1, g_->orp.get(), len, s_);
+        exclusive_scan_i32(len, prefix, mine, tmp, s_);
+        kernels_ += 4;
+    }
     int64_t hi = mine;
     while (hi > 0) {
         const Arena::Mark mark = arena_.mark();
-        const int64_t room = (int64_t)(arena_.avail() / 3);
-        const int64_t maxw = o_.window > 0 ? o_.window : hi;
-        launch_find_window(prefix, hi, std::max<int64_t>(0, hi - maxw), room, row_bytes, per_root, win, s_);
-        ++kernels_;
-        int64_t *hw = g_->host.get<int64_t>(2);
-        MCE_CUDA(cudaMemcpyAsync(hw, win, 2 * sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
-        stream_sync(s_);
-        const int64_t lo = hw[0], rows = hw[1];
+        int64_t lo = 0, rows = 0;
+        if (one_window) {
+            rows = mine * std::max(g_->max_out, 1);
+        } else {
+            const int64_t room = (int64_t)(arena_.avail() / 3);
+            const int64_t maxw = o_.window > 0 ? o_.window : hi;
+            launch_find_window(prefix, hi, std::max<int64_t>(0, hi - maxw), room, row_bytes, per_root, win, s_);
+            ++kernels_;
+            int64_t *hw = g_->host.get<int64_t>(2);
+            MCE_CUDA(cudaMemcpyAsync(hw, win, 2 * sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
+            stream_sync(s_);
+            lo = hw[0];
+            rows = hw[1];
+        }
         const int64_t nw = hi - lo;
         RootArgs ra{};
         ra.list = base + lo;
