@@ -70,6 +70,10 @@ __global__ void build_adj_w1(const RootInfo *__restrict__ roots, int64_t nroots,
 // the spans are short); otherwise binary search in the staged V.  Bits go to
 // a shared-memory bit matrix when it fits (SMEM), else straight to the
 // (zeroed) global matrix.
+#ifndef ADJ_CHUNKS
+#define ADJ_CHUNKS 4
+#endif
+constexpr int kAdjChunks = ADJ_CHUNKS;
 constexpr int kSpanBits = 1 << 18;
 constexpr int kSpanWords = kSpanBits / 32;
 template <bool SMEM>
@@ -110,10 +114,23 @@ __global__ void build_adj_block(const RootInfo *__restrict__ roots, int64_t nroo
         for (int i = wib; i < L; i += nwb) {
             const int32_t a = sV[i];
             const int64_t pb = __ldg(orp + a), pe = __ldg(orp + a + 1);
-            for (int64_t p0 = pb; p0 < pe; p0 += 32) {
-                const int64_t p = p0 + lane;
-                const int32_t u = p < pe ? __ldg(ocol + p) : INT32_MAX;
-                if (__shfl_sync(0xffffffffu, u, 0) > vmax) break;
+            // kAdjChunks chunks of 32 ids loaded before any is looked up (the
+            // row scan is bound by its load latency, one chunk per trip)
+            bool stop = false;
+            for (int64_t q0 = pb; q0 < pe && !stop; q0 += 32 * kAdjChunks) {
+              int32_t uu[kAdjChunks];
+#pragma unroll
+              for (int k = 0; k < kAdjChunks; ++k) {
+                  const int64_t p = q0 + 32 * k + lane;
+                  uu[k] = p < pe ? __ldg(ocol + p) : INT32_MAX;
+              }
+#pragma unroll
+              for (int k = 0; k < kAdjChunks; ++k) {
+                const int32_t u = uu[k];
+                if (__shfl_sync(0xffffffffu, u, 0) > vmax) {
+                    stop = true;
+                    break;
+                }
                 int c = -1;
                 if (map) {
                     if (u >= vmin && u <= vmax) {
@@ -137,6 +154,7 @@ __global__ void build_adj_block(const RootInfo *__restrict__ roots, int64_t nroo
                     atomicOr(A + (int64_t)li * 2 * W + (lc >> 5), 1u << (lc & 31));
                     atomicOr(A + (int64_t)lc * 2 * W + (li >> 5), 1u << (li & 31));
                 }
+              }
             }
         }
         __syncthreads();
