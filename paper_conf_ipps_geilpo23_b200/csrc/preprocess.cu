@@ -343,7 +343,7 @@ struct Tile {
 // the start of v's own undirected row in `stage` (rowptr-indexed), their
 // number at odeg[pid[v]]; orient_copy moves them to the oriented CSR once the
 // out-degrees are scanned (one gather pass over rank/pid instead of two)
-template <int G>
+template <int G, int KL>
 __device__ void stage_one(int64_t v, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
                           const int32_t *__restrict__ rank, const int32_t *__restrict__ pid, int32_t *odeg,
                           int32_t *stage) {
@@ -351,18 +351,31 @@ __device__ void stage_one(int64_t v, const int64_t *__restrict__ rowptr, const i
     const int32_t r = rank[v];
     const int64_t eb = rowptr[v], ee = rowptr[v + 1];
     int64_t out = eb;
-    for (int64_t e0 = eb; e0 < ee; e0 += G) {
-        const int64_t e = e0 + t.gl;
-        const int32_t u = e < ee ? col[e] : 0;
-        const bool up = e < ee && rank[u] > r;
-        const unsigned m = t.ballot(up);
-        if (up) stage[out + __popc(m & t.lt())] = pid[u];
-        out += __popc(m);
+    // whole warps (long rows): KL chunks' ids and ranks gathered before any
+    // is used, so a long row costs one gather latency per KL chunks
+    constexpr int K = G == 32 ? KL : 1;
+    for (int64_t e0 = eb; e0 < ee; e0 += G * K) {
+        int32_t u[K];
+        bool up[K];
+#pragma unroll
+        for (int k = 0; k < K; ++k) {
+            const int64_t e = e0 + G * k + t.gl;
+            u[k] = e < ee ? col[e] : 0;
+        }
+#pragma unroll
+        for (int k = 0; k < K; ++k) up[k] = e0 + G * k + t.gl < ee && rank[u[k]] > r;
+#pragma unroll
+        for (int k = 0; k < K; ++k) {
+            const unsigned m = t.ballot(up[k]);
+            if (up[k]) stage[out + __popc(m & t.lt())] = pid[u[k]];
+            out += __popc(m);
+        }
     }
     if (t.gl == 0) odeg[pid[v]] = (int32_t)(out - eb);
 }
 
 // Warp w takes vertices [4w, 4w+4): 8-lane tiles when all four have degree <= 64, else a warp each
+template <int KL>
 __global__ void __launch_bounds__(256) orient_stage_kernel(int64_t n, const int64_t *__restrict__ rowptr,
                                                            const int32_t *__restrict__ col,
                                                            const int32_t *__restrict__ rank,
@@ -375,9 +388,9 @@ __global__ void __launch_bounds__(256) orient_stage_kernel(int64_t n, const int6
         const int64_t v = v0 + (lane >> 3);
         const int64_t d = v < n ? rowptr[v + 1] - rowptr[v] : 0;
         if (__all_sync(0xffffffffu, d <= 64)) {
-            if (v < n) stage_one<8>(v, rowptr, col, rank, pid, odeg, stage);
+            if (v < n) stage_one<8, 1>(v, rowptr, col, rank, pid, odeg, stage);
         } else {
-            for (int t = 0; t < 4 && v0 + t < n; ++t) stage_one<32>(v0 + t, rowptr, col, rank, pid, odeg, stage);
+            for (int t = 0; t < 4 && v0 + t < n; ++t) stage_one<32, KL>(v0 + t, rowptr, col, rank, pid, odeg, stage);
         }
         __syncwarp();
     }
@@ -652,7 +665,15 @@ void orient(mce_graph *g, int orientation) {
     }
     int32_t *odeg = g->pool.take<int32_t>(n);
     int32_t *stage = g->pool.take<int32_t>(std::max<int64_t>(g->nnz, 1));
-    orient_stage_kernel<<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), g->rank.get(),
+    // Long rows (degree > 64, a warp each) gather 4 chunks per trip when they
+    // are rare (mean degree <= 16: ba1m preprocessing 1.27 -> 1.17 ms); with
+    // many (rmat22, mean 31) the wider gathers slow the greedy heuristic that
+    // runs beside this pass more than they gain (step 82.6 -> 88-93 ms)
+    if (g->nnz <= 16 * n)
+        orient_stage_kernel<4><<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), g->rank.get(),
+                                                              g->pid.get(), odeg, stage);
+    else
+        orient_stage_kernel<1><<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), g->rank.get(),
                                                               g->pid.get(), odeg, stage);
     MCE_LAUNCH_CHECK();
     exclusive_scan_i32(odeg, g->orp.get(), n, g->pool.take<int64_t>(scan_tmp_items(n)), s);
