@@ -56,7 +56,10 @@ constexpr int kPeelThreads = 1024;  // launch bound; the launch uses kcore_threa
 // Work items are int64 (vertex | chunk << 32), -1 = empty; levels alternate
 // between two lists so one can be cleared while the other fills.
 // ---------------------------------------------------------------------------
-constexpr int64_t kChunk = 128;  // edges per work item
+#ifndef KCORE_CHUNK
+#define KCORE_CHUNK 32  // measured: 128 / 64 / 32 / 16 / 8 = ba1m 1.49 / 1.46 / 1.43 / 1.44 / 1.50 ms, rmat22 82.5 / 81.8 / 82.1 / 81.4 / - ms
+#endif
+constexpr int64_t kChunk = KCORE_CHUNK;  // edges per work item
 
 __device__ __forceinline__ unsigned long long ld_relaxed(const unsigned long long *p) {
     unsigned long long v;
