@@ -56,6 +56,9 @@ constexpr int kPeelThreads = 1024;  // launch bound; the launch uses kcore_threa
 // Work items are int64 (vertex | chunk << 32), -1 = empty; levels alternate
 // between two lists so one can be cleared while the other fills.
 // ---------------------------------------------------------------------------
+#ifndef ORIENT_KL
+#define ORIENT_KL 4
+#endif
 #ifndef KCORE_CHUNK
 #define KCORE_CHUNK 32  // measured: 128 / 64 / 32 / 16 / 8 = ba1m 1.49 / 1.46 / 1.43 / 1.44 / 1.50 ms, rmat22 82.5 / 81.8 / 82.1 / 81.4 / - ms
 #endif
@@ -673,7 +676,7 @@ void orient(mce_graph *g, int orientation) {
     // many (rmat22, mean 31) the wider gathers slow the greedy heuristic that
     // runs beside this pass more than they gain (step 82.6 -> 88-93 ms)
     if (g->nnz <= 16 * n)
-        orient_stage_kernel<4><<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), g->rank.get(),
+        orient_stage_kernel<ORIENT_KL><<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), g->rank.get(),
                                                               g->pid.get(), odeg, stage);
     else
         orient_stage_kernel<1><<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), g->rank.get(),
