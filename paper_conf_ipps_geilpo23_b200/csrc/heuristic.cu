@@ -227,7 +227,10 @@ __device__ int32_t greedy_run(int32_t s, const int64_t *__restrict__ rowptr, con
 // and an order-preserving in-place compaction.  Hub seeds (degree > kBigSeed)
 // run this way so a long run is not serialised on one warp; the replay of the
 // winning run uses it too, writing the clique (in order added).
-constexpr int kBlockRun = 512;
+#ifndef BLOCK_RUN
+#define BLOCK_RUN 512  // measured on rmat22: 256 / 512 / 1024 threads = 95.4 / 81.8 / 90.7 ms per step
+#endif
+constexpr int kBlockRun = BLOCK_RUN;
 constexpr int64_t kBigSeed = 1024;
 template <int NT>
 __device__ int32_t block_run(int32_t s, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
