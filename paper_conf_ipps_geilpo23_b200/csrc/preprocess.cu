@@ -59,6 +59,9 @@ constexpr int kPeelThreads = 1024;  // launch bound; the launch uses kcore_threa
 #ifndef ORIENT_KL
 #define ORIENT_KL 4
 #endif
+#ifndef KCORE_OVL_PCT
+#define KCORE_OVL_PCT 50  // percent of the SMs the peel takes beside the heuristic; measured 35 / 50 / 65 = ba1m 1.51 / 1.43 / 1.49 ms, rmat22 81.5 / 81.7 / 83.9 ms
+#endif
 #ifndef KCORE_CHUNK
 #define KCORE_CHUNK 32  // measured: 128 / 64 / 32 / 16 / 8 = ba1m 1.49 / 1.46 / 1.43 / 1.44 / 1.50 ms, rmat22 82.5 / 81.8 / 82.1 / 81.4 / - ms
 #endif
@@ -586,7 +589,7 @@ void kcore(mce_graph *g) {
     int blocks_per_sm = 0;
     MCE_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm, kcore_async, threads, 0));
     if (blocks_per_sm < 1) fail(2, "kcore: cooperative kernel does not fit an SM");
-    const int grid = half ? std::max(1, num_sms() / 2) : num_sms();
+    const int grid = half ? std::max(1, num_sms() * KCORE_OVL_PCT / 100) : num_sms();
     int64_t n_arg = n;
     const int64_t *rp = g->rowptr.get();
     const int32_t *cl = g->col.get();
