@@ -9,6 +9,7 @@ follows and tests/test_oracle.py for the pins.
 
 from .oracle import (  # noqa: F401
     build,
+    count_max_cliques,
     core_numbers,
     default_threshold,
     greedy,

@@ -236,12 +236,18 @@ typedef struct {
     int32_t *out;      /* found cliques of size best, flat */
     int64_t out_count;
     int64_t out_cap;
+    int32_t count_only; /* 1: count the cliques of size best, store none */
+    int32_t tight;      /* 1: apply the tight-node rule (see expand) */
 } mce_ctx;
 
 static void record(mce_ctx *x, int32_t size) {
     if (size > x->best) {
         x->best = size;
         x->out_count = 0;
+    }
+    if (x->count_only) {
+        x->out_count++;
+        return;
     }
     if ((x->out_count + 1) * (int64_t)size > x->out_cap) {
         int64_t cap = x->out_cap ? x->out_cap * 2 : 1024;
@@ -267,6 +273,29 @@ static void expand(mce_ctx *x, int32_t csize) {
     int32_t *ord = x->ord + (int64_t)csize * x->L;
     int32_t *colr = x->colr + (int64_t)csize * x->L;
     int32_t np = 0;
+    if (x->tight && popcount_set(P, W) + csize == x->best) {
+        /* Tight node (a direct consequence of the |C|+|P| bound, II-B-3 line
+         * 63): every clique below (C, P) is C + S with S a clique inside P, so
+         * the only one that can have the size sought, |C| + |P|, is C + P
+         * itself -- a maximum clique iff P is a clique.  Checked pair by pair
+         * instead of expanding the |P| levels of single-child branches. */
+        int32_t k = csize;
+        for (int32_t w = 0; w < W; ++w) {
+            uint64_t b = P[w];
+            while (b) {
+                int32_t v = w * 64 + __builtin_ctzll(b);
+                b &= b - 1;
+                for (int32_t j = 0; j < W; ++j) {
+                    uint64_t miss = P[j] & ~x->A[(int64_t)v * W + j];
+                    if (j == (v >> 6)) miss &= ~(1ULL << (v & 63));
+                    if (miss) return; /* P is not a clique: nothing of size best here */
+                }
+                x->stack[k++] = x->V[x->L - 1 - v];
+            }
+        }
+        record(x, k);
+        return;
+    }
     if (x->bound == 1) { /* greedy sequential colouring of P */
         uint64_t *U = x->scratch, *S = x->scratch + W;
         memcpy(U, P, sizeof(uint64_t) * W);
@@ -334,10 +363,15 @@ static int32_t g_res_omega = 0;
 
 /* Returns the number of maximum cliques; *omega_out = clique number.
  * lb: initial lower bound (0 = none).  bound: 0 = |C|+|P|, 1 = colouring.
+ * flags bit 0 (count_only): count the maximum cliques without storing them
+ * (graphs whose multiplicity does not fit in memory, e.g. R-MAT scale 22);
+ * bit 1 (tight): apply the tight-node rule of expand() (same answer, fewer
+ * levels on long single-child chains).
  * The cliques are kept until oracle_mce_fetch() copies them out.
  * Returns -1 if some root has more than 65536 later neighbours. */
-int64_t oracle_mce(int64_t n, const int64_t *rowptr, const int32_t *col, int32_t lb, int32_t bound,
-                   int32_t *omega_out) {
+int64_t oracle_mce_ex(int64_t n, const int64_t *rowptr, const int32_t *col, int32_t lb, int32_t bound,
+                      int32_t flags, int32_t *omega_out) {
+    const int32_t count_only = flags & 1, tight = (flags >> 1) & 1;
     free(g_res);
     g_res = NULL;
     g_res_count = 0;
@@ -386,6 +420,8 @@ int64_t oracle_mce(int64_t n, const int64_t *rowptr, const int32_t *col, int32_t
     memset(&x, 0, sizeof(x));
     x.best = lb > 1 ? lb : 1;
     x.bound = bound;
+    x.count_only = count_only;
+    x.tight = tight;
     uint64_t *A = (uint64_t *)malloc(sizeof(uint64_t) * (maxout + 1) * Wmax);
     x.stack = (int32_t *)malloc(sizeof(int32_t) * (maxout + 2));
     x.pool = (uint64_t *)malloc(sizeof(uint64_t) * (maxout + 3) * Wmax);
@@ -432,6 +468,14 @@ int64_t oracle_mce(int64_t n, const int64_t *rowptr, const int32_t *col, int32_t
     }
     int32_t k = x.best;
     if (x.out_count == 0) k = 0; /* lb was above omega: nothing of size >= lb */
+    if (count_only) {
+        *omega_out = k;
+        g_res_count = x.out_count;
+        g_res_omega = k;
+        free(A); free(x.stack); free(x.pool); free(x.ord); free(x.colr); free(x.scratch);
+        free(core); free(order); free(pos); free(loc); free(orp); free(ocol);
+        return g_res_count;
+    }
     for (int64_t c = 0; c < x.out_count; ++c) qsort(x.out + c * k, (size_t)k, sizeof(int32_t), cmp_i32);
     g_k = k;
     if (k > 0) qsort(x.out, (size_t)x.out_count, sizeof(int32_t) * k, cmp_clique);
@@ -442,6 +486,11 @@ int64_t oracle_mce(int64_t n, const int64_t *rowptr, const int32_t *col, int32_t
     free(A); free(x.stack); free(x.pool); free(x.ord); free(x.colr); free(x.scratch);
     free(core); free(order); free(pos); free(loc); free(orp); free(ocol);
     return g_res_count;
+}
+
+int64_t oracle_mce(int64_t n, const int64_t *rowptr, const int32_t *col, int32_t lb, int32_t bound,
+                   int32_t *omega_out) {
+    return oracle_mce_ex(n, rowptr, col, lb, bound, 0, omega_out);
 }
 
 /* Copy the cliques of the last oracle_mce() call (count * omega int32). */
@@ -496,4 +545,149 @@ int32_t oracle_kclique_counts(int64_t n, const int64_t *rowptr, const int32_t *c
     for (int32_t k = 0; k < kmax; ++k)
         if (counts[k]) top = k + 1;
     return top;
+}
+
+/* ------------------------------------------------------------------------ */
+/* oracle_mce_plain -- the SAME problem (PAPER.md II line 47: omega and all   */
+/* cliques of size omega) by the most literal form of the basic branching    */
+/* algorithm of II-A (lines 51-53) with the "most straightforward" bound of  */
+/* II-B-3 (line 63: "the size of C plus the size of P").  It is written to   */
+/* share nothing with oracle_mce above, nor with the CUDA path: no k-core,   */
+/* no orientation by rank, no bitsets, no local index space, no colouring.   */
+/*                                                                            */
+/* A vertex order "<" is fixed first: plain vertex id (order = 0), or the    */
+/* paper's own orientation of IV-C (line 131: "keep the edge where the       */
+/* source vertex has lower degree"; order = 1: by (degree, id)).             */
+/*   for every vertex v in that order:  C = {v},  P = {u in N(v) : u > v}     */
+/*   EXPAND(C, P): for the i-th vertex w of P (ascending id):                 */
+/*       if |C| + (|P| - i) < best: stop  (C + the vertices of P from w on    */
+/*                                         cannot reach best)                 */
+/*       Q = {u in P : u > w, u adjacent to w}   (list in "<" order, edge     */
+/*                                 test by binary search in w's CSR row)     */
+/*       Q empty  -> C + w is a clique no later vertex extends: note it       */
+/*       else     -> EXPAND(C + w, Q)                                         */
+/*                                                                            */
+/* Every clique K = {k1 < ... < kt} is visited exactly once (root k1, then   */
+/* k2, ...), and a maximum clique is always a leaf, so the cliques noted at   */
+/* the final best size are exactly the maximum cliques.  Pruning is strict   */
+/* (<), so cliques of size equal to best survive.                            */
+/* count_only = 1 counts instead of storing.  Results are read back with     */
+/* oracle_mce_fetch (same canonical order as oracle_mce).                    */
+/* ------------------------------------------------------------------------ */
+typedef struct {
+    const int64_t *rowptr;
+    const int32_t *col;
+    int32_t best;
+    int32_t count_only;
+    int32_t *C;         /* current clique, vertex ids */
+    int32_t **lists;    /* one candidate list per depth */
+    int32_t *out;
+    int64_t out_count;
+    int64_t out_cap;
+} plain_ctx;
+
+static void plain_note(plain_ctx *x, int32_t size) {
+    if (size < x->best) return;
+    if (size > x->best) {
+        x->best = size;
+        x->out_count = 0;
+    }
+    if (!x->count_only) {
+        if ((x->out_count + 1) * (int64_t)size > x->out_cap) {
+            int64_t cap = x->out_cap ? x->out_cap * 2 : 1024;
+            while ((x->out_count + 1) * (int64_t)size > cap) cap *= 2;
+            x->out = (int32_t *)realloc(x->out, sizeof(int32_t) * cap);
+            x->out_cap = cap;
+        }
+        memcpy(x->out + x->out_count * size, x->C, sizeof(int32_t) * size);
+    }
+    x->out_count++;
+}
+
+static void plain_expand(plain_ctx *x, int32_t csize, const int32_t *P, int64_t np) {
+    int32_t *Q = x->lists[csize + 1];
+    for (int64_t i = 0; i < np; ++i) {
+        if (csize + (np - i) < x->best) return;
+        int32_t w = P[i];
+        x->C[csize] = w;
+        int64_t nq = 0;
+        for (int64_t j = i + 1; j < np; ++j)
+            if (has_edge(x->rowptr, x->col, w, P[j])) Q[nq++] = P[j];
+        if (nq == 0)
+            plain_note(x, csize + 1);
+        else
+            plain_expand(x, csize + 1, Q, nq);
+    }
+}
+
+static const int64_t *g_rank;
+static int cmp_by_rank(const void *a, const void *b) {
+    int64_t x = g_rank[*(const int32_t *)a], y = g_rank[*(const int32_t *)b];
+    return (x > y) - (x < y);
+}
+
+int64_t oracle_mce_plain(int64_t n, const int64_t *rowptr, const int32_t *col, int32_t lb,
+                         int32_t order, int32_t count_only, int32_t *omega_out) {
+    free(g_res);
+    g_res = NULL;
+    g_res_count = 0;
+    g_res_omega = 0;
+    if (n == 0) { /* the empty clique is the only clique of the null graph */
+        *omega_out = 0;
+        g_res_count = 1;
+        return 1;
+    }
+    int64_t maxdeg = 0;
+    for (int64_t v = 0; v < n; ++v)
+        if (rowptr[v + 1] - rowptr[v] > maxdeg) maxdeg = rowptr[v + 1] - rowptr[v];
+    plain_ctx x;
+    memset(&x, 0, sizeof(x));
+    x.rowptr = rowptr;
+    x.col = col;
+    x.best = lb > 1 ? lb : 1;
+    x.count_only = count_only;
+    /* rank[v] = position of v in the order "<": key (degree, id) or id */
+    int64_t *rank = (int64_t *)malloc(sizeof(int64_t) * n);
+    for (int64_t v = 0; v < n; ++v) rank[v] = order == 1 ? (rowptr[v + 1] - rowptr[v]) * n + v : v;
+    x.C = (int32_t *)malloc(sizeof(int32_t) * (maxdeg + 2));
+    x.lists = (int32_t **)malloc(sizeof(int32_t *) * (maxdeg + 3));
+    for (int64_t d = 0; d < maxdeg + 3; ++d) x.lists[d] = NULL;
+    for (int64_t v = 0; v < n; ++v) {
+        int64_t np = 0;
+        for (int64_t e = rowptr[v]; e < rowptr[v + 1]; ++e) np += rank[col[e]] > rank[v];
+        if (1 + np < x.best) continue;
+        x.C[0] = (int32_t)v;
+        if (np == 0) {
+            plain_note(&x, 1);
+            continue;
+        }
+        /* lists are allocated lazily, one per depth, each of the root's size */
+        for (int64_t d = 1; d <= np + 1; ++d)
+            if (!x.lists[d]) x.lists[d] = (int32_t *)malloc(sizeof(int32_t) * (maxdeg + 1));
+        int32_t *P = x.lists[1];
+        np = 0;
+        for (int64_t e = rowptr[v]; e < rowptr[v + 1]; ++e)
+            if (rank[col[e]] > rank[v]) P[np++] = col[e];
+        g_rank = rank;
+        qsort(P, (size_t)np, sizeof(int32_t), cmp_by_rank);
+        plain_expand(&x, 1, P, np);
+    }
+    int32_t k = x.best;
+    if (x.out_count == 0) k = 0;
+    if (!count_only) {
+        for (int64_t c = 0; c < x.out_count; ++c) qsort(x.out + c * k, (size_t)k, sizeof(int32_t), cmp_i32);
+        g_k = k;
+        if (k > 0) qsort(x.out, (size_t)x.out_count, sizeof(int32_t) * k, cmp_clique);
+        g_res = x.out;
+    } else {
+        free(x.out);
+    }
+    g_res_count = x.out_count;
+    g_res_omega = k;
+    *omega_out = k;
+    for (int64_t d = 0; d < maxdeg + 3; ++d) free(x.lists[d]);
+    free(x.lists);
+    free(x.C);
+    free(rank);
+    return g_res_count;
 }

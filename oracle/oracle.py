@@ -39,6 +39,12 @@ def _load():
         lib.oracle_greedy.argtypes = [ctypes.c_int64, _i64p, _i32p, _i64p, ctypes.c_int64, _i32p, _i32p]
         lib.oracle_mce.restype = ctypes.c_int64
         lib.oracle_mce.argtypes = [ctypes.c_int64, _i64p, _i32p, ctypes.c_int32, ctypes.c_int32, _i32p]
+        lib.oracle_mce_ex.restype = ctypes.c_int64
+        lib.oracle_mce_ex.argtypes = [ctypes.c_int64, _i64p, _i32p, ctypes.c_int32, ctypes.c_int32,
+                                      ctypes.c_int32, _i32p]
+        lib.oracle_mce_plain.restype = ctypes.c_int64
+        lib.oracle_mce_plain.argtypes = [ctypes.c_int64, _i64p, _i32p, ctypes.c_int32, ctypes.c_int32,
+                                         ctypes.c_int32, _i32p]
         lib.oracle_mce_fetch.restype = None
         lib.oracle_mce_fetch.argtypes = [_i32p]
         lib.oracle_kclique_counts.restype = ctypes.c_int32
@@ -86,24 +92,56 @@ def greedy(rowptr, col, threshold, h: int) -> Tuple[int, np.ndarray, np.ndarray]
     return int(w), runs[:h], best[:w]
 
 
-def max_cliques(rowptr, col, lb: int = 0, bound: str = "color") -> Tuple[int, np.ndarray]:
+def max_cliques(rowptr, col, lb: int = 0, bound: str = "color", tight: bool = False) -> Tuple[int, np.ndarray]:
     """(omega, all maximum cliques as a sorted int32 [count, omega] array).
 
     bound: "size" = |C|+|P| (PAPER.md II-B-3 first option), "color" = greedy
-    colouring bound (II-B-3 "tighter upper bound ... vertex coloring").
+    colouring bound (II-B-3 "tighter upper bound ... vertex coloring"), both
+    on oracle_mce's degeneracy-ordered bitset search; "plain" = oracle_mce_plain,
+    the literal list-based II-A search with the |C|+|P| bound over the
+    paper's degree orientation (IV-C, line 131), "plain_id" the same in
+    vertex-id order (no k-core, no bitsets, no colouring: independent of
+    both the other oracle and the CUDA path's layout).
     """
     rowptr, col = _csr(rowptr, col)
     n = rowptr.size - 1
     lib = _load()
     om = ctypes.c_int32(0)
-    b = {"size": 0, "color": 1}[bound]
-    cnt = lib.oracle_mce(n, _p64(rowptr), _p32(col), int(lb), b, ctypes.byref(om))
+    if bound in ("plain", "plain_id"):
+        cnt = lib.oracle_mce_plain(n, _p64(rowptr), _p32(col), int(lb), int(bound == "plain"), 0,
+                                   ctypes.byref(om))
+    else:
+        b = {"size": 0, "color": 1}[bound]
+        cnt = lib.oracle_mce_ex(n, _p64(rowptr), _p32(col), int(lb), b, 2 * int(tight), ctypes.byref(om))
     if cnt < 0:
         raise ValueError("oracle: a vertex has more than 65536 later neighbours")
     omega = int(om.value)
     out = np.zeros((cnt, omega), dtype=np.int32)
     lib.oracle_mce_fetch(_p32(out) if out.size else None)
     return omega, out
+
+
+def count_max_cliques(rowptr, col, lb: int = 0, bound: str = "color", tight: bool = False) -> Tuple[int, int]:
+    """(omega, multiplicity) without storing the cliques (count-only mode).
+
+    Same searches as max_cliques; for graphs whose maximum cliques do not fit
+    in host memory (R-MAT scale 22: 3 * 2^26 cliques of 223 vertices).
+    tight (colour / size bounds only): stop at a node where |C| + |P| equals
+    the size sought and test P for being a clique (mce_oracle.c expand()).
+    """
+    rowptr, col = _csr(rowptr, col)
+    n = rowptr.size - 1
+    lib = _load()
+    om = ctypes.c_int32(0)
+    if bound in ("plain", "plain_id"):
+        cnt = lib.oracle_mce_plain(n, _p64(rowptr), _p32(col), int(lb), int(bound == "plain"), 1,
+                                   ctypes.byref(om))
+    else:
+        b = {"size": 0, "color": 1}[bound]
+        cnt = lib.oracle_mce_ex(n, _p64(rowptr), _p32(col), int(lb), b, 1 | (2 * int(tight)), ctypes.byref(om))
+    if cnt < 0:
+        raise ValueError("oracle: a vertex has more than 65536 later neighbours")
+    return int(om.value), int(cnt)
 
 
 def kclique_counts(rowptr, col, kmax: int) -> np.ndarray:

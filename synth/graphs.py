@@ -247,6 +247,19 @@ def plant_cliques(g: Graph, count: int, size: int, seed: int) -> Graph:
     return out
 
 
+def cocktail_party_join(j: int, t: int, seed: int) -> Graph:
+    """Cocktail-party graph CP(j) (K_2j minus a perfect matching) joined with K_t,
+    vertex ids permuted with a seeded permutation.  Closed form (test pin):
+    omega = j + t with 2^j maximum cliques (one vertex of every non-adjacent
+    pair), the structure of the R-MAT hub core."""
+    n = 2 * j + t
+    u, v = np.triu_indices(n, 1)
+    keep = ~((u < 2 * j) & (v < 2 * j) & (u // 2 == v // 2))
+    perm = torch.argsort(rand_u64(seed, 7, torch.arange(n, dtype=torch.int64))).numpy()
+    return from_edges(n, torch.from_numpy(perm[u[keep]].astype(np.int64)),
+                      torch.from_numpy(perm[v[keep]].astype(np.int64)), name=f"CP({j})+K{t}")
+
+
 def barabasi_albert(n: int, m: int, seed: int) -> Graph:
     """Barabasi-Albert preferential attachment (networkx-style, sequential).
 

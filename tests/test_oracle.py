@@ -19,7 +19,7 @@ from synth import graphs as G
 from tests import bruteforce as bf
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-BOUNDS = ["size", "color"]
+BOUNDS = ["size", "color", "plain", "plain_id"]  # oracle_mce (two bounds), oracle_mce_plain (two orders)
 
 
 def csr_from_edges(n, edges):
@@ -71,13 +71,17 @@ def test_core_numbers_vs_definition(seed):
     assert sorted(order.tolist()) == list(range(n))
 
 
-def test_lower_bound_does_not_change_answer():
+@pytest.mark.parametrize("bound", BOUNDS)
+def test_lower_bound_does_not_change_answer(bound):
     edges = random_small_graph(16, 0.6, 7)
     rp, col = csr_from_edges(16, edges)
     om, cl = oracle.max_cliques(rp, col)
     for lb in range(0, om + 1):
-        om2, cl2 = oracle.max_cliques(rp, col, lb=lb)
+        om2, cl2 = oracle.max_cliques(rp, col, lb=lb, bound=bound)
         assert om2 == om and cl2.tolist() == cl.tolist()
+    # a lower bound above omega: nothing of that size exists
+    om3, cl3 = oracle.max_cliques(rp, col, lb=om + 1, bound=bound)
+    assert om3 == 0 and cl3.shape[0] == 0
 
 
 # ---------------------------------------------------------------------------
@@ -91,6 +95,7 @@ def test_complete_graph(n, bound):
     g = G.complete_graph(n)
     om, cl = oracle.max_cliques(*g.numpy(), bound=bound)
     assert om == n and cl.tolist() == [list(range(n))]
+    assert oracle.count_max_cliques(*g.numpy(), bound=bound) == (n, 1)
     counts = oracle.kclique_counts(*g.numpy(), n + 1)
     assert counts.tolist() == [math.comb(n, k) for k in range(1, n + 2)]
 
@@ -243,3 +248,110 @@ def test_greedy_closed_forms():
     rp, col = g.numpy()
     w, runs, _ = oracle.greedy(rp, col, np.diff(rp), g.n)
     assert w == 4 and set(runs.tolist()) == {4}
+
+
+# ---------------------------------------------------------------------------
+# the two oracles against each other, and the multi-word (out-degree > 64)
+# bitset path of oracle_mce against closed forms
+# ---------------------------------------------------------------------------
+
+# graphs of the GPU parity set the list-based oracle finishes in < 1 s
+CROSS = {
+    "ER60": lambda: G.erdos_renyi(60, 0.3, seed=4),
+    "ER300": lambda: G.erdos_renyi(300, 0.1, seed=5),
+    "ER150d": lambda: G.erdos_renyi(150, 0.5, seed=6),
+    "ER400d": lambda: G.erdos_renyi(400, 0.35, seed=7),
+    "RMAT11": lambda: G.rmat(11, 8, 0.57, 0.19, 0.19, seed=3),
+    "RMAT13": lambda: G.rmat(13, 8, 0.45, 0.2, 0.2, seed=2),
+    "BA5k": lambda: G.barabasi_albert(5000, 4, seed=2),
+    "BA3k_m1": lambda: G.barabasi_albert(3000, 1, seed=11),
+    "planted": lambda: G.plant_cliques(G.erdos_renyi(3000, 0.004, seed=9), 3, 9, seed=9),
+    "T(36,12)": lambda: G.turan_graph(36, 12),
+    # out-degree > 64 after orientation: oracle_mce's multi-word bitsets
+    "ER200x": lambda: G.erdos_renyi(200, 0.5, seed=3),  # degeneracy 84, W = 2
+    "ER150x": lambda: G.erdos_renyi(150, 0.6, seed=3),  # degeneracy 77, 96 maximum cliques
+    "ER300x": lambda: G.erdos_renyi(300, 0.4, seed=3),  # degeneracy 101
+}
+
+
+@pytest.mark.parametrize("key", list(CROSS))
+def test_colour_oracle_vs_plain_oracle(key):
+    """oracle_mce (degeneracy order, root-local bitsets, colouring bound) and
+    oracle_mce_plain (degree order, sorted lists, |C|+|P| bound) share no
+    search code: they must agree clique for clique."""
+    rp, col = CROSS[key]().numpy()
+    om, cl = oracle.max_cliques(rp, col, bound="color")
+    om_p, cl_p = oracle.max_cliques(rp, col, bound="plain")
+    assert om == om_p and np.array_equal(cl, cl_p)
+    om_t, cl_t = oracle.max_cliques(rp, col, bound="color", tight=True)
+    assert om_t == om and np.array_equal(cl_t, cl)
+    assert oracle.count_max_cliques(rp, col, bound="color", tight=True) == (om, len(cl))
+    assert oracle.count_max_cliques(rp, col, bound="plain") == (om, len(cl))
+    # invariants: cliques of size omega, none bigger
+    for c in cl[:50]:
+        assert oracle.is_clique(rp, col, c)
+    kc = oracle.kclique_counts(rp, col, om + 1) if key not in ("T(36,12)",) else None
+    if kc is not None:
+        assert kc[om - 1] == len(cl) and kc[om] == 0
+
+
+@pytest.mark.parametrize("bound", ["size", "color", "plain"])
+@pytest.mark.parametrize("n", [65, 130, 300])
+def test_complete_graph_multiword(n, bound):
+    """K_n with n - 1 > 64 later neighbours at the root: W = 2, 3, 5 words."""
+    om, cl = oracle.max_cliques(*G.complete_graph(n).numpy(), bound=bound)
+    assert om == n and cl.tolist() == [list(range(n))]
+
+
+@pytest.mark.parametrize("tight", [False, True])
+@pytest.mark.parametrize("j,t", [(3, 1), (13, 5), (6, 60), (12, 300), (16, 50), (8, 600)])
+def test_cocktail_party_join_closed_form(j, t, tight):
+    """CP(j) + K_t: omega = j + t, exactly 2^j maximum cliques, each taking
+    one vertex of every non-adjacent pair.  (8, 600): root out-degree 615,
+    the (512, 1024] width class of R-MAT scale 22/26 roots."""
+    g = G.cocktail_party_join(j, t, seed=j * 1000 + t)
+    rp, col = g.numpy()
+    om, cl = oracle.max_cliques(rp, col, tight=tight)
+    assert om == j + t and len(cl) == 2 ** j
+    assert len({tuple(c) for c in cl}) == len(cl)
+    deg = np.diff(rp)
+    # the non-adjacent pairs are the only vertices of degree n - 2
+    paired = set(np.nonzero(deg == g.n - 2)[0].tolist())
+    assert len(paired) == 2 * j
+    for c in cl[:64]:
+        assert len(set(c.tolist()) & paired) == j  # one of each pair
+        assert oracle.is_clique(rp, col, c)
+    assert oracle.count_max_cliques(rp, col, tight=tight) == (j + t, 2 ** j)
+
+
+def test_turan_multiword():
+    """T(150, 3): parts of 50, out-degree up to 100 (W = 2), 50^3 maximum cliques."""
+    rp, col = G.turan_graph(150, 3).numpy()
+    for bound in ("color", "plain"):
+        assert oracle.count_max_cliques(rp, col, bound=bound) == (3, 125000)
+
+
+def test_is_clique_negative():
+    """oracle_is_clique must reject non-cliques (every find-one check relies on it)."""
+    g = G.cocktail_party_join(4, 6, seed=1)
+    rp, col = g.numpy()
+    deg = np.diff(rp)
+    paired = np.nonzero(deg == g.n - 2)[0]
+    a = int(paired[0])
+    row = set(col[rp[a]:rp[a + 1]].tolist())
+    b = next(int(v) for v in paired if int(v) != a and int(v) not in row)  # a's non-neighbour
+    others = [v for v in range(g.n) if v not in set(paired.tolist())]  # the K_t part: adjacent to all
+    assert not oracle.is_clique(rp, col, [a, b])
+    assert not oracle.is_clique(rp, col, others[:5] + [a, b])
+    assert not oracle.is_clique(rp, col, [b] + others[:3] + [a])
+    assert oracle.is_clique(rp, col, [a] + others[:5])
+    assert oracle.is_clique(rp, col, [a])
+    assert oracle.is_clique(rp, col, [])
+    # against brute force on every subset of a small random graph
+    edges = random_small_graph(9, 0.5, 3)
+    rp2, col2 = csr_from_edges(9, edges)
+    es = {tuple(e) for e in edges}
+    for mask in range(1 << 9):
+        vs = [v for v in range(9) if mask >> v & 1]
+        truth = all((u, w) in es for u, w in combinations(vs, 2))
+        assert oracle.is_clique(rp2, col2, vs) == truth
