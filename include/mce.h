@@ -40,7 +40,8 @@ typedef enum {
     MCE_ERR_CUDA = 2,     /* CUDA runtime error (incl. no device) */
     MCE_ERR_NOMEM = 3,    /* device allocation failed */
     MCE_ERR_BUDGET = 4,   /* a single frontier entry set cannot fit the memory budget */
-    MCE_ERR_STATE = 5     /* call out of order (e.g. result already fetched) */
+    MCE_ERR_STATE = 5,    /* call out of order (e.g. result already fetched) */
+    MCE_ERR_SYNC = 6      /* the bound_sync callback reported a failure (negative return) */
 } mce_status;
 
 typedef struct mce_graph mce_graph;   /* device-resident graph + preprocessing */
@@ -50,8 +51,13 @@ enum { MCE_WHERE_HOST = 0, MCE_WHERE_DEVICE = 1 };
 
 /* Vertex ordering used to orient edges (PAPER.md IV-C line 131: "we use only
  * one of the two directed edges that represent each undirected edge"). */
-enum { MCE_ORIENT_DEGENERACY = 0, /* k-core peel order (north star) */
-       MCE_ORIENT_DEGREE = 1 };   /* (degree, id) order (the paper's choice) */
+enum { MCE_ORIENT_DEGENERACY = 0,     /* k-core peel order (north star); the asynchronous
+                                         peel's order within a level depends on timing */
+       MCE_ORIENT_DEGREE = 1,         /* (degree, id) order (the paper's choice) */
+       MCE_ORIENT_DEGENERACY_DET = 2  /* a degeneracy order that is a function of the graph
+                                         alone: (core, synchronous round of the peel of the
+                                         core's shell, id); every process computes the same
+                                         one (multi-GPU sharding, no broadcast) */ };
 
 /* Greedy heuristic for the initial lower bound (PAPER.md IV-A, Table I). */
 enum { MCE_HEUR_NONE = 0,
@@ -81,8 +87,16 @@ typedef struct {
     int32_t shard_count;     /*   roots with index % shard_count == shard_rank (<=1: all) */
     /* Optional per-step bound exchange (multi-GPU).  Called after every
      * expansion step with this shard's best clique size and whether it still
-     * has work; must return the global best and set *global_active to 1 while
-     * any shard has work.  All shards call it the same number of times. */
+     * has work; must return the global best (>= 0) and set *global_active to 1
+     * while any shard has work.  Shards call it a DIFFERENT number of times
+     * (one call per level / window / chunk of their own work): the exchange
+     * is a collective that pairs the k-th calls of all shards, whatever step
+     * each is at; a shard that has finished keeps calling it with
+     * local_active = 0 until *global_active comes back 0, so every shard
+     * leaves in the same collective round.  A negative return means the
+     * exchange failed (e.g. a peer is gone): the call stops with
+     * MCE_ERR_SYNC.  The returned bound only ever raises the pruning bound to
+     * a size some shard has found, so the pairing does not affect results. */
     int32_t (*bound_sync)(int32_t local_best, int32_t local_active, int32_t *global_active, void *user);
     void *bound_sync_user;
     int32_t verbose;         /* >0: per-level statistics on stderr */
@@ -105,7 +119,9 @@ typedef struct {
                                 id; d >= 2: every shard expands all roots through level d - 1 and
                                 keeps the level-d candidates (d-cliques) whose vertex-path hash
                                 % shard_count == shard_rank (balances work that sits under a few
-                                hub roots); cliques found above level d are reported by shard 0 */
+                                hub roots); cliques found above level d (leaves: clique /
+                                pair completions are off above the split, their firing
+                                depends on the shard's bound) are reported by shard 0 */
     int32_t no_overlap;      /* 0 (default): the degree heuristics run on a second stream and host
                                 thread while the k-core / orientation preprocessing runs (they
                                 share no data); 1: one after the other */

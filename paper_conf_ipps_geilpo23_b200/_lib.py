@@ -18,9 +18,9 @@ HEADER = os.path.join(os.path.dirname(_HERE), "include", "mce.h")
 
 MCE_OK = 0
 STATUS = {0: "MCE_OK", 1: "MCE_ERR_INVALID", 2: "MCE_ERR_CUDA", 3: "MCE_ERR_NOMEM", 4: "MCE_ERR_BUDGET",
-          5: "MCE_ERR_STATE"}
+          5: "MCE_ERR_STATE", 6: "MCE_ERR_SYNC"}
 WHERE_HOST, WHERE_DEVICE = 0, 1
-ORIENT = {"degeneracy": 0, "degree": 1}
+ORIENT = {"degeneracy": 0, "degree": 1, "degeneracy_det": 2}
 HEURISTIC = {"none": 0, "single_degree": 1, "single_core": 2, "multi_degree": 3, "multi_core": 4}
 BOUND = {"size": 0, "color": 1}
 

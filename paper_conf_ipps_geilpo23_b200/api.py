@@ -82,14 +82,36 @@ def make_options(orientation="degeneracy", heuristic="multi_degree", heuristic_r
     o.shard_depth = int(shard_depth)
     keep = None
     if bound_sync is not None:
-        def _cb(local_best, local_active, gactive, _user):
-            gb, ga = bound_sync(int(local_best), int(local_active))
-            gactive[0] = int(ga)
-            return int(gb)
+        errors = []
 
-        keep = BOUND_SYNC(_cb)
-        o.bound_sync = keep
+        def _cb(local_best, local_active, gactive, _user):
+            # an exception must not unwind through the C frames: report it with
+            # the negative sentinel (the engine stops with MCE_ERR_SYNC) and
+            # re-raise it from the Python call (SyncGuard)
+            try:
+                gb, ga = bound_sync(int(local_best), int(local_active))
+                gactive[0] = int(ga)
+                return max(int(gb), 0)
+            except BaseException as e:  # noqa: BLE001
+                errors.append(e)
+                gactive[0] = 0
+                return -1
+
+        keep = _SyncGuard(BOUND_SYNC(_cb), errors)
+        o.bound_sync = keep.fn
     return o, keep
+
+
+class _SyncGuard:
+    """Keeps the ctypes callback alive for the call and re-raises what it caught."""
+
+    def __init__(self, fn, errors):
+        self.fn = fn
+        self.errors = errors
+
+    def reraise(self):
+        if self.errors:
+            raise self.errors[0]
 
 
 class Graph:
@@ -183,15 +205,19 @@ class Graph:
     def enumerate(self, **opts) -> Result:
         o, keep = make_options(**opts)
         h = ctypes.c_void_p()
-        check(lib().mce_enumerate(self._h, ctypes.byref(o), ctypes.byref(h)))
-        del keep
+        st = lib().mce_enumerate(self._h, ctypes.byref(o), ctypes.byref(h))
+        if keep is not None:
+            keep.reraise()
+        check(st)
         return self._result(h)
 
     def find_one(self, window: int = 0, **opts) -> Result:
         o, keep = make_options(**opts)
         h = ctypes.c_void_p()
-        check(lib().mce_find_one(self._h, int(window), ctypes.byref(o), ctypes.byref(h)))
-        del keep
+        st = lib().mce_find_one(self._h, int(window), ctypes.byref(o), ctypes.byref(h))
+        if keep is not None:
+            keep.reraise()
+        check(st)
         return self._result(h)
 
 

@@ -231,7 +231,7 @@ mce_status mce_preprocess(mce_graph *g, int32_t orientation, int32_t *core_out, 
                           int32_t *degeneracy_out) {
     return run_guarded([&] {
         if (!g) fail(MCE_ERR_INVALID, "graph is NULL");
-        if (orientation != MCE_ORIENT_DEGENERACY && orientation != MCE_ORIENT_DEGREE)
+        if (orientation < MCE_ORIENT_DEGENERACY || orientation > MCE_ORIENT_DEGENERACY_DET)
             fail(MCE_ERR_INVALID, "bad orientation");
         MCE_CUDA(cudaSetDevice(g->device));
         preprocess(g, orientation);
@@ -263,7 +263,7 @@ mce_status mce_heuristic(mce_graph *g, int32_t kind, int64_t h, int32_t *omega_b
 
 static void check_options(const mce_options *o) {
     if (!o) fail(MCE_ERR_INVALID, "options are NULL");
-    if (o->orientation != MCE_ORIENT_DEGENERACY && o->orientation != MCE_ORIENT_DEGREE)
+    if (o->orientation < MCE_ORIENT_DEGENERACY || o->orientation > MCE_ORIENT_DEGENERACY_DET)
         fail(MCE_ERR_INVALID, "bad orientation");
     if (o->heuristic < MCE_HEUR_NONE || o->heuristic > MCE_HEUR_MULTI_CORE) fail(MCE_ERR_INVALID, "bad heuristic");
     if (o->bound != MCE_BOUND_SIZE && o->bound != MCE_BOUND_COLOR) fail(MCE_ERR_INVALID, "bad bound");

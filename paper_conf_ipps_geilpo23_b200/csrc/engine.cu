@@ -252,6 +252,7 @@ void Engine::sync_bound(bool active) {
     if (!o_.bound_sync) return;
     int32_t gactive = 0;
     int32_t gb = o_.bound_sync(best_, active ? 1 : 0, &gactive, o_.bound_sync_user);
+    if (gb < 0) fail(MCE_ERR_SYNC, "bound_sync reported a failed exchange");
     if (gb > best_) best_ = gb;
 }
 
@@ -260,7 +261,13 @@ void Engine::leaf_args(ExpandArgs &a) const {
     a.leaf_slot = leaf_slot_;
     a.leaf_rows = g_->stage.get();
     a.leaf_cap = stage_rows_;
-    a.shortcut = o_.no_clique_shortcut ? 0 : 1;
+    // No clique / pair completions above the split depth of the level-d deal:
+    // whether a completion fires depends on this shard's bound (k + |P| ==
+    // need), so a clique could be completed above the split on one shard and
+    // reached below it on another.  Without them, what is found above the split
+    // (leaves only) does not depend on the bound, and every deeper clique sits
+    // under exactly one dealt level-d entry.
+    a.shortcut = (o_.no_clique_shortcut || (entry_shard_ && !split_)) ? 0 : 1;
     a.clq_total = clq_total_;
     a.clq_slot = clq_slot_;
     a.clq_rows = g_->cstage.get();
@@ -1033,6 +1040,7 @@ mce_result *Engine::run() {
         int guard = 0;
         while (gactive && guard++ < (1 << 30)) {
             int32_t gb = o_.bound_sync(best_, 0, &gactive, o_.bound_sync_user);
+            if (gb < 0) fail(MCE_ERR_SYNC, "bound_sync reported a failed exchange");
             if (gb > best_) best_ = gb;
         }
     }

@@ -535,6 +535,151 @@ __global__ void long_rows_kernel(int64_t n, const int64_t *__restrict__ orp, int
     if (lane == 0 && mx) atomicMax(max_out, mx);
 }
 
+// ---------------------------------------------------------------------------
+// Deterministic degeneracy order (MCE_ORIENT_DEGENERACY_DET, multi-GPU): the
+// asynchronous peel above gives every vertex its (unique) core number but a
+// peel ORDER that depends on timing, and root / candidate sharding needs every
+// rank to orient the edges identically.  With the core numbers known, shell c
+// (the vertices of core c) is peeled inside the c-core H_c in synchronous
+// rounds, every shell at once:
+//   d(v)  = neighbours w with core(w) >= core(v)        (degree inside H_c)
+//   round t removes every alive v with d(v) <= core(v) (a set fixed by the
+//           state at the start of the round), then decrements d(w) for the
+//           alive neighbours w of the same shell
+// Each round's set, hence round(v), is a function of the graph alone.  Order
+// = (core, round, id): when v goes (round t) every later neighbour -- higher
+// core, or same shell with round >= t -- was alive and counted in d(v) <=
+// core(v), so out-degrees along the order stay <= core (a degeneracy order).
+// One cooperative launch, two grid barriers per round; frontier lists
+// alternate.  ctrl[0] = rounds, ctrl[2 + (t & 1)] = size of frontier t.
+// ---------------------------------------------------------------------------
+__global__ void __launch_bounds__(512)
+    shell_round_peel(int64_t n, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
+                     const int32_t *__restrict__ core, int32_t *d, int32_t *round, int32_t *fa, int32_t *fb,
+                     unsigned long long *ctrl) {
+    cg::grid_group grid = cg::this_grid();
+    const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t nthreads = (int64_t)gridDim.x * blockDim.x;
+    const int lane = threadIdx.x & 31;
+    // d(v) and frontier 0: a warp per 32 vertices, 8-lane tiles over the rows
+    for (int64_t v0 = (tid >> 5) * 32; v0 < n; v0 += (nthreads >> 5) * 32) {
+        for (int q = 0; q < 32; q += 4) {
+            const int64_t v = v0 + q + (lane >> 3);
+            int32_t cnt = 0, c = 0;
+            if (v < n) {
+                c = core[v];
+                for (int64_t e = rowptr[v] + (lane & 7); e < rowptr[v + 1]; e += 8) cnt += core[col[e]] >= c;
+            }
+            cnt += __shfl_xor_sync(0xffffffffu, cnt, 1);
+            cnt += __shfl_xor_sync(0xffffffffu, cnt, 2);
+            cnt += __shfl_xor_sync(0xffffffffu, cnt, 4);
+            const bool take = v < n && (lane & 7) == 0 && cnt <= c;
+            if (v < n && (lane & 7) == 0) {
+                d[v] = cnt;
+                round[v] = -1;
+            }
+            const unsigned m = __ballot_sync(0xffffffffu, take);
+            unsigned long long b = 0;
+            if (lane == 0 && m) b = atomicAdd(ctrl + 2, (unsigned long long)__popc(m));
+            b = __shfl_sync(0xffffffffu, b, 0);
+            if (take) fa[b + __popc(m & lanemask_lt())] = (int32_t)v;
+        }
+    }
+    grid.sync();
+    int32_t *cur = fa, *nxt = fb;
+    for (int32_t t = 0;; ++t) {
+        const int64_t nf = (int64_t)__ldcg(ctrl + 2 + (t & 1));
+        if (nf == 0) {
+            if (tid == 0) ctrl[0] = (unsigned long long)t;
+            break;
+        }
+        for (int64_t i = tid; i < nf; i += nthreads) round[cur[i]] = t;
+        if (tid == 0) ctrl[2 + ((t + 1) & 1)] = 0;
+        grid.sync();
+        // decrements: 8-lane tile per frontier vertex
+        for (int64_t b0 = (tid >> 5) * 4; b0 < nf; b0 += (nthreads >> 5) * 4) {  // warp-uniform trip count
+            const int64_t i = b0 + (lane >> 3);
+            int32_t v = -1, c = 0;
+            int64_t eb = 0, ee = 0;
+            if (i < nf) {
+                v = cur[i];
+                c = core[v];
+                eb = rowptr[v];
+                ee = rowptr[v + 1];
+            }
+            const int iters = __reduce_max_sync(0xffffffffu, (unsigned)((ee - eb + 7) >> 3));
+            for (int it = 0; it < iters; ++it) {
+                const int64_t e = eb + it * 8 + (lane & 7);
+                bool fell = false;
+                int32_t w = -1;
+                if (e < ee) {
+                    w = col[e];
+                    if (core[w] == c && __ldcg(round + w) < 0) fell = atomicSub(d + w, 1) == c + 1;
+                }
+                const unsigned m = __ballot_sync(0xffffffffu, fell);
+                unsigned long long b = 0;
+                if (lane == 0 && m) b = atomicAdd(ctrl + 2 + ((t + 1) & 1), (unsigned long long)__popc(m));
+                b = __shfl_sync(0xffffffffu, b, 0);
+                if (fell) nxt[b + __popc(m & lanemask_lt())] = w;
+            }
+        }
+        grid.sync();
+        int32_t *tmp = cur;
+        cur = nxt;
+        nxt = tmp;
+    }
+}
+
+// sort key of the deterministic order: core * (rounds + 1) + round (stable radix sort: ties by id)
+__global__ void shell_keys_kernel(int64_t n, const int32_t *__restrict__ core, const int32_t *__restrict__ round,
+                                  uint64_t span, uint64_t *keys, int32_t *vals) {
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+        keys[v] = (uint64_t)(uint32_t)core[v] * span + (uint64_t)(uint32_t)round[v];
+        vals[v] = (int32_t)v;
+    }
+}
+
+// stable radix sort of `keys` (values: vertex ids ascending) into `out`
+void sort_by_key_stable(uint64_t *keys, uint64_t *keys_out, int32_t *vals, int32_t *out, int64_t n, uint64_t kmax,
+                        mce::Pool &pool, cudaStream_t s) {
+    int end_bit = 1;
+    while (end_bit < 64 && (1ull << end_bit) <= kmax) ++end_bit;
+    size_t tmp_bytes = 0;
+    MCE_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tmp_bytes, keys, keys_out, vals, out, (int)n, 0, end_bit, s));
+    void *tmp = pool.take<uint8_t>((int64_t)tmp_bytes);
+    MCE_CUDA(cub::DeviceRadixSort::SortPairs(tmp, tmp_bytes, keys, keys_out, vals, out, (int)n, 0, end_bit, s));
+}
+
+// g->order = the deterministic degeneracy order (needs g->core)
+void deterministic_order(mce_graph *g) {
+    const int64_t n = g->n;
+    cudaStream_t s = g->stream;
+    int32_t *d = g->pool.take<int32_t>(n), *round = g->pool.take<int32_t>(n);
+    int32_t *fa = g->pool.take<int32_t>(n), *fb = g->pool.take<int32_t>(n);
+    unsigned long long *ctrl = g->pool.take<unsigned long long>(4);
+    MCE_CUDA(cudaMemsetAsync(ctrl, 0, 4 * sizeof(unsigned long long), s));
+    int blocks_per_sm = 0;
+    MCE_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm, shell_round_peel, 512, 0));
+    if (blocks_per_sm < 1) fail(2, "shell_round_peel: cooperative kernel does not fit an SM");
+    const int grid = num_sms() * std::min(blocks_per_sm, 2);
+    int64_t n_arg = n;
+    const int64_t *rp = g->rowptr.get();
+    const int32_t *cl = g->col.get(), *co = g->core.get();
+    unsigned long long *ct = ctrl;
+    void *args[] = {&n_arg, &rp, &cl, &co, &d, &round, &fa, &fb, &ct};
+    MCE_CUDA(cudaLaunchCooperativeKernel((void *)shell_round_peel, grid, 512, args, 0, s));
+    unsigned long long *h = g->host.get<unsigned long long>(1);
+    MCE_CUDA(cudaMemcpyAsync(h, ctrl, sizeof(unsigned long long), cudaMemcpyDeviceToHost, s));
+    stream_sync(s);
+    const uint64_t span = h[0] + 1;
+    uint64_t *keys = g->pool.take<uint64_t>(n), *keys_out = g->pool.take<uint64_t>(n);
+    int32_t *vals = g->pool.take<int32_t>(n);
+    shell_keys_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->core.get(), round, span, keys, vals);
+    MCE_LAUNCH_CHECK();
+    sort_by_key_stable(keys, keys_out, vals, g->order.get(), n, ((uint64_t)g->degeneracy + 1) * span, g->pool, s);
+    g->kernels += 4;
+}
+
 }  // namespace
 
 int num_sms() {
@@ -631,6 +776,8 @@ void orient(mce_graph *g, int orientation) {
     if (g->order_given) {  // mce_set_order: g->order already holds the order
     } else if (orientation == 0) {  // degeneracy: the peel queue
         MCE_CUDA(cudaMemcpyAsync(g->order.get(), g->peel.get(), sizeof(int32_t) * n, cudaMemcpyDeviceToDevice, s));
+    } else if (orientation == 2) {  // deterministic degeneracy order: (core, shell round, id)
+        deterministic_order(g);
     } else {  // degree order
         int64_t nb = g->max_deg + 1;
         int32_t *bins = g->pool.take<int32_t>(nb);
@@ -649,7 +796,7 @@ void orient(mce_graph *g, int orientation) {
     // id space of the oriented CSR (reading 5): degeneracy -> vertices
     // sorted by (core, degree) ascending, so the reverse local order of a root
     // meets high-core, then high-degree vertices first; degree -> the rank itself
-    if (orientation == 0) {
+    if (orientation != 1) {
         uint64_t *keys = g->pool.take<uint64_t>(n), *keys_out = g->pool.take<uint64_t>(n);
         int32_t *vals = g->pool.take<int32_t>(n);
         const uint64_t span = (uint64_t)g->max_deg + 1;

@@ -4,12 +4,15 @@ North star: "Work is partitioned ... by sharding first-level root vertices,
 whose subtrees are independent, with a small NCCL max-allreduce of the omega
 lower bound each level and a final gather of the cliques over NVLink."
 
- * every rank loads the whole graph and runs the same preprocessing, then
-   takes rank 0's orientation order (agree_orientation: the peel order is not
-   deterministic across processes, and clique ownership depends on it);
+ * every rank loads the whole graph and runs the whole preprocessing itself,
+   concurrently, with the DETERMINISTIC degeneracy orientation
+   (MCE_ORIENT_DEGENERACY_DET: order (core, shell round, id), a function of
+   the graph alone), so every rank orients the edges identically with no
+   broadcast and no second k-core -- clique ownership depends on it;
  * heuristic seeds are dealt cyclically (seed position % world == rank) and
    root vertices by CSR id (id % world == rank) inside the library
-   (mce_options.shard_rank / shard_count);
+   (mce_options.shard_rank / shard_count), or level-d candidates by path hash
+   (shard_depth d >= 2);
  * after every expansion step the library calls `bound_sync`, which
    max-allreduces (best clique size, still-active flag) across ranks, so a
    clique found on one GPU tightens the pruning bound on all of them and the
@@ -49,7 +52,7 @@ def make_bound_sync(group=None):
     return sync
 
 
-def gather_result(res: Result, group=None, find_one: bool = False) -> Result:
+def gather_result(res: Result, group=None, find_one: bool = False, max_cliques: int = 0) -> Result:
     """Combine per-rank results: global omega, summed multiplicity, all cliques."""
     dev = _device(group)
     world = dist.get_world_size(group)
@@ -72,7 +75,8 @@ def gather_result(res: Result, group=None, find_one: bool = False) -> Result:
         dist.broadcast(buf, src=dist.get_global_rank(group, src) if group is not None else src, group=group)
         cl = buf[:omega].cpu().numpy().astype(np.int32).reshape(1, omega)
         return Result(omega, 1, cl, False, res.levels, res.timing)
-    c = torch.tensor([count, int(res.truncated)], dtype=torch.int64, device=dev)
+    # only ranks holding cliques of the global omega count (their lists are the ones kept)
+    c = torch.tensor([count, int(res.truncated) if res.omega == omega else 0], dtype=torch.int64, device=dev)
     dist.all_reduce(c, op=dist.ReduceOp.SUM, group=group)
     total, trunc = (int(x) for x in c.tolist())
     n_local = torch.tensor([mine.shape[0]], dtype=torch.int64, device=dev)
@@ -90,14 +94,23 @@ def gather_result(res: Result, group=None, find_one: bool = False) -> Result:
     allrows = np.concatenate(rows, 0).astype(np.int32) if rows else np.zeros((0, omega), np.int32)
     if allrows.shape[0] > 1 and omega > 0:
         allrows = allrows[np.lexsort(allrows.T[::-1])]
+    if max_cliques > 0 and allrows.shape[0] > max_cliques:  # each rank stored up to max_cliques
+        allrows = allrows[:max_cliques]
+        trunc = 1
     return Result(omega, total, allrows, bool(trunc), res.levels, res.timing)
 
 
+def sharded_orientation(orientation: str, world: int) -> str:
+    """The orientation every rank uses: the asynchronous peel's order depends
+    on timing, so a multi-rank degeneracy run takes the deterministic one."""
+    return "degeneracy_det" if world > 1 and orientation == "degeneracy" else orientation
+
+
 def agree_orientation(graph: Graph, group=None, orientation: str = "degeneracy"):
-    """Make every rank orient the edges like rank 0.  The asynchronous k-core
-    peel is not deterministic across processes, and the root of a clique (its
-    lowest-rank vertex) -- hence the rank that owns it -- depends on the
-    order: rank 0's order is broadcast and set on the others."""
+    """Fallback for callers that need rank 0's own (asynchronous-peel) order on
+    every rank: broadcast it and set it on the others.  enumerate_distributed /
+    find_one_distributed do not use it (each rank computes the deterministic
+    order itself)."""
     if dist.get_world_size(group) == 1 or graph.n == 0:
         return
     dev = _device(group)
@@ -116,15 +129,15 @@ def agree_orientation(graph: Graph, group=None, orientation: str = "degeneracy")
 def enumerate_distributed(graph: Graph, group=None, **opts) -> Result:
     rank = dist.get_rank(group)
     world = dist.get_world_size(group)
-    agree_orientation(graph, group, opts.get("orientation", "degeneracy"))
+    opts["orientation"] = sharded_orientation(opts.get("orientation", "degeneracy"), world)
     res = graph.enumerate(shard_rank=rank, shard_count=world, bound_sync=make_bound_sync(group), **opts)
-    return gather_result(res, group)
+    return gather_result(res, group, max_cliques=int(opts.get("max_cliques", 0) or 0))
 
 
 def find_one_distributed(graph: Graph, window: int = 0, group=None, **opts) -> Result:
     rank = dist.get_rank(group)
     world = dist.get_world_size(group)
-    agree_orientation(graph, group, opts.get("orientation", "degeneracy"))
+    opts["orientation"] = sharded_orientation(opts.get("orientation", "degeneracy"), world)
     res = graph.find_one(window=window, shard_rank=rank, shard_count=world, bound_sync=make_bound_sync(group),
                          **opts)
     return gather_result(res, group, find_one=True)

@@ -36,14 +36,14 @@ def _run(rank, world, port, fn, q):
         dist.destroy_process_group()
 
 
-def spawn(fn, world=2):
+def spawn(fn, world=2, timeout=120):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
     procs = [ctx.Process(target=_run, args=(r, world, port, fn, q)) for r in range(world)]
     for p in procs:
         p.start()
-    out = dict(q.get(timeout=120) for _ in procs)
+    out = dict(q.get(timeout=timeout) for _ in procs)
     for p in procs:
         p.join(timeout=60)
         assert p.exitcode == 0
@@ -81,6 +81,18 @@ def _gather_mixed_omega_body(rank, world):
     return g.omega, g.count, g.cliques.tolist(), g.truncated
 
 
+def _gather_trunc_body(rank, world):
+    # rank 1 is truncated but below the global omega: its list is dropped, so
+    # the result is not truncated; max_cliques caps the merged list
+    if rank == 0:
+        r = Result(3, 3, np.array([[0, 1, 2], [1, 2, 3], [4, 5, 6]], np.int32), False, [], {})
+    else:
+        r = Result(2, 9, np.array([[7, 8]], np.int32), True, [], {})
+    a = mdist.gather_result(r)
+    b = mdist.gather_result(r, max_cliques=2)
+    return (a.omega, a.count, a.truncated, len(a.cliques)), (b.omega, b.count, b.truncated, b.cliques.tolist())
+
+
 def _find_one_body(rank, world):
     r = Result(3, 1, np.array([[9, 10, 11]], np.int32), False, [], {}) if rank == 1 else \
         Result(2, 1, np.array([[0, 1]], np.int32), False, [], {})
@@ -108,6 +120,39 @@ def test_gather_drops_smaller_local_results():
         assert omega == 4 and count == 1 and cliques == [[5, 6, 7, 8]] and trunc
 
 
+def test_gather_truncation_only_from_omega_holders():
+    out = spawn(_gather_trunc_body)
+    for a, b in out:
+        assert a == (3, 3, False, 3)
+        assert b == (3, 3, True, [[0, 1, 2], [1, 2, 3]])
+
+
+def _sync_raises_body(rank, world):
+    """A failing exchange must surface as a Python exception through the
+    ctypes callback wrapper (make_options), not a hang or a silent 0."""
+    from paper_conf_ipps_geilpo23_b200 import api
+
+    calls = []
+
+    def bad(best, active):
+        calls.append(best)
+        raise ConnectionError("peer gone")
+
+    o, keep = api.make_options(bound_sync=bad)
+    ga = (api.ctypes.c_int32 * 1)(1)
+    ret = o.bound_sync(5, 1, ga, None)
+    try:
+        keep.reraise()
+    except ConnectionError as e:
+        return ret, ga[0], str(e), len(calls)
+    return ret, ga[0], None, len(calls)
+
+
+def test_bound_sync_exception_is_reported():
+    for ret, ga, err, n in spawn(_sync_raises_body):
+        assert ret == -1 and ga == 0 and err == "peer gone" and n == 1
+
+
 def test_find_one_gather_takes_a_holder_of_omega():
     out = spawn(_find_one_body)
     for omega, count, cliques in out:
@@ -133,12 +178,8 @@ def test_shards_union_is_the_full_answer(key, shards, depth):
     shard_depth d >= 2, every root down to level d - 1 and its hash share of
     the level-d candidates (heuristic seeds dealt either way); merged like
     gather_result, the shards give the oracle's answer."""
-    if (key, shards, depth) == ("BA5k", 3, 3):
-        # Known bug (DESIGN.md §(f), found late in round 1, present before the
-        # round's last session): with the level-d deal and NO bound exchange
-        # between the shards (this one-process simulation), BA5k's single
-        # maximum clique is reported by two shards (multiplicity 2 vs 1).
-        pytest.xfail("level-d deal without bound sync double-reports a clique on BA5k (3 shards, depth 3)")
+    # (BA5k, 3 shards, depth 3) was the round-1 double report: completions above
+    # the split fired on one shard's bound and not another's (fixed: none above it)
     import oracle
     from tests.test_gpu_parity import GRAPHS
 
@@ -209,3 +250,98 @@ def test_shards_on_separate_handles_agree_after_set_order(key, depth):
     rows = np.concatenate([p.cliques for p in parts if p.omega == omega], 0)
     rows = rows[np.lexsort(rows.T[::-1])]
     assert omega == om and count == len(cl) and np.array_equal(rows, cl)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("depth", [0, 2, 3])
+@pytest.mark.parametrize("key", ["planted", "RMAT13", "BA5k", "T(30,6)", "ER400d", "RMAT11"])
+def test_shards_with_different_bounds(key, depth):
+    """Shards whose lower bounds differ (one with no heuristic and no bound,
+    one told omega, one told omega - 1) still partition the maximum cliques
+    exactly: nothing reported twice, nothing lost (pre-split
+    reporting must not depend on the shard's bound)."""
+    import oracle
+    from tests.test_gpu_parity import GRAPHS
+
+    import paper_conf_ipps_geilpo23_b200 as m
+
+    g = GRAPHS[key]()
+    om, cl = oracle.max_cliques(*g.numpy(), bound="plain")
+    settings = [dict(heuristic="none"), dict(lower_bound=om), dict(lower_bound=max(om - 1, 0), heuristic="single_degree")]
+    gg = m.Graph(g.rowptr, g.col)
+    for shards in (2, 3):
+        parts = [gg.enumerate(shard_rank=r, shard_count=shards, shard_depth=depth, **settings[r % 3])
+                 for r in range(shards)]
+        omega = max(p.omega for p in parts)
+        count = sum(p.count for p in parts if p.omega == omega)
+        rows = np.concatenate([p.cliques for p in parts if p.omega == omega], 0)
+        rows = rows[np.lexsort(rows.T[::-1])]
+        assert omega == om and count == len(cl) and np.array_equal(rows, cl), (shards, omega, count)
+    gg.close()
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("key", ["RMAT13", "BA5k", "planted", "ER400d", "RMAT15"])
+def test_deterministic_orientation(key):
+    """MCE_ORIENT_DEGENERACY_DET: two handles (two processes' worth of state)
+    compute the same order, bit for bit, and it is a degeneracy order
+    (out-degree <= core number, checked against the oracle's cores)."""
+    import oracle
+    from tests.test_gpu_parity import GRAPHS
+
+    import paper_conf_ipps_geilpo23_b200 as m
+
+    g = GRAPHS[key]()
+    rp, col = g.numpy()
+    core_o, _, d_o = oracle.core_numbers(rp, col)
+    orders = []
+    for _ in range(2):
+        h = m.Graph(g.rowptr, g.col)
+        core, order, d = h.preprocess("degeneracy_det")
+        h.close()
+        assert np.array_equal(core, core_o) and d == d_o
+        orders.append(order)
+    assert np.array_equal(orders[0], orders[1])
+    order = orders[0]
+    assert sorted(order.tolist()) == list(range(g.n))
+    rank = np.empty(g.n, np.int64)
+    rank[order] = np.arange(g.n)
+    src = np.repeat(np.arange(g.n), np.diff(rp))
+    up = rank[col] > rank[src]
+    assert np.all(np.bincount(src[up], minlength=g.n) <= core_o)
+    # cores never decrease along the order
+    assert np.all(np.diff(core_o[order]) >= 0)
+
+
+def _enumerate_mp_body(rank, world):
+    import oracle
+    from tests.test_gpu_parity import GRAPHS
+
+    import paper_conf_ipps_geilpo23_b200 as m
+
+    out = []
+    for key in ("planted", "RMAT13", "BA5k", "ER400d"):
+        g = GRAPHS[key]()
+        om, cl = oracle.max_cliques(*g.numpy(), bound="plain")
+        gg = m.Graph(g.rowptr.cuda(), g.col.cuda())
+        for depth in (0, 3):
+            gg.clear_cache()
+            r = mdist.enumerate_distributed(gg, shard_depth=depth)
+            ok = r.omega == om and r.count == len(cl) and np.array_equal(r.cliques, cl)
+            f = mdist.find_one_distributed(gg, window=8, shard_depth=depth)
+            okf = f.omega == om and oracle.is_clique(*g.numpy(), f.cliques[0])
+            out.append((key, depth, bool(ok), bool(okf), r.omega, r.count))
+        gg.close()
+    return out
+
+
+@pytest.mark.gpu
+def test_enumerate_distributed_end_to_end():
+    """Two processes (gloo process group, both on cuda:0) run the whole
+    sharded path -- deterministic orientation computed by each rank, cyclic
+    root deal or level-3 hash deal, per-step bound all-reduce, final gather --
+    and get the oracle's answer (PAPER.md IV-E line 146: root subsets are
+    independent)."""
+    for rank_out in spawn(_enumerate_mp_body, timeout=900):
+        for key, depth, ok, okf, om, cnt in rank_out:
+            assert ok and okf, (key, depth, om, cnt)
