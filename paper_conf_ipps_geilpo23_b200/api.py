@@ -60,7 +60,8 @@ def _current_stream(device: int):
 def make_options(orientation="degeneracy", heuristic="multi_degree", heuristic_runs=0, bound="color",
                  lower_bound=0, window=0, budget_bytes=0, max_cliques=0, shard_rank=0, shard_count=1,
                  bound_sync: Optional[Callable[[int, int], tuple]] = None, verbose=0, legacy_roots=False,
-                 fused_levels=True, clique_shortcut=True, fused_expand=True, overlap=True, shard_depth=0):
+                 fused_levels=True, clique_shortcut=True, fused_expand=True, overlap=True, shard_depth=0,
+                 smem_expand=True):
     o = Options()
     lib().mce_default_options(ctypes.byref(o))
     o.orientation = ORIENT[orientation]
@@ -80,6 +81,7 @@ def make_options(orientation="degeneracy", heuristic="multi_degree", heuristic_r
     o.no_fused_expand = int(not fused_expand)
     o.no_overlap = int(not overlap)
     o.shard_depth = int(shard_depth)
+    o.no_smem_expand = int(not smem_expand)
     keep = None
     if bound_sync is not None:
         errors = []

@@ -10,6 +10,7 @@
 //           Windowing"), so the frontier never exceeds the budget.
 #include <algorithm>
 #include <chrono>
+#include <cstdlib>
 #include <exception>
 #include <thread>
 #include <cstdio>
@@ -212,6 +213,11 @@ class Engine {
     int32_t *maxbit_ = nullptr;                 // g->misc[4]
     unsigned long long *out_count_ = nullptr;   // g->misc[5] fused-pass children
     unsigned long long *pair_n_ = nullptr;      // g->misc[6] pair-completion descriptors
+    unsigned long long *chunk_ctr_ = nullptr;   // g->misc[7] work counter of the shared-memory count pass
+    int64_t nroots_ = 0;                        // roots of the current window (slots 0 .. nroots_ - 1)
+    int smem_min_w_ = 8;                        // narrowest level width taking the shared-memory count pass
+    int64_t smem_min_n_ = 2048;                 // ... and fewest entries (small levels: rows stay L1/L2 hits)
+    int64_t smem_per_root_ = 16;                // ... and fewest entries per root of the window on average
     int64_t pair_cap_ = 0;
     int64_t stage_rows_ = 0;
     int64_t cstage_rows_ = 0;
@@ -514,6 +520,21 @@ void Engine::process(int32_t k, const Level &L) {
     a.maxbit = maxbit_;
     leaf_args(a);
     a.chain = chain_dev_;
+    // shared-memory count pass (expand_smem): the level's entries grouped by
+    // root slot so a block stages one root's matrix per run of its candidates
+    // (only when a root has many candidates on average: one entry per root, as at
+    // level 1, gains nothing from staging 64 W rows and loses the L2's parallelism)
+    if (!o_.no_smem_expand && smem_width(L.W) && L.W >= smem_min_w_ && N >= smem_min_n_ && nroots_ > 0 &&
+        N >= smem_per_root_ * nroots_) {
+        int32_t *hist = arena_.alloc<int32_t>(nroots_);
+        int64_t *hoffs = arena_.alloc<int64_t>(nroots_ + 1);
+        int64_t *htmp = arena_.alloc<int64_t>(scan_tmp_items(nroots_));
+        int32_t *perm = arena_.alloc<int32_t>(N);
+        launch_group_by_slot(L.slot, N, (int32_t)nroots_, hist, hoffs, htmp, perm, s_);
+        kernels_ += 5;
+        a.perm = perm;
+        a.chunk_ctr = chunk_ctr_;
+    }
 
     // Fused count + write: the children are written by the count pass into
     // arrays sized for half of the free budget; if they fit they are compacted
@@ -574,8 +595,9 @@ void Engine::process(int32_t k, const Level &L) {
     while (Wc * 64 <= maxbit && Wc < L.W) Wc <<= 1;
     a.Wc = Wc;
     if (o_.verbose > 0)
-        fprintf(stderr, "[mce] level k=%d entries=%lld children=%lld leaves=%llu need=%d%s\n", k, (long long)N,
-                (long long)total, leaves, a.need, fused ? (total <= fcap ? " fused" : " fused-overflow") : "");
+        fprintf(stderr, "[mce] level k=%d entries=%lld W=%d children=%lld leaves=%llu completions=%lld need=%d%s%s\n",
+                k, (long long)N, L.W, (long long)total, leaves, (long long)completions, a.need,
+                fused ? (total <= fcap ? " fused" : " fused-overflow") : "", a.perm ? " smem" : "");
     const int32_t need_counted = a.need;
     a.fused = 0;  // a count-pass replay (staging growth) must not write children again
     if (leaves) handle_leaves(k + 1, (int64_t)leaves, a, 0);
@@ -656,6 +678,7 @@ void Engine::process(int32_t k, const Level &L) {
         C.parent = arena_.alloc<int32_t>(cnt);
         C.vloc = arena_.alloc<int32_t>(cnt);
         ExpandArgs w = a;
+        w.perm = nullptr;
         w.begin = a0;
         w.end = b;
         w.offsets = offs;
@@ -781,6 +804,7 @@ void Engine::do_class_w1(const int32_t *list, int64_t count) {
         if (entries > 0) {
             roots_ = ra.roots;
             adj_ = ra.adj;
+            nroots_ = nw;
             Level L2;
             L2.count = entries;
             L2.W = 1;
@@ -837,6 +861,7 @@ void Engine::do_class(int32_t cls, const int32_t *list, int64_t count) {
         kernels_ += 2;
         roots_ = roots;
         adj_ = adj;
+        nroots_ = nw;
         Level L1;
         L1.count = nw;
         L1.W = W_;
@@ -973,6 +998,10 @@ mce_result *Engine::run() {
     maxbit_ = reinterpret_cast<int32_t *>(leaf_total_ + 4);
     out_count_ = leaf_total_ + 5;
     pair_n_ = leaf_total_ + 6;
+    chunk_ctr_ = leaf_total_ + 7;
+    if (const char *sw = getenv("MCE_SMEM_MIN_W")) smem_min_w_ = atoi(sw);  // tuning hooks (A/B runs)
+    if (const char *sn = getenv("MCE_SMEM_MIN_N")) smem_min_n_ = atoll(sn);
+    if (const char *sp = getenv("MCE_SMEM_PER_ROOT")) smem_per_root_ = atoll(sp);
     pair_cap_ = std::max<int64_t>(4096, (int64_t)g_->pdesc.n / 3);
     g_->pdesc.ensure((size_t)pair_cap_ * 3);
     chain_dev_ = reinterpret_cast<LevelLink *>(g_->misc.get() + 256);

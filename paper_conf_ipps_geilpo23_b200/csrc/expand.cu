@@ -953,6 +953,237 @@ __global__ void expand_tile(const ExpandArgs a, int max_l) {
     if (!WRITE) flush_counters(a, nleaf, nclq, hb, ub);
 }
 
+// ---------------------------------------------------------------------------
+// Levels >= 2 with the root's adjacency matrix staged in shared memory
+// (W = G words per candidate set, G in {4, 8, 16}: at most 64 G rows of G
+// words, 128 KB for G = 16).  The level is visited through `perm`, which
+// groups its entries by root slot (launch_group_by_slot), so a block loads a
+// root's matrix once per run of that root's candidates and every colouring /
+// branching row read is a shared-memory hit instead of a dependent L2 trip.
+// A tile of G lanes per candidate (lane gl owns word gl), 32 / G candidates
+// per warp.  Count pass + fused child write (as expand_tile), leaves, clique
+// completions (reading 10) and pair completions (reading 13).
+//   The colouring order is kept per tile in shared memory as u16 local
+// indices with bit 15 marking the first vertex of each colour class (the
+// colour of position i is recovered while walking the order backwards).
+// ---------------------------------------------------------------------------
+constexpr uint16_t kClassStart = 0x8000u;
+
+template <int G>
+__device__ __forceinline__ int tile_sum(int x, unsigned gmask) {
+#pragma unroll
+    for (int o = G / 2; o > 0; o >>= 1) x += __shfl_xor_sync(gmask, x, o, G);
+    return x;
+}
+
+template <int G>
+__global__ void __launch_bounds__(512) expand_smem(const ExpandArgs a, int64_t nchunks) {
+    extern __shared__ uint64_t sA[];  // [64 G rows][G words], then the tiles' colouring orders
+    uint16_t *sOrd = reinterpret_cast<uint16_t *>(sA + 64 * G * G);
+    __shared__ int64_t s_chunk;
+    const int lane = threadIdx.x & 31;
+    const int gl = lane & (G - 1), gbase = lane & ~(G - 1);
+    const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << gbase);
+    const int tib = threadIdx.x / G, ntb = blockDim.x / G;
+    uint16_t *ord = sOrd + (int64_t)tib * 64 * G;
+    const int32_t k = a.k, need = a.need;
+    int32_t loaded = -1;
+    unsigned nleaf = 0;
+    unsigned long long nclq = 0;
+    int hb = -1, ub = 0;
+    for (;;) {
+        if (threadIdx.x == 0) s_chunk = (int64_t)atomicAdd(a.chunk_ctr, 1ull);
+        __syncthreads();
+        const int64_t c = s_chunk;
+        __syncthreads();
+        if (c >= nchunks) break;
+        const int64_t p1 = min(a.end, a.begin + (c + 1) * (int64_t)a.chunk);
+        for (int64_t q0 = a.begin + c * (int64_t)a.chunk; q0 < p1;) {
+            const int32_t slot = a.slot[a.perm[q0]];
+            int64_t lo = q0 + 1, hi = p1;  // end of this slot's run (positions are grouped by slot)
+            while (lo < hi) {
+                const int64_t mid = (lo + hi) >> 1;
+                if (a.slot[a.perm[mid]] == slot)
+                    lo = mid + 1;
+                else
+                    hi = mid;
+            }
+            const int64_t q1 = lo;
+            const RootInfo ri = a.roots[slot];
+            if (slot != loaded) {  // stage the root's rows (only the first G words matter: P < 64 G bits)
+                __syncthreads();
+                const int rows = min(ri.L, 64 * G);
+                const uint64_t *gA = a.adj + ri.abase;
+                for (int w = threadIdx.x; w < rows * G; w += blockDim.x)
+                    sA[w] = __ldg(gA + (int64_t)(w / G) * a.Wa + (w % G));
+                __syncthreads();
+                loaded = slot;
+            }
+            for (int64_t q = q0 + tib; q < q1; q += ntb) {
+                const int64_t e = a.perm[q];
+                const uint64_t P = a.P[e * a.Ps + gl];
+                // ---- colouring (bound 1) or plain order (bound 0)
+                int np = 0, ncol = 0;
+                if (a.bound == 1) {
+                    uint64_t U = P;
+                    while (__ballot_sync(gmask, U != 0ull) & gmask) {
+                        ++ncol;
+                        uint64_t Q = U;
+                        uint16_t first = kClassStart;
+                        while (true) {
+                            const unsigned m = (__ballot_sync(gmask, Q != 0ull) & gmask) >> gbase;
+                            if (!m) break;
+                            const int src = __ffs(m) - 1;
+                            const int bit = __shfl_sync(gmask, __ffsll((long long)Q) - 1, src, G);
+                            const int v = src * 64 + bit;
+                            Q &= ~sA[v * G + gl];
+                            if (gl == src) {
+                                Q &= ~(1ull << bit);
+                                U &= ~(1ull << bit);
+                            }
+                            if (gl == 0) ord[np] = (uint16_t)v | first;
+                            first = 0;
+                            ++np;
+                        }
+                    }
+                } else {
+                    const int pc = __popcll(P);
+                    int incl = pc;
+#pragma unroll
+                    for (int o = 1; o < G; o <<= 1) {
+                        const int y = __shfl_up_sync(gmask, incl, o, G);
+                        if (gl >= o) incl += y;
+                    }
+                    int pos = incl - pc;
+                    uint64_t q2 = P;
+                    while (q2) {  // every vertex its own "class": colour of position i = i + 1
+                        const int b = __ffsll((long long)q2) - 1;
+                        q2 &= q2 - 1;
+                        ord[pos++] = (uint16_t)(gl * 64 + b) | kClassStart;
+                    }
+                    np = __shfl_sync(gmask, incl, G - 1, G);
+                    ncol = np;
+                }
+                __syncwarp(gmask);
+                // ---- completions: P a clique (reading 10), or P's complement a matching (reading 13)
+                if (a.shortcut && a.bound == 1 && np >= 2 && ncol == np && k + np == need) {
+                    if (gl == 0) {
+                        ++nclq;
+                        a.counts[e] = 0;
+                    }
+                    uint64_t Pa[1] = {P};
+                    store_clique_leaf<G, 1>(a, e, Pa, ri, gmask);
+                    __syncwarp(gmask);
+                    continue;
+                }
+                if (a.shortcut && a.bound == 1 && ncol < np && np - ncol <= 40 && k + ncol == need && need <= 4096) {
+                    bool matching = true;
+                    for (int i = 0; i < np && matching; ++i) {
+                        const int v = ord[i] & 0x7fff;
+                        uint64_t nb = P & ~sA[v * G + gl];
+                        if (gl == (v >> 6)) nb &= ~(1ull << (v & 63));
+                        matching = tile_sum<G>(__popcll(nb), gmask) <= 1;
+                    }
+                    if (matching) {
+                        if (gl == 0) {
+                            nclq += 1ull << (np - ncol);
+                            reserve_pair_completions(a, e, np - ncol);
+                            a.counts[e] = 0;
+                        }
+                        __syncwarp(gmask);
+                        continue;
+                    }
+                }
+                // ---- branching from the last position (highest colour) down
+                int32_t cnt = 0;
+                if (k + ncol >= need) {
+                    uint64_t R = P;
+                    int col = ncol;
+                    for (int i = np - 1; i >= 0; --i) {
+                        if (k + col < need) break;
+                        const uint16_t o = ord[i];
+                        const int v = o & 0x7fff;
+                        if (o & kClassStart) --col;  // (after this vertex the next class down starts)
+                        const uint64_t C = R & sA[v * G + gl];
+                        const int pc = tile_sum<G>(__popcll(C), gmask);
+                        if (gl == (v >> 6)) R &= ~(1ull << (v & 63));
+                        if (pc == 0) {
+                            if (k + 1 >= need && gl == 0) {
+                                ++nleaf;
+                                store_leaf(a, e, v, ri);
+                            }
+                        } else if (k + 1 + pc >= need) {
+                            if (C) hb = max(hb, gl * 64 + 63 - __clzll((long long)C));
+                            ub = max(ub, k + 1 + pc);
+                            ++cnt;
+                        }
+                    }
+                }
+                if (gl == 0) a.counts[e] = cnt;
+                if (a.fused && cnt > 0) {  // reserve the children's slots, replay the branching, write them
+                    unsigned long long base = 0;
+                    if (gl == 0) base = atomicAdd(a.out_count, (unsigned long long)cnt);
+                    base = __shfl_sync(gmask, base, 0, G);
+                    if ((int64_t)(base + cnt) <= a.out_cap) {
+                        uint64_t R = P;
+                        int col = ncol;
+                        int64_t cpos = (int64_t)base;
+                        for (int i = np - 1; i >= 0; --i) {
+                            if (k + col < need) break;
+                            const uint16_t o = ord[i];
+                            const int v = o & 0x7fff;
+                            if (o & kClassStart) --col;
+                            const uint64_t C = R & sA[v * G + gl];
+                            const int pc = tile_sum<G>(__popcll(C), gmask);
+                            if (gl == (v >> 6)) R &= ~(1ull << (v & 63));
+                            if (pc > 0 && k + 1 + pc >= need) {
+                                a.cP[cpos * G + gl] = C;
+                                if (gl == 0) {
+                                    a.cslot[cpos] = slot;
+                                    a.cparent[cpos] = (int32_t)e;
+                                    a.cvloc[cpos] = v;
+                                }
+                                ++cpos;
+                            }
+                        }
+                    }
+                }
+                __syncwarp(gmask);
+            }
+            q0 = q1;
+        }
+    }
+    flush_counters(a, nleaf, nclq, hb, ub);
+}
+
+// counting sort of a level's entries by root slot (order inside a slot is
+// arbitrary).  Few slots take millions of entries, so the atomics are
+// aggregated over the lanes of a warp holding the same slot (__match_any_sync).
+__global__ void slot_hist_kernel(const int32_t *__restrict__ slot, int64_t n, int32_t *hist) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t i0 = (int64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31); i0 < n; i0 += stride) {
+        const int64_t i = i0 + (threadIdx.x & 31);
+        const int32_t sl = i < n ? slot[i] : -1;
+        const unsigned same = __match_any_sync(0xffffffffu, sl);
+        if (sl >= 0 && (threadIdx.x & 31) == __ffs(same) - 1) atomicAdd(hist + sl, __popc(same));
+    }
+}
+__global__ void slot_scatter_kernel(const int32_t *__restrict__ slot, int64_t n, unsigned long long *cursor,
+                                    int32_t *perm) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    const int lane = threadIdx.x & 31;
+    for (int64_t i0 = (int64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31); i0 < n; i0 += stride) {
+        const int64_t i = i0 + lane;
+        const int32_t sl = i < n ? slot[i] : -1;
+        const unsigned same = __match_any_sync(0xffffffffu, sl);
+        const int leader = __ffs(same) - 1;
+        unsigned long long base = 0;
+        if (sl >= 0 && lane == leader) base = atomicAdd(cursor + sl, (unsigned long long)__popc(same));
+        base = __shfl_sync(0xffffffffu, base, leader);
+        if (sl >= 0) perm[base + __popc(same & lanemask_lt())] = (int32_t)i;
+    }
+}
+
 __device__ __forceinline__ uint64_t mix64(uint64_t z) {
     z += 0x9E3779B97F4A7C15ull;
     z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
@@ -1147,9 +1378,38 @@ void launch_thread(const ExpandArgs &a, bool write_pass, cudaStream_t s) {
     MCE_LAUNCH_CHECK();
 }
 
+template <int G>
+void launch_smem(const ExpandArgs &a0, cudaStream_t s) {
+    constexpr int threads = 512;
+    ExpandArgs a = a0;
+    const int64_t n = a.end - a.begin;
+    const size_t smem = (size_t)64 * G * G * 8 + (size_t)(threads / G) * 64 * G * 2;
+    static int per_sm = 0;
+    if (!per_sm) {
+        MCE_CUDA(cudaFuncSetAttribute(expand_smem<G>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        MCE_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, expand_smem<G>, threads, smem));
+        per_sm = std::max(per_sm, 1);
+    }
+    const int64_t slots = (int64_t)num_sms() * per_sm;
+    // ~8 chunks per resident block (dynamic balance), at most 16 positions per tile; a
+    // small level (one entry per root at k = 1) takes chunks of one entry, spread over SMs
+    a.chunk = (int32_t)std::max<int64_t>(1, std::min<int64_t>(16 * (threads / G), ceil_div(n, 8 * slots)));
+    MCE_CUDA(cudaMemsetAsync(a.chunk_ctr, 0, sizeof(unsigned long long), s));
+    const int64_t nchunks = ceil_div(n, a.chunk);
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(nchunks, slots));
+    expand_smem<G><<<grid, threads, smem, s>>>(a, nchunks);
+    MCE_LAUNCH_CHECK();
+}
+
 void launch_expand(const ExpandArgs &a, bool write_pass, cudaStream_t s) {
     const int64_t items = a.end - a.begin;
     if (items <= 0) return;
+    if (!write_pass && a.perm) {  // shared-memory count pass (the caller grouped the level by slot)
+        if (a.Wp == 4) return launch_smem<4>(a, s);
+        if (a.Wp == 8) return launch_smem<8>(a, s);
+        if (a.Wp == 16) return launch_smem<16>(a, s);
+        fail(1, "internal: shared-memory expansion for an unsupported width");
+    }
     if (a.Wp == 1) {
         launch_thread<1>(a, write_pass, s);
     } else if (a.Wp == 2) {
@@ -1168,6 +1428,18 @@ void launch_expand(const ExpandArgs &a, bool write_pass, cudaStream_t s) {
     } else {
         launch_tile<32, 8>(a, write_pass, s);
     }
+}
+
+void launch_group_by_slot(const int32_t *slot, int64_t n, int32_t nslots, int32_t *hist, int64_t *offs,
+                          int64_t *scan_tmp, int32_t *perm, cudaStream_t s) {
+    if (n <= 0) return;
+    MCE_CUDA(cudaMemsetAsync(hist, 0, sizeof(int32_t) * std::max<int32_t>(nslots, 1), s));
+    slot_hist_kernel<<<grid_for(n, 256), 256, 0, s>>>(slot, n, hist);
+    MCE_LAUNCH_CHECK();
+    exclusive_scan_i32(hist, offs, nslots, scan_tmp, s);
+    slot_scatter_kernel<<<grid_for(n, 256), 256, 0, s>>>(slot, n, reinterpret_cast<unsigned long long *>(offs),
+                                                          perm);
+    MCE_LAUNCH_CHECK();
 }
 
 void launch_materialize_pairs(const ExpandArgs &a, int64_t n, cudaStream_t s) {

@@ -84,6 +84,12 @@ struct ExpandArgs {
     int32_t fused;
     unsigned long long *out_count;
     int64_t out_cap;
+    // shared-memory path (expand_smem, count pass only): position q of the
+    // level is entry perm[q] (entries grouped by root slot); blocks take
+    // chunks of `chunk` positions from *chunk_ctr (zeroed by the caller)
+    const int32_t *perm;
+    unsigned long long *chunk_ctr;
+    int32_t chunk;
 };
 
 // Fused root level for W == 1 roots (roots.cu): one warp per root builds the
@@ -147,6 +153,11 @@ void launch_build_adj(const RootInfo *roots, int64_t nroots, int W, const int64_
 void launch_init_level1(const RootInfo *roots, int64_t nroots, int W, uint64_t *P, int32_t *slot, int32_t *parent,
                         int32_t *vloc, cudaStream_t s);
 void launch_expand(const ExpandArgs &a, bool write_pass, cudaStream_t s);
+// widths the shared-memory count pass handles (the root's matrix, 64 W rows x W words, staged per block)
+inline bool smem_width(int W) { return W == 4 || W == 8 || W == 16; }
+// perm = the level's entries [0, n) grouped by slot (counting sort: hist over nslots, scan, scatter)
+void launch_group_by_slot(const int32_t *slot, int64_t n, int32_t nslots, int32_t *hist, int64_t *offs,
+                          int64_t *scan_tmp, int32_t *perm, cudaStream_t s);
 void launch_classify_roots(int64_t n, const int64_t *orp, int32_t min_len, int32_t shard_rank, int32_t shard_count,
                            int32_t *cls, int64_t *hist, cudaStream_t s);
 void launch_find_window(const int64_t *prefix, int64_t hi, int64_t lo_min, int64_t room, int64_t row_bytes,

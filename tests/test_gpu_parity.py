@@ -7,6 +7,8 @@ rest is checked for validity).
 """
 
 import functools
+import json
+import os
 
 import numpy as np
 import pytest
@@ -359,3 +361,103 @@ def test_overlap_off_matches(key):
         m = mce()
         f = m.Graph(g.rowptr, g.col).find_one(window=8)
         assert f.omega == om and oracle.is_clique(*g.numpy(), f.cliques[0])
+
+
+@pytest.mark.parametrize("min_w", [4, 8, 16, 99])
+@pytest.mark.parametrize("key", ["ER400d", "ER150d", "RMAT13", "RMAT15", "K257", "K130", "T(36,12)", "CP8+K600",
+                                 "CP12+K300", "planted", "Paley17"])
+def test_smem_expand_widths(key, min_w, monkeypatch):
+    """The shared-memory count pass (expand_smem, root matrix staged per block,
+    entries grouped by slot) from width min_w up, against the oracle; 99 = off
+    (global-memory tile / thread kernels)."""
+    monkeypatch.setenv("MCE_SMEM_MIN_W", str(min_w))
+    monkeypatch.setenv("MCE_SMEM_MIN_N", "1")  # every level of the width, however small
+    monkeypatch.setenv("MCE_SMEM_PER_ROOT", "0")
+    g = GRAPHS[key]()
+    om, cl = oracle_answer(key)
+    for kw in (dict(), dict(fused_levels=False), dict(clique_shortcut=False), dict(bound="size", heuristic="none")):
+        if kw.get("bound") == "size" and key in ("RMAT15", "RMAT13", "CP8+K600", "CP12+K300", "K257", "ER400d"):
+            continue
+        r = run_enum(g, **kw)
+        assert (r.omega, r.count) == (om, len(cl)) and np.array_equal(r.cliques, cl), kw
+    r = run_enum(g, smem_expand=False)
+    assert (r.omega, r.count) == (om, len(cl)) and np.array_equal(r.cliques, cl)
+    f = mce().Graph(g.rowptr, g.col).find_one(window=4)
+    assert f.omega == om and oracle.is_clique(*g.numpy(), f.cliques[0])
+
+
+GOLDEN = os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden")
+
+
+def golden(name):
+    path = os.path.join(GOLDEN, f"{name}.json")
+    if not os.path.exists(path):
+        pytest.skip(f"{path} not written yet (scripts/make_golden_rmat.py)")
+    with open(path) as f:
+        return json.load(f)
+
+
+def rmat_graph(name, device):
+    if name in ("rmat22", "rmat26"):
+        return G.make_config(name, device=device)
+    return G.rmat(int(name[4:]), 16, 0.57, 0.19, 0.19, seed=1, device=device)
+
+
+def check_stored_rows(rows, omega, rp, col, sample=64):
+    """Every stored row: omega distinct ascending vertices, rows distinct and in
+    lexicographic order; a spread sample is checked to be a clique."""
+    assert rows.ndim == 2 and rows.shape[1] == omega
+    assert np.all(np.diff(rows, axis=1) > 0)
+    if rows.shape[0] > 1:
+        order = np.lexsort(rows.T[::-1])
+        assert np.array_equal(order, np.arange(rows.shape[0]))
+        assert np.all(np.any(rows[1:] != rows[:-1], axis=1))
+    for i in np.linspace(0, rows.shape[0] - 1, min(sample, rows.shape[0])).astype(np.int64):
+        assert oracle.is_clique(rp, col, rows[i])
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("name", ["rmat20", "rmat22"])
+def test_config_rmat_golden(name):
+    """BASELINE configs[2] (rmat22) and the same recipe at scale 20: omega and
+    the exact multiplicity against the oracle's count (tests/golden, written by
+    scripts/make_golden_rmat.py from oracle/ only); the 2^16 stored rows are
+    valid, distinct maximum cliques."""
+    gd = golden(name)
+    g = rmat_graph(name, "cuda")
+    r = run_enum(g, max_cliques=1 << 16)
+    assert (r.omega, r.count) == (gd["omega"], gd["multiplicity"])
+    assert r.cliques.shape[0] == min(1 << 16, gd["multiplicity"])
+    rp, col = g.rowptr.cpu().numpy(), g.col.cpu().numpy()
+    check_stored_rows(r.cliques, r.omega, rp, col)
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("depth", [0, 3])
+def test_config_rmat22_shards(depth):
+    """configs[2] at "2 GPUs": two graph handles (two processes' state), the
+    deterministic orientation computed by each, root (depth 0) or level-3 hash
+    deal: the shards' multiplicities add up to the oracle's."""
+    gd = golden("rmat22")
+    g = rmat_graph("rmat22", "cuda")
+    m = mce()
+    parts = []
+    for rank in range(2):
+        h = m.Graph(g.rowptr, g.col)
+        parts.append(h.enumerate(orientation="degeneracy_det", shard_rank=rank, shard_count=2, shard_depth=depth,
+                                 max_cliques=1 << 10))
+        h.close()
+    omega = max(p.omega for p in parts)
+    assert omega == gd["omega"]
+    assert sum(p.count for p in parts if p.omega == omega) == gd["multiplicity"]
+
+
+@pytest.mark.slow
+def test_config_rmat26_golden():
+    """BASELINE configs[4] on one GPU against the oracle's count (when the
+    oracle run has been committed)."""
+    gd = golden("rmat26")
+    g = rmat_graph("rmat26", "cuda")
+    r = run_enum(g, max_cliques=1 << 12)
+    assert (r.omega, r.count) == (gd["omega"], gd["multiplicity"])
+    check_stored_rows(r.cliques, r.omega, g.rowptr.cpu().numpy(), g.col.cpu().numpy(), sample=16)
