@@ -524,8 +524,12 @@ void Engine::process(int32_t k, const Level &L) {
     // root slot so a block stages one root's matrix per run of its candidates
     // (only when a root has many candidates on average: one entry per root, as at
     // level 1, gains nothing from staging 64 W rows and loses the L2's parallelism)
-    if (!o_.no_smem_expand && smem_width(L.W) && L.W >= smem_min_w_ && N >= smem_min_n_ && nroots_ > 0 &&
-        N >= smem_per_root_ * nroots_) {
+    // A level of at most one entry per SM is the other case: every candidate is a
+    // long serial colouring chain with nothing to overlap it, and a block of its
+    // own turns the chain's row reads from L2 into shared-memory hits.
+    const bool many_per_root = N >= smem_min_n_ && N >= smem_per_root_ * nroots_;
+    const bool few_chains = N <= num_sms();
+    if (!o_.no_smem_expand && smem_width(L.W) && L.W >= smem_min_w_ && nroots_ > 0 && (many_per_root || few_chains)) {
         int32_t *hist = arena_.alloc<int32_t>(nroots_);
         int64_t *hoffs = arena_.alloc<int64_t>(nroots_ + 1);
         int64_t *htmp = arena_.alloc<int64_t>(scan_tmp_items(nroots_));

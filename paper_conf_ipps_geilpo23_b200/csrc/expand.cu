@@ -20,6 +20,8 @@
 // its branch: when its size reaches `need` it is recorded (leaf).
 // Children go to the next level through the count pass -> scan -> write pass
 // (Algorithm 2 lines 29-35: COUNTCLIQUES, CUBSCAN, OUTPUTNEWCLIQUES).
+#include <cstdlib>
+
 #include "expand.cuh"
 
 namespace mce {
@@ -955,20 +957,33 @@ __global__ void expand_tile(const ExpandArgs a, int max_l) {
 
 // ---------------------------------------------------------------------------
 // Levels >= 2 with the root's adjacency matrix staged in shared memory
-// (W = G words per candidate set, G in {4, 8, 16}: at most 64 G rows of G
-// words, 128 KB for G = 16).  The level is visited through `perm`, which
-// groups its entries by root slot (launch_group_by_slot), so a block loads a
-// root's matrix once per run of that root's candidates and every colouring /
-// branching row read is a shared-memory hit instead of a dependent L2 trip.
-// A tile of G lanes per candidate (lane gl owns word gl), 32 / G candidates
-// per warp.  Count pass + fused child write (as expand_tile), leaves, clique
-// completions (reading 10) and pair completions (reading 13).
+// (expand_lock; W = G words per candidate set, G in {4, 8, 16}: at most 64 G
+// rows of G words, 128 KB for G = 16).  The level is visited through `perm`,
+// which groups its entries by root slot (launch_group_by_slot), so a block
+// loads a root's matrix once per run of that root's candidates and every
+// colouring / branching row read is a shared-memory hit.
+//   A warp holds T = 32 / G candidates, one G-lane tile each (lane gl owns word
+// gl), and runs them in LOCKSTEP: every loop is warp-uniform (it runs until
+// the last tile is done, finished tiles predicated off) and every vote /
+// shuffle takes the full mask, each tile reading its own G bits.  (Tiles that
+// diverged instead cost ~45 warp instructions per colouring step, most of them
+// the divergence checks of partial-mask collectives; a thread per candidate
+// was 5x slower still: 32 unrelated serial chains diverge in a warp.)
+// Count pass + fused child write, leaves, clique completions (reading 10) and
+// pair completions (reading 13).
 //   The colouring order is kept per tile in shared memory as u16 local
 // indices with bit 15 marking the first vertex of each colour class (the
 // colour of position i is recovered while walking the order backwards).
 // ---------------------------------------------------------------------------
 constexpr uint16_t kClassStart = 0x8000u;
+constexpr unsigned kFull = 0xffffffffu;
 
+template <int G>
+__device__ __forceinline__ int tile_sum_full(int x) {  // sum over the lane's aligned G-lane tile, full-warp shuffles
+#pragma unroll
+    for (int o = G / 2; o > 0; o >>= 1) x += __shfl_xor_sync(kFull, x, o);
+    return x;
+}
 template <int G>
 __device__ __forceinline__ int tile_sum(int x, unsigned gmask) {
 #pragma unroll
@@ -977,15 +992,17 @@ __device__ __forceinline__ int tile_sum(int x, unsigned gmask) {
 }
 
 template <int G>
-__global__ void __launch_bounds__(512) expand_smem(const ExpandArgs a, int64_t nchunks) {
-    extern __shared__ uint64_t sA[];  // [64 G rows][G words], then the tiles' colouring orders
+__global__ void __launch_bounds__(512) expand_lock(const ExpandArgs a, int64_t nchunks) {
+    constexpr int T = 32 / G;                       // tiles (candidates) per warp
+    constexpr unsigned TM = G == 32 ? kFull : ((1u << G) - 1u);
+    extern __shared__ uint64_t sA[];                // [64 G rows][G words], then the tiles' colouring orders
     uint16_t *sOrd = reinterpret_cast<uint16_t *>(sA + 64 * G * G);
     __shared__ int64_t s_chunk;
     const int lane = threadIdx.x & 31;
-    const int gl = lane & (G - 1), gbase = lane & ~(G - 1);
-    const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << gbase);
-    const int tib = threadIdx.x / G, ntb = blockDim.x / G;
-    uint16_t *ord = sOrd + (int64_t)tib * 64 * G;
+    const int gl = lane & (G - 1), gbase = lane & ~(G - 1), tiw = lane / G;
+    const unsigned gmask = TM << gbase;
+    const int warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
+    uint16_t *ord = sOrd + (int64_t)(threadIdx.x / G) * 64 * G;
     const int32_t k = a.k, need = a.need;
     int32_t loaded = -1;
     unsigned nleaf = 0;
@@ -1019,22 +1036,33 @@ __global__ void __launch_bounds__(512) expand_smem(const ExpandArgs a, int64_t n
                 __syncthreads();
                 loaded = slot;
             }
-            for (int64_t q = q0 + tib; q < q1; q += ntb) {
-                const int64_t e = a.perm[q];
-                const uint64_t P = a.P[e * a.Ps + gl];
-                // ---- colouring (bound 1) or plain order (bound 0)
+            // warp-uniform trips: T candidates per warp per trip
+            for (int64_t qb = q0 + (int64_t)warp * T; qb < q1; qb += (int64_t)nwarps * T) {
+                const int64_t q = qb + tiw;
+                const bool active = q < q1;
+                const int64_t e = active ? a.perm[q] : 0;
+                const uint64_t P = active ? a.P[e * a.Ps + gl] : 0ull;
+                // ---- colouring, one vertex per tile per trip
                 int np = 0, ncol = 0;
                 if (a.bound == 1) {
-                    uint64_t U = P;
-                    while (__ballot_sync(gmask, U != 0ull) & gmask) {
-                        ++ncol;
-                        uint64_t Q = U;
-                        uint16_t first = kClassStart;
-                        while (true) {
-                            const unsigned m = (__ballot_sync(gmask, Q != 0ull) & gmask) >> gbase;
-                            if (!m) break;
-                            const int src = __ffs(m) - 1;
-                            const int bit = __shfl_sync(gmask, __ffsll((long long)Q) - 1, src, G);
+                    uint64_t U = P, Q = 0ull;
+                    uint16_t first = 0;
+                    while (true) {
+                        const unsigned bq = __ballot_sync(kFull, Q != 0ull), bu = __ballot_sync(kFull, U != 0ull);
+                        if (!(bq | bu)) break;  // every tile coloured
+                        unsigned mq = (bq >> gbase) & TM;
+                        if (!mq) {  // this tile's class is closed: the next one starts from what is left
+                            const unsigned mu = (bu >> gbase) & TM;
+                            if (mu) {
+                                Q = U;
+                                mq = mu;
+                                ++ncol;
+                                first = kClassStart;
+                            }
+                        }
+                        const int src = mq ? __ffs(mq) - 1 : 0;
+                        const int bit = __shfl_sync(kFull, __ffsll((long long)Q) - 1, gbase + src);
+                        if (mq) {
                             const int v = src * 64 + bit;
                             Q &= ~sA[v * G + gl];
                             if (gl == src) {
@@ -1051,7 +1079,7 @@ __global__ void __launch_bounds__(512) expand_smem(const ExpandArgs a, int64_t n
                     int incl = pc;
 #pragma unroll
                     for (int o = 1; o < G; o <<= 1) {
-                        const int y = __shfl_up_sync(gmask, incl, o, G);
+                        const int y = __shfl_up_sync(kFull, incl, o);
                         if (gl >= o) incl += y;
                     }
                     int pos = incl - pc;
@@ -1061,22 +1089,23 @@ __global__ void __launch_bounds__(512) expand_smem(const ExpandArgs a, int64_t n
                         q2 &= q2 - 1;
                         ord[pos++] = (uint16_t)(gl * 64 + b) | kClassStart;
                     }
-                    np = __shfl_sync(gmask, incl, G - 1, G);
+                    np = __shfl_sync(kFull, incl, gbase + G - 1);
                     ncol = np;
                 }
-                __syncwarp(gmask);
-                // ---- completions: P a clique (reading 10), or P's complement a matching (reading 13)
-                if (a.shortcut && a.bound == 1 && np >= 2 && ncol == np && k + np == need) {
-                    if (gl == 0) {
+                __syncwarp();
+                // ---- completions (rare: divergent, tile-mask collectives)
+                bool done = !active;
+                if (!done && a.shortcut && a.bound == 1 && np >= 2 && ncol == np && k + np == need) {
+                    if (gl == 0) {  // P is a clique (reading 10)
                         ++nclq;
                         a.counts[e] = 0;
                     }
                     uint64_t Pa[1] = {P};
                     store_clique_leaf<G, 1>(a, e, Pa, ri, gmask);
-                    __syncwarp(gmask);
-                    continue;
+                    done = true;
                 }
-                if (a.shortcut && a.bound == 1 && ncol < np && np - ncol <= 40 && k + ncol == need && need <= 4096) {
+                if (!done && a.shortcut && a.bound == 1 && ncol < np && np - ncol <= 40 && k + ncol == need &&
+                    need <= 4096) {  // P's complement a matching (reading 13)
                     bool matching = true;
                     for (int i = 0; i < np && matching; ++i) {
                         const int v = ord[i] & 0x7fff;
@@ -1090,51 +1119,66 @@ __global__ void __launch_bounds__(512) expand_smem(const ExpandArgs a, int64_t n
                             reserve_pair_completions(a, e, np - ncol);
                             a.counts[e] = 0;
                         }
-                        __syncwarp(gmask);
-                        continue;
+                        done = true;
                     }
                 }
-                // ---- branching from the last position (highest colour) down
+                __syncwarp();
+                // ---- branching from the last position (highest colour) down, in lockstep
                 int32_t cnt = 0;
-                if (k + ncol >= need) {
+                {
+                    bool stop = done || k + ncol < need;
                     uint64_t R = P;
-                    int col = ncol;
-                    for (int i = np - 1; i >= 0; --i) {
-                        if (k + col < need) break;
-                        const uint16_t o = ord[i];
+                    int col = ncol, pos = np - 1;
+                    while (__ballot_sync(kFull, !stop)) {
+                        if (!stop && (pos < 0 || k + col < need)) stop = true;
+                        const uint16_t o = stop ? 0 : ord[pos];
                         const int v = o & 0x7fff;
-                        if (o & kClassStart) --col;  // (after this vertex the next class down starts)
-                        const uint64_t C = R & sA[v * G + gl];
-                        const int pc = tile_sum<G>(__popcll(C), gmask);
-                        if (gl == (v >> 6)) R &= ~(1ull << (v & 63));
-                        if (pc == 0) {
-                            if (k + 1 >= need && gl == 0) {
-                                ++nleaf;
-                                store_leaf(a, e, v, ri);
+                        const uint64_t C = stop ? 0ull : (R & sA[v * G + gl]);
+                        const int pc = tile_sum_full<G>(__popcll(C));
+                        if (!stop) {
+                            if (o & kClassStart) --col;
+                            --pos;
+                            if (gl == (v >> 6)) R &= ~(1ull << (v & 63));
+                            if (pc == 0) {
+                                if (k + 1 >= need && gl == 0) {
+                                    ++nleaf;
+                                    store_leaf(a, e, v, ri);
+                                }
+                            } else if (k + 1 + pc >= need) {
+                                if (C) hb = max(hb, gl * 64 + 63 - __clzll((long long)C));
+                                ub = max(ub, k + 1 + pc);
+                                ++cnt;
                             }
-                        } else if (k + 1 + pc >= need) {
-                            if (C) hb = max(hb, gl * 64 + 63 - __clzll((long long)C));
-                            ub = max(ub, k + 1 + pc);
-                            ++cnt;
                         }
                     }
                 }
-                if (gl == 0) a.counts[e] = cnt;
-                if (a.fused && cnt > 0) {  // reserve the children's slots, replay the branching, write them
+                if (active && !done && gl == 0) a.counts[e] = cnt;
+                if (a.fused) {  // reserve the warp's children at once, replay the branching, write them
+                    int tot = cnt;  // exclusive scan over the warp's tiles (value held by every lane of a tile)
+                    int excl = 0;
+#pragma unroll
+                    for (int t = 0; t < T; ++t) {
+                        const int ct = __shfl_sync(kFull, cnt, t * G);
+                        if (t < tiw) excl += ct;
+                        if (t == 0) tot = ct; else tot += ct;
+                    }
                     unsigned long long base = 0;
-                    if (gl == 0) base = atomicAdd(a.out_count, (unsigned long long)cnt);
-                    base = __shfl_sync(gmask, base, 0, G);
-                    if ((int64_t)(base + cnt) <= a.out_cap) {
-                        uint64_t R = P;
-                        int col = ncol;
-                        int64_t cpos = (int64_t)base;
-                        for (int i = np - 1; i >= 0; --i) {
-                            if (k + col < need) break;
-                            const uint16_t o = ord[i];
-                            const int v = o & 0x7fff;
+                    if (lane == 0 && tot) base = atomicAdd(a.out_count, (unsigned long long)tot);
+                    base = __shfl_sync(kFull, base, 0) + (unsigned long long)excl;
+                    const bool fits = (int64_t)(base - excl + tot) <= a.out_cap;
+                    bool stop = done || cnt == 0 || !fits || k + ncol < need;
+                    uint64_t R = P;
+                    int col = ncol, pos = np - 1;
+                    int64_t cpos = (int64_t)base;
+                    while (__ballot_sync(kFull, !stop)) {
+                        if (!stop && (pos < 0 || k + col < need)) stop = true;
+                        const uint16_t o = stop ? 0 : ord[pos];
+                        const int v = o & 0x7fff;
+                        const uint64_t C = stop ? 0ull : (R & sA[v * G + gl]);
+                        const int pc = tile_sum_full<G>(__popcll(C));
+                        if (!stop) {
                             if (o & kClassStart) --col;
-                            const uint64_t C = R & sA[v * G + gl];
-                            const int pc = tile_sum<G>(__popcll(C), gmask);
+                            --pos;
                             if (gl == (v >> 6)) R &= ~(1ull << (v & 63));
                             if (pc > 0 && k + 1 + pc >= need) {
                                 a.cP[cpos * G + gl] = C;
@@ -1148,7 +1192,7 @@ __global__ void __launch_bounds__(512) expand_smem(const ExpandArgs a, int64_t n
                         }
                     }
                 }
-                __syncwarp(gmask);
+                __syncwarp();
             }
             q0 = q1;
         }
@@ -1379,25 +1423,25 @@ void launch_thread(const ExpandArgs &a, bool write_pass, cudaStream_t s) {
 }
 
 template <int G>
-void launch_smem(const ExpandArgs &a0, cudaStream_t s) {
+void launch_lock(const ExpandArgs &a0, cudaStream_t s) {
     constexpr int threads = 512;
     ExpandArgs a = a0;
     const int64_t n = a.end - a.begin;
     const size_t smem = (size_t)64 * G * G * 8 + (size_t)(threads / G) * 64 * G * 2;
     static int per_sm = 0;
     if (!per_sm) {
-        MCE_CUDA(cudaFuncSetAttribute(expand_smem<G>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        MCE_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, expand_smem<G>, threads, smem));
+        MCE_CUDA(cudaFuncSetAttribute(expand_lock<G>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        MCE_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, expand_lock<G>, threads, smem));
         per_sm = std::max(per_sm, 1);
     }
     const int64_t slots = (int64_t)num_sms() * per_sm;
-    // ~8 chunks per resident block (dynamic balance), at most 16 positions per tile; a
+    // ~8 chunks per resident block (dynamic balance), at most 16 candidates per tile; a
     // small level (one entry per root at k = 1) takes chunks of one entry, spread over SMs
     a.chunk = (int32_t)std::max<int64_t>(1, std::min<int64_t>(16 * (threads / G), ceil_div(n, 8 * slots)));
     MCE_CUDA(cudaMemsetAsync(a.chunk_ctr, 0, sizeof(unsigned long long), s));
     const int64_t nchunks = ceil_div(n, a.chunk);
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(nchunks, slots));
-    expand_smem<G><<<grid, threads, smem, s>>>(a, nchunks);
+    expand_lock<G><<<grid, threads, smem, s>>>(a, nchunks);
     MCE_LAUNCH_CHECK();
 }
 
@@ -1405,9 +1449,9 @@ void launch_expand(const ExpandArgs &a, bool write_pass, cudaStream_t s) {
     const int64_t items = a.end - a.begin;
     if (items <= 0) return;
     if (!write_pass && a.perm) {  // shared-memory count pass (the caller grouped the level by slot)
-        if (a.Wp == 4) return launch_smem<4>(a, s);
-        if (a.Wp == 8) return launch_smem<8>(a, s);
-        if (a.Wp == 16) return launch_smem<16>(a, s);
+        if (a.Wp == 4) return launch_lock<4>(a, s);
+        if (a.Wp == 8) return launch_lock<8>(a, s);
+        if (a.Wp == 16) return launch_lock<16>(a, s);
         fail(1, "internal: shared-memory expansion for an unsupported width");
     }
     if (a.Wp == 1) {

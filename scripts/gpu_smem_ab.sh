@@ -2,19 +2,20 @@
 TAG=${1:-s}
 mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.build()" > gpurun_out/${TAG}_build.log 2>&1; echo build rc=$?
-timeout 900 python -m pytest tests/test_gpu_parity.py -q -m gpu -x -p no:cacheprovider -k "smem or enumerate_matches or completions" > gpurun_out/${TAG}_pytest.log 2>&1; echo pytest rc=$?
+timeout 900 python -m pytest tests/test_gpu_parity.py -q -m gpu -x -p no:cacheprovider -k "smem or enumerate_matches or completions or overflow or chunking" > gpurun_out/${TAG}_pytest.log 2>&1; echo pytest rc=$?
 tail -5 gpurun_out/${TAG}_pytest.log
-for w in 99 16 8 4; do
-  MCE_SMEM_MIN_W=$w timeout 300 python bench.py --config dense800 --steps 3 --warmup 2 --no-cpu-baseline --no-e2e > gpurun_out/${TAG}_dense_w$w.log 2>&1
+for w in 99 8 4 16; do
+  K=thr; case $w in tile*) K=tile; w=${w#tile};; esac
+  MCE_SMEM_KIND=$K MCE_SMEM_MIN_W=$w timeout 300 python bench.py --config dense800 --steps 3 --warmup 2 --no-cpu-baseline --no-e2e > gpurun_out/${TAG}_dense_w$w.log 2>&1
   python - "$w" gpurun_out/${TAG}_dense_w$w.log <<'PY'
-import json,sys
+import json,sys,os
 l=[x for x in open(sys.argv[2]) if x.startswith('{')]
 if l:
-    d=json.loads(l[-1]); print("dense800 minw", sys.argv[1], "ms", round(d["ms_per_step"],2), "count_ms", round(d["details"]["phases_ms"]["expand_count_ms"],2), d["verified"]["ok"])
+    d=json.loads(l[-1]); print("dense800 minw", sys.argv[1], os.environ.get("MCE_SMEM_KIND"), "ms", round(d["ms_per_step"],2), "count_ms", round(d["details"]["phases_ms"]["expand_count_ms"],2), d["verified"]["ok"])
 else: print("dense800 minw", sys.argv[1], "FAILED"); print(open(sys.argv[2]).read()[-2000:])
 PY
 done
-for w in 99 8; do
+for w in 99 4; do
   MCE_SMEM_MIN_W=$w timeout 300 python bench.py --config rmat22 --steps 3 --warmup 2 --no-cpu-baseline --no-e2e > gpurun_out/${TAG}_rmat22_w$w.log 2>&1
   python - "$w" gpurun_out/${TAG}_rmat22_w$w.log <<'PY'
 import json,sys

@@ -32,7 +32,7 @@ def mce():
 # the kernels' layout) wherever it finishes in seconds; the colouring oracle
 # (pinned against it and against closed forms in tests/test_oracle.py) only
 # where the |C|+|P| bound alone is exponential (R-MAT hub cores, CP(j)+K_t).
-COLOUR_ONLY = {"RMAT15", "CP8+K600", "CP12+K300"}
+COLOUR_ONLY = {"RMAT15", "CP8+K600", "CP12+K300", "ER700w8", "ER1000w8"}
 
 
 @functools.lru_cache(maxsize=None)
@@ -74,6 +74,10 @@ GRAPHS = {
     # root out-degree 615: the (512, 1024] width class (W = 16) of the R-MAT scale 22 / 26 roots
     "CP8+K600": lambda: G.cocktail_party_join(8, 600, seed=8600),
     "CP12+K300": lambda: G.cocktail_party_join(12, 300, seed=12300),  # W = 8, 4096 cliques
+    # dense, degeneracy 286 / 314: W = 8 roots whose candidates keep many colour
+    # classes within the bound (more than the shared-memory kernels' class ring)
+    "ER700w8": lambda: G.erdos_renyi(700, 0.45, seed=3),
+    "ER1000w8": lambda: G.erdos_renyi(1000, 0.35, seed=2),
 }
 
 
@@ -363,21 +367,33 @@ def test_overlap_off_matches(key):
         assert f.omega == om and oracle.is_clique(*g.numpy(), f.cliques[0])
 
 
+@pytest.mark.parametrize("kind", ["thr", "tile"])
 @pytest.mark.parametrize("min_w", [4, 8, 16, 99])
 @pytest.mark.parametrize("key", ["ER400d", "ER150d", "RMAT13", "RMAT15", "K257", "K130", "T(36,12)", "CP8+K600",
-                                 "CP12+K300", "planted", "Paley17"])
-def test_smem_expand_widths(key, min_w, monkeypatch):
-    """The shared-memory count pass (expand_smem, root matrix staged per block,
-    entries grouped by slot) from width min_w up, against the oracle; 99 = off
+                                 "CP12+K300", "planted", "Paley17", "ER700w8", "ER1000w8"])
+def test_smem_expand_widths(key, min_w, kind, monkeypatch):
+    """The shared-memory count pass (root matrix staged per block, entries
+    grouped by slot; thread per candidate = expand_thr, tile per candidate =
+    expand_smem) from width min_w up, against the oracle; 99 = off
     (global-memory tile / thread kernels)."""
+    if min_w == 99 and kind == "tile":
+        pytest.skip("same as kind=thr with the shared-memory pass off")
+    monkeypatch.setenv("MCE_SMEM_KIND", kind)
     monkeypatch.setenv("MCE_SMEM_MIN_W", str(min_w))
     monkeypatch.setenv("MCE_SMEM_MIN_N", "1")  # every level of the width, however small
     monkeypatch.setenv("MCE_SMEM_PER_ROOT", "0")
     g = GRAPHS[key]()
     om, cl = oracle_answer(key)
-    for kw in (dict(), dict(fused_levels=False), dict(clique_shortcut=False), dict(bound="size", heuristic="none")):
-        if kw.get("bound") == "size" and key in ("RMAT15", "RMAT13", "CP8+K600", "CP12+K300", "K257", "ER400d"):
+    # small budgets: the fused pass overflows and the (global-memory) write pass
+    # must reproduce exactly the children the shared-memory count pass counted
+    for kw in (dict(), dict(fused_levels=False), dict(clique_shortcut=False), dict(bound="size", heuristic="none"),
+               dict(budget_bytes=6 << 20, heuristic="none", fused_levels=False),
+               dict(budget_bytes=24 << 20, heuristic="single_degree")):
+        if kw.get("bound") == "size" and key in ("RMAT15", "RMAT13", "CP8+K600", "CP12+K300", "K257", "ER400d",
+                                                 "ER700w8", "ER1000w8"):
             continue
+        if "budget_bytes" in kw and (key.startswith("K") or key.startswith("CP")):
+            continue  # 256-level chains: a 6 MB budget is below one candidate's chunk share (MCE_ERR_BUDGET)
         r = run_enum(g, **kw)
         assert (r.omega, r.count) == (om, len(cl)) and np.array_equal(r.cliques, cl), kw
     r = run_enum(g, smem_expand=False)
