@@ -49,6 +49,7 @@ class Options(ctypes.Structure):
         ("no_fused_expand", ctypes.c_int32),
         ("shard_depth", ctypes.c_int32),
         ("no_overlap", ctypes.c_int32),
+        ("no_reroot", ctypes.c_int32),
         ("no_smem_expand", ctypes.c_int32),
     ]
 

@@ -125,6 +125,7 @@ void mce_default_options(mce_options *o) {
     o->no_fused_expand = 0;
     o->no_overlap = 0;
     o->no_smem_expand = 0;
+    o->no_reroot = 0;
     o->shard_depth = 0;
 }
 

@@ -181,6 +181,7 @@ class Engine {
     int32_t need() const { return find_one_ ? best_ + 1 : best_; }
     void process(int32_t k, const Level &L);
     bool run_small(int32_t k, const Level &L);
+    bool reroot(int32_t k, const Level &L);
     void do_class(int32_t cls, const int32_t *list, int64_t count);
     void do_class_w1(const int32_t *list, int64_t count);
     void handle_leaves(int32_t size, int64_t cnt, ExpandArgs &a, int kind = 0);
@@ -215,6 +216,11 @@ class Engine {
     unsigned long long *pair_n_ = nullptr;      // g->misc[6] pair-completion descriptors
     unsigned long long *chunk_ctr_ = nullptr;   // g->misc[7] work counter of the shared-memory count pass
     int64_t nroots_ = 0;                        // roots of the current window (slots 0 .. nroots_ - 1)
+    const int32_t *vtab_ = nullptr;             // vertex table of the window's roots (g->ocol, or re-rooted lists)
+    const int32_t *prefix_ = nullptr;           // re-rooted window: per-root clique prefix (k0_ vertices each)
+    int32_t k0_ = 0;
+    int reroot_min_w_ = 32;                     // levels this wide re-root their candidates (0: never)
+    int32_t no_reroot_level_ = -1;              // the level being processed in a re-rooted space
     int smem_min_w_ = 8;                        // narrowest level width taking the shared-memory count pass
     int64_t smem_min_n_ = 2048;                 // ... and fewest entries (small levels: rows stay L1/L2 hits)
     int64_t smem_per_root_ = 16;                // ... and fewest entries per root of the window on average
@@ -394,8 +400,10 @@ bool Engine::run_small(int32_t k, const Level &L) {
     a.Wc = L.W;
     a.roots = roots_;
     a.adj = adj_;
-    a.ocol = g_->ocol.get();
+    a.ocol = vtab_;
     a.order = g_->vid.get();
+    a.prefix = prefix_;
+    a.k0 = k0_;
     a.maxbit = maxbit_;
     leaf_args(a);
     a.chain = chain_dev_;
@@ -449,6 +457,143 @@ bool Engine::run_small(int32_t k, const Level &L) {
     return true;
 }
 
+// Re-rooting (expand.cuh launch_reroot_build): the candidates of a wide level
+// (W >= reroot_min_w_ words, e.g. R-MAT scale 26's 2048-4096-vertex roots)
+// whose sets hold at most 1024 vertices become roots of their own over P,
+// grouped by the width of |P|; each group is processed as a window of its own
+// (level k, the same candidates) at that width.  Candidates with larger sets
+// stay in the old space.  Returns false (nothing done) when the derived arrays
+// would not fit half of the free budget.
+bool Engine::reroot(int32_t k, const Level &L) {
+    const int64_t N = L.count;
+    if (N <= 0) return false;
+    const Arena::Mark mark = arena_.mark();
+    const int32_t Ps = L.Ps > 0 ? L.Ps : L.W;
+    int32_t *Lp = arena_.alloc<int32_t>(N);
+    int32_t *cls = arena_.alloc<int32_t>(N);
+    int64_t *hist = arena_.alloc<int64_t>(kMaxClass + 1);
+    MCE_CUDA(cudaMemsetAsync(hist, 0, sizeof(int64_t) * (kMaxClass + 1), s_));
+    launch_reroot_sizes(L.P, Ps, L.W, N, Lp, cls, hist, s_);
+    int64_t *hh = g_->host.get<int64_t>(kMaxClass + 1);
+    MCE_CUDA(cudaMemcpyAsync(hh, hist, sizeof(int64_t) * (kMaxClass + 1), cudaMemcpyDeviceToHost, s_));
+    stream_sync(s_);
+    kernels_ += 1;
+    std::vector<int64_t> counts(hh, hh + kMaxClass + 1);
+    // derived bytes: per re-rooted candidate L' (4 + 8 Wn) + 8 Wn + ~64; bound it by the sizes' upper end
+    int64_t need_bytes = 0, moved = 0;
+    for (int c = 0; c <= 4 && c <= kMaxClass; ++c) {
+        const int64_t Wn = 1ll << c;
+        need_bytes += counts[c] * (64 * Wn * (4 + 8 * Wn) + 8 * Wn + 64 + 4 * k);
+        moved += counts[c];
+    }
+    if (moved == 0 || need_bytes > (int64_t)(arena_.avail() / 4)) {  // (the subtrees below need the rest)
+        arena_.reset(mark);
+        return false;
+    }
+    if ((int64_t)level_entries_.size() <= k) level_entries_.resize(k + 1, 0);
+    // the saved window state (the caller's siblings continue in the old space)
+    const RootInfo *sroots = roots_;
+    const uint64_t *sadj = adj_;
+    const int32_t *svtab = vtab_, *sprefix = prefix_;
+    const int32_t sk0 = k0_, sW = W_;
+    const int64_t snroots = nroots_;
+    int32_t *flag = arena_.alloc<int32_t>(N);
+    int64_t *pos = arena_.alloc<int64_t>(N + 1);
+    int64_t *tmp = arena_.alloc<int64_t>(scan_tmp_items(N));
+    ExpandArgs ra{};
+    ra.P = L.P;
+    ra.slot = L.slot;
+    ra.Wp = L.W;
+    ra.Ps = Ps;
+    ra.Wa = W_;
+    ra.k = k;
+    ra.roots = roots_;
+    ra.adj = adj_;
+    ra.ocol = vtab_;
+    ra.order = g_->vid.get();
+    ra.chain = chain_dev_;
+    ra.prefix = prefix_;
+    ra.k0 = k0_;
+    if (k + 2 > chain_cap_) fail(MCE_ERR_INVALID, "clique depth above the supported maximum");
+    const LevelLink link{L.parent, L.vloc};  // the candidates' own level (read-out of their prefixes)
+    for (int c = 0; c <= kMaxClass; ++c) {
+        if (counts[c] == 0) continue;
+        const Arena::Mark cmark = arena_.mark();
+        const int64_t cnt = counts[c];
+        int32_t *list = arena_.alloc<int32_t>(cnt);
+        launch_flag_eq(N, cls, c, flag, s_);
+        exclusive_scan_i32(flag, pos, N, tmp, s_);
+        launch_compact(N, flag, pos, list, s_);
+        kernels_ += 5;
+        if (c > 4) {  // sets above 1024 vertices: the old space, at the old width
+            Level O;
+            O.count = cnt;
+            O.W = L.W;
+            O.P = arena_.alloc<uint64_t>(cnt * L.W);
+            O.slot = arena_.alloc<int32_t>(cnt);
+            O.parent = arena_.alloc<int32_t>(cnt);
+            O.vloc = arena_.alloc<int32_t>(cnt);
+            launch_gather_level(N, flag, pos, L.W, Ps, L.P, L.slot, L.parent, L.vloc, O.P, O.slot, O.parent, O.vloc, s_);
+            kernels_ += 1;
+            const int32_t saved = no_reroot_level_;
+            no_reroot_level_ = k;  // (no second attempt on these)
+            level_entries_[k] -= cnt;  // (counted again by process)
+            process(k, O);
+            no_reroot_level_ = saved;
+            arena_.reset(cmark);
+            continue;
+        }
+        const int Wn = 1 << c;
+        int32_t *lens = arena_.alloc<int32_t>(cnt);
+        int64_t *voff = arena_.alloc<int64_t>(cnt + 1);
+        int64_t *tmp2 = arena_.alloc<int64_t>(scan_tmp_items(cnt));
+        launch_gather_i32(Lp, list, cnt, lens, s_);
+        exclusive_scan_i32(lens, voff, cnt, tmp2, s_);
+        int64_t *hv = g_->host.get<int64_t>(1);
+        MCE_CUDA(cudaMemcpyAsync(hv, voff + cnt, sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
+        stream_sync(s_);
+        const int64_t total = hv[0];
+        int32_t *nV = arena_.alloc<int32_t>(total);
+        uint64_t *nA = arena_.alloc<uint64_t>(total * Wn);
+        RootInfo *nroots = arena_.alloc<RootInfo>(cnt);
+        int32_t *nprefix = arena_.alloc<int32_t>(cnt * k);
+        Level D;
+        D.count = cnt;
+        D.W = Wn;
+        D.P = arena_.alloc<uint64_t>(cnt * Wn);
+        D.slot = arena_.alloc<int32_t>(cnt);
+        D.parent = arena_.alloc<int32_t>(cnt);
+        D.vloc = arena_.alloc<int32_t>(cnt);
+        // (a previous group's process(k, ...) replaced chain[k]: the prefixes read the candidates' own links)
+        MCE_CUDA(cudaMemcpyAsync(chain_dev_ + k, &link, sizeof(link), cudaMemcpyHostToDevice, s_));
+        launch_reroot_build(ra, list, cnt, voff, Wn, nV, nA, nroots, D.P, D.slot, D.parent, D.vloc, nprefix, s_);
+        kernels_ += 4;
+        roots_ = nroots;
+        adj_ = nA;
+        vtab_ = nV;
+        prefix_ = nprefix;
+        k0_ = k;
+        W_ = Wn;
+        nroots_ = cnt;
+        level_entries_[k] -= cnt;  // (counted again by process)
+        const int32_t saved = no_reroot_level_;
+        no_reroot_level_ = k;  // the derived level itself is not re-rooted again (deeper levels may be)
+        process(k, D);
+        no_reroot_level_ = saved;
+        roots_ = sroots;
+        adj_ = sadj;
+        vtab_ = svtab;
+        prefix_ = sprefix;
+        k0_ = sk0;
+        W_ = sW;
+        nroots_ = snroots;
+        arena_.reset(cmark);
+    }
+    level_entries_[k] += N;
+    arena_.reset(mark);
+    return true;
+}
+
 void Engine::process(int32_t k, const Level &L) {
     if (entry_shard_ && !split_ && k >= o_.shard_depth) {  // deal this level's entries by path hash
         if (k + 2 > chain_cap_) fail(MCE_ERR_INVALID, "clique depth above the supported maximum");
@@ -460,7 +605,15 @@ void Engine::process(int32_t k, const Level &L) {
         int32_t *flag = arena_.alloc<int32_t>(N);
         int64_t *pos = arena_.alloc<int64_t>(N + 1);
         int64_t *tmp = arena_.alloc<int64_t>(scan_tmp_items(N));
-        launch_shard_flags(roots_, L.slot, chain_dev_, N, k, (int32_t)offset_, (int32_t)stride_, flag, s_);
+        ExpandArgs sa{};
+        sa.roots = roots_;
+        sa.slot = L.slot;
+        sa.chain = chain_dev_;
+        sa.ocol = vtab_;
+        sa.order = g_->vid.get();
+        sa.prefix = prefix_;
+        sa.k0 = k0_;
+        launch_shard_flags(sa, N, k, (int32_t)offset_, (int32_t)stride_, flag, s_);
         exclusive_scan_i32(flag, pos, N, tmp, s_);
         int64_t *h = g_->host.get<int64_t>(1);
         MCE_CUDA(cudaMemcpyAsync(h, pos + N, sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
@@ -483,6 +636,9 @@ void Engine::process(int32_t k, const Level &L) {
         arena_.reset(mark);
         return;
     }
+    if (k >= 2 && k != no_reroot_level_ && reroot_min_w_ > 0 && L.W >= reroot_min_w_ && !o_.no_reroot &&
+        reroot(k, L))
+        return;
     const bool pre_split = entry_shard_ && !split_;  // fused tiny levels would run past the split depth
     if (!pre_split && !o_.no_fused_levels && L.count <= kSmallMax && L.W <= 4 && run_small(k, L)) return;
     if ((int64_t)level_entries_.size() <= k) level_entries_.resize(k + 1, 0);
@@ -514,8 +670,10 @@ void Engine::process(int32_t k, const Level &L) {
     a.Wc = L.W;
     a.roots = roots_;
     a.adj = adj_;
-    a.ocol = g_->ocol.get();
+    a.ocol = vtab_;
     a.order = g_->vid.get();
+    a.prefix = prefix_;
+    a.k0 = k0_;
     a.counts = counts;
     a.maxbit = maxbit_;
     leaf_args(a);
@@ -796,6 +954,8 @@ void Engine::do_class_w1(const int32_t *list, int64_t count) {
         if (leaves > 0) {
             ExpandArgs la{};
             la.k = 1;
+            la.ocol = g_->ocol.get();
+            la.order = g_->vid.get();
             leaf_args(la);
             la.leaf_rows = ra.leaf_rows;
             la.leaf_cap = ra.leaf_cap;
@@ -809,6 +969,9 @@ void Engine::do_class_w1(const int32_t *list, int64_t count) {
             roots_ = ra.roots;
             adj_ = ra.adj;
             nroots_ = nw;
+            vtab_ = g_->ocol.get();
+            prefix_ = nullptr;
+            k0_ = 0;
             Level L2;
             L2.count = entries;
             L2.W = 1;
@@ -866,6 +1029,9 @@ void Engine::do_class(int32_t cls, const int32_t *list, int64_t count) {
         roots_ = roots;
         adj_ = adj;
         nroots_ = nw;
+        vtab_ = g_->ocol.get();
+        prefix_ = nullptr;
+        k0_ = 0;
         Level L1;
         L1.count = nw;
         L1.W = W_;
@@ -1006,9 +1172,11 @@ mce_result *Engine::run() {
     if (const char *sw = getenv("MCE_SMEM_MIN_W")) smem_min_w_ = atoi(sw);  // tuning hooks (A/B runs)
     if (const char *sn = getenv("MCE_SMEM_MIN_N")) smem_min_n_ = atoll(sn);
     if (const char *sp = getenv("MCE_SMEM_PER_ROOT")) smem_per_root_ = atoll(sp);
+    if (const char *rr = getenv("MCE_REROOT_MIN_W")) reroot_min_w_ = atoi(rr);
     pair_cap_ = std::max<int64_t>(4096, (int64_t)g_->pdesc.n / 3);
     g_->pdesc.ensure((size_t)pair_cap_ * 3);
     chain_dev_ = reinterpret_cast<LevelLink *>(g_->misc.get() + 256);
+    vtab_ = g_->ocol.get();
     stage_max_rows_ = std::max<int64_t>(1ll << 20, budget / 4 / (4ll * std::max<int32_t>(g_->max_out + 2, 2)));
     // staging rows: whatever the buffers kept from earlier calls hold (a count
     // pass is replayed when the staging is too small, so reuse avoids replays)

@@ -186,6 +186,26 @@ __global__ void init_level1_kernel(const RootInfo *__restrict__ roots, int64_t n
 // by the caller (aggregated per warp); a staging slot is taken only while the
 // staging area has room, so a level with 10^8 maximum cliques does not
 // serialise on one counter.
+// Vertices (original ids) of entry e's clique C (|C| = a.k) into row[0 .. k-1]:
+// the levels above the root's own space come from its prefix (a re-rooted
+// candidate, reroot_build_kernel: prefix[slot * k0 ..] holds its first k0
+// vertices), the rest from the chain of parent links (PAPER.md IV-B read-out).
+__device__ __forceinline__ void write_path(const ExpandArgs &a, int64_t e, const RootInfo &ri, int32_t *row) {
+    const int32_t *V = a.ocol + ri.vbase;
+    int64_t cur = e;
+    const int32_t stop = a.k0 > 0 ? a.k0 : 1;
+    for (int32_t lev = a.k; lev > stop; --lev) {
+        row[lev - 1] = a.order[V[ri.L - 1 - a.chain[lev].vloc[cur]]];
+        cur = a.chain[lev].parent[cur];
+    }
+    if (a.k0 > 0) {
+        const int32_t *pre = a.prefix + (int64_t)a.slot[e] * a.k0;
+        for (int32_t j = 0; j < a.k0; ++j) row[j] = pre[j];
+    } else {
+        row[0] = a.order[ri.r];
+    }
+}
+
 __device__ void store_leaf(const ExpandArgs &a, int64_t e, int32_t v, const RootInfo &ri) {
     if (*(volatile unsigned long long *)a.leaf_slot >= (unsigned long long)a.leaf_cap) return;
     const unsigned long long idx = atomicAdd(a.leaf_slot, 1ull);
@@ -194,12 +214,7 @@ __device__ void store_leaf(const ExpandArgs &a, int64_t e, int32_t v, const Root
     int32_t *row = a.leaf_rows + (int64_t)idx * size;
     const int32_t *V = a.ocol + ri.vbase;
     row[a.k] = a.order[V[ri.L - 1 - v]];
-    int64_t cur = e;
-    for (int32_t lev = a.k; lev >= 2; --lev) {
-        row[lev - 1] = a.order[V[ri.L - 1 - a.chain[lev].vloc[cur]]];
-        cur = a.chain[lev].parent[cur];
-    }
-    row[0] = a.order[ri.r];
+    write_path(a, e, ri, row);
 }
 
 // Store one clique completion C + P of size a.need (count pass): the caller
@@ -222,14 +237,7 @@ __device__ void store_clique_leaf(const ExpandArgs &a, int64_t e, const uint64_t
     if (idx == ~0ull) return;
     int32_t *row = a.clq_rows + (int64_t)idx * a.need;
     const int32_t *V = a.ocol + ri.vbase;
-    if (gl == 0) {
-        int64_t cur = e;
-        for (int32_t lev = a.k; lev >= 2; --lev) {
-            row[lev - 1] = a.order[V[ri.L - 1 - a.chain[lev].vloc[cur]]];
-            cur = a.chain[lev].parent[cur];
-        }
-        row[0] = a.order[ri.r];
-    }
+    if (gl == 0) write_path(a, e, ri, row);
     int pc = 0;
 #pragma unroll
     for (int t = 0; t < WPL; ++t) pc += __popcll(P[t]);
@@ -318,12 +326,7 @@ __global__ void __launch_bounds__(kMatThreads) materialize_pairs_kernel(const Ex
             const RootInfo ri = a.roots[a.slot[e]];
             const int32_t *V = a.ocol + ri.vbase;
             const uint64_t *A = a.adj + ri.abase;
-            int64_t cur = e;
-            for (int32_t lev = a.k; lev >= 2; --lev) {
-                tmpl[lev - 1] = a.order[V[ri.L - 1 - a.chain[lev].vloc[cur]]];
-                cur = a.chain[lev].parent[cur];
-            }
-            tmpl[0] = a.order[ri.r];
+            write_path(a, e, ri, tmpl);
             int pos = a.k, np2 = 0;
             for (int w = 0; w < a.Wp; ++w) {
                 uint64_t q = a.P[e * a.Ps + w];
@@ -1200,6 +1203,110 @@ __global__ void __launch_bounds__(512) expand_lock(const ExpandArgs a, int64_t n
     flush_counters(a, nleaf, nclq, hb, ub);
 }
 
+// ---------------------------------------------------------------------------
+// Re-rooting (see expand.cuh launch_reroot_build): a candidate whose set P is
+// a few hundred bits scattered over a wide root space (R-MAT scale 26: roots
+// of 2048-4096 out-neighbours, W = 64) becomes a root of its own over P, so
+// its subtree runs at the width of |P| (4-16 words, the shared-memory pass)
+// instead of the root's.  Exact: the new space keeps the old relative order,
+// so colouring and branching are the same sequence of sets.
+// ---------------------------------------------------------------------------
+__global__ void reroot_sizes_kernel(const uint64_t *__restrict__ P, int Ps, int W, int64_t n, int32_t *Lp,
+                                    int32_t *cls, unsigned long long *hist) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t e0 = (int64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31); e0 < n; e0 += stride) {
+        const int64_t e = e0 + (threadIdx.x & 31);
+        int32_t c = -1;
+        if (e < n) {
+            int pc = 0;
+            for (int w = 0; w < W; ++w) pc += __popcll(P[e * Ps + w]);
+            Lp[e] = pc;
+            c = 0;
+            while ((64 << c) < pc) ++c;
+            cls[e] = c;
+        }
+        const unsigned same = __match_any_sync(0xffffffffu, c);
+        if (c >= 0 && (threadIdx.x & 31) == __ffs(same) - 1) atomicAdd(hist + c, (unsigned long long)__popc(same));
+    }
+}
+
+__global__ void gather_i32_kernel(const int32_t *__restrict__ src, const int32_t *__restrict__ idx, int64_t n,
+                                  int32_t *dst) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        dst[i] = src[idx[i]];
+}
+
+constexpr int kRerootWarps = 8;
+constexpr int kRerootMaxL = 1024;  // re-rooted spaces of at most 16 words
+__global__ void __launch_bounds__(32 * kRerootWarps)
+    reroot_build_kernel(const ExpandArgs a, const int32_t *__restrict__ list, int64_t cnt,
+                        const int64_t *__restrict__ voff, int Wn, int32_t *nV, uint64_t *nA, RootInfo *nroots,
+                        uint64_t *nP, int32_t *nslot, int32_t *nparent, int32_t *nvloc, int32_t *nprefix) {
+    __shared__ uint16_t spos[kRerootWarps][kRerootMaxL];
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    uint16_t *pos = spos[wib];
+    for (int64_t i = (int64_t)blockIdx.x * kRerootWarps + wib; i < cnt; i += (int64_t)gridDim.x * kRerootWarps) {
+        const int64_t e = list[i];
+        const RootInfo ri = a.roots[a.slot[e]];
+        const int32_t *Vo = a.ocol + ri.vbase;
+        const uint64_t *Ao = a.adj + ri.abase;
+        const int64_t base = voff[i];
+        const int Lp = (int)(voff[i + 1] - base);
+        // positions of P's bits, ascending (the new local indices 0 .. Lp-1)
+        int np = 0;
+        for (int w = 0; w < a.Wp; ++w) {
+            const uint64_t word = a.P[e * a.Ps + w];
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+                const uint32_t m = (uint32_t)(word >> (32 * h));
+                if ((m >> lane) & 1u) pos[np + __popc(m & lanemask_lt())] = (uint16_t)(w * 64 + h * 32 + lane);
+                np += __popc(m);
+            }
+        }
+        __syncwarp();
+        for (int j = lane; j < Lp; j += 32) nV[base + (Lp - 1 - j)] = Vo[ri.L - 1 - pos[j]];
+        // rows: A'[j] = A[pos[j]] compressed to P's bits
+        uint64_t *Arow = nA + base * Wn;
+        const int wused = (Lp + 63) >> 6;  // words beyond are zero
+        for (int j = 0; j < Lp; ++j) {
+            const uint64_t *row = Ao + (int64_t)pos[j] * a.Wa;
+            uint32_t lo = 0;
+            if (lane >= wused && lane < Wn) Arow[(int64_t)j * Wn + lane] = 0ull;
+            for (int t0 = 0; t0 < 64 * wused; t0 += 32) {
+                const int t = t0 + lane;
+                bool bit = false;
+                if (t < Lp) {
+                    const int u = pos[t];
+                    bit = (__ldg(row + (u >> 6)) >> (u & 63)) & 1ull;
+                }
+                const uint32_t m = __ballot_sync(0xffffffffu, bit);
+                if ((t0 & 32) == 0) {
+                    lo = m;
+                } else if (lane == 0) {
+                    Arow[(int64_t)j * Wn + (t0 >> 6)] = ((uint64_t)m << 32) | lo;
+                }
+            }
+        }
+        if (lane < Wn) {
+            const int lo = lane * 64;
+            nP[i * Wn + lane] = Lp >= lo + 64 ? ~0ull : (Lp > lo ? ((1ull << (Lp - lo)) - 1) : 0ull);
+        }
+        if (lane == 0) {
+            RootInfo nr;
+            nr.r = ri.r;
+            nr.L = Lp;
+            nr.vbase = base;
+            nr.abase = base * Wn;
+            nroots[i] = nr;
+            nslot[i] = (int32_t)i;
+            nparent[i] = -1;
+            nvloc[i] = -1;
+            write_path(a, e, ri, nprefix + i * a.k);
+        }
+        __syncwarp();
+    }
+}
+
 // counting sort of a level's entries by root slot (order inside a slot is
 // arbitrary).  Few slots take millions of entries, so the atomics are
 // aggregated over the lanes of a warp holding the same slot (__match_any_sync).
@@ -1235,15 +1342,26 @@ __device__ __forceinline__ uint64_t mix64(uint64_t z) {
     return z ^ (z >> 31);
 }
 
-__global__ void shard_flags_kernel(const RootInfo *__restrict__ roots, const int32_t *__restrict__ slot,
-                                   const LevelLink *__restrict__ chain, int64_t n, int32_t k, int32_t rank,
-                                   int32_t count, int32_t *flag) {
+// hash of entry e's vertex path (original vertex ids, root first, then levels
+// k .. 2): the same on every shard whatever local space (root or re-rooted
+// candidate) the entry lives in
+__global__ void shard_flags_kernel(const ExpandArgs a, int64_t n, int32_t k, int32_t rank, int32_t count,
+                                   int32_t *flag) {
     for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x) {
-        uint64_t h = mix64((uint64_t)(uint32_t)roots[slot[e]].r);
+        const RootInfo ri = a.roots[a.slot[e]];
+        const int32_t *V = a.ocol + ri.vbase;
+        const int32_t *pre = a.k0 > 0 ? a.prefix + (int64_t)a.slot[e] * a.k0 : nullptr;
+        uint64_t h = mix64((uint64_t)(uint32_t)(pre ? pre[0] : a.order[ri.r]));
         int64_t cur = e;
         for (int32_t lev = k; lev >= 2; --lev) {
-            h = mix64(h ^ (uint64_t)(uint32_t)chain[lev].vloc[cur]);
-            cur = chain[lev].parent[cur];
+            int32_t v;
+            if (pre && lev <= a.k0) {
+                v = pre[lev - 1];
+            } else {
+                v = a.order[V[ri.L - 1 - a.chain[lev].vloc[cur]]];
+                cur = a.chain[lev].parent[cur];
+            }
+            h = mix64(h ^ (uint64_t)(uint32_t)v);
         }
         flag[e] = (int32_t)(h % (uint64_t)count) == rank;
     }
@@ -1486,6 +1604,28 @@ void launch_group_by_slot(const int32_t *slot, int64_t n, int32_t nslots, int32_
     MCE_LAUNCH_CHECK();
 }
 
+void launch_reroot_sizes(const uint64_t *P, int Ps, int W, int64_t n, int32_t *Lp, int32_t *cls, int64_t *hist,
+                         cudaStream_t s) {
+    if (n <= 0) return;
+    reroot_sizes_kernel<<<grid_for(n, 256), 256, 0, s>>>(P, Ps, W, n, Lp, cls, reinterpret_cast<unsigned long long *>(hist));
+    MCE_LAUNCH_CHECK();
+}
+void launch_gather_i32(const int32_t *src, const int32_t *idx, int64_t n, int32_t *dst, cudaStream_t s) {
+    if (n <= 0) return;
+    gather_i32_kernel<<<grid_for(n, 256), 256, 0, s>>>(src, idx, n, dst);
+    MCE_LAUNCH_CHECK();
+}
+void launch_reroot_build(const ExpandArgs &a, const int32_t *list, int64_t cnt, const int64_t *voff, int Wn,
+                         int32_t *nV, uint64_t *nA, RootInfo *nroots, uint64_t *nP, int32_t *nslot, int32_t *nparent,
+                         int32_t *nvloc, int32_t *nprefix, cudaStream_t s) {
+    if (cnt <= 0) return;
+    if (Wn > kRerootMaxL / 64) fail(1, "internal: re-rooted space wider than 16 words");
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(cnt, kRerootWarps), (int64_t)num_sms() * 8));
+    reroot_build_kernel<<<grid, 32 * kRerootWarps, 0, s>>>(a, list, cnt, voff, Wn, nV, nA, nroots, nP, nslot, nparent,
+                                                            nvloc, nprefix);
+    MCE_LAUNCH_CHECK();
+}
+
 void launch_materialize_pairs(const ExpandArgs &a, int64_t n, cudaStream_t s) {
     if (n <= 0) return;
     materialize_pairs_kernel<<<(int)std::min<int64_t>(n, (int64_t)num_sms() * 8), kMatThreads, 0, s>>>(a, n);
@@ -1498,10 +1638,10 @@ void launch_expand_small(const ExpandArgs &a, uint8_t *scratch, int64_t scratch_
     MCE_LAUNCH_CHECK();
 }
 
-void launch_shard_flags(const RootInfo *roots, const int32_t *slot, const LevelLink *chain, int64_t n, int32_t k,
-                        int32_t rank, int32_t count, int32_t *flag, cudaStream_t s) {
+void launch_shard_flags(const ExpandArgs &a, int64_t n, int32_t k, int32_t rank, int32_t count, int32_t *flag,
+                        cudaStream_t s) {
     if (n <= 0) return;
-    shard_flags_kernel<<<grid_for(n, 256), 256, 0, s>>>(roots, slot, chain, n, k, rank, count, flag);
+    shard_flags_kernel<<<grid_for(n, 256), 256, 0, s>>>(a, n, k, rank, count, flag);
     MCE_LAUNCH_CHECK();
 }
 void launch_gather_level(int64_t n, const int32_t *flag, const int64_t *pos, int W, int Ps, const uint64_t *P,

@@ -90,6 +90,11 @@ struct ExpandArgs {
     const int32_t *perm;
     unsigned long long *chunk_ctr;
     int32_t chunk;
+    // re-rooted candidates (reroot_build_kernel): every root of this window is a
+    // former candidate whose first k0 clique vertices (original ids) are
+    // prefix[slot * k0 ..]; k0 = 0: ordinary roots (the clique starts at r)
+    const int32_t *prefix;
+    int32_t k0;
 };
 
 // Fused root level for W == 1 roots (roots.cu): one warp per root builds the
@@ -171,8 +176,21 @@ void launch_root_lengths(const int32_t *list, int64_t count, int64_t stride, con
 // depth-d entry sharding (mce_options.shard_depth): flag[e] = 1 when the hash
 // of entry e's vertex path (root CSR id, then the local vertices of levels
 // 2..k) modulo `count` is `rank`; chain[2..k] must be set
-void launch_shard_flags(const RootInfo *roots, const int32_t *slot, const LevelLink *chain, int64_t n, int32_t k,
-                        int32_t rank, int32_t count, int32_t *flag, cudaStream_t s);
+// (a: roots, slot, chain, ocol, order, prefix / k0 of the level)
+void launch_shard_flags(const ExpandArgs &a, int64_t n, int32_t k, int32_t rank, int32_t count, int32_t *flag,
+                        cudaStream_t s);
+// Re-rooting: each listed entry e of a level
+// (candidate set P over its root's space of W words) becomes a root of its
+// own whose space is P: L' = |P|, vertices V' (CSR ids, local index i <-> V'[L'-1-i],
+// the old relative order kept), adjacency A' = the old rows of P's vertices
+// compressed to P's bits (L' rows x Wn words), candidate set all of V', and a
+// prefix of the entry's k clique vertices.  voff: exclusive scan of L' over the list.
+void launch_reroot_sizes(const uint64_t *P, int Ps, int W, int64_t n, int32_t *Lp, int32_t *cls, int64_t *hist,
+                         cudaStream_t s);
+void launch_gather_i32(const int32_t *src, const int32_t *idx, int64_t n, int32_t *dst, cudaStream_t s);
+void launch_reroot_build(const ExpandArgs &a, const int32_t *list, int64_t cnt, const int64_t *voff, int Wn,
+                         int32_t *nV, uint64_t *nA, RootInfo *nroots, uint64_t *nP, int32_t *nslot, int32_t *nparent,
+                         int32_t *nvloc, int32_t *nprefix, cudaStream_t s);
 // out = the flagged entries of a level (P re-strided from Ps to W words)
 void launch_gather_level(int64_t n, const int32_t *flag, const int64_t *pos, int W, int Ps, const uint64_t *P,
                          const int32_t *slot, const int32_t *parent, const int32_t *vloc, uint64_t *oP,

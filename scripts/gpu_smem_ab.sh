@@ -2,7 +2,7 @@
 TAG=${1:-s}
 mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.build()" > gpurun_out/${TAG}_build.log 2>&1; echo build rc=$?
-timeout 900 python -m pytest tests/test_gpu_parity.py -q -m gpu -x -p no:cacheprovider -k "smem or enumerate_matches or completions or overflow or chunking" > gpurun_out/${TAG}_pytest.log 2>&1; echo pytest rc=$?
+timeout 1200 python -m pytest tests/test_gpu_parity.py tests/test_distributed.py -q -m gpu -x -p no:cacheprovider -k "smem or enumerate_matches or completions or overflow or chunking or reroot or different_bounds or shards" > gpurun_out/${TAG}_pytest.log 2>&1; echo pytest rc=$?
 tail -5 gpurun_out/${TAG}_pytest.log
 for w in 99 8 4 16; do
   K=thr; case $w in tile*) K=tile; w=${w#tile};; esac
@@ -35,3 +35,7 @@ g=G.make_config('rmat22', device='cuda'); gg=m.Graph(g.rowptr, g.col)
 r=gg.enumerate(max_cliques=1<<16); print(r.omega, r.count)
 " > gpurun_out/${TAG}_verbose.log 2>&1; echo verbose rc=$?
 grep -c level gpurun_out/${TAG}_verbose.log
+if [ -n "$RMAT26" ]; then
+  MCE_VERBOSE=1 timeout 900 python scripts/dense_once.py rmat26 > gpurun_out/${TAG}_rmat26.log 2>&1; echo rmat26 rc=$?
+  tail -1 gpurun_out/${TAG}_rmat26.log
+fi

@@ -255,7 +255,7 @@ def test_shards_on_separate_handles_agree_after_set_order(key, depth):
 @pytest.mark.gpu
 @pytest.mark.parametrize("depth", [0, 2, 3])
 @pytest.mark.parametrize("key", ["planted", "RMAT13", "BA5k", "T(30,6)", "ER400d", "RMAT11"])
-def test_shards_with_different_bounds(key, depth):
+def test_shards_with_different_bounds(key, depth, monkeypatch):
     """Shards whose lower bounds differ (one with no heuristic and no bound,
     one told omega, one told omega - 1) still partition the maximum cliques
     exactly: nothing reported twice, nothing lost (pre-split
@@ -268,6 +268,8 @@ def test_shards_with_different_bounds(key, depth):
     g = GRAPHS[key]()
     om, cl = oracle.max_cliques(*g.numpy(), bound="plain")
     settings = [dict(heuristic="none"), dict(lower_bound=om), dict(lower_bound=max(om - 1, 0), heuristic="single_degree")]
+    if depth == 3:  # re-rooted spaces above the split on every level (hash on vertex ids, not local indices)
+        monkeypatch.setenv("MCE_REROOT_MIN_W", "1")
     gg = m.Graph(g.rowptr, g.col)
     for shards in (2, 3):
         parts = [gg.enumerate(shard_rank=r, shard_count=shards, shard_depth=depth, **settings[r % 3])

@@ -477,3 +477,24 @@ def test_config_rmat26_golden():
     r = run_enum(g, max_cliques=1 << 12)
     assert (r.omega, r.count) == (gd["omega"], gd["multiplicity"])
     check_stored_rows(r.cliques, r.omega, g.rowptr.cpu().numpy(), g.col.cpu().numpy(), sample=16)
+
+
+@pytest.mark.parametrize("min_w", [1, 2, 8])
+@pytest.mark.parametrize("key", ["ER400d", "RMAT13", "RMAT15", "K130", "K257", "T(36,12)", "CP8+K600", "CP12+K300",
+                                 "planted", "ER700w8", "er2000", "BA5k"])
+def test_reroot(key, min_w, monkeypatch):
+    """Re-rooted candidates (every level >= 2 of at least min_w words becomes a
+    set of roots over the candidates' own sets, nested level after level with
+    min_w = 1): same answer as the oracle, with and without completions, and
+    under a small budget (chunked levels), and find-one."""
+    monkeypatch.setenv("MCE_REROOT_MIN_W", str(min_w))
+    g = GRAPHS[key]()
+    om, cl = oracle_answer(key)
+    for kw in (dict(), dict(clique_shortcut=False), dict(fused_levels=False), dict(smem_expand=False),
+               dict(budget_bytes=24 << 20, heuristic="single_degree")):
+        if "budget_bytes" in kw and (key.startswith("K") or key.startswith("CP") or min_w == 1):
+            continue  # (nested re-rooting on every level holds every level's derived arrays)
+        r = run_enum(g, **kw)
+        assert (r.omega, r.count) == (om, len(cl)) and np.array_equal(r.cliques, cl), kw
+    f = mce().Graph(g.rowptr, g.col).find_one(window=4)
+    assert f.omega == om and oracle.is_clique(*g.numpy(), f.cliques[0])
