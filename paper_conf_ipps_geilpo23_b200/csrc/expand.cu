@@ -221,8 +221,8 @@ __device__ void store_leaf(const ExpandArgs &a, int64_t e, int32_t v, const Root
 // checked that P is a clique and k + |P| == need.  G lanes of a tile hold the
 // words of P (lane gl: words gl, gl + G, ...; WPL per lane); returns with the
 // row written by the whole tile.
-template <int G, int WPL>
-__device__ void store_clique_leaf(const ExpandArgs &a, int64_t e, const uint64_t (&P)[WPL], const RootInfo &ri,
+template <int G, int WPL, bool CONTIG = false>  // CONTIG: lane gl holds words gl*WPL .. (else gl + G t)
+__device__ __forceinline__ void store_clique_leaf(const ExpandArgs &a, int64_t e, const uint64_t (&P)[WPL], const RootInfo &ri,
                                   unsigned gmask) {
     const int gl = (threadIdx.x & 31) & (G - 1);
     unsigned long long idx = 0;
@@ -254,7 +254,7 @@ __device__ void store_clique_leaf(const ExpandArgs &a, int64_t e, const uint64_t
         while (q) {
             const int b = __ffsll((long long)q) - 1;
             q &= q - 1;
-            row[pos++] = a.order[V[ri.L - 1 - ((gl + G * t) * 64 + b)]];
+            row[pos++] = a.order[V[ri.L - 1 - ((CONTIG ? gl * WPL + t : gl + G * t) * 64 + b)]];
         }
     }
 }
@@ -1307,6 +1307,266 @@ __global__ void __launch_bounds__(32 * kRerootWarps)
     }
 }
 
+// ---------------------------------------------------------------------------
+// Wide levels (W = G * WPL >= 32 words: roots of more than 1024 out-neighbours,
+// R-MAT scale 26) with rows read from global memory (the L2; a 64-word root
+// matrix is 2 MB): expand_lock's lockstep tiles with WPL contiguous words per
+// lane (vector row loads), T = 32 / G candidates per warp in flight, and work
+// taken dynamically in chunks (a static grid stride left most warps idle
+// behind a few long candidates: 16% achieved occupancy, ncu).  The colouring
+// order is kept only for the vertices the branching can visit (colour >= need
+// - k), in per-tile global scratch (the L2), so shared memory does not cap the
+// warps per SM.
+// ---------------------------------------------------------------------------
+template <int G, int WPL>
+__global__ void __launch_bounds__(256) expand_wide(const ExpandArgs a, int64_t nchunks, uint16_t *__restrict__ scratch) {
+    constexpr int T = 32 / G;
+    constexpr int W = G * WPL;
+    constexpr unsigned TM = G == 32 ? kFull : ((1u << G) - 1u);
+    __shared__ int64_t s_chunk;
+    const int lane = threadIdx.x & 31;
+    const int gl = lane & (G - 1), gbase = lane & ~(G - 1), tiw = lane / G;
+    const unsigned gmask = TM << gbase;
+    const int warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
+    uint16_t *ord = scratch + ((int64_t)blockIdx.x * (blockDim.x / G) + threadIdx.x / G) * (64 * W);
+    const int32_t k = a.k, need = a.need, cmin = need - k;
+    unsigned nleaf = 0;
+    unsigned long long nclq = 0;
+    int hb = -1, ub = 0;
+    for (;;) {
+        if (threadIdx.x == 0) s_chunk = (int64_t)atomicAdd(a.chunk_ctr, 1ull);
+        __syncthreads();
+        const int64_t c = s_chunk;
+        __syncthreads();
+        if (c >= nchunks) break;
+        const int64_t q0 = a.begin + c * (int64_t)a.chunk, q1 = min(a.end, q0 + (int64_t)a.chunk);
+        for (int64_t qb = q0 + (int64_t)warp * T; qb < q1; qb += (int64_t)nwarps * T) {
+            const int64_t q = qb + tiw;
+            const bool active = q < q1;
+            const int64_t e = active ? (a.perm ? (int64_t)a.perm[q] : q) : 0;
+            uint64_t P[WPL];
+#pragma unroll
+            for (int t = 0; t < WPL; ++t) P[t] = active ? a.P[e * a.Ps + gl * WPL + t] : 0ull;
+            const int32_t slot = active ? a.slot[e] : 0;
+            const RootInfo ri = a.roots[slot];
+            const uint64_t *A = a.adj + ri.abase;
+            // ---- colouring; the order is stored from colour cmin up
+            int np = 0, ncol = 0, ns = 0;
+            if (a.bound == 1) {
+                uint64_t U[WPL], Q[WPL];
+#pragma unroll
+                for (int t = 0; t < WPL; ++t) {
+                    U[t] = P[t];
+                    Q[t] = 0ull;
+                }
+                uint16_t first = 0;
+                while (true) {
+                    bool qn = false, un = false;
+#pragma unroll
+                    for (int t = 0; t < WPL; ++t) {
+                        qn |= Q[t] != 0ull;
+                        un |= U[t] != 0ull;
+                    }
+                    const unsigned bq = __ballot_sync(kFull, qn), bu = __ballot_sync(kFull, un);
+                    if (!(bq | bu)) break;
+                    unsigned mq = (bq >> gbase) & TM;
+                    if (!mq) {
+                        const unsigned mu = (bu >> gbase) & TM;
+                        if (mu) {
+#pragma unroll
+                            for (int t = 0; t < WPL; ++t) Q[t] = U[t];
+                            mq = mu;
+                            ++ncol;
+                            first = kClassStart;
+                        }
+                    }
+                    const int src = mq ? __ffs(mq) - 1 : 0;
+                    int lb = 0;  // this lane's lowest set bit (word-major)
+#pragma unroll
+                    for (int t = WPL - 1; t >= 0; --t)
+                        if (Q[t]) lb = t * 64 + __ffsll((long long)Q[t]) - 1;
+                    lb = __shfl_sync(kFull, lb, gbase + src);
+                    if (mq) {
+                        const int v = src * 64 * WPL + lb;
+                        const uint64_t *row = A + (int64_t)v * a.Wa + gl * WPL;
+#pragma unroll
+                        for (int t = 0; t < WPL; ++t) Q[t] &= ~__ldg(row + t);
+                        if (gl == src) {
+#pragma unroll
+                            for (int t = 0; t < WPL; ++t)
+                                if (t == (lb >> 6)) {
+                                    Q[t] &= ~(1ull << (lb & 63));
+                                    U[t] &= ~(1ull << (lb & 63));
+                                }
+                        }
+                        if (ncol >= cmin) {
+                            if (gl == 0) ord[ns] = (uint16_t)v | first;
+                            ++ns;
+                        }
+                        first = 0;
+                        ++np;
+                    }
+                }
+            } else {  // |C| + |P|: positions in ascending bit order, colour of position i = i + 1
+                int pc = 0;
+#pragma unroll
+                for (int t = 0; t < WPL; ++t) pc += __popcll(P[t]);
+                int incl = pc;
+#pragma unroll
+                for (int o = 1; o < G; o <<= 1) {
+                    const int y = __shfl_up_sync(kFull, incl, o);
+                    if (gl >= o) incl += y;
+                }
+                int pos = incl - pc;
+#pragma unroll
+                for (int t = 0; t < WPL; ++t) {
+                    uint64_t q2 = P[t];
+                    while (q2) {
+                        const int b = __ffsll((long long)q2) - 1;
+                        q2 &= q2 - 1;
+                        ord[pos++] = (uint16_t)((gl * WPL + t) * 64 + b) | kClassStart;
+                    }
+                }
+                np = __shfl_sync(kFull, incl, gbase + G - 1);
+                ncol = np;
+                ns = np;
+            }
+            __syncwarp();
+            __threadfence_block();
+            // ---- completions (rare: divergent, tile-mask collectives)
+            bool done = !active;
+            if (!done && a.shortcut && a.bound == 1 && np >= 2 && ncol == np && k + np == need) {
+                if (gl == 0) {
+                    ++nclq;
+                    a.counts[e] = 0;
+                }
+                store_clique_leaf<G, WPL, true>(a, e, P, ri, gmask);
+                done = true;
+            }
+            if (!done && a.shortcut && a.bound == 1 && ncol < np && np - ncol <= 40 && k + ncol == need &&
+                need <= 4096) {  // P's complement a matching (reading 13): every vertex of P, one by one
+                bool matching = true;
+                uint64_t X[WPL];
+#pragma unroll
+                for (int t = 0; t < WPL; ++t) X[t] = P[t];
+                while (matching) {
+                    bool xn = false;
+#pragma unroll
+                    for (int t = 0; t < WPL; ++t) xn |= X[t] != 0ull;
+                    const unsigned mx = (__ballot_sync(gmask, xn) & gmask) >> gbase;
+                    if (!mx) break;
+                    const int src = __ffs(mx) - 1;
+                    int lb = 0;
+#pragma unroll
+                    for (int t = WPL - 1; t >= 0; --t)
+                        if (X[t]) lb = t * 64 + __ffsll((long long)X[t]) - 1;
+                    lb = __shfl_sync(gmask, lb, src, G);
+                    const int v = src * 64 * WPL + lb;
+                    const uint64_t *row = A + (int64_t)v * a.Wa + gl * WPL;
+                    int miss = 0;
+#pragma unroll
+                    for (int t = 0; t < WPL; ++t) {
+                        uint64_t nb = P[t] & ~__ldg(row + t);
+                        if (gl == src && t == (lb >> 6)) {
+                            nb &= ~(1ull << (lb & 63));
+                            X[t] &= ~(1ull << (lb & 63));
+                        }
+                        miss += __popcll(nb);
+                    }
+                    matching = tile_sum<G>(miss, gmask) <= 1;
+                }
+                if (matching) {
+                    if (gl == 0) {
+                        nclq += 1ull << (np - ncol);
+                        reserve_pair_completions(a, e, np - ncol);
+                        a.counts[e] = 0;
+                    }
+                    done = true;
+                }
+            }
+            __syncwarp();
+            // ---- branching over the stored positions, highest colour first, in lockstep:
+            // pass 0 counts (+ leaves), pass 1 (fused) writes the warp's reserved children
+            int32_t cnt = 0;
+            for (int pass = 0; pass < (a.fused ? 2 : 1); ++pass) {
+                int64_t at = -1;
+                if (pass == 1) {
+                    int tot = 0, excl = 0;
+#pragma unroll
+                    for (int t = 0; t < T; ++t) {
+                        const int ct = __shfl_sync(kFull, cnt, t * G);
+                        if (t < tiw) excl += ct;
+                        tot += ct;
+                    }
+                    unsigned long long wbase = 0;
+                    if (lane == 0 && tot) wbase = atomicAdd(a.out_count, (unsigned long long)tot);
+                    wbase = __shfl_sync(kFull, wbase, 0);
+                    if (cnt > 0 && (int64_t)(wbase + tot) <= a.out_cap) at = (int64_t)(wbase + excl);
+                }
+                const bool write = pass == 1;
+                int32_t c2 = 0;
+                bool stop = done || k + ncol < need || (write && at < 0);
+                uint64_t R[WPL];
+#pragma unroll
+                for (int t = 0; t < WPL; ++t) R[t] = P[t];
+                int col = ncol, pos = ns - 1;
+                while (__ballot_sync(kFull, !stop)) {
+                    if (!stop && (pos < 0 || k + col < need)) stop = true;
+                    const uint16_t o = stop ? 0 : ord[pos];
+                    const int v = o & 0x7fff;
+                    uint64_t C[WPL];
+                    int pc = 0;
+                    const uint64_t *row = A + (int64_t)v * a.Wa + gl * WPL;
+#pragma unroll
+                    for (int t = 0; t < WPL; ++t) {
+                        C[t] = stop ? 0ull : (R[t] & __ldg(row + t));
+                        pc += __popcll(C[t]);
+                    }
+                    pc = tile_sum_full<G>(pc);
+                    if (!stop) {
+                        if (o & kClassStart) --col;
+                        --pos;
+                        if (gl == (v >> 6) / WPL) {
+#pragma unroll
+                            for (int t = 0; t < WPL; ++t)
+                                if (t == (v >> 6) % WPL) R[t] &= ~(1ull << (v & 63));
+                        }
+                        if (pc == 0) {
+                            if (!write && k + 1 >= need && gl == 0) {
+                                ++nleaf;
+                                store_leaf(a, e, v, ri);
+                            }
+                        } else if (k + 1 + pc >= need) {
+                            if (write) {
+                                const int64_t cp = at + c2;
+#pragma unroll
+                                for (int t = 0; t < WPL; ++t) a.cP[cp * W + gl * WPL + t] = C[t];
+                                if (gl == 0) {
+                                    a.cslot[cp] = slot;
+                                    a.cparent[cp] = (int32_t)e;
+                                    a.cvloc[cp] = v;
+                                }
+                            } else {
+#pragma unroll
+                                for (int t = 0; t < WPL; ++t)
+                                    if (C[t]) hb = max(hb, (gl * WPL + t) * 64 + 63 - __clzll((long long)C[t]));
+                                ub = max(ub, k + 1 + pc);
+                            }
+                            ++c2;
+                        }
+                    }
+                }
+                if (pass == 0) {
+                    cnt = c2;
+                    if (active && !done && gl == 0) a.counts[e] = cnt;
+                }
+            }
+            __syncwarp();
+        }
+    }
+    flush_counters(a, nleaf, nclq, hb, ub);
+}
+
 // counting sort of a level's entries by root slot (order inside a slot is
 // arbitrary).  Few slots take millions of entries, so the atomics are
 // aggregated over the lanes of a warp holding the same slot (__match_any_sync).
@@ -1563,9 +1823,62 @@ void launch_lock(const ExpandArgs &a0, cudaStream_t s) {
     MCE_LAUNCH_CHECK();
 }
 
+template <int G, int WPL>
+void launch_wide(const ExpandArgs &a0, cudaStream_t s) {
+    constexpr int threads = 256, W = G * WPL;
+    ExpandArgs a = a0;
+    const int64_t n = a.end - a.begin;
+    static int per_sm = 0;
+    if (!per_sm) {
+        MCE_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, expand_wide<G, WPL>, threads, 0));
+        per_sm = std::max(per_sm, 1);
+    }
+    const int64_t slots = (int64_t)num_sms() * per_sm;
+    a.chunk = (int32_t)std::max<int64_t>(1, std::min<int64_t>(4 * (threads / G), ceil_div(n, 16 * slots)));
+    MCE_CUDA(cudaMemsetAsync(a.chunk_ctr, 0, sizeof(unsigned long long), s));
+    const int64_t nchunks = ceil_div(n, a.chunk);
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(nchunks, slots));
+    // per-tile colouring orders (64 W u16 each) in the caller's scratch: at most as many blocks as it holds
+    const int64_t per_block = (int64_t)(threads / G) * 64 * W;
+    const int g2 = (int)std::min<int64_t>(grid, a.wscratch_n / per_block);
+    if (g2 < 1) fail(4, "wide expansion: scratch below one block's colouring orders");
+    expand_wide<G, WPL><<<g2, threads, 0, s>>>(a, nchunks, a.wscratch);
+    MCE_LAUNCH_CHECK();
+}
+
+static int wide_kind() {  // lanes per candidate for the wide pass (MCE_WIDE_G = 8 / 16 / 32; 0 = off)
+    static int g = -1;
+    if (g < 0) {
+        const char *e = getenv("MCE_WIDE_G");
+        g = e ? atoi(e) : 16;
+    }
+    return g;
+}
+
+int wide_min_w() {  // narrowest level the wide pass takes (MCE_WIDE_MIN_W; default 32 words)
+    static int w = -1;
+    if (w < 0) {
+        const char *e = getenv("MCE_WIDE_MIN_W");
+        w = e ? atoi(e) : 32;
+        if (wide_kind() <= 0) w = 1 << 30;
+    }
+    return w;
+}
+
 void launch_expand(const ExpandArgs &a, bool write_pass, cudaStream_t s) {
     const int64_t items = a.end - a.begin;
     if (items <= 0) return;
+    if (!write_pass && !a.perm && a.wscratch && a.Wp >= wide_min_w() && a.Wp <= 64) {
+        const int g = wide_kind();
+        switch (a.Wp) {
+            case 4: return launch_wide<4, 1>(a, s);
+            case 8: return g == 4 ? launch_wide<4, 2>(a, s) : launch_wide<8, 1>(a, s);
+            case 16: return g == 8 ? launch_wide<8, 2>(a, s) : launch_wide<16, 1>(a, s);
+            case 32: return g == 8 ? launch_wide<8, 4>(a, s) : (g == 32 ? launch_wide<32, 1>(a, s) : launch_wide<16, 2>(a, s));
+            case 64: return g == 8 ? launch_wide<8, 8>(a, s) : (g == 32 ? launch_wide<32, 2>(a, s) : launch_wide<16, 4>(a, s));
+            default: break;
+        }
+    }
     if (!write_pass && a.perm) {  // shared-memory count pass (the caller grouped the level by slot)
         if (a.Wp == 4) return launch_lock<4>(a, s);
         if (a.Wp == 8) return launch_lock<8>(a, s);

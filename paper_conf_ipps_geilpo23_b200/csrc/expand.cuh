@@ -95,6 +95,9 @@ struct ExpandArgs {
     // prefix[slot * k0 ..]; k0 = 0: ordinary roots (the clique starts at r)
     const int32_t *prefix;
     int32_t k0;
+    // wide count pass (expand_wide, W >= 32): per-tile colouring-order scratch (u16 entries)
+    uint16_t *wscratch;
+    int64_t wscratch_n;
 };
 
 // Fused root level for W == 1 roots (roots.cu): one warp per root builds the
@@ -160,6 +163,8 @@ void launch_init_level1(const RootInfo *roots, int64_t nroots, int W, uint64_t *
 void launch_expand(const ExpandArgs &a, bool write_pass, cudaStream_t s);
 // widths the shared-memory count pass handles (the root's matrix, 64 W rows x W words, staged per block)
 inline bool smem_width(int W) { return W == 4 || W == 8 || W == 16; }
+// narrowest width the wide (global-row, lockstep) count pass takes: 32 words unless MCE_WIDE_MIN_W says otherwise
+int wide_min_w();
 // perm = the level's entries [0, n) grouped by slot (counting sort: hist over nslots, scan, scatter)
 void launch_group_by_slot(const int32_t *slot, int64_t n, int32_t nslots, int32_t *hist, int64_t *offs,
                           int64_t *scan_tmp, int32_t *perm, cudaStream_t s);

@@ -498,3 +498,28 @@ def test_reroot(key, min_w, monkeypatch):
         assert (r.omega, r.count) == (om, len(cl)) and np.array_equal(r.cliques, cl), kw
     f = mce().Graph(g.rowptr, g.col).find_one(window=4)
     assert f.omega == om and oracle.is_clique(*g.numpy(), f.cliques[0])
+
+
+@pytest.mark.parametrize("g", ["16", "8", "32"])
+@pytest.mark.parametrize("key", ["ER400d", "RMAT13", "RMAT15", "K130", "K257", "T(36,12)", "CP8+K600", "CP12+K300",
+                                 "planted", "ER700w8", "Paley17"])
+def test_wide_lockstep(key, g, monkeypatch):
+    """The wide count pass (expand_wide: global rows, lockstep G-lane tiles with
+    W / G words per lane, order stored from colour need - k up) forced onto
+    every level of 4 words or more (shared-memory pass off), against the oracle."""
+    monkeypatch.setenv("MCE_WIDE_MIN_W", "4")
+    monkeypatch.setenv("MCE_WIDE_G", g)
+    monkeypatch.setenv("MCE_SMEM_MIN_W", "99")
+    g_ = GRAPHS[key]()
+    om, cl = oracle_answer(key)
+    for kw in (dict(), dict(clique_shortcut=False), dict(fused_levels=False), dict(reroot=False),
+               dict(budget_bytes=24 << 20, heuristic="single_degree"), dict(bound="size", heuristic="none")):
+        if "budget_bytes" in kw and (key.startswith("K") or key.startswith("CP")):
+            continue
+        if kw.get("bound") == "size" and key in ("RMAT15", "RMAT13", "CP8+K600", "CP12+K300", "K257", "ER400d",
+                                                 "ER700w8"):
+            continue
+        r = run_enum(g_, **kw)
+        assert (r.omega, r.count) == (om, len(cl)) and np.array_equal(r.cliques, cl), kw
+    f = mce().Graph(g_.rowptr, g_.col).find_one(window=4)
+    assert f.omega == om and oracle.is_clique(*g_.numpy(), f.cliques[0])
