@@ -699,11 +699,14 @@ void Engine::process(int32_t k, const Level &L) {
     }
 
     a.chunk_ctr = chunk_ctr_;  // (dynamic work counter of the shared-memory and wide count passes)
-    if (!a.perm && L.W >= wide_min_w() && L.W <= 64) {  // expand_wide's colouring orders: 64 W u16 per tile
-        const int64_t want = (int64_t)num_sms() * 8 * 32 * 64 * L.W;
-        const int64_t room = (int64_t)(arena_.avail() / 8) / 2;
-        a.wscratch_n = std::max<int64_t>(std::min<int64_t>(want, room), 32ll * 64 * L.W);
-        a.wscratch = arena_.alloc<uint16_t>(a.wscratch_n);
+    if (!a.perm && L.W >= wide_min_w() && L.W <= 64) {
+        // expand_wide's colouring orders (64 W u16 per tile): a workspace kept on the graph
+        // (like the leaf staging, outside the frontier budget); the launch takes as many
+        // blocks as it holds, at most 64 MB
+        const int64_t want = std::min<int64_t>((int64_t)num_sms() * 8 * 32 * 64 * L.W, 32ll << 20);
+        g_->wide.ensure((size_t)want);
+        a.wscratch = g_->wide.get();
+        a.wscratch_n = (int64_t)g_->wide.n;
     }
 
     // Fused count + write: the children are written by the count pass into

@@ -1323,7 +1323,6 @@ __global__ void __launch_bounds__(256) expand_wide(const ExpandArgs a, int64_t n
     constexpr int T = 32 / G;
     constexpr int W = G * WPL;
     constexpr unsigned TM = G == 32 ? kFull : ((1u << G) - 1u);
-    __shared__ int64_t s_chunk;
     const int lane = threadIdx.x & 31;
     const int gl = lane & (G - 1), gbase = lane & ~(G - 1), tiw = lane / G;
     const unsigned gmask = TM << gbase;
@@ -1333,14 +1332,17 @@ __global__ void __launch_bounds__(256) expand_wide(const ExpandArgs a, int64_t n
     unsigned nleaf = 0;
     unsigned long long nclq = 0;
     int hb = -1, ub = 0;
+    (void)warp;
+    (void)nwarps;
+    // every warp takes its own chunks of positions (no block barrier: a block's
+    // warps never wait for its slowest candidate)
     for (;;) {
-        if (threadIdx.x == 0) s_chunk = (int64_t)atomicAdd(a.chunk_ctr, 1ull);
-        __syncthreads();
-        const int64_t c = s_chunk;
-        __syncthreads();
-        if (c >= nchunks) break;
-        const int64_t q0 = a.begin + c * (int64_t)a.chunk, q1 = min(a.end, q0 + (int64_t)a.chunk);
-        for (int64_t qb = q0 + (int64_t)warp * T; qb < q1; qb += (int64_t)nwarps * T) {
+        unsigned long long c = 0;
+        if (lane == 0) c = atomicAdd(a.chunk_ctr, 1ull);
+        c = __shfl_sync(kFull, c, 0);
+        if ((int64_t)c >= nchunks) break;
+        const int64_t q0 = a.begin + (int64_t)c * a.chunk, q1 = min(a.end, q0 + (int64_t)a.chunk);
+        for (int64_t qb = q0; qb < q1; qb += T) {
             const int64_t q = qb + tiw;
             const bool active = q < q1;
             const int64_t e = active ? (a.perm ? (int64_t)a.perm[q] : q) : 0;
@@ -1391,13 +1393,15 @@ __global__ void __launch_bounds__(256) expand_wide(const ExpandArgs a, int64_t n
                         const uint64_t *row = A + (int64_t)v * a.Wa + gl * WPL;
 #pragma unroll
                         for (int t = 0; t < WPL; ++t) Q[t] &= ~__ldg(row + t);
-                        if (gl == src) {
+                        {  // clear v (select form: no dynamically indexed array, so no local memory)
+                            const uint64_t bit = gl == src ? 1ull << (lb & 63) : 0ull;
+                            const int wsel = lb >> 6;
 #pragma unroll
-                            for (int t = 0; t < WPL; ++t)
-                                if (t == (lb >> 6)) {
-                                    Q[t] &= ~(1ull << (lb & 63));
-                                    U[t] &= ~(1ull << (lb & 63));
-                                }
+                            for (int t = 0; t < WPL; ++t) {
+                                const uint64_t m = wsel == t ? bit : 0ull;
+                                Q[t] &= ~m;
+                                U[t] &= ~m;
+                            }
                         }
                         if (ncol >= cmin) {
                             if (gl == 0) ord[ns] = (uint16_t)v | first;
@@ -1464,13 +1468,12 @@ __global__ void __launch_bounds__(256) expand_wide(const ExpandArgs a, int64_t n
                     const int v = src * 64 * WPL + lb;
                     const uint64_t *row = A + (int64_t)v * a.Wa + gl * WPL;
                     int miss = 0;
+                    const uint64_t bit = gl == src ? 1ull << (lb & 63) : 0ull;
 #pragma unroll
                     for (int t = 0; t < WPL; ++t) {
-                        uint64_t nb = P[t] & ~__ldg(row + t);
-                        if (gl == src && t == (lb >> 6)) {
-                            nb &= ~(1ull << (lb & 63));
-                            X[t] &= ~(1ull << (lb & 63));
-                        }
+                        const uint64_t m = (lb >> 6) == t ? bit : 0ull;
+                        const uint64_t nb = P[t] & ~__ldg(row + t) & ~m;
+                        X[t] &= ~m;
                         miss += __popcll(nb);
                     }
                     matching = tile_sum<G>(miss, gmask) <= 1;
@@ -1526,10 +1529,11 @@ __global__ void __launch_bounds__(256) expand_wide(const ExpandArgs a, int64_t n
                     if (!stop) {
                         if (o & kClassStart) --col;
                         --pos;
-                        if (gl == (v >> 6) / WPL) {
+                        {
+                            const uint64_t bit = gl == (v >> 6) / WPL ? 1ull << (v & 63) : 0ull;
+                            const int wsel = (v >> 6) % WPL;
 #pragma unroll
-                            for (int t = 0; t < WPL; ++t)
-                                if (t == (v >> 6) % WPL) R[t] &= ~(1ull << (v & 63));
+                            for (int t = 0; t < WPL; ++t) R[t] &= ~(wsel == t ? bit : 0ull);
                         }
                         if (pc == 0) {
                             if (!write && k + 1 >= need && gl == 0) {
@@ -1834,7 +1838,9 @@ void launch_wide(const ExpandArgs &a0, cudaStream_t s) {
         per_sm = std::max(per_sm, 1);
     }
     const int64_t slots = (int64_t)num_sms() * per_sm;
-    a.chunk = (int32_t)std::max<int64_t>(1, std::min<int64_t>(4 * (threads / G), ceil_div(n, 16 * slots)));
+    // per-warp chunks: T candidates (one trip) or a few trips when the level is large
+    const int64_t warps = slots * (threads / 32);
+    a.chunk = (int32_t)((32 / G) * std::max<int64_t>(1, std::min<int64_t>(4, n / (warps * 8 * (32 / G)))));
     MCE_CUDA(cudaMemsetAsync(a.chunk_ctr, 0, sizeof(unsigned long long), s));
     const int64_t nchunks = ceil_div(n, a.chunk);
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(nchunks, slots));

@@ -53,6 +53,7 @@ struct mce_graph {
     mce::DevBuf<int32_t> cstage;   // engine: staged clique completions of one launch (grow-only)
     mce::DevBuf<int64_t> pdesc;    // engine: pair-completion descriptors of one launch (grow-only)
     mce::DevBuf<int32_t> store;    // engine: stored maximum cliques of the run (grow-only)
+    mce::DevBuf<uint16_t> wide;    // engine: colouring-order scratch of the wide count pass (grow-only)
 };
 
 namespace mce {
