@@ -9,6 +9,7 @@ pass (cold-cache, serialised: compare SHARES of the step, not absolutes).
 """
 
 import collections
+import gzip
 import csv
 import io
 import re
@@ -32,7 +33,7 @@ KEYS = [
 
 
 def launches(path):
-    rows = list(csv.reader(open(path)))
+    rows = list(csv.reader(gzip.open(path, 'rt') if path.endswith('.gz') else open(path)))
     hi = [i for i, r in enumerate(rows) if "Kernel Name" in r][0]
     h = rows[hi]
     ki, vi, ui = h.index("Kernel Name"), h.index("Metric Value"), h.index("Metric Unit")
