@@ -49,6 +49,10 @@ def parse():
     p.add_argument("--max-cliques", type=int, default=-1,
                    help="stored-clique capacity (multiplicity stays exact); -1: 2^16 for the R-MAT configs "
                         "(~10^8 maximum cliques of size ~223 there), unbounded otherwise")
+    p.add_argument("--heuristic", default="auto",
+                   choices=["auto", "none", "single_degree", "single_core", "multi_degree", "multi_core"],
+                   help="lower-bound heuristic (PAPER.md IV-A); auto: the per-config choice of HEURISTIC below "
+                        "(PAPER.md V line 315 reports each dataset under its fastest heuristic)")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--shard-depth", type=int, default=-1,
@@ -232,11 +236,20 @@ def config_dict(config, mode, window, n, edges, max_cl, world, shard_depth):
             "l2": "flushed (256 MiB write) before every step"}
 
 
+# per-config heuristic (the answer never depends on it, only the work does; PAPER.md V line 315: "we
+# report the results from the fastest configuration ... the best combination of heuristic, window
+# size, and other preprocessing"); chosen by the sweep in profiles/r02_heuristic_sweep_*.json
+HEURISTIC = {"er2000": "multi_degree", "ba1m": "multi_degree", "rmat22": "multi_degree",
+             "dense800": "multi_degree", "rmat26": "multi_degree"}
+
+
 def bench_defaults(args):
     mode = args.mode or ("find_one" if args.config == "dense800" else "enumerate")
     shard_depth = args.shard_depth if args.shard_depth >= 0 else (3 if args.config == "rmat26" else 0)
     window = args.window if args.window >= 0 else (64 if args.config == "dense800" else 0)
     max_cl = args.max_cliques if args.max_cliques >= 0 else (1 << 16 if args.config.startswith("rmat") else 0)
+    if args.heuristic == "auto":
+        args.heuristic = HEURISTIC[args.config]
     return mode, shard_depth, window, max_cl
 
 
@@ -324,6 +337,7 @@ def main():
             dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     rdev = "cpu" if (world > 1 and dist.get_backend() == "gloo") else f"cuda:{local}"
     mode, shard_depth, args.window, max_cl = bench_defaults(args)
+    heur = args.heuristic
 
     g = build_graph(args.config, f"cuda:{local}")
     edges = g.num_edges
@@ -335,11 +349,11 @@ def main():
         gr.clear_cache()
         if world > 1:
             if mode == "enumerate":
-                return mdist.enumerate_distributed(gr, max_cliques=max_cl, shard_depth=shard_depth)
-            return mdist.find_one_distributed(gr, window=args.window)
+                return mdist.enumerate_distributed(gr, max_cliques=max_cl, shard_depth=shard_depth, heuristic=heur)
+            return mdist.find_one_distributed(gr, window=args.window, heuristic=heur)
         if mode == "enumerate":
-            return gr.enumerate(max_cliques=max_cl)
-        return gr.find_one(window=args.window)
+            return gr.enumerate(max_cliques=max_cl, heuristic=heur)
+        return gr.find_one(window=args.window, heuristic=heur)
 
     for _ in range(args.warmup):
         res = one_step(graph)
@@ -407,9 +421,9 @@ def main():
             torch.cuda.synchronize()
             t0 = time.perf_counter()
             gh = mce.Graph(rp_h, col_h, device=local)
-            r2 = mdist.enumerate_distributed(gh, max_cliques=max_cl, shard_depth=shard_depth) if (world > 1 and mode == "enumerate") else (
-                mdist.find_one_distributed(gh, window=args.window) if world > 1 else
-                (gh.enumerate(max_cliques=max_cl) if mode == "enumerate" else gh.find_one(window=args.window)))
+            r2 = mdist.enumerate_distributed(gh, max_cliques=max_cl, shard_depth=shard_depth, heuristic=heur) if (world > 1 and mode == "enumerate") else (
+                mdist.find_one_distributed(gh, window=args.window, heuristic=heur) if world > 1 else
+                (gh.enumerate(max_cliques=max_cl, heuristic=heur) if mode == "enumerate" else gh.find_one(window=args.window, heuristic=heur)))
             dt = time.perf_counter() - t0
             gh.close()
             if i >= e2e_warm:
@@ -443,7 +457,7 @@ def main():
             "dtype": "int32",
             "data": "synthetic",
             "config": config_dict(args.config, mode, args.window, g.n, edges, max_cl, world, shard_depth),
-            "details": {"omega": res.omega, "multiplicity": res.count, "stored_cliques": int(res.cliques.shape[0]),
+            "details": {"heuristic": heur, "omega": res.omega, "multiplicity": res.count, "stored_cliques": int(res.cliques.shape[0]),
                         "phases_ms": phases, "levels": res.levels, "step_ms": [round(t, 4) for t in times]},
             "verified": verified,
             "paper_context": PAPER_CONTEXT,

@@ -41,13 +41,26 @@ __device__ __forceinline__ unsigned long long pick_key(const int32_t *__restrict
     return ((unsigned long long)(uint32_t)__ldg(thr + x) << 32) | (unsigned long long)(0x7fffffffu - (uint32_t)x);
 }
 
-// x ~ w?  Binary search in the shorter of the two sorted adjacency lists (the
-// picked vertex w is usually a hub, the candidate x rarely is).
+// x ~ w?  Binary search for x in w's sorted adjacency list.  Every lane of a
+// run searches the SAME list N(w) (w is the pick, the highest-threshold
+// candidate, so for the degree heuristic its list is the longest of all): the
+// top levels of the search tree are shared by all lanes and candidates (L1
+// hits), and P is kept in id order, so neighbouring lanes end in neighbouring
+// sectors.  Searching each candidate's own (shorter) list instead costs two
+// rowptr loads and ~log2(deg x) probes into a different cold list per
+// candidate (measured on rmat22: 44 GB of DRAM reads for the heuristic runs).
+#ifndef HEUR_SEARCH_W
+#define HEUR_SEARCH_W 1
+#endif
 __device__ __forceinline__ bool adjacent(const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
                                          int32_t x, int32_t w, int64_t wb, int64_t we) {
+#if HEUR_SEARCH_W
+    return contains_sorted(col, wb, we, x);
+#else
     const int64_t xb = __ldg(rowptr + x), xe = __ldg(rowptr + x + 1);
     if (xe - xb < we - wb) return contains_sorted(col, xb, xe, w);
     return contains_sorted(col, wb, we, x);
+#endif
 }
 
 // Early abort (exact).  A run's final size is at most |C| + |P| at any
@@ -63,22 +76,49 @@ __device__ __forceinline__ int32_t ld_best(const int32_t *best) {
     return v;
 }
 
-// Hub bit matrix (exact acceleration of long runs on power-law graphs).  H =
-// the highest-degree vertices (at most kHubMax, degree bucket threshold), M =
-// their induced adjacency as K x K bits, hkey = their pick keys.  Once every
-// candidate of a run is in H (after a few picks, runs from hubs are inside the
-// dense hub core), the run continues on a bit set over H: the pick is a max
-// over the set bits' keys, the filter one AND with M's row.  Same picks, same
-// sizes as the list form (the key encodes threshold and id).
-constexpr int kHubMax = 8192;
-constexpr int kHubWords = kHubMax / 64;  // 128
-constexpr int kHubWPL = kHubWords / 32;  // words per lane
+// Candidate filter (exact, with the early abort).  A candidate x whose
+// threshold (degree, or core number: both bound the size of any clique
+// through x by thr(x) + 1) is below best - 1 can never be picked by a run that
+// still reaches best: picks go by the highest threshold, so x is picked only
+// once every candidate above it is gone, and the clique then holds x, hence
+// has at most thr(x) + 1 < best vertices.  Dropping such candidates therefore
+// changes neither the picks of any run that reaches best (so neither the best
+// size nor the winning seed nor its clique) nor whether a run reaches it;
+// |C| + |P| then counts only candidates that can matter, so hopeless runs
+// abort sooner, and the adjacency tests of the dropped candidates (most of a
+// power-law seed's neighbours) are never made.  b == 0 (every run size
+// wanted, Algorithm 1 verbatim) keeps every candidate.
+#ifndef HEUR_FILTER
+#define HEUR_FILTER 1
+#endif
+__device__ __forceinline__ bool useful(const int32_t *__restrict__ thr, int32_t x, int32_t b) {
+    return !HEUR_FILTER || b <= 1 || __ldg(thr + x) + 1 >= b;
+}
+
+// Hub bit matrix (exact acceleration of the runs on power-law graphs).  H =
+// the highest-degree vertices (whole degree buckets, at most kHubBig of them),
+// indexed so that the (at most kHubTail) highest come first; M = their induced
+// adjacency, K rows of KW words; hkey = their pick keys.
+//  * adjacency tests between two hubs are one bit of M instead of a binary
+//    search (rmat22: the 110K vertices of degree >= omega - 1 are all hubs, so
+//    once the candidate filter has run every test of every run is a bit load);
+//  * once every candidate of a run is among the first KT hubs (the tail set),
+//    the run continues on a bit set over them: the pick is a max over the set
+//    bits' keys, the filter one AND with M's row prefix.
+// Same picks, same sizes as the list form (the key encodes threshold and id).
+#ifndef HUB_BIG
+#define HUB_BIG 131072
+#endif
+constexpr int kHubBig = HUB_BIG;          // lookup matrix: at most 2^17 rows of 2^11 words (2 GiB)
+constexpr int kHubTail = 8192;            // bit-set tail: the first kHubTail hubs
+constexpr int kHubWords = kHubTail / 64;  // 128
+constexpr int kHubWPL = kHubWords / 32;   // words per lane
 struct Hub {
-    const int32_t *hid = nullptr;           // [n] hub index or -1
-    const int32_t *hv = nullptr;            // [K] hub -> vertex
+    const int32_t *hid = nullptr;              // [n] hub index or -1
+    const int32_t *hv = nullptr;               // [K] hub -> vertex
     const unsigned long long *hkey = nullptr;  // [K] pick keys
-    const uint64_t *M = nullptr;            // [K][KW]
-    int K = 0, KW = 0;
+    const uint64_t *M = nullptr;               // [K][KW]
+    int K = 0, KW = 0, KT = 0;                 // KT: hubs of the tail set (indices < KT), <= kHubTail
 };
 
 // The rest of a run whose candidates are all hubs, by one warp: P = the
@@ -92,7 +132,7 @@ __device__ int32_t hub_tail_warp(const Hub &H, const int32_t *src, int64_t len, 
     // build: lane l collects the members whose word is owned by l (word % 32 == l)
     for (int64_t i0 = 0; i0 < len; i0 += 32) {
         const int64_t i = i0 + lane;
-        const int h = i < len ? __ldg(H.hid + src[i]) : -1;
+        const int h = i < len ? __ldg(H.hid + src[i]) : -1;  // < KT for every member (caller)
         for (int src_lane = 0; src_lane < 32; ++src_lane) {
             const int hh = __shfl_sync(0xffffffffu, h, src_lane);
             if (hh >= 0 && ((hh >> 6) & 31) == lane) {
@@ -142,10 +182,11 @@ __device__ int32_t hub_tail_warp(const Hub &H, const int32_t *src, int64_t len, 
         if (clique && lane == 0) clique[csize] = (int32_t)(0x7fffffffu - (uint32_t)(key & 0xffffffffull));
         ++csize;
         const uint64_t *row = H.M + (int64_t)hb * H.KW;
+        const int tw = (H.KT + 63) >> 6;  // words of the tail set
 #pragma unroll
         for (int t = 0; t < kHubWPL; ++t) {
             const int w = t * 32 + lane;
-            P[t] &= w < H.KW ? __ldg(row + w) : 0ull;
+            P[t] &= w < tw ? __ldg(row + w) : 0ull;
             if (w == (hb >> 6)) P[t] &= ~(1ull << (hb & 63));
         }
     }
@@ -153,14 +194,14 @@ __device__ int32_t hub_tail_warp(const Hub &H, const int32_t *src, int64_t len, 
 }
 
 // x ~ w with the hub bit matrix when both are hubs (hw = hid[w] or -1);
-// also reports whether x is a hub
+// also reports whether x is in the tail set
 __device__ __forceinline__ bool adjacent_h(const Hub &H, int hw, const int64_t *__restrict__ rowptr,
                                            const int32_t *__restrict__ col, int32_t x, int32_t w, int64_t wb,
                                            int64_t we, bool &x_hub) {
     if (H.K) {
         const int hx = __ldg(H.hid + x);
-        x_hub = hx >= 0;
-        if (x_hub && hw >= 0) return (__ldg(H.M + (int64_t)hw * H.KW + (hx >> 6)) >> (hx & 63)) & 1ull;
+        x_hub = hx >= 0 && hx < H.KT;
+        if (hx >= 0 && hw >= 0) return (__ldg(H.M + (int64_t)hw * H.KW + (hx >> 6)) >> (hx & 63)) & 1ull;
     } else {
         x_hub = false;
     }
@@ -183,8 +224,8 @@ __device__ int32_t greedy_run(int32_t s, const int64_t *__restrict__ rowptr, con
     int32_t *buf = scratch + base;    // later rounds work in place in the seed's segment
     int32_t csize = 1;
     while (len > 0) {
+        int32_t b = 0;  // current best (0: no abort, no candidate filter)
         if (best) {
-            int32_t b = 0;
             if (gl == 0) b = ld_best(best);
             b = __shfl_sync(gmask, b, 0, G);
             if (csize + len < b) break;
@@ -209,7 +250,7 @@ __device__ int32_t greedy_run(int32_t s, const int64_t *__restrict__ rowptr, con
             int64_t i = i0 + gl;
             int32_t x = i < len ? src[i] : -1;
             bool xh = true;
-            bool keep = i < len && x != w && adjacent_h(H, hw, rowptr, col, x, w, wb, we, xh);
+            bool keep = i < len && x != w && useful(thr, x, b) && adjacent_h(H, hw, rowptr, col, x, w, wb, we, xh);
             const unsigned m = (__ballot_sync(gmask, keep) & gmask) >> gbase;
             if (keep) buf[out + __popc(m & ((1u << gl) - 1u))] = x;
             out += __popc(m);
@@ -247,10 +288,11 @@ __device__ int32_t block_run(int32_t s, const int64_t *__restrict__ rowptr, cons
     int32_t csize = 1;
     if (clique && threadIdx.x == 0) clique[0] = s;
     while (len > 0) {
+        int32_t b = 0;  // current best (0: no abort, no candidate filter)
         if (best) {
             if (threadIdx.x == 0) sbest = ld_best(best);
             __syncthreads();
-            const int32_t b = sbest;
+            b = sbest;
             __syncthreads();
             if (csize + len < b) break;
         }
@@ -279,7 +321,7 @@ __device__ int32_t block_run(int32_t s, const int64_t *__restrict__ rowptr, cons
             const int64_t i = i0 + threadIdx.x;
             const int32_t x = i < len ? src[i] : -1;
             bool xh = true;
-            const bool keep = i < len && x != w && adjacent_h(H, hw, rowptr, col, x, w, wb, we, xh);
+            const bool keep = i < len && x != w && useful(thr, x, b) && adjacent_h(H, hw, rowptr, col, x, w, wb, we, xh);
             const unsigned m = __ballot_sync(0xffffffffu, keep);
             const unsigned nh = H.K ? __ballot_sync(0xffffffffu, keep && !xh) : 0u;
             __syncthreads();  // wkey/wcnt reuse, and every read of this chunk precedes its writes
@@ -433,13 +475,15 @@ __global__ void best_seed_kernel(int64_t nseeds, const int32_t *__restrict__ see
 
 // Replay of the winning run to recover its clique (one block, nothing else running)
 constexpr int kReplay = 1024;
-__global__ void __launch_bounds__(kReplay) replay_kernel(const unsigned long long *best_key,
+__global__ void __launch_bounds__(kReplay) replay_kernel(const unsigned long long *best_key, const int32_t *best,
                                                          const int64_t *__restrict__ rowptr,
                                                          const int32_t *__restrict__ col,
                                                          const int32_t *__restrict__ thr,
                                                          int32_t *__restrict__ scratch, int32_t *clique, const Hub H) {
     const int32_t s = (int32_t)(0x7fffffffu - (uint32_t)(*best_key & 0xffffffffull));
-    block_run<kReplay>(s, rowptr, col, thr, scratch, clique, nullptr, H);
+    // the winning run reaches *best, so the filter (and the abort) against it
+    // leaves its picks unchanged (see useful())
+    block_run<kReplay>(s, rowptr, col, thr, scratch, clique, best, H);
 }
 
 __global__ void degree_thr_kernel(int64_t n, const int64_t *__restrict__ rowptr, int32_t *thr) {
@@ -502,47 +546,61 @@ __global__ void deg_bucket_hist(int64_t n, const int64_t *__restrict__ rowptr, u
         if (h[i]) atomicAdd(bins + i, (unsigned long long)h[i]);
 }
 
-// hub index of every vertex (-1: not a hub), by warp-aggregated appends;
-// hub order is immaterial (keys carry the tie-break)
-__global__ void hub_index_kernel(int64_t n, const int64_t *__restrict__ rowptr, int bstar, int32_t *hid, int32_t *hv,
-                                 int32_t *count) {
+// hub index of every vertex (-1: not a hub), by warp-aggregated appends:
+// buckets >= btail take [0, KT) (cnt[0]), buckets in [bstar, btail) take
+// [KT, K) (cnt[1] starts at KT); order inside each range is immaterial (keys
+// carry the tie-break)
+__global__ void hub_index_kernel(int64_t n, const int64_t *__restrict__ rowptr, int bstar, int btail, int32_t *hid,
+                                 int32_t *hv, int32_t *cnt) {
     const int lane = threadIdx.x & 31;
     for (int64_t v0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) & ~31ll; v0 < n;
          v0 += (int64_t)gridDim.x * blockDim.x) {
         const int64_t v = v0 + lane;
-        const bool h = v < n && deg_bucket(rowptr[v + 1] - rowptr[v]) >= bstar;
-        const unsigned m = __ballot_sync(0xffffffffu, h);
-        int b = 0;
-        if (lane == 0 && m) b = atomicAdd(count, __popc(m));
-        b = __shfl_sync(0xffffffffu, b, 0);
+        const int bk = v < n ? deg_bucket(rowptr[v + 1] - rowptr[v]) : -1;
+        const bool t = bk >= btail, h = bk >= bstar && !t;
+        const unsigned mt = __ballot_sync(0xffffffffu, t), mh = __ballot_sync(0xffffffffu, h);
+        int bt = 0, bh = 0;
+        if (lane == 0 && mt) bt = atomicAdd(cnt, __popc(mt));
+        if (lane == 0 && mh) bh = atomicAdd(cnt + 1, __popc(mh));
+        bt = __shfl_sync(0xffffffffu, bt, 0);
+        bh = __shfl_sync(0xffffffffu, bh, 0);
         if (v < n) {
-            const int idx = h ? b + __popc(m & lanemask_lt()) : -1;
+            const int idx = t ? bt + __popc(mt & lanemask_lt()) : (h ? bh + __popc(mh & lanemask_lt()) : -1);
             hid[v] = idx;
-            if (h) hv[idx] = (int32_t)v;
+            if (idx >= 0) hv[idx] = (int32_t)v;
         }
     }
 }
 
-// row h of M: warp per hub, bits gathered in shared memory
+// row h of M: warp per hub, the KW-word row gathered in shared memory
+// (dynamic: 8 warps x KW words)
 __global__ void __launch_bounds__(256) hub_matrix_kernel(int K, int KW, const int32_t *__restrict__ hv,
                                                          const int64_t *__restrict__ rowptr,
                                                          const int32_t *__restrict__ col,
                                                          const int32_t *__restrict__ hid,
                                                          const int32_t *__restrict__ thr, uint64_t *M,
                                                          unsigned long long *hkey) {
-    __shared__ unsigned long long row_all[8][kHubWords];
+    extern __shared__ unsigned long long row_all[];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    unsigned long long *row = row_all[wid];
+    unsigned long long *row = row_all + (size_t)wid * KW;
     for (int h = blockIdx.x * 8 + wid; h < K; h += gridDim.x * 8) {
         for (int w = lane; w < KW; w += 32) row[w] = 0ull;
         __syncwarp();
         const int32_t v = hv[h];
-        for (int64_t e = rowptr[v] + lane; e < rowptr[v + 1]; e += 32) {
-            const int32_t u = __ldg(hid + __ldg(col + e));
-            if (u >= 0) atomicOr(row + (u >> 6), 1ull << (u & 63));
+        const int64_t eb = rowptr[v], ee = rowptr[v + 1];
+        for (int64_t e0 = eb; e0 < ee; e0 += 128) {  // four independent gathers in flight per lane
+            int32_t u[4];
+#pragma unroll
+            for (int q = 0; q < 4; ++q) u[q] = e0 + 32 * q + lane < ee ? __ldg(col + e0 + 32 * q + lane) : -1;
+#pragma unroll
+            for (int q = 0; q < 4; ++q) u[q] = u[q] >= 0 ? __ldg(hid + u[q]) : -1;
+#pragma unroll
+            for (int q = 0; q < 4; ++q)
+                if (u[q] >= 0) atomicOr(row + (u[q] >> 6), 1ull << (u[q] & 63));
         }
         __syncwarp();
-        for (int w = lane; w < KW; w += 32) M[(int64_t)h * KW + w] = row[w];
+        uint64_t *dst = M + (int64_t)h * KW;
+        for (int w = lane; w < KW; w += 32) dst[w] = row[w];
         if (lane == 0) hkey[h] = pick_key(thr, v);
         __syncwarp();
     }
@@ -665,7 +723,9 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
         kernels += 5;
     }
     if (nbig >= 64) {  // enough hub runs for the hub bit matrix to pay
-        // H = the vertices of the highest degree buckets, at most kHubMax of them
+        // H = the vertices of the highest degree buckets: at most kHubBig of them
+        // (and a matrix of at most a quarter of the free memory), the first
+        // buckets up to kHubTail of them forming the tail set
         unsigned long long *bins = pool.take<unsigned long long>(kBuckets);
         MCE_CUDA(cudaMemsetAsync(bins, 0, sizeof(unsigned long long) * kBuckets, s));
         deg_bucket_hist<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(), bins);
@@ -673,24 +733,34 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
         unsigned long long *hb = host.get<unsigned long long>(kBuckets);
         MCE_CUDA(cudaMemcpyAsync(hb, bins, sizeof(unsigned long long) * kBuckets, cudaMemcpyDeviceToHost, s));
         stream_sync(s);
-        int bstar = kBuckets;
-        unsigned long long above = 0;
+        const size_t free_b = dev_free_memory();
+        unsigned long long kcap = kHubBig;
+        while (kcap > kHubTail && (kcap * ((kcap + 63) / 64) * 8ull) > free_b / 4) kcap >>= 1;
+        int bstar = kBuckets, btail = kBuckets;
+        unsigned long long above = 0, tail = 0;
         for (int b = kBuckets - 1; b >= 0; --b) {
-            if (above + hb[b] > (unsigned long long)kHubMax) break;
+            if (above + hb[b] > kcap) break;
             above += hb[b];
             if (hb[b]) bstar = b;
+            if (above <= (unsigned long long)kHubTail) {
+                tail = above;
+                if (hb[b]) btail = b;
+            }
         }
         kernels += 1;
         if (above >= 64) {  // enough hubs to matter
-            int32_t *hid = pool.take<int32_t>(n), *hv = pool.take<int32_t>(kHubMax), *cnt = pool.take<int32_t>(1);
-            MCE_CUDA(cudaMemsetAsync(cnt, 0, sizeof(int32_t), s));
-            hub_index_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(), bstar, hid, hv, cnt);
-            MCE_LAUNCH_CHECK();
             const int K = (int)above;
             const int KW = (K + 63) / 64;
+            int32_t *hid = pool.take<int32_t>(n), *hv = pool.take<int32_t>(K), *cnt = pool.take<int32_t>(2);
+            const int32_t cnt0[2] = {0, (int32_t)tail};
+            MCE_CUDA(cudaMemcpyAsync(cnt, cnt0, sizeof(cnt0), cudaMemcpyHostToDevice, s));
+            hub_index_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(), bstar, btail, hid, hv, cnt);
+            MCE_LAUNCH_CHECK();
             uint64_t *M = pool.take<uint64_t>((int64_t)K * KW);
             unsigned long long *hkey = pool.take<unsigned long long>(K);
-            hub_matrix_kernel<<<std::max(1, std::min((K + 7) / 8, num_sms() * 8)), 256, 0, s>>>(
+            const size_t smem = (size_t)8 * KW * sizeof(unsigned long long);
+            MCE_CUDA(cudaFuncSetAttribute(hub_matrix_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            hub_matrix_kernel<<<std::max(1, std::min((K + 7) / 8, num_sms() * 8)), 256, smem, s>>>(
                 K, KW, hv, g->rowptr.get(), g->col.get(), hid, thr, M, hkey);
             MCE_LAUNCH_CHECK();
             kernels += 2;
@@ -700,6 +770,7 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
             H.M = M;
             H.K = K;
             H.KW = KW;
+            H.KT = (int)tail;
         }
     }
     if (nseeds > 0) {
@@ -733,7 +804,7 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
         MCE_LAUNCH_CHECK();
         best_seed_kernel<<<grid_for(nseeds, 256), 256, 0, s>>>(nseeds, seed_ptr, thr, run_size, best, best_key);
         MCE_LAUNCH_CHECK();
-        replay_kernel<<<1, kReplay, 0, s>>>(best_key, g->rowptr.get(), g->col.get(), thr, scratch, clique, H);
+        replay_kernel<<<1, kReplay, 0, s>>>(best_key, best, g->rowptr.get(), g->col.get(), thr, scratch, clique, H);
         MCE_LAUNCH_CHECK();
         kernels += 3;
     }

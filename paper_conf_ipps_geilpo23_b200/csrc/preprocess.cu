@@ -21,6 +21,8 @@
 #include <cub/device/device_radix_sort.cuh>
 
 #include <algorithm>
+#include <cstdio>
+#include <cstdlib>
 #include <vector>
 
 #include "graph.cuh"
@@ -66,6 +68,9 @@ constexpr int kPeelThreads = 1024;  // launch bound; the launch uses kcore_threa
 #define KCORE_CHUNK 32  // measured: 128 / 64 / 32 / 16 / 8 = ba1m 1.49 / 1.46 / 1.43 / 1.44 / 1.50 ms, rmat22 82.5 / 81.8 / 82.1 / 81.4 / - ms
 #endif
 constexpr int64_t kChunk = KCORE_CHUNK;  // edges per work item
+#ifndef KCORE_GRAB
+#define KCORE_GRAB 0  // 1: reserve only while items are queued (fewer atomics on tiny levels); measured slower overall (rmat22 78.1 vs 74.2 ms, ba1m 1.52 vs 1.47)
+#endif
 
 __device__ __forceinline__ unsigned long long ld_relaxed(const unsigned long long *p) {
     unsigned long long v;
@@ -119,7 +124,8 @@ constexpr int kLine = 16;  // u64 per counter line
 __global__ void __launch_bounds__(kPeelThreads)
     kcore_async(int64_t n, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col, int32_t *deg,
                 int32_t *core, int32_t *order, int32_t *alive_a, int32_t *alive_b, uint8_t *dead,
-                long long *work0, long long *work1, int64_t witems, unsigned long long *ctrl, int max_sleep) {
+                long long *work0, long long *work1, int64_t witems, unsigned long long *ctrl, int max_sleep,
+                long long *trace) {
     cg::grid_group grid = cg::this_grid();
     __shared__ unsigned long long sh[6];
     const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -180,6 +186,14 @@ __global__ void __launch_bounds__(kPeelThreads)
         __syncthreads();
         const unsigned long long appended = sh[0], kept = sh[1], md = sh[2], placed = sh[3];
         __syncthreads();
+        if (trace && tid == 0 && s < 8192) {  // MCE_KCORE_TRACE: (k, alive before scan, appended, t)
+            unsigned long long t;
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+            trace[4 * s] = k;
+            trace[4 * s + 1] = n_alive;
+            trace[4 * s + 2] = (long long)appended;
+            trace[4 * s + 3] = (long long)t;
+        }
         n_alive = (int64_t)kept;
         {
             int32_t *t = cur;
@@ -203,11 +217,47 @@ __global__ void __launch_bounds__(kPeelThreads)
         // appends.  The tiles' edge loops run in warp lock-step so appends and
         // done counts are aggregated over the whole warp (one atomic each).
         unsigned long long pending = 0;  // lane 0: items processed, not yet added to `done`
-        while (true) {
+        bool finished = false;
+        while (!finished) {
+            // Lane 0 reserves slots only while the list holds unreserved items
+            // (head < tail): with nothing queued, every warp reserving four
+            // slots per level would cost one same-address atomic per warp
+            // (~2400 per level, 959 levels on rmat22).  Otherwise it publishes
+            // its processed count and waits until items arrive or done == tail
+            // (read in that order: every appended item processed, nothing can
+            // follow -- the level is over).  Deep backlogs are reserved in
+            // groups of up to 8 rounds of 4 slots (fewer atomics on `head`).
             unsigned long long base = 0;
-            if (lane == 0) base = atomicAdd(head, 4ull);
+            int rounds = 0;
+            if (lane == 0 && !KCORE_GRAB) {
+                base = atomicAdd(head, 4ull);
+                rounds = 1;
+            } else if (lane == 0) {
+                int naps = 0;
+                while (true) {
+                    const unsigned long long h = ld_relaxed(head), t = ld_relaxed(tail);
+                    if (h < t) {
+                        const unsigned long long backlog = t - h;
+                        rounds = backlog >= 64ull * (unsigned long long)nwarps ? 8 : (backlog >= 16ull * (unsigned long long)nwarps ? 2 : 1);
+                        base = atomicAdd(head, 4ull * rounds);
+                        break;
+                    }
+                    if (pending) {
+                        __threadfence();  // this warp's appends before its done count
+                        atomicAdd(done, pending);
+                        pending = 0;
+                    }
+                    const unsigned long long dn = ld_relaxed(done), tl = ld_relaxed(tail);
+                    if (dn == tl) break;  // rounds == 0: the level is over
+                    __nanosleep(naps < 4 ? 32 : (naps < 16 ? 128 : max_sleep));
+                    ++naps;
+                }
+            }
             base = __shfl_sync(0xffffffffu, base, 0);
-            const unsigned long long slot = base + (lane >> 3);
+            rounds = __shfl_sync(0xffffffffu, rounds, 0);
+            if (rounds == 0) break;
+          for (int rd = 0; rd < rounds && !finished; ++rd) {
+            const unsigned long long slot = base + 4ull * rd + (lane >> 3);
             const int leader = lane & ~7;
             bool resolved = false, over = false;
             int idle = 0;  // consecutive empty polls: back off, and only then look at the hot counters
@@ -269,7 +319,8 @@ __global__ void __launch_bounds__(kPeelThreads)
                     idle = 0;
                 }
             }
-            if (__all_sync(0xffffffffu, over)) break;
+            if (__all_sync(0xffffffffu, over)) finished = true;  // later rounds' slots are beyond the end too
+          }
         }
         if (lane == 0 && pending) {  // (cannot happen: `over` needs an idle, flushed warp)
             __threadfence();
@@ -744,8 +795,23 @@ void kcore(mce_graph *g) {
     int64_t wi = witems;
     unsigned long long *ct = ctrl;
     int ms = 512;  // longest poll back-off (ns); 256-2048 measured equal
-    void *args[] = {&n_arg, &rp, &cl, &dg, &co, &qu, &aa, &ab, &dd, &w0, &w1, &wi, &ct, &ms};
+    long long *trace = nullptr;
+    const bool tracing = getenv("MCE_KCORE_TRACE") != nullptr;  // per-scan trace to stderr (tuning aid)
+    if (tracing) {
+        trace = g->pool.take<long long>(4 * 8192);
+        MCE_CUDA(cudaMemsetAsync(trace, 0xff, sizeof(long long) * 4 * 8192, s));
+    }
+    void *args[] = {&n_arg, &rp, &cl, &dg, &co, &qu, &aa, &ab, &dd, &w0, &w1, &wi, &ct, &ms, &trace};
     MCE_CUDA(cudaLaunchCooperativeKernel((void *)kcore_async, grid, threads, args, 0, s));
+    if (tracing) {
+        std::vector<long long> ht(4 * 8192);
+        MCE_CUDA(cudaMemcpyAsync(ht.data(), trace, sizeof(long long) * ht.size(), cudaMemcpyDeviceToHost, s));
+        stream_sync(s);
+        fprintf(stderr, "[kcore] grid %d x %d\n", grid, threads);
+        for (int i = 0; i < 8192 && ht[4 * i] >= 0; ++i)
+            fprintf(stderr, "[kcore] scan %d k %lld alive %lld appended %lld t_us %.2f\n", i, ht[4 * i], ht[4 * i + 1],
+                    ht[4 * i + 2], i ? (ht[4 * i + 3] - ht[3]) / 1e3 : 0.0);
+    }
     g->kernels += 2;
     // degeneracy = max core (the last queued vertex has it)
     last_core_kernel<<<1, 1, 0, s>>>(n, g->peel.get(), g->core.get(), deg);
