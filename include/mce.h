@@ -133,6 +133,13 @@ typedef struct {
                                 root and expanded with the root's adjacency matrix staged in
                                 shared memory (expand_smem); 1: rows read from global memory
                                 (expand_tile; A/B tests) */
+    int32_t no_root_colour;  /* 0 (default, colouring bound only): when many vertices can be in a
+                                clique of the size sought (core >= need - 1, PAPER.md II-B-2), they
+                                are greedily coloured once in reverse degeneracy order on the device
+                                and a root whose out-neighbourhood meets fewer than need - 1
+                                colours is dropped before its adjacency matrix is built (a proper
+                                colouring of G restricted to N+(r) bounds every clique there;
+                                DESIGN.md reading 14); 1: off (A/B tests) */
 } mce_options;
 
 /* Fill `opt` with defaults: degeneracy orientation, multi-run degree heuristic

@@ -51,6 +51,7 @@ class Options(ctypes.Structure):
         ("no_overlap", ctypes.c_int32),
         ("no_reroot", ctypes.c_int32),
         ("no_smem_expand", ctypes.c_int32),
+        ("no_root_colour", ctypes.c_int32),
     ]
 
 

@@ -61,7 +61,7 @@ def make_options(orientation="degeneracy", heuristic="multi_degree", heuristic_r
                  lower_bound=0, window=0, budget_bytes=0, max_cliques=0, shard_rank=0, shard_count=1,
                  bound_sync: Optional[Callable[[int, int], tuple]] = None, verbose=0, legacy_roots=False,
                  fused_levels=True, clique_shortcut=True, fused_expand=True, overlap=True, shard_depth=0,
-                 smem_expand=True, reroot=True):
+                 smem_expand=True, reroot=True, root_colour=True):
     o = Options()
     lib().mce_default_options(ctypes.byref(o))
     o.orientation = ORIENT[orientation]
@@ -83,6 +83,7 @@ def make_options(orientation="degeneracy", heuristic="multi_degree", heuristic_r
     o.shard_depth = int(shard_depth)
     o.no_smem_expand = int(not smem_expand)
     o.no_reroot = int(not reroot)
+    o.no_root_colour = int(not root_colour) or int(os.environ.get("MCE_NO_ROOT_COLOUR", "0") or 0)
     keep = None
     if bound_sync is not None:
         errors = []

@@ -34,6 +34,10 @@ constexpr size_t kAlign = 256;
 // small problems stay small while an exploding frontier may use the whole
 // budget.  Allocation is stack-like: mark() / reset(mark).
 constexpr size_t kBigSeg = 4ull << 30;
+// the root colour filter runs when at least this many vertices can be in a
+// clique of the size sought (below it the colouring costs more than it saves;
+// MCE_ROOT_COLOUR_MIN_S overrides, for tests)
+constexpr int64_t kRootColourMinS = 4096;
 struct Arena {
     struct Mark {
         size_t seg, off, before;
@@ -1210,10 +1214,31 @@ mce_result *Engine::run() {
         int64_t *tmp = arena_.alloc<int64_t>(scan_tmp_items(n));
         int64_t *hist = arena_.alloc<int64_t>(kMaxClass + 1);
         MCE_CUDA(cudaMemsetAsync(hist, 0, sizeof(int64_t) * (kMaxClass + 1), s_));
+        // root colour filter (colour.cu, reading 14): roots whose
+        // out-neighbourhood meets fewer than need - 1 colours of a greedy
+        // colouring of the vertices of core >= need - 1 are dropped here
+        const uint8_t *rkeep = nullptr;
+        int64_t rT = 0;
+        if (o_.bound == MCE_BOUND_COLOR && !o_.no_root_colour && g_->max_out >= 64) {
+            uint8_t *keepb = arena_.alloc<uint8_t>(n);
+            const Arena::Mark cm = arena_.mark();
+            int32_t *colr = arena_.alloc<int32_t>(n);
+            int64_t *scr = arena_.alloc<int64_t>(4);
+            int64_t kept = 0;
+            const char *ms = getenv("MCE_ROOT_COLOUR_MIN_S");
+            if (root_colour_filter(g_, need(), ms ? atoll(ms) : kRootColourMinS, keepb, colr, scr, s_, &rT, &kept)) {
+                rkeep = keepb;
+                kernels_ += 4;
+                if (o_.verbose > 0)
+                    fprintf(stderr, "[mce] root colour filter: %lld vertices of core >= %d, %lld roots kept\n",
+                            (long long)(n - rT), need() - 1, (long long)kept);
+            }
+            arena_.reset(cm);
+        }
         // roots are dealt to shards by CSR id (r % shard_count): independent of the
         // lower bound, so ranks whose bounds differ still partition the roots exactly
         launch_classify_roots(n, g_->orp.get(), std::max<int32_t>(need() - 1, 1), entry_shard_ ? 0 : (int32_t)offset_,
-                              entry_shard_ ? 1 : (int32_t)stride_, cls, hist, s_);
+                              entry_shard_ ? 1 : (int32_t)stride_, rkeep, rT, cls, hist, s_);
         ++kernels_;
         int64_t *hh = g_->host.get<int64_t>(kMaxClass + 1);
         MCE_CUDA(cudaMemcpyAsync(hh, hist, sizeof(int64_t) * (kMaxClass + 1), cudaMemcpyDeviceToHost, s_));

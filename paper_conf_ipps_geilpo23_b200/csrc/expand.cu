@@ -75,6 +75,9 @@ __global__ void build_adj_w1(const RootInfo *__restrict__ roots, int64_t nroots,
 #ifndef ADJ_CHUNKS
 #define ADJ_CHUNKS 4
 #endif
+#ifndef ADJ_VEC
+#define ADJ_VEC 1  // bit-map rows scanned with 16-byte loads (0: 32-bit loads, ADJ_CHUNKS per trip)
+#endif
 constexpr int kAdjChunks = ADJ_CHUNKS;
 constexpr int kSpanBits = 1 << 18;
 constexpr int kSpanWords = kSpanBits / 32;
@@ -116,6 +119,36 @@ __global__ void build_adj_block(const RootInfo *__restrict__ roots, int64_t nroo
         for (int i = wib; i < L; i += nwb) {
             const int32_t a = sV[i];
             const int64_t pb = __ldg(orp + a), pe = __ldg(orp + a + 1);
+            if (map && ADJ_VEC) {
+                // aligned 16-byte loads: a lane takes 4 consecutive ids, the warp 128
+                // per trip (elements outside [pb, pe) are masked; ocol is padded by 4)
+                const int li = L - 1 - i;
+                for (int64_t q0 = pb & ~3ll; q0 < pe; q0 += 128) {
+                    const int64_t q = q0 + 4 * lane;
+                    int4 v4 = make_int4(INT32_MAX, INT32_MAX, INT32_MAX, INT32_MAX);
+                    if (q < pe) v4 = __ldg(reinterpret_cast<const int4 *>(ocol + q));
+                    const int32_t uu[4] = {q >= pb ? v4.x : INT32_MIN, q + 1 >= pb ? v4.y : INT32_MIN,
+                                           q + 2 >= pb ? v4.z : INT32_MIN, v4.w};
+                    bool past = false;
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) {
+                        const int32_t u = q + j < pe ? uu[j] : INT32_MAX;
+                        past |= u > vmax;
+                        if (u >= vmin && u <= vmax) {
+                            const uint32_t off = (uint32_t)(u - vmin);
+                            const int w = off >> 5;
+                            const uint32_t bits = sMap[w], bit = 1u << (off & 31);
+                            if (bits & bit) {  // local indices L-1-position (expand.cuh)
+                                const int lc = L - 1 - (sRank[w] + __popc(bits & (bit - 1u)));
+                                atomicOr(A + (int64_t)li * 2 * W + (lc >> 5), 1u << (lc & 31));
+                                atomicOr(A + (int64_t)lc * 2 * W + (li >> 5), 1u << (li & 31));
+                            }
+                        }
+                    }
+                    if (__any_sync(0xffffffffu, past)) break;  // sorted row: the rest is beyond V
+                }
+                continue;
+            }
             // kAdjChunks chunks of 32 ids loaded before any is looked up (the
             // row scan is bound by its load latency, one chunk per trip)
             bool stop = false;
@@ -387,17 +420,28 @@ __device__ __forceinline__ unsigned long long warp_excl_u64(unsigned long long x
 // slots reserved for the whole warp with one atomicAdd, by replaying the
 // cheap branching loop after the colouring (which the separate write pass
 // would recompute).
-template <int W, bool WRITE>
+// adjacency row word: read-only global (LDG) or a copy in shared memory (SROWS)
+template <bool SROWS>
+__device__ __forceinline__ uint64_t ldrow(const uint64_t *p) {
+    if constexpr (SROWS)
+        return *p;
+    else
+        return __ldg(p);
+}
+
+// SROWS: the root's rows 0 .. 64 W - 1 (first W words each) are staged at
+// srows with stride W (expand_small, every candidate under one root)
+template <int W, bool WRITE, bool SROWS = false>
 __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, int64_t out, unsigned &nleaf,
                                                 unsigned long long &nclq, int &hb, int &ub, bool active = true,
-                                                bool fused = false) {
+                                                bool fused = false, const uint64_t *srows = nullptr) {
     uint64_t P[W];
 #pragma unroll
     for (int w = 0; w < W; ++w) P[w] = active ? a.P[e * a.Ps + w] : 0ull;
     RootInfo ri{};
     if (active) ri = a.roots[a.slot[e]];
-    const uint64_t *A = a.adj + ri.abase;
-    const int Wa = a.Wa;
+    const uint64_t *A = SROWS ? srows : a.adj + ri.abase;
+    const int Wa = SROWS ? W : a.Wa;
     uint8_t ord[64 * W];
     uint8_t colr[64 * W];  // colour - 1 (a full 4-word set has 256 colours)
     int np = 0;
@@ -422,7 +466,7 @@ __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, 
                     const int v = w * 64 + b;
                     const uint64_t *row = A + (int64_t)v * Wa;
 #pragma unroll
-                    for (int x = 0; x < W; ++x) Q[x] &= ~__ldg(row + x);
+                    for (int x = 0; x < W; ++x) Q[x] &= ~ldrow<SROWS>(row + x);
                     Q[w] &= ~(1ull << b);
                     U[w] &= ~(1ull << b);
                     ord[np] = (uint8_t)v;
@@ -467,7 +511,7 @@ __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, 
             int miss = 0;
 #pragma unroll
             for (int x = 0; x < W; ++x) {
-                uint64_t nb = P[x] & ~__ldg(row + x);
+                uint64_t nb = P[x] & ~ldrow<SROWS>(row + x);
                 if (x == (v >> 6)) nb &= ~(1ull << (v & 63));
                 miss += __popcll(nb);
             }
@@ -498,7 +542,7 @@ __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, 
             int pc = 0;
 #pragma unroll
             for (int w = 0; w < W; ++w) {
-                C[w] = R[w] & __ldg(row + w);
+                C[w] = R[w] & ldrow<SROWS>(row + w);
                 pc += __popcll(C[w]);
             }
             R[v >> 6] &= ~(1ull << (v & 63));
@@ -576,7 +620,13 @@ constexpr int kSmallThreads = 1024;
 template <bool WRITE>
 __device__ __forceinline__ int32_t expand_entry_w(int W, const ExpandArgs &a, int64_t e, int64_t out,
                                                   unsigned &nleaf, unsigned long long &nclq, int &hb, int &ub,
-                                                  bool active = true, bool fused = false) {
+                                                  bool active = true, bool fused = false,
+                                                  const uint64_t *srows = nullptr) {
+    if (srows) {
+        if (W == 1) return expand_entry<1, WRITE, true>(a, e, out, nleaf, nclq, hb, ub, active, fused, srows);
+        if (W == 2) return expand_entry<2, WRITE, true>(a, e, out, nleaf, nclq, hb, ub, active, fused, srows);
+        return expand_entry<4, WRITE, true>(a, e, out, nleaf, nclq, hb, ub, active, fused, srows);
+    }
     if (W == 1) return expand_entry<1, WRITE>(a, e, out, nleaf, nclq, hb, ub, active, fused);
     if (W == 2) return expand_entry<2, WRITE>(a, e, out, nleaf, nclq, hb, ub, active, fused);
     return expand_entry<4, WRITE>(a, e, out, nleaf, nclq, hb, ub, active, fused);
@@ -591,6 +641,8 @@ __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a
     __shared__ int64_t s_end;
     __shared__ int s_hb, s_ub;
     __shared__ int64_t s_used;
+    __shared__ int s_smin, s_smax;
+    __shared__ uint64_t s_rows[256 * 4];  // one root's rows 0 .. 64 W - 1, W words each (W <= 4)
     const int t = threadIdx.x;
     if (t == 0) {
         A = a0;
@@ -645,10 +697,35 @@ __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a
             s_end = p - scratch;
         }
         __syncthreads();
+        // every candidate under one root (the deep chains of a hub root): its
+        // rows are staged in shared memory, so the colouring's dependent row
+        // loads are shared-memory hits instead of L2 round trips
+        if (t == 0) {
+            s_smin = INT32_MAX;
+            s_smax = -1;
+        }
+        __syncthreads();
+        if (t < N) {
+            const int32_t sl = A.slot[A.begin + t];
+            atomicMin(&s_smin, sl);
+            atomicMax(&s_smax, sl);
+        }
+        __syncthreads();
+        const bool one_root = s_smin == s_smax;
+        if (one_root) {
+            const RootInfo ri = A.roots[s_smin];
+            const int nr = min(64 * W, ri.L);
+            for (int q = t; q < nr * W; q += blockDim.x) {
+                const int r = q / W, x = q - r * W;
+                s_rows[q] = __ldg(A.adj + ri.abase + (int64_t)r * A.Wa + x);
+            }
+        }
+        __syncthreads();
         unsigned nleaf = 0;
         unsigned long long nclq = 0;
         int hb = -1, ub = 0;
-        const int32_t cnt = expand_entry_w<false>(W, A, A.begin + t, 0, nleaf, nclq, hb, ub, t < N, true);
+        const int32_t cnt = expand_entry_w<false>(W, A, A.begin + t, 0, nleaf, nclq, hb, ub, t < N, true,
+                                                  one_root ? s_rows : nullptr);
         (void)cnt;
         if (nleaf) atomicAdd(&s_leaf, nleaf);
         if (nclq) atomicAdd(&s_clq, nclq);
@@ -1646,15 +1723,16 @@ __global__ void gather_level_kernel(int64_t n, const int32_t *__restrict__ flag,
 }
 
 __global__ void classify_roots_kernel(int64_t n, const int64_t *__restrict__ orp, int32_t min_len,
-                                      int32_t shard_rank, int32_t shard_count, int32_t *cls,
-                                      unsigned long long *hist) {
+                                      int32_t shard_rank, int32_t shard_count, const uint8_t *__restrict__ keep,
+                                      int64_t keep_T, int32_t *cls, unsigned long long *hist) {
     __shared__ unsigned int h[kMaxClass + 1];
     for (int i = threadIdx.x; i <= kMaxClass; i += blockDim.x) h[i] = 0;
     __syncthreads();
     for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < n; r += (int64_t)gridDim.x * blockDim.x) {
         const int64_t L = orp[r + 1] - orp[r];
         int32_t c = -1;
-        if (L >= min_len && L > 0 && (shard_count <= 1 || r % shard_count == shard_rank)) {
+        if (L >= min_len && L > 0 && (shard_count <= 1 || r % shard_count == shard_rank) &&
+            (!keep || (r >= keep_T && keep[r - keep_T]))) {
             const int64_t words = (L + 63) / 64;
             c = 0;
             while ((1ll << c) < words) ++c;
@@ -1972,9 +2050,9 @@ void launch_gather_level(int64_t n, const int32_t *flag, const int64_t *pos, int
     MCE_LAUNCH_CHECK();
 }
 void launch_classify_roots(int64_t n, const int64_t *orp, int32_t min_len, int32_t shard_rank, int32_t shard_count,
-                           int32_t *cls, int64_t *hist, cudaStream_t s) {
-    classify_roots_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, orp, min_len, shard_rank, shard_count, cls,
-                                                           (unsigned long long *)hist);
+                           const uint8_t *keep, int64_t keep_T, int32_t *cls, int64_t *hist, cudaStream_t s) {
+    classify_roots_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, orp, min_len, shard_rank, shard_count, keep, keep_T,
+                                                           cls, (unsigned long long *)hist);
     MCE_LAUNCH_CHECK();
 }
 void launch_find_window(const int64_t *prefix, int64_t hi, int64_t lo_min, int64_t room, int64_t row_bytes,

@@ -1,7 +1,7 @@
 // Frontier layout and expansion kernels (the hot path).
 #pragma once
 
-#include "common.cuh"
+#include "graph.cuh"
 
 namespace mce {
 
@@ -168,8 +168,12 @@ int wide_min_w();
 // perm = the level's entries [0, n) grouped by slot (counting sort: hist over nslots, scan, scatter)
 void launch_group_by_slot(const int32_t *slot, int64_t n, int32_t nslots, int32_t *hist, int64_t *offs,
                           int64_t *scan_tmp, int32_t *perm, cudaStream_t s);
+// keep != nullptr: only CSR ids r >= keep_T with keep[r - keep_T] are roots (root colour filter, colour.cu)
 void launch_classify_roots(int64_t n, const int64_t *orp, int32_t min_len, int32_t shard_rank, int32_t shard_count,
-                           int32_t *cls, int64_t *hist, cudaStream_t s);
+                           const uint8_t *keep, int64_t keep_T, int32_t *cls, int64_t *hist, cudaStream_t s);
+// colour.cu: greedy colouring of the vertices of core >= need - 1 and the per-root colour bound
+bool root_colour_filter(mce_graph *g, int32_t need, int64_t min_s, uint8_t *keep, int32_t *colr, int64_t *scratch,
+                        cudaStream_t s, int64_t *T_out, int64_t *kept_out);
 void launch_find_window(const int64_t *prefix, int64_t hi, int64_t lo_min, int64_t room, int64_t row_bytes,
                         int64_t per_root, int64_t *out, cudaStream_t s);
 void launch_flag_eq(int64_t n, const int32_t *cls, int32_t c, int32_t *flag, cudaStream_t s);

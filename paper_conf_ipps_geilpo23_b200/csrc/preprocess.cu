@@ -118,8 +118,8 @@ __device__ __forceinline__ void async_append(bool take, int32_t u, const int64_t
 
 // ctrl (u64, one counter per 128-byte line so the hot counters do not share an
 // L2 sector / slice): line 0 peel-order tail; lines 1..3 + 3 * (L % 2): work
-// head, tail, done of level L; lines 8..10 + 3 * (s % 3): scan s appended /
-// kept-alive count / min kept degree
+// head, tail, done of level L; lines 8..11 + 4 * (s % 3): scan s appended /
+// kept-alive count / min kept degree / dead entries seen
 constexpr int kLine = 16;  // u64 per counter line
 __global__ void __launch_bounds__(kPeelThreads)
     kcore_async(int64_t n, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col, int32_t *deg,
@@ -127,10 +127,9 @@ __global__ void __launch_bounds__(kPeelThreads)
                 long long *work0, long long *work1, int64_t witems, unsigned long long *ctrl, int max_sleep,
                 long long *trace) {
     cg::grid_group grid = cg::this_grid();
-    __shared__ unsigned long long sh[6];
+    __shared__ unsigned long long sh[8];
     const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const int64_t nthreads = (int64_t)gridDim.x * blockDim.x;
-    const int64_t warp = tid >> 5;
     const int64_t nwarps = nthreads >> 5;
     const int lane = threadIdx.x & 31;
     unsigned long long *otail = ctrl;
@@ -140,51 +139,102 @@ __global__ void __launch_bounds__(kPeelThreads)
     int64_t n_alive = n;
     int32_t *cur = alive_a, *nxt = alive_b;
     int32_t k = 0;
+    bool compact = true;  // block-uniform: decided from counters every block reads after a grid barrier
+    __shared__ unsigned swcnt[32];
+    __shared__ unsigned long long sbase, sred[3][32];
+    const int wib = threadIdx.x >> 5, nwb = blockDim.x >> 5;
     while (true) {
         unsigned long long *head = CTR(1 + 3 * (L & 1)), *tail = CTR(2 + 3 * (L & 1)), *done = CTR(3 + 3 * (L & 1));
-        unsigned long long *sapp = CTR(8 + 3 * (s % 3)), *skept = CTR(9 + 3 * (s % 3)), *smin = CTR(10 + 3 * (s % 3));
+        unsigned long long *sapp = CTR(8 + 4 * (s % 3)), *skept = CTR(9 + 4 * (s % 3)), *smin = CTR(10 + 4 * (s % 3)),
+                           *sdead = CTR(11 + 4 * (s % 3));
         long long *work = (L & 1) ? work1 : work0;
         if (tid == 0) {  // scan counters of s+1 (last read before scan s began)
-            *CTR(8 + 3 * ((s + 1) % 3)) = 0;
-            *CTR(9 + 3 * ((s + 1) % 3)) = 0;
-            *CTR(10 + 3 * ((s + 1) % 3)) = ~0ull;
+            *CTR(8 + 4 * ((s + 1) % 3)) = 0;
+            *CTR(9 + 4 * ((s + 1) % 3)) = 0;
+            *CTR(10 + 4 * ((s + 1) % 3)) = ~0ull;
+            *CTR(11 + 4 * ((s + 1) % 3)) = 0;
         }
-        // ---- scan: append every alive vertex of degree <= k, compact the rest
+        // ---- scan: append every alive vertex of degree <= k; the rest is
+        // compacted into the next list only when enough of the list has died
+        // (else the list is scanned in place next time, dead entries skipped).
+        // Counts are aggregated per block (one atomic per block per scan, and
+        // per block-iteration for the compaction offsets): same-address
+        // atomics per warp cost ~n_alive / 32 serialised L2 operations per
+        // scan, the larger part of a scan on rmat22 (260 scans, ~50 us each).
         int32_t dmin = INT32_MAX;
-        for (int64_t i0 = warp * 32; i0 < n_alive; i0 += nwarps * 32) {
-            const int64_t i = i0 + lane;
+        unsigned napp = 0, ndead = 0;
+        for (int64_t b0 = (int64_t)blockIdx.x * blockDim.x; b0 < n_alive; b0 += (int64_t)gridDim.x * blockDim.x) {
+            const int64_t i = b0 + threadIdx.x;
             int32_t v = -1, d = 0;
             bool live = false;
             if (i < n_alive) {
                 v = cur[i];
                 live = !dead[v];
                 if (live) d = deg[v];
+                else ++ndead;
             }
             const bool q = live && d <= k;
             const bool keep = live && d > k;
-            const unsigned qm = __ballot_sync(0xffffffffu, q);
-            if (lane == 0 && qm) atomicAdd(sapp, (unsigned long long)__popc(qm));
+            napp += q;
             async_append<32>(q, v, rowptr, core, order, dead, work, otail, tail, k);
-            const unsigned km = __ballot_sync(0xffffffffu, keep);
-            unsigned long long kb = 0;
-            if (lane == 0 && km) kb = atomicAdd(skept, (unsigned long long)__popc(km));
-            kb = __shfl_sync(0xffffffffu, kb, 0);
-            if (keep) {
-                nxt[kb + __popc(km & lanemask_lt())] = v;
-                dmin = min(dmin, d);
+            if (keep) dmin = min(dmin, d);
+            if (compact) {
+                const unsigned km = __ballot_sync(0xffffffffu, keep);
+                if (lane == 0) swcnt[wib] = __popc(km);
+                __syncthreads();
+                if (wib == 0) {  // exclusive prefix over the block's warps, one atomic
+                    const unsigned c = lane < nwb ? swcnt[lane] : 0u;
+                    unsigned incl = c;
+#pragma unroll
+                    for (int o = 1; o < 32; o <<= 1) {
+                        const unsigned y = __shfl_up_sync(0xffffffffu, incl, o);
+                        if (lane >= o) incl += y;
+                    }
+                    if (lane < nwb) swcnt[lane] = incl - c;
+                    const unsigned tot = __shfl_sync(0xffffffffu, incl, 31);
+                    if (lane == 0) sbase = tot ? atomicAdd(skept, (unsigned long long)tot) : 0ull;
+                }
+                __syncthreads();
+                if (keep) nxt[sbase + swcnt[wib] + __popc(km & lanemask_lt())] = v;
+                __syncthreads();  // swcnt / sbase reuse
             }
         }
-        dmin = __reduce_min_sync(0xffffffffu, dmin);
-        if (lane == 0 && dmin != INT32_MAX) atomicMin(smin, (unsigned long long)dmin);
+        {  // block totals: appended, dead entries seen, smallest kept degree
+            const unsigned wa = __reduce_add_sync(0xffffffffu, napp), wd = __reduce_add_sync(0xffffffffu, ndead);
+            const int32_t wm = __reduce_min_sync(0xffffffffu, dmin);
+            if (lane == 0) {
+                sred[0][wib] = wa;
+                sred[1][wib] = wd;
+                sred[2][wib] = (unsigned long long)(uint32_t)wm;
+            }
+            __syncthreads();
+            if (wib == 0) {
+                unsigned long long a = lane < nwb ? sred[0][lane] : 0ull, dd = lane < nwb ? sred[1][lane] : 0ull;
+                unsigned long long m = lane < nwb ? sred[2][lane] : (unsigned long long)INT32_MAX;
+#pragma unroll
+                for (int o = 16; o > 0; o >>= 1) {
+                    a += __shfl_xor_sync(0xffffffffu, a, o);
+                    dd += __shfl_xor_sync(0xffffffffu, dd, o);
+                    const unsigned long long y = __shfl_xor_sync(0xffffffffu, m, o);
+                    m = y < m ? y : m;
+                }
+                if (lane == 0) {
+                    if (a) atomicAdd(sapp, a);
+                    if (dd) atomicAdd(sdead, dd);
+                    if (m != (unsigned long long)INT32_MAX) atomicMin(smin, m);
+                }
+            }
+        }
         grid.sync();
         if (threadIdx.x == 0) {
             sh[0] = __ldcg(sapp);
             sh[1] = __ldcg(skept);
             sh[2] = __ldcg(smin);
             sh[3] = __ldcg(otail);
+            sh[4] = __ldcg(sdead);
         }
         __syncthreads();
-        const unsigned long long appended = sh[0], kept = sh[1], md = sh[2], placed = sh[3];
+        const unsigned long long appended = sh[0], kept = sh[1], md = sh[2], placed = sh[3], ndead_all = sh[4];
         __syncthreads();
         if (trace && tid == 0 && s < 8192) {  // MCE_KCORE_TRACE: (k, alive before scan, appended, t)
             unsigned long long t;
@@ -194,11 +244,14 @@ __global__ void __launch_bounds__(kPeelThreads)
             trace[4 * s + 2] = (long long)appended;
             trace[4 * s + 3] = (long long)t;
         }
-        n_alive = (int64_t)kept;
-        {
+        if (compact) {
+            n_alive = (int64_t)kept;
             int32_t *t = cur;
             cur = nxt;
             nxt = t;
+            compact = false;
+        } else {
+            compact = (ndead_all + appended) * 8 >= (unsigned long long)n_alive;
         }
         ++s;
         if ((int64_t)placed >= n) break;  // every vertex has its core number
@@ -771,8 +824,8 @@ void kcore(mce_graph *g) {
     MCE_CUDA(cudaMemsetAsync(work0, 0xff, sizeof(long long) * witems, s));
     MCE_CUDA(cudaMemsetAsync(work1, 0xff, sizeof(long long) * witems, s));
     MCE_CUDA(cudaMemsetAsync(ctrl, 0, kLine * 20 * sizeof(unsigned long long), s));
-    for (int i = 0; i < 3; ++i)
-        MCE_CUDA(cudaMemsetAsync(ctrl + kLine * (10 + 3 * i), 0xff, sizeof(unsigned long long), s));
+    for (int i = 0; i < 3; ++i)  // smin of the three scan counter sets
+        MCE_CUDA(cudaMemsetAsync(ctrl + kLine * (10 + 4 * i), 0xff, sizeof(unsigned long long), s));
     degrees_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(), deg, alive_a);
     MCE_LAUNCH_CHECK();
     // launch shape (measured on B200, ba1m / rmat22): alone, one 512-thread

@@ -523,3 +523,25 @@ def test_wide_lockstep(key, g, monkeypatch):
         assert (r.omega, r.count) == (om, len(cl)) and np.array_equal(r.cliques, cl), kw
     f = mce().Graph(g_.rowptr, g_.col).find_one(window=4)
     assert f.omega == om and oracle.is_clique(*g_.numpy(), f.cliques[0])
+
+
+@pytest.mark.parametrize("key", ["RMAT15", "RMAT13", "CP8+K600", "CP12+K300", "K130", "ER400d", "ER700w8", "planted",
+                                 "T(36,12)", "Paley17", "BA5k", "er2000"])
+def test_root_colour_filter(key, monkeypatch):
+    """Root colour filter (colour.cu, reading 14) forced on at every size (MCE_ROOT_COLOUR_MIN_S=1):
+    the greedy colouring of the vertices of core >= need - 1 and the per-root colour bound drop roots, never a
+    maximum clique; enumeration (several heuristics: different need) and find-one against the oracle, and the
+    filter off gives the same answer."""
+    monkeypatch.setenv("MCE_ROOT_COLOUR_MIN_S", "1")
+    g = GRAPHS[key]()
+    om, cl = oracle_answer(key)
+    for kw in (dict(), dict(heuristic="single_degree"), dict(heuristic="none"), dict(root_colour=False),
+               dict(orientation="degeneracy_det")):
+        if kw.get("heuristic") == "none" and key not in ("RMAT13", "planted", "BA5k", "er2000", "ER400d"):
+            continue  # (no bound: exponential on the dense and hub-core graphs)
+        r = run_enum(g, **kw)
+        assert (r.omega, r.count) == (om, len(cl)) and np.array_equal(r.cliques, cl), kw
+    m = mce()
+    gg = m.Graph(g.rowptr, g.col)
+    r = gg.find_one(window=4)
+    assert r.omega == om and oracle.is_clique(*g.numpy(), r.cliques[0])
