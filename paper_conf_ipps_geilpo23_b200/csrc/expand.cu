@@ -616,6 +616,7 @@ __global__ void __launch_bounds__(256) expand_thread(const ExpandArgs a) {
 // small-frontier fused levels (see expand.cuh)
 // ---------------------------------------------------------------------------
 constexpr int kSmallThreads = 1024;
+constexpr int kSmallRoots = 4;  // roots whose rows expand_small stages in shared memory (8 KB each)
 
 template <bool WRITE>
 __device__ __forceinline__ int32_t expand_entry_w(int W, const ExpandArgs &a, int64_t e, int64_t out,
@@ -641,8 +642,8 @@ __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a
     __shared__ int64_t s_end;
     __shared__ int s_hb, s_ub;
     __shared__ int64_t s_used;
-    __shared__ int s_smin, s_smax;
-    __shared__ uint64_t s_rows[256 * 4];  // one root's rows 0 .. 64 W - 1, W words each (W <= 4)
+    __shared__ int s_slots[kSmallRoots], s_over;
+    __shared__ uint64_t s_rows[kSmallRoots][256 * 4];  // per root: rows 0 .. 64 W - 1, W words each (W <= 4)
     const int t = threadIdx.x;
     if (t == 0) {
         A = a0;
@@ -697,27 +698,33 @@ __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a
             s_end = p - scratch;
         }
         __syncthreads();
-        // every candidate under one root (the deep chains of a hub root): its
-        // rows are staged in shared memory, so the colouring's dependent row
-        // loads are shared-memory hits instead of L2 round trips
-        if (t == 0) {
-            s_smin = INT32_MAX;
-            s_smax = -1;
-        }
+        // candidates under at most kSmallRoots roots (the deep chains below the
+        // hub roots): the roots' rows are staged in shared memory, so the
+        // colouring's dependent row loads are shared-memory hits instead of
+        // L2 round trips
+        if (t < kSmallRoots) s_slots[t] = -1;
+        if (t == 0) s_over = 0;
         __syncthreads();
+        int my = -1;
         if (t < N) {
             const int32_t sl = A.slot[A.begin + t];
-            atomicMin(&s_smin, sl);
-            atomicMax(&s_smax, sl);
+            for (int j = 0; j < kSmallRoots && my < 0; ++j) {
+                const int old = atomicCAS(&s_slots[j], -1, sl);
+                if (old == -1 || old == sl) my = j;
+            }
+            if (my < 0) s_over = 1;
         }
         __syncthreads();
-        const bool one_root = s_smin == s_smax;
-        if (one_root) {
-            const RootInfo ri = A.roots[s_smin];
-            const int nr = min(64 * W, ri.L);
-            for (int q = t; q < nr * W; q += blockDim.x) {
-                const int r = q / W, x = q - r * W;
-                s_rows[q] = __ldg(A.adj + ri.abase + (int64_t)r * A.Wa + x);
+        const bool staged = !s_over;
+        if (staged) {
+            for (int j = 0; j < kSmallRoots; ++j) {
+                if (s_slots[j] < 0) break;
+                const RootInfo ri = A.roots[s_slots[j]];
+                const int nr = min(64 * W, ri.L);
+                for (int q = t; q < nr * W; q += blockDim.x) {
+                    const int r = q / W, x = q - r * W;
+                    s_rows[j][q] = __ldg(A.adj + ri.abase + (int64_t)r * A.Wa + x);
+                }
             }
         }
         __syncthreads();
@@ -725,7 +732,7 @@ __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a
         unsigned long long nclq = 0;
         int hb = -1, ub = 0;
         const int32_t cnt = expand_entry_w<false>(W, A, A.begin + t, 0, nleaf, nclq, hb, ub, t < N, true,
-                                                  one_root ? s_rows : nullptr);
+                                                  staged ? s_rows[max(my, 0)] : nullptr);  // block-uniform path
         (void)cnt;
         if (nleaf) atomicAdd(&s_leaf, nleaf);
         if (nclq) atomicAdd(&s_clq, nclq);

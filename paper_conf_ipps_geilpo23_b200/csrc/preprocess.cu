@@ -239,10 +239,10 @@ __global__ void __launch_bounds__(kPeelThreads)
         if (trace && tid == 0 && s < 8192) {  // MCE_KCORE_TRACE: (k, alive before scan, appended, t)
             unsigned long long t;
             asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-            trace[4 * s] = k;
-            trace[4 * s + 1] = n_alive;
-            trace[4 * s + 2] = (long long)appended;
-            trace[4 * s + 3] = (long long)t;
+            trace[8 * s] = k;
+            trace[8 * s + 1] = n_alive;
+            trace[8 * s + 2] = (long long)appended;
+            trace[8 * s + 3] = (long long)t;
         }
         if (compact) {
             n_alive = (int64_t)kept;
@@ -389,6 +389,13 @@ __global__ void __launch_bounds__(kPeelThreads)
         const int64_t extent = min((int64_t)max(sh[4], sh[5]), witems);
         const int64_t placed2 = (int64_t)__ldcg(otail);
         __syncthreads();
+        if (trace && tid == 0 && s - 1 < 8192) {  // drain end, items drained, vertices placed
+            unsigned long long t;
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+            trace[8 * (s - 1) + 4] = (long long)t;
+            trace[8 * (s - 1) + 5] = (long long)sh[5];
+            trace[8 * (s - 1) + 6] = placed2;
+        }
         for (int64_t i = tid; i < extent; i += nthreads) work[i] = -1;
         ++L;
         ++k;
@@ -851,19 +858,20 @@ void kcore(mce_graph *g) {
     long long *trace = nullptr;
     const bool tracing = getenv("MCE_KCORE_TRACE") != nullptr;  // per-scan trace to stderr (tuning aid)
     if (tracing) {
-        trace = g->pool.take<long long>(4 * 8192);
-        MCE_CUDA(cudaMemsetAsync(trace, 0xff, sizeof(long long) * 4 * 8192, s));
+        trace = g->pool.take<long long>(8 * 8192);
+        MCE_CUDA(cudaMemsetAsync(trace, 0xff, sizeof(long long) * 8 * 8192, s));
     }
     void *args[] = {&n_arg, &rp, &cl, &dg, &co, &qu, &aa, &ab, &dd, &w0, &w1, &wi, &ct, &ms, &trace};
     MCE_CUDA(cudaLaunchCooperativeKernel((void *)kcore_async, grid, threads, args, 0, s));
     if (tracing) {
-        std::vector<long long> ht(4 * 8192);
+        std::vector<long long> ht(8 * 8192);
         MCE_CUDA(cudaMemcpyAsync(ht.data(), trace, sizeof(long long) * ht.size(), cudaMemcpyDeviceToHost, s));
         stream_sync(s);
         fprintf(stderr, "[kcore] grid %d x %d\n", grid, threads);
-        for (int i = 0; i < 8192 && ht[4 * i] >= 0; ++i)
-            fprintf(stderr, "[kcore] scan %d k %lld alive %lld appended %lld t_us %.2f\n", i, ht[4 * i], ht[4 * i + 1],
-                    ht[4 * i + 2], i ? (ht[4 * i + 3] - ht[3]) / 1e3 : 0.0);
+        for (int i = 0; i < 8192 && ht[8 * i] >= 0; ++i)
+            fprintf(stderr, "[kcore] scan %d k %lld alive %lld appended %lld t_us %.2f drain_end_us %.2f items %lld placed %lld\n",
+                    i, ht[8 * i], ht[8 * i + 1], ht[8 * i + 2], (ht[8 * i + 3] - ht[3]) / 1e3,
+                    ht[8 * i + 4] >= 0 ? (ht[8 * i + 4] - ht[3]) / 1e3 : -1.0, ht[8 * i + 5], ht[8 * i + 6]);
     }
     g->kernels += 2;
     // degeneracy = max core (the last queued vertex has it)

@@ -3,6 +3,7 @@
 
     python scripts/make_golden_rmat.py rmat22      # ~15 min on one core
     python scripts/make_golden_rmat.py rmat20      # same recipe at scale 20 (~8 min)
+    python scripts/make_golden_rmat.py rmat26s20   # configs[4]'s recipe (50 planted 20-cliques) at scale 20
 
 The R-MAT workloads have too many maximum cliques to store (rmat22: 3 * 2^26
 cliques of 223 vertices), so the colouring oracle runs in count-only mode
@@ -30,6 +31,10 @@ from synth import graphs as G  # noqa: E402
 def graph(name):
     if name in ("rmat22", "rmat26"):
         return G.make_config(name), f"synth.graphs.make_config('{name}')"
+    if name.startswith("rmat26s"):  # the rmat26 recipe (50 planted 20-cliques) at a scale the oracle finishes
+        scale = int(name[7:])
+        return (G.make_config("rmat26", scale_override=scale),
+                f"synth.graphs.make_config('rmat26', scale_override={scale})")
     scale = int(name[4:])
     return G.rmat(scale, 16, 0.57, 0.19, 0.19, seed=1), f"synth.graphs.rmat({scale}, 16, 0.57, 0.19, 0.19, seed=1)"
 

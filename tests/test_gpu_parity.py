@@ -416,6 +416,8 @@ def golden(name):
 def rmat_graph(name, device):
     if name in ("rmat22", "rmat26"):
         return G.make_config(name, device=device)
+    if name.startswith("rmat26s"):  # configs[4]'s recipe (50 planted 20-cliques) at a smaller scale
+        return G.make_config("rmat26", device=device, scale_override=int(name[7:]))
     return G.rmat(int(name[4:]), 16, 0.57, 0.19, 0.19, seed=1, device=device)
 
 
@@ -433,7 +435,7 @@ def check_stored_rows(rows, omega, rp, col, sample=64):
 
 
 @pytest.mark.slow
-@pytest.mark.parametrize("name", ["rmat20", "rmat22"])
+@pytest.mark.parametrize("name", ["rmat20", "rmat22", "rmat26s20"])
 def test_config_rmat_golden(name):
     """BASELINE configs[2] (rmat22) and the same recipe at scale 20: omega and
     the exact multiplicity against the oracle's count (tests/golden, written by
