@@ -400,6 +400,7 @@ def main():
               "heuristic_ms": statistics.mean(t["heuristic_ms"] for t in timings),
               "expand_ms": statistics.mean(t["expand_ms"] for t in timings),
               "expand_count_ms": cnt_ms, "root_kernel_ms": root_ms,
+              "root_setup_ms": statistics.mean(t.get("root_setup_ms", 0.0) for t in timings),
               "host_call_ms": statistics.mean(t["host_total_ms"] for t in timings),
               "host_preprocess_ms": statistics.mean(t["host_preprocess_ms"] for t in timings),
               "host_heuristic_ms": statistics.mean(t["host_heuristic_ms"] for t in timings),

@@ -233,7 +233,9 @@ mce_status mce_result_levels(const mce_result *r, int64_t *entries, int32_t cap,
  * [10] host wall time of the whole call, [11] of its preprocessing, [12] of
  * its heuristic, [13] host<->device synchronisations it made, [14] host
  * time of the budget / workspace setup, [15] of the root classes + levels,
- * [16] of the canonical read-out of the stored cliques (device sort + copy). */
+ * [16] of the canonical read-out of the stored cliques (device sort + copy),
+ * [17] device time of the root setup: root colour filter and the root /
+ * re-root adjacency matrix builds (not part of [2]). */
 mce_status mce_result_timing(const mce_result *r, double *t, int32_t cap);
 void mce_result_free(mce_result *r);
 

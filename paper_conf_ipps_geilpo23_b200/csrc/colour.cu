@@ -52,6 +52,9 @@ __global__ void core_threshold_kernel(int64_t n, const int32_t *__restrict__ vid
 }
 
 constexpr int kColWarps = 8;  // warps per block of both kernels
+#ifndef COL_SPIN
+#define COL_SPIN 0  // polls of the pending list before the first back-off sleep
+#endif
 
 // greedy colouring of the top m ranks (= CSR ids [T, n)), colr[id - T].
 // Per vertex: one pass over its out-row with independent loads ORs every
@@ -112,7 +115,10 @@ __global__ void __launch_bounds__(32 * kColWarps) colour_dataflow_kernel(
                 left += __popc(pm);
             }
             np = left;
-            if (np > 0) __nanosleep(naps++ < 8 ? 32 : 128);
+            if (np > 0) {
+                if (naps >= COL_SPIN) __nanosleep(naps < COL_SPIN + 8 ? 32 : 128);
+                ++naps;
+            }
         }
         __syncwarp();
         int first = INT32_MAX;

@@ -139,7 +139,8 @@ class LaunchClock {
             cudaEventDestroy(e.b);
         }
     }
-    // kind: 0 count pass, 1 write pass, 2 fused root level
+    // kind: 0 count pass, 1 write pass, 2 fused root level, 3 root setup (root
+    // colour filter, root / re-root matrix builds; not part of the expansion total)
     int start(int kind) {
         if (used_ == ev_.size()) {
             Pair p;
@@ -153,10 +154,14 @@ class LaunchClock {
     }
     void stop(int i) { MCE_CUDA(cudaEventRecord(ev_[i].b, s_)); }
     // call after a stream sync that covers every recorded pair
-    void collect(double &all_ms, double &count_ms, double &root_ms) {
+    void collect(double &all_ms, double &count_ms, double &root_ms, double &setup_ms) {
         for (size_t i = 0; i < used_; ++i) {
             float ms = 0;
             MCE_CUDA(cudaEventElapsedTime(&ms, ev_[i].a, ev_[i].b));
+            if (ev_[i].kind == 3) {
+                setup_ms += ms;
+                continue;
+            }
             all_ms += ms;
             if (ev_[i].kind == 0) count_ms += ms;
             if (ev_[i].kind == 2) root_ms += ms;
@@ -247,7 +252,7 @@ class Engine {
 
     // stats
     std::vector<int64_t> level_entries_;
-    double t_expand_ms_ = 0.0, t_count_ms_ = 0.0, t_root_ms_ = 0.0;
+    double t_expand_ms_ = 0.0, t_count_ms_ = 0.0, t_root_ms_ = 0.0, t_setup_ms_ = 0.0;
     int64_t count_launches_ = 0, kernels_ = 0, root_launches_ = 0;
     double count_bytes_ = 0.0, root_bytes_ = 0.0;
 };
@@ -570,7 +575,9 @@ bool Engine::reroot(int32_t k, const Level &L) {
         D.vloc = arena_.alloc<int32_t>(cnt);
         // (a previous group's process(k, ...) replaced chain[k]: the prefixes read the candidates' own links)
         MCE_CUDA(cudaMemcpyAsync(chain_dev_ + k, &link, sizeof(link), cudaMemcpyHostToDevice, s_));
+        const int tcl = clock_.start(3);
         launch_reroot_build(ra, list, cnt, voff, Wn, nV, nA, nroots, D.P, D.slot, D.parent, D.vloc, nprefix, s_);
+        clock_.stop(tcl);
         kernels_ += 4;
         roots_ = nroots;
         adj_ = nA;
@@ -1039,7 +1046,9 @@ void Engine::do_class(int32_t cls, const int32_t *list, int64_t count) {
         RootInfo *roots = arena_.alloc<RootInfo>(nw);
         uint64_t *adj = arena_.alloc<uint64_t>(rows * W_);
         launch_make_roots(base + lo, nw, 1, W_, g_->orp.get(), prefix + lo, roots, s_);
+        const int tcl = clock_.start(3);
         launch_build_adj(roots, nw, W_, g_->orp.get(), g_->ocol.get(), adj, rows * W_, s_);
+        clock_.stop(tcl);
         kernels_ += 2;
         roots_ = roots;
         adj_ = adj;
@@ -1226,7 +1235,10 @@ mce_result *Engine::run() {
             int64_t *scr = arena_.alloc<int64_t>(4);
             int64_t kept = 0;
             const char *ms = getenv("MCE_ROOT_COLOUR_MIN_S");
-            if (root_colour_filter(g_, need(), ms ? atoll(ms) : kRootColourMinS, keepb, colr, scr, s_, &rT, &kept)) {
+            const int tcl = clock_.start(3);
+            const bool ran = root_colour_filter(g_, need(), ms ? atoll(ms) : kRootColourMinS, keepb, colr, scr, s_, &rT, &kept);
+            clock_.stop(tcl);
+            if (ran) {
                 rkeep = keepb;
                 kernels_ += 4;
                 if (o_.verbose > 0)
@@ -1270,7 +1282,7 @@ mce_result *Engine::run() {
     res->t_pre_ms = preprocess_ms(g_);  // (the preprocessing finished long ago; no extra wait)
     stream_sync(s_);
     res->t_enum_ms = tt.collect();
-    clock_.collect(t_expand_ms_, t_count_ms_, t_root_ms_);
+    clock_.collect(t_expand_ms_, t_count_ms_, t_root_ms_, t_setup_ms_);
     // keep answering the other shards until everyone is done
     if (o_.bound_sync) {
         int32_t gactive = 1;
@@ -1316,6 +1328,7 @@ mce_result *Engine::run() {
     res->count_bytes = count_bytes_;
     res->t_expand_ms = t_expand_ms_;
     res->t_root_ms = t_root_ms_;
+    res->t_setup_ms = t_setup_ms_;
     res->root_launches = root_launches_;
     res->root_bytes = root_bytes_;
     res->kernels = kernels_;

@@ -18,6 +18,7 @@ struct mce_result {
     double t_pre_ms = 0, t_heur_ms = 0, t_enum_ms = 0, t_expand_ms = 0, t_count_ms = 0, count_bytes = 0;
     int64_t count_launches = 0, kernels = 0;
     double t_root_ms = 0, root_bytes = 0;  // fused root-level kernel
+    double t_setup_ms = 0;                 // root colour filter + root / re-root matrix builds
     int64_t root_launches = 0;
     double h_total_ms = 0, h_pre_ms = 0, h_heur_ms = 0;  // host wall time of the call / its phases
     double h_setup_ms = 0, h_enum_ms = 0, h_readout_ms = 0;

@@ -68,6 +68,13 @@ constexpr int kPeelThreads = 1024;  // launch bound; the launch uses kcore_threa
 #define KCORE_CHUNK 32  // measured: 128 / 64 / 32 / 16 / 8 = ba1m 1.49 / 1.46 / 1.43 / 1.44 / 1.50 ms, rmat22 82.5 / 81.8 / 82.1 / 81.4 / - ms
 #endif
 constexpr int64_t kChunk = KCORE_CHUNK;  // edges per work item
+#ifndef KCORE_LOCAL
+#define KCORE_LOCAL 0  // 1: fallen vertices continued by the same warp from a shared-memory stack (append_local); measured: rmat22 same, ba1m 1.40 -> 1.47-1.65 ms (20 ms without the batch cap: one warp serialises a long cascade)
+#endif
+#ifndef KCORE_LOCAL_BATCHES
+#define KCORE_LOCAL_BATCHES 4
+#endif
+constexpr int kLocal = 96;  // items per warp-local continuation stack (32 warps x 768 B)
 #ifndef KCORE_GRAB
 #define KCORE_GRAB 0  // 1: reserve only while items are queued (fewer atomics on tiny levels); measured slower overall (rmat22 78.1 vs 74.2 ms, ba1m 1.52 vs 1.47)
 #endif
@@ -116,6 +123,55 @@ __device__ __forceinline__ void async_append(bool take, int32_t u, const int64_t
     }
 }
 
+// The drain's variant (whole warp): the vertices that fell are appended to
+// the peel order as above, but their work items go to the warp's local stack
+// (shared memory) while it has room -- the warp continues the cascade itself,
+// depth first, instead of a round trip through the global list and another
+// warp's poll (a cascade step then costs one warp's dependent loads).  Items
+// that do not fit go to the global list.  lcount is warp-uniform.
+__device__ __forceinline__ void append_local(bool take, int32_t u, const int64_t *__restrict__ rowptr, int32_t *core,
+                                             int32_t *order, uint8_t *dead, long long *work,
+                                             unsigned long long *otail, unsigned long long *wtail, int32_t k,
+                                             long long *lstack, int &lcount, int lcap) {
+    const int lane = threadIdx.x & 31;
+    const unsigned m = __ballot_sync(0xffffffffu, take);
+    if (!m) return;
+    int items = 0;
+    if (take) {
+        const int64_t d = rowptr[u + 1] - rowptr[u];
+        items = (int)((d + kChunk - 1) / kChunk);
+    }
+    int inc = items;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int y = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= o) inc += y;
+    }
+    const int total = __shfl_sync(0xffffffffu, inc, 31);
+    const bool local = lcount + total <= lcap;
+    unsigned long long ob = 0, wb = 0;
+    if (lane == 0) {
+        ob = atomicAdd(otail, (unsigned long long)__popc(m));
+        if (total && !local) wb = atomicAdd(wtail, (unsigned long long)total);
+    }
+    ob = __shfl_sync(0xffffffffu, ob, 0);
+    wb = __shfl_sync(0xffffffffu, wb, 0);
+    if (take) {
+        order[ob + __popc(m & lanemask_lt())] = u;
+        core[u] = k;
+        dead[u] = 1;
+        for (int c = 0; c < items; ++c) {
+            const long long it = (long long)(uint32_t)u | ((long long)c << 32);
+            if (local)
+                lstack[lcount + inc - items + c] = it;
+            else
+                work[wb + inc - items + c] = it;
+        }
+    }
+    if (local) lcount += total;
+    __syncwarp();
+}
+
 // ctrl (u64, one counter per 128-byte line so the hot counters do not share an
 // L2 sector / slice): line 0 peel-order tail; lines 1..3 + 3 * (L % 2): work
 // head, tail, done of level L; lines 8..11 + 4 * (s % 3): scan s appended /
@@ -128,6 +184,7 @@ __global__ void __launch_bounds__(kPeelThreads)
                 long long *trace) {
     cg::grid_group grid = cg::this_grid();
     __shared__ unsigned long long sh[8];
+    __shared__ long long lstack_all[(kPeelThreads / 32) * kLocal];
     const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const int64_t nthreads = (int64_t)gridDim.x * blockDim.x;
     const int64_t nwarps = nthreads >> 5;
@@ -271,6 +328,58 @@ __global__ void __launch_bounds__(kPeelThreads)
         // done counts are aggregated over the whole warp (one atomic each).
         unsigned long long pending = 0;  // lane 0: items processed, not yet added to `done`
         bool finished = false;
+        // warp-local continuation stack (append_local); pending is never
+        // published while it holds items, so done < tail until it is empty
+        long long *lst = lstack_all + (size_t)(threadIdx.x >> 5) * kLocal;
+        int lcount = 0;
+        // the edges of up to four items (one per 8-lane tile; -1: none), fallen
+        // neighbours to the local stack
+        auto run_items = [&](long long item) {
+            int64_t eb = 0, ee = 0;
+            if (item != -1) {
+                const int32_t v = (int32_t)(item & 0xffffffffll);
+                const int64_t c = item >> 32;
+                eb = rowptr[v] + c * kChunk;
+                ee = min(rowptr[v + 1], eb + kChunk);
+            }
+            const int iters = __reduce_max_sync(0xffffffffu, (unsigned)((ee - eb + 7) >> 3));
+            for (int it = 0; it < iters; ++it) {
+                const int64_t e = eb + it * 8 + (lane & 7);
+                bool fell = false;
+                int32_t u = -1;
+                if (e < ee) {
+                    u = col[e];
+                    if (!dead[u]) fell = atomicSub(deg + u, 1) == k + 1;
+                }
+                if (KCORE_LOCAL)
+                    append_local(fell, u, rowptr, core, order, dead, work, otail, tail, k, lst, lcount, kLocal);
+                else
+                    async_append<32>(fell, u, rowptr, core, order, dead, work, otail, tail, k);
+            }
+        };
+        // pop up to four local items (one per tile) and run them, at most
+        // KCORE_LOCAL_BATCHES times; what is left goes to the global list (a
+        // long cascade must not serialise on one warp while others idle)
+        auto drain_local = [&]() {
+            int batches = 0;
+            while (lcount > 0 && batches < KCORE_LOCAL_BATCHES) {
+                const int take = min(lcount, 4);
+                const int t = lane >> 3;
+                const long long item = t < take ? lst[lcount - 1 - t] : -1ll;
+                __syncwarp();
+                lcount -= take;
+                run_items(item);
+                ++batches;
+            }
+            if (lcount > 0) {  // spill
+                unsigned long long wb = 0;
+                if (lane == 0) wb = atomicAdd(tail, (unsigned long long)lcount);
+                wb = __shfl_sync(0xffffffffu, wb, 0);
+                for (int i = lane; i < lcount; i += 32) work[wb + i] = lst[i];
+                __syncwarp();
+                lcount = 0;
+            }
+        };
         while (!finished) {
             // Lane 0 reserves slots only while the list holds unreserved items
             // (head < tail): with nothing queued, every warp reserving four
@@ -332,24 +441,8 @@ __global__ void __launch_bounds__(kPeelThreads)
                 item = __shfl_sync(0xffffffffu, item, leader);
                 dead_slot = __shfl_sync(0xffffffffu, dead_slot, leader);
                 const bool work_now = !resolved && item != -1;
-                int64_t eb = 0, ee = 0;
-                if (work_now) {
-                    const int32_t v = (int32_t)(item & 0xffffffffll);
-                    const int64_t c = item >> 32;
-                    eb = rowptr[v] + c * kChunk;
-                    ee = min(rowptr[v + 1], eb + kChunk);
-                }
-                const int iters = __reduce_max_sync(0xffffffffu, (unsigned)((ee - eb + 7) >> 3));
-                for (int it = 0; it < iters; ++it) {
-                    const int64_t e = eb + it * 8 + (lane & 7);
-                    bool fell = false;
-                    int32_t u = -1;
-                    if (e < ee) {
-                        u = col[e];
-                        if (!dead[u]) fell = atomicSub(deg + u, 1) == k + 1;
-                    }
-                    async_append<32>(fell, u, rowptr, core, order, dead, work, otail, tail, k);
-                }
+                run_items(work_now ? item : -1ll);
+                drain_local();  // the cascade below these items, in this warp
                 const unsigned done_m = __ballot_sync(0xffffffffu, work_now && (lane & 7) == 0);
                 if (lane == 0) pending += (unsigned long long)__popc(done_m);
                 if (work_now) resolved = true;

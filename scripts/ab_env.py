@@ -23,7 +23,7 @@ for spec in sys.argv[2:]:
         r = gg.find_one(window=64) if cfg == "dense800" else gg.enumerate(max_cliques=1 << 16)
         dt = time.perf_counter() - t0
         tm = r.timing
-        print(f"{spec or 'default'} rep{rep}: {dt * 1e3:.1f} ms omega {r.omega} count {r.count} pre {tm['preprocess_ms']:.1f} "
+        print(f"{spec or 'default'} rep{rep}: {dt * 1e3:.1f} ms omega {r.omega} count {r.count} setup {tm['root_setup_ms']:.1f} pre {tm['preprocess_ms']:.1f} "
               f"heur {tm['heuristic_ms']:.1f} enum(host) {tm['host_enum_ms']:.1f} expand {tm['expand_ms']:.1f}", flush=True)
         gg.close()
     for k, v in old.items():

@@ -3,6 +3,7 @@
 
     python scripts/ncu_summary.py launches <launches.csv>          # per-kernel device time (launch list)
     python scripts/ncu_summary.py full <report.ncu-rep> [regex]    # key counters + hottest source lines
+    python scripts/ncu_summary.py longest <report.ncu-rep> [regex] # the same for the longest matching launch only
 
 The launch list is the `--metrics gpu__time_duration.sum --clock-control none`
 pass (cold-cache, serialised: compare SHARES of the step, not absolutes).
@@ -29,6 +30,8 @@ KEYS = [
     ("launch__grid_size", "grid"),
     ("launch__block_size", "block"),
     ("smsp__inst_executed.sum", "warp instructions"),
+    ("sass__inst_executed_local_loads", "local-memory loads (spills)"),
+    ("sass__inst_executed_local_stores", "local-memory stores (spills)"),
 ]
 
 
@@ -56,11 +59,17 @@ def launches(path):
     print(f"\n{sum(c for c, _ in agg.values())} launches, {total:.1f} us total")
 
 
-def full(path, regex=None):
+def full(path, regex=None, longest=False):
     raw = subprocess.check_output(["ncu", "-i", path, "--page", "raw", "--csv"], stderr=subprocess.DEVNULL).decode()
     rows = list(csv.reader(io.StringIO(raw)))
     h, units = rows[0], rows[1]
-    for r in rows[2:]:
+    body = rows[2:]
+    if longest:  # only the longest launch (of the kernels matching regex)
+        di = h.index("gpu__time_duration.sum")
+        cand = [r for r in body if not regex or re.search(regex, r[h.index("Kernel Name")])]
+        body = [max(cand, key=lambda r: float(r[di].replace(",", "")))] if cand else []
+        print(f"(longest of {len(cand)} captured launches)\n")
+    for r in body:
         name = r[h.index("Kernel Name")]
         if regex and not re.search(regex, name):
             continue
@@ -97,4 +106,4 @@ if __name__ == "__main__":
     if sys.argv[1] == "launches":
         launches(sys.argv[2])
     else:
-        full(sys.argv[2], sys.argv[3] if len(sys.argv) > 3 else None)
+        full(sys.argv[2], sys.argv[3] if len(sys.argv) > 3 else None, longest=sys.argv[1] == "longest")
