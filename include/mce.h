@@ -125,10 +125,11 @@ typedef struct {
     int32_t no_overlap;      /* 0 (default): the degree heuristics run on a second stream and host
                                 thread while the k-core / orientation preprocessing runs (they
                                 share no data); 1: one after the other */
-    int32_t no_reroot;       /* 0 (default): candidates of levels >= 2 that are 32 or more words wide
-                                (roots of more than 1024 out-neighbours) become roots of their own
-                                over their candidate set P (at the width of |P|); 1: they stay in
-                                the root's space (A/B tests) */
+    int32_t no_reroot;       /* 0 (default): candidates of levels >= 2 at least MCE_REROOT_MIN_W
+                                words wide (environment; unset = never, the measured best: on
+                                R-MAT scale 26 the re-root matrix builds cost more than the
+                                narrower expansion saves) become roots of their own over their
+                                candidate set P (at the width of |P|); 1: never (A/B tests) */
     int32_t no_smem_expand;  /* 0 (default): levels of 8 or 16 words per candidate set are grouped by
                                 root and expanded with the root's adjacency matrix staged in
                                 shared memory (expand_smem); 1: rows read from global memory

@@ -179,6 +179,27 @@ class LaunchClock {
     size_t used_ = 0;
 };
 
+// verbose > 1: device time of one step, synchronously (diagnostics only)
+template <typename F>
+double timed_step(cudaStream_t s, bool on, F &&f) {
+    if (!on) {
+        f();
+        return 0.0;
+    }
+    cudaEvent_t a, b;
+    MCE_CUDA(cudaEventCreate(&a));
+    MCE_CUDA(cudaEventCreate(&b));
+    MCE_CUDA(cudaEventRecord(a, s));
+    f();
+    MCE_CUDA(cudaEventRecord(b, s));
+    MCE_CUDA(cudaEventSynchronize(b));
+    float ms = 0;
+    MCE_CUDA(cudaEventElapsedTime(&ms, a, b));
+    cudaEventDestroy(a);
+    cudaEventDestroy(b);
+    return ms;
+}
+
 class Engine {
    public:
     Engine(mce_graph *g, const mce_options &o, bool find_one)
@@ -228,7 +249,10 @@ class Engine {
     const int32_t *vtab_ = nullptr;             // vertex table of the window's roots (g->ocol, or re-rooted lists)
     const int32_t *prefix_ = nullptr;           // re-rooted window: per-root clique prefix (k0_ vertices each)
     int32_t k0_ = 0;
-    int reroot_min_w_ = 32;                     // levels this wide re-root their candidates (0: never)
+    // levels this wide re-root their candidates (0: never, the default: on rmat26
+    // the re-root matrix builds cost 17.5 s for no expansion gain -- 48.7 s vs
+    // 30.2 s per step, 40.8 s with 64; MCE_REROOT_MIN_W sets it, tests force it)
+    int reroot_min_w_ = 0;
     int32_t no_reroot_level_ = -1;              // the level being processed in a re-rooted space
     int smem_min_w_ = 8;                        // narrowest level width taking the shared-memory count pass
     int64_t smem_min_n_ = 2048;                 // ... and fewest entries (small levels: rows stay L1/L2 hits)
@@ -576,8 +600,12 @@ bool Engine::reroot(int32_t k, const Level &L) {
         // (a previous group's process(k, ...) replaced chain[k]: the prefixes read the candidates' own links)
         MCE_CUDA(cudaMemcpyAsync(chain_dev_ + k, &link, sizeof(link), cudaMemcpyHostToDevice, s_));
         const int tcl = clock_.start(3);
-        launch_reroot_build(ra, list, cnt, voff, Wn, nV, nA, nroots, D.P, D.slot, D.parent, D.vloc, nprefix, s_);
+        const double bms = timed_step(s_, o_.verbose > 1, [&] {
+            launch_reroot_build(ra, list, cnt, voff, Wn, nV, nA, nroots, D.P, D.slot, D.parent, D.vloc, nprefix, s_);
+        });
         clock_.stop(tcl);
+        if (o_.verbose > 1)
+            fprintf(stderr, "[mce] re-root build k=%d Wn=%d candidates=%lld: %.3f ms\n", k, (int)Wn, (long long)cnt, bms);
         kernels_ += 4;
         roots_ = nroots;
         adj_ = nA;
@@ -1047,8 +1075,13 @@ void Engine::do_class(int32_t cls, const int32_t *list, int64_t count) {
         uint64_t *adj = arena_.alloc<uint64_t>(rows * W_);
         launch_make_roots(base + lo, nw, 1, W_, g_->orp.get(), prefix + lo, roots, s_);
         const int tcl = clock_.start(3);
-        launch_build_adj(roots, nw, W_, g_->orp.get(), g_->ocol.get(), adj, rows * W_, s_);
+        const double bms = timed_step(s_, o_.verbose > 1, [&] {
+            launch_build_adj(roots, nw, W_, g_->orp.get(), g_->ocol.get(), adj, rows * W_, s_);
+        });
         clock_.stop(tcl);
+        if (o_.verbose > 1)
+            fprintf(stderr, "[mce] root build W=%d roots=%lld rows=%lld: %.3f ms\n", W_, (long long)nw, (long long)rows,
+                    bms);
         kernels_ += 2;
         roots_ = roots;
         adj_ = adj;
@@ -1236,8 +1269,12 @@ mce_result *Engine::run() {
             int64_t kept = 0;
             const char *ms = getenv("MCE_ROOT_COLOUR_MIN_S");
             const int tcl = clock_.start(3);
-            const bool ran = root_colour_filter(g_, need(), ms ? atoll(ms) : kRootColourMinS, keepb, colr, scr, s_, &rT, &kept);
+            bool ran = false;
+            const double fms = timed_step(s_, o_.verbose > 1, [&] {
+                ran = root_colour_filter(g_, need(), ms ? atoll(ms) : kRootColourMinS, keepb, colr, scr, s_, &rT, &kept);
+            });
             clock_.stop(tcl);
+            if (o_.verbose > 1) fprintf(stderr, "[mce] root colour filter: %.3f ms\n", fms);
             if (ran) {
                 rkeep = keepb;
                 kernels_ += 4;
