@@ -236,7 +236,10 @@ mce_status mce_result_levels(const mce_result *r, int64_t *entries, int32_t cap,
  * time of the budget / workspace setup, [15] of the root classes + levels,
  * [16] of the canonical read-out of the stored cliques (device sort + copy),
  * [17] device time of the root setup: root colour filter and the root /
- * re-root adjacency matrix builds (not part of [2]). */
+ * re-root adjacency matrix builds (not part of [2]), [18] of the root matrix
+ * builds alone (build_adj_block), [19] their launches, [20] their
+ * algorithmic bytes (V and row bounds 20 B per member, every out-row id the
+ * scan reads 4 B, the matrix 8 W B per row). */
 mce_status mce_result_timing(const mce_result *r, double *t, int32_t cap);
 void mce_result_free(mce_result *r);
 

@@ -194,14 +194,15 @@ class Graph:
             nl = ctypes.c_int32()
             ent = (ctypes.c_int64 * 512)()
             check(L.mce_result_levels(handle, ent, 512, ctypes.byref(nl)))
-            tm = (ctypes.c_double * 18)()
-            check(L.mce_result_timing(handle, tm, 18))
+            tm = (ctypes.c_double * 21)()
+            check(L.mce_result_timing(handle, tm, 21))
             timing = dict(preprocess_ms=tm[0], heuristic_ms=tm[1], expand_ms=tm[2], count_kernel_ms=tm[3],
                           count_launches=int(tm[4]), count_kernel_bytes=tm[5], kernels=int(tm[6]),
                           root_kernel_ms=tm[7], root_launches=int(tm[8]), root_kernel_bytes=tm[9],
                           host_total_ms=tm[10], host_preprocess_ms=tm[11], host_heuristic_ms=tm[12],
                           syncs=int(tm[13]), host_setup_ms=tm[14], host_enum_ms=tm[15], host_readout_ms=tm[16],
-                          root_setup_ms=tm[17])
+                          root_setup_ms=tm[17], build_kernel_ms=tm[18], build_launches=int(tm[19]),
+                          build_kernel_bytes=tm[20])
             return Result(om.value, cnt.value, cl, bool(tr.value), [int(ent[i]) for i in range(min(nl.value, 512))],
                           timing)
         finally:

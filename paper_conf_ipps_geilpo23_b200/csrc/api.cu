@@ -393,12 +393,13 @@ mce_status mce_result_levels(const mce_result *r, int64_t *entries, int32_t cap,
 mce_status mce_result_timing(const mce_result *r, double *t, int32_t cap) {
     return run_guarded([&] {
         if (!r || !t) fail(MCE_ERR_INVALID, "NULL argument");
-        double v[18] = {r->t_pre_ms,    r->t_heur_ms,     r->t_expand_ms,          r->t_count_ms,
+        double v[21] = {r->t_pre_ms,    r->t_heur_ms,     r->t_expand_ms,          r->t_count_ms,
                         (double)r->count_launches, r->count_bytes, (double)r->kernels, r->t_root_ms,
                         (double)r->root_launches,  r->root_bytes,  r->h_total_ms, r->h_pre_ms,
                         r->h_heur_ms,              (double)r->syncs, r->h_setup_ms, r->h_enum_ms,
-                        r->h_readout_ms,           r->t_setup_ms};
-        for (int32_t i = 0; i < std::min(cap, 18); ++i) t[i] = v[i];
+                        r->h_readout_ms,           r->t_setup_ms,    r->t_build_ms,
+                        (double)r->build_launches, r->build_bytes};
+        for (int32_t i = 0; i < std::min(cap, 21); ++i) t[i] = v[i];
     });
 }
 

@@ -140,7 +140,8 @@ class LaunchClock {
         }
     }
     // kind: 0 count pass, 1 write pass, 2 fused root level, 3 root setup (root
-    // colour filter, root / re-root matrix builds; not part of the expansion total)
+    // colour filter, re-root matrix builds), 4 root matrix builds (build_adj_block);
+    // 3 and 4 are not part of the expansion total
     int start(int kind) {
         if (used_ == ev_.size()) {
             Pair p;
@@ -154,12 +155,13 @@ class LaunchClock {
     }
     void stop(int i) { MCE_CUDA(cudaEventRecord(ev_[i].b, s_)); }
     // call after a stream sync that covers every recorded pair
-    void collect(double &all_ms, double &count_ms, double &root_ms, double &setup_ms) {
+    void collect(double &all_ms, double &count_ms, double &root_ms, double &setup_ms, double &build_ms) {
         for (size_t i = 0; i < used_; ++i) {
             float ms = 0;
             MCE_CUDA(cudaEventElapsedTime(&ms, ev_[i].a, ev_[i].b));
-            if (ev_[i].kind == 3) {
+            if (ev_[i].kind >= 3) {
                 setup_ms += ms;
+                if (ev_[i].kind == 4) build_ms += ms;
                 continue;
             }
             all_ms += ms;
@@ -243,6 +245,8 @@ class Engine {
     unsigned long long *clq_slot_ = nullptr;    // g->misc[3]
     int32_t *maxbit_ = nullptr;                 // g->misc[4]
     unsigned long long *out_count_ = nullptr;   // g->misc[5] fused-pass children
+    unsigned long long *build_bytes_ = nullptr; // g->misc[8] algorithmic bytes of the root matrix builds
+    int64_t build_launches_ = 0;
     unsigned long long *pair_n_ = nullptr;      // g->misc[6] pair-completion descriptors
     unsigned long long *chunk_ctr_ = nullptr;   // g->misc[7] work counter of the shared-memory count pass
     int64_t nroots_ = 0;                        // roots of the current window (slots 0 .. nroots_ - 1)
@@ -276,7 +280,7 @@ class Engine {
 
     // stats
     std::vector<int64_t> level_entries_;
-    double t_expand_ms_ = 0.0, t_count_ms_ = 0.0, t_root_ms_ = 0.0, t_setup_ms_ = 0.0;
+    double t_expand_ms_ = 0.0, t_count_ms_ = 0.0, t_root_ms_ = 0.0, t_setup_ms_ = 0.0, t_build_ms_ = 0.0;
     int64_t count_launches_ = 0, kernels_ = 0, root_launches_ = 0;
     double count_bytes_ = 0.0, root_bytes_ = 0.0;
 };
@@ -1074,10 +1078,11 @@ void Engine::do_class(int32_t cls, const int32_t *list, int64_t count) {
         RootInfo *roots = arena_.alloc<RootInfo>(nw);
         uint64_t *adj = arena_.alloc<uint64_t>(rows * W_);
         launch_make_roots(base + lo, nw, 1, W_, g_->orp.get(), prefix + lo, roots, s_);
-        const int tcl = clock_.start(3);
+        const int tcl = clock_.start(4);
         const double bms = timed_step(s_, o_.verbose > 1, [&] {
-            launch_build_adj(roots, nw, W_, g_->orp.get(), g_->ocol.get(), adj, rows * W_, s_);
+            launch_build_adj(roots, nw, W_, g_->orp.get(), g_->ocol.get(), adj, rows * W_, s_, build_bytes_);
         });
+        ++build_launches_;
         clock_.stop(tcl);
         if (o_.verbose > 1)
             fprintf(stderr, "[mce] root build W=%d roots=%lld rows=%lld: %.3f ms\n", W_, (long long)nw, (long long)rows,
@@ -1226,6 +1231,8 @@ mce_result *Engine::run() {
     out_count_ = leaf_total_ + 5;
     pair_n_ = leaf_total_ + 6;
     chunk_ctr_ = leaf_total_ + 7;
+    build_bytes_ = leaf_total_ + 8;
+    MCE_CUDA(cudaMemsetAsync(build_bytes_, 0, sizeof(unsigned long long), s_));
     if (const char *sw = getenv("MCE_SMEM_MIN_W")) smem_min_w_ = atoi(sw);  // tuning hooks (A/B runs)
     if (const char *sn = getenv("MCE_SMEM_MIN_N")) smem_min_n_ = atoll(sn);
     if (const char *sp = getenv("MCE_SMEM_PER_ROOT")) smem_per_root_ = atoll(sp);
@@ -1319,7 +1326,7 @@ mce_result *Engine::run() {
     res->t_pre_ms = preprocess_ms(g_);  // (the preprocessing finished long ago; no extra wait)
     stream_sync(s_);
     res->t_enum_ms = tt.collect();
-    clock_.collect(t_expand_ms_, t_count_ms_, t_root_ms_, t_setup_ms_);
+    clock_.collect(t_expand_ms_, t_count_ms_, t_root_ms_, t_setup_ms_, t_build_ms_);
     // keep answering the other shards until everyone is done
     if (o_.bound_sync) {
         int32_t gactive = 1;
@@ -1366,6 +1373,14 @@ mce_result *Engine::run() {
     res->t_expand_ms = t_expand_ms_;
     res->t_root_ms = t_root_ms_;
     res->t_setup_ms = t_setup_ms_;
+    res->t_build_ms = t_build_ms_;
+    res->build_launches = build_launches_;
+    if (build_launches_ > 0) {
+        unsigned long long *hb = g_->host.get<unsigned long long>(1);
+        MCE_CUDA(cudaMemcpyAsync(hb, build_bytes_, sizeof(unsigned long long), cudaMemcpyDeviceToHost, s_));
+        stream_sync(s_);
+        res->build_bytes = (double)hb[0];
+    }
     res->root_launches = root_launches_;
     res->root_bytes = root_bytes_;
     res->kernels = kernels_;

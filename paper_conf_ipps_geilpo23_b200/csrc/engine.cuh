@@ -19,6 +19,8 @@ struct mce_result {
     int64_t count_launches = 0, kernels = 0;
     double t_root_ms = 0, root_bytes = 0;  // fused root-level kernel
     double t_setup_ms = 0;                 // root colour filter + root / re-root matrix builds
+    double t_build_ms = 0, build_bytes = 0;  // root matrix builds (build_adj_block) and their algorithmic bytes
+    int64_t build_launches = 0;
     int64_t root_launches = 0;
     double h_total_ms = 0, h_pre_ms = 0, h_heur_ms = 0;  // host wall time of the call / its phases
     double h_setup_ms = 0, h_enum_ms = 0, h_readout_ms = 0;

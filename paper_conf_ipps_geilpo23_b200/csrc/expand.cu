@@ -84,8 +84,12 @@ constexpr int kSpanWords = kSpanBits / 32;
 template <bool SMEM>
 __global__ void build_adj_block(const RootInfo *__restrict__ roots, int64_t nroots, int W,
                                 const int64_t *__restrict__ orp, const int32_t *__restrict__ ocol,
-                                uint64_t *__restrict__ adj, int Lmax, int use_map) {
+                                uint64_t *__restrict__ adj, int Lmax, int use_map, unsigned long long *bytes) {
     extern __shared__ int32_t dsm[];
+    // algorithmic bytes: V and the row bounds of its members
+    // (4 + 16 per member), every out-row id the scan must read (4 each; a row
+    // stops at the first chunk beyond V's largest id) and the matrix (8 W L)
+    unsigned long long nbytes = 0;
     const int lane = threadIdx.x & 31;
     const int wib = threadIdx.x >> 5, nwb = blockDim.x >> 5;
     int32_t *sV = dsm;
@@ -123,7 +127,9 @@ __global__ void build_adj_block(const RootInfo *__restrict__ roots, int64_t nroo
                 // aligned 16-byte loads: a lane takes 4 consecutive ids, the warp 128
                 // per trip (elements outside [pb, pe) are masked; ocol is padded by 4)
                 const int li = L - 1 - i;
+                int64_t q_end = pb;
                 for (int64_t q0 = pb & ~3ll; q0 < pe; q0 += 128) {
+                    q_end = min(pe, q0 + 128);
                     const int64_t q = q0 + 4 * lane;
                     int4 v4 = make_int4(INT32_MAX, INT32_MAX, INT32_MAX, INT32_MAX);
                     if (q < pe) v4 = __ldg(reinterpret_cast<const int4 *>(ocol + q));
@@ -147,12 +153,15 @@ __global__ void build_adj_block(const RootInfo *__restrict__ roots, int64_t nroo
                     }
                     if (__any_sync(0xffffffffu, past)) break;  // sorted row: the rest is beyond V
                 }
+                if (lane == 0) nbytes += 20 + 4 * (unsigned long long)(q_end - pb);
                 continue;
             }
             // kAdjChunks chunks of 32 ids loaded before any is looked up (the
             // row scan is bound by its load latency, one chunk per trip)
             bool stop = false;
+            int64_t q_last = pb;
             for (int64_t q0 = pb; q0 < pe && !stop; q0 += 32 * kAdjChunks) {
+              q_last = min(pe, q0 + 32 * kAdjChunks);
               int32_t uu[kAdjChunks];
 #pragma unroll
               for (int k = 0; k < kAdjChunks; ++k) {
@@ -191,13 +200,16 @@ __global__ void build_adj_block(const RootInfo *__restrict__ roots, int64_t nroo
                 }
               }
             }
+            if (lane == 0) nbytes += 20 + 4 * (unsigned long long)(q_last - pb);
         }
         __syncthreads();
         if (SMEM) {
             for (int64_t w = threadIdx.x; w < (int64_t)L * W * 2; w += blockDim.x) gA[w] = sA[w];
         }
+        if (threadIdx.x == 0) nbytes += 8ull * L * W;
         __syncthreads();
     }
+    if (bytes && (threadIdx.x & 31) == 0 && nbytes) atomicAdd(bytes, nbytes);
 }
 
 __global__ void init_level1_kernel(const RootInfo *__restrict__ roots, int64_t nroots, int W, uint64_t *P,
@@ -1836,7 +1848,7 @@ void launch_tile(const ExpandArgs &a, bool write_pass, cudaStream_t s) {
 }  // namespace
 
 void launch_build_adj(const RootInfo *roots, int64_t nroots, int W, const int64_t *orp, const int32_t *ocol,
-                      uint64_t *adj, int64_t adj_words, cudaStream_t s) {
+                      uint64_t *adj, int64_t adj_words, cudaStream_t s, unsigned long long *bytes) {
     if (nroots <= 0) return;
     if (W == 1) {
         build_adj_w1<<<grid_for(nroots * 32, 256, 16), 256, 0, s>>>(roots, nroots, orp, ocol, adj);
@@ -1855,7 +1867,7 @@ void launch_build_adj(const RootInfo *roots, int64_t nroots, int W, const int64_
                 attr_set = smem;
             }
             build_adj_block<true><<<grid_for(nroots, 1, 8), 1024, smem, s>>>(roots, nroots, W, orp, ocol, adj,
-                                                                              (int)Lmax, 1);
+                                                                              (int)Lmax, 1, bytes);
         } else {
             const size_t smem = base + map_bytes;
             static size_t attr_set = 0;
@@ -1866,7 +1878,7 @@ void launch_build_adj(const RootInfo *roots, int64_t nroots, int W, const int64_
             }
             MCE_CUDA(cudaMemsetAsync(adj, 0, sizeof(uint64_t) * (size_t)adj_words, s));
             build_adj_block<false><<<grid_for(nroots, 1, 8), 1024, smem, s>>>(roots, nroots, W, orp, ocol, adj,
-                                                                               (int)Lmax, 1);
+                                                                               (int)Lmax, 1, bytes);
         }
     }
     MCE_LAUNCH_CHECK();

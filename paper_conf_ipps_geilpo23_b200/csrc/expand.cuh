@@ -156,8 +156,9 @@ void launch_expand_small(const ExpandArgs &a, uint8_t *scratch, int64_t scratch_
 // W classes: 0 -> 1 word, 1 -> 2, 2 -> 4, ... (W = 1 << class); L <= 64 W
 constexpr int kMaxClass = 9;  // W up to 256 words (L <= 16384)
 
+// bytes (optional): += the build's algorithmic bytes (build_adj_block, W >= 2)
 void launch_build_adj(const RootInfo *roots, int64_t nroots, int W, const int64_t *orp, const int32_t *ocol,
-                      uint64_t *adj, int64_t adj_words, cudaStream_t s);
+                      uint64_t *adj, int64_t adj_words, cudaStream_t s, unsigned long long *bytes = nullptr);
 void launch_init_level1(const RootInfo *roots, int64_t nroots, int W, uint64_t *P, int32_t *slot, int32_t *parent,
                         int32_t *vloc, cudaStream_t s);
 void launch_expand(const ExpandArgs &a, bool write_pass, cudaStream_t s);
