@@ -328,6 +328,7 @@ __global__ void __launch_bounds__(kPeelThreads)
         // done counts are aggregated over the whole warp (one atomic each).
         unsigned long long pending = 0;  // lane 0: items processed, not yet added to `done`
         bool finished = false;
+        int next_rounds = 1;  // KCORE_GRAB == 2: rounds of 4 slots of the next reservation (lane 0)
         // warp-local continuation stack (append_local); pending is never
         // published while it holds items, so done < tail until it is empty
         long long *lst = lstack_all + (size_t)(threadIdx.x >> 5) * kLocal;
@@ -391,7 +392,10 @@ __global__ void __launch_bounds__(kPeelThreads)
             // groups of up to 8 rounds of 4 slots (fewer atomics on `head`).
             unsigned long long base = 0;
             int rounds = 0;
-            if (lane == 0 && !KCORE_GRAB) {
+            if (lane == 0 && KCORE_GRAB == 2) {  // adaptive: grow while every slot was ready at once
+                rounds = next_rounds;
+                base = atomicAdd(head, 4ull * rounds);
+            } else if (lane == 0 && !KCORE_GRAB) {
                 base = atomicAdd(head, 4ull);
                 rounds = 1;
             } else if (lane == 0) {
@@ -423,6 +427,7 @@ __global__ void __launch_bounds__(kPeelThreads)
             const int leader = lane & ~7;
             bool resolved = false, over = false;
             int idle = 0;  // consecutive empty polls: back off, and only then look at the hot counters
+            int polls = 0;
             while (true) {
                 long long item = -1;
                 bool dead_slot = false;
@@ -450,6 +455,7 @@ __global__ void __launch_bounds__(kPeelThreads)
                     resolved = true;
                     over = true;
                 }
+                ++polls;
                 if (__all_sync(0xffffffffu, resolved)) break;
                 if (!done_m) {
                     // about to wait: publish the processed count first (a warp with work
@@ -466,6 +472,7 @@ __global__ void __launch_bounds__(kPeelThreads)
                 }
             }
             if (__all_sync(0xffffffffu, over)) finished = true;  // later rounds' slots are beyond the end too
+            if (KCORE_GRAB == 2 && lane == 0) next_rounds = polls == 1 ? min(8, next_rounds * 2) : 1;
           }
         }
         if (lane == 0 && pending) {  // (cannot happen: `over` needs an idle, flushed warp)
