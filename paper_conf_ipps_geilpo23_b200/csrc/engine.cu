@@ -34,6 +34,7 @@ constexpr size_t kAlign = 256;
 // small problems stay small while an exploding frontier may use the whole
 // budget.  Allocation is stack-like: mark() / reset(mark).
 constexpr size_t kBigSeg = 4ull << 30;
+constexpr int64_t kLevelReserve = 12 * (int64_t)kAlign;  // see process(): chunk sizing (the fixed allocations of one level)
 // the root colour filter runs when at least this many vertices can be in a
 // clique of the size sought (below it the colouring costs more than it saves;
 // MCE_ROOT_COLOUR_MIN_S overrides, for tests)
@@ -865,8 +866,13 @@ void Engine::process(int32_t k, const Level &L) {
     const int64_t depth_left = std::max<int64_t>(1, (int64_t)maxub - (k + 1));
     int64_t a0 = 0;
     while (total > 0 && a0 < N) {
-        const int64_t share = total * per_child2 <= (int64_t)(arena_.avail() / 2) ? 2 : depth_left + 1;
-        const int64_t cap = (int64_t)(arena_.avail() / share) / per_child2;
+        // kLevelReserve stays free for the fixed small allocations of the levels
+        // below (every arena allocation is rounded to kAlign bytes, which the
+        // per-child share does not cover: under a few-MB budget a deep chain of
+        // chunked levels otherwise ends on a 256-byte allocation with nothing left)
+        const int64_t usable = std::max<int64_t>(0, (int64_t)arena_.avail() - kLevelReserve);
+        const int64_t share = total * per_child2 <= usable / 2 ? 2 : depth_left + 1;
+        const int64_t cap = (usable / share) / per_child2;
         int64_t b, cnt, base;
         if (a0 == 0 && total <= cap) {
             b = N;
@@ -881,6 +887,17 @@ void Engine::process(int32_t k, const Level &L) {
             b = hc[0];
             cnt = hc[1];
             base = hc[2];
+            if (b == a0 && share > 2) {
+                // one candidate's children exceed this level's share: let that chunk
+                // take half of what is left (the levels below it still get the rest)
+                launch_find_chunk_end(offs, a0, N, (usable / 2) / per_child2, chunk, s_);
+                ++kernels_;
+                MCE_CUDA(cudaMemcpyAsync(hc, chunk, 3 * sizeof(int64_t), cudaMemcpyDeviceToHost, s_));
+                stream_sync(s_);
+                b = hc[0];
+                cnt = hc[1];
+                base = hc[2];
+            }
             if (b == a0)
                 fail(MCE_ERR_BUDGET, "the children of one candidate at level " + std::to_string(k) +
                                          " exceed the frontier budget");

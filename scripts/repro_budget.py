@@ -11,7 +11,7 @@ from synth import graphs as G  # noqa: E402
 
 g = G.rmat(15, 16, 0.57, 0.19, 0.19, seed=5).to("cuda")
 cases = [dict(), dict(fused_levels=False), dict(clique_shortcut=False),
-         dict(budget_bytes=6 << 20, heuristic="none", fused_levels=False),
+         dict(budget_bytes=8 << 20, heuristic="none", fused_levels=False),
          dict(budget_bytes=24 << 20, heuristic="single_degree")]
 fails = 0
 for it in range(int(sys.argv[1]) if len(sys.argv) > 1 else 20):
