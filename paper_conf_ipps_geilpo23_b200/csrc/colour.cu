@@ -22,6 +22,8 @@
 // warps, so the wait always ends), and publish their own.  The critical path is
 // the longest chain of the orientation DAG inside S (2581 vertices on rmat22,
 // whose 35.5K-vertex S prunes 27K of its 35K roots of out-degree >= 222).
+#include <cooperative_groups.h>
+
 #include "graph.cuh"
 
 namespace mce {
@@ -52,6 +54,12 @@ __global__ void core_threshold_kernel(int64_t n, const int32_t *__restrict__ vid
 }
 
 constexpr int kColWarps = 8;  // warps per block of both kernels
+#ifndef COL_CLUSTER
+#define COL_CLUSTER 1  // S small enough for shared memory: colour inside one 8-CTA cluster (DSMEM)
+#endif
+#ifndef COL_BACKOFF
+#define COL_BACKOFF 1  // poll back-off by the number of colours still missing (0: fixed 32 / 128 ns)
+#endif
 #ifndef COL_SPIN
 #define COL_SPIN 0  // polls of the pending list before the first back-off sleep
 #endif
@@ -80,17 +88,17 @@ __global__ void __launch_bounds__(32 * kColWarps) colour_dataflow_kernel(
         for (int w = lane; w < MW; w += 32) mask[w] = 0u;
         __syncwarp();
         int np = 0;  // pending entries (warp-uniform)
-        for (int64_t e0 = rb; e0 < re; e0 += 128) {
-            int32_t u[4], c[4];
+        for (int64_t e0 = rb; e0 < re; e0 += 256) {
+            int32_t u[8], c[8];
 #pragma unroll
-            for (int q = 0; q < 4; ++q) {
+            for (int q = 0; q < 8; ++q) {
                 const int64_t e = e0 + 32 * q + lane;
                 u[q] = e < re ? __ldg(ocol + e) : -1;
             }
 #pragma unroll
-            for (int q = 0; q < 4; ++q) c[q] = u[q] >= 0 ? ld_relaxed_i32(colr + (u[q] - T)) : -2;
+            for (int q = 0; q < 8; ++q) c[q] = u[q] >= 0 ? ld_relaxed_i32(colr + (u[q] - T)) : -2;
 #pragma unroll
-            for (int q = 0; q < 4; ++q) {
+            for (int q = 0; q < 8; ++q) {
                 if (c[q] >= 0) atomicOr(mask + (c[q] >> 5), 1u << (c[q] & 31));
                 const unsigned pm = __ballot_sync(0xffffffffu, c[q] == -1);
                 if (c[q] == -1) pend[np + __popc(pm & lanemask_lt())] = u[q];
@@ -116,7 +124,14 @@ __global__ void __launch_bounds__(32 * kColWarps) colour_dataflow_kernel(
             }
             np = left;
             if (np > 0) {
-                if (naps >= COL_SPIN) __nanosleep(naps < COL_SPIN + 8 ? 32 : 128);
+                // back off in proportion to how much is still missing: a warp waiting
+                // for many predecessors is far from the chain's head, and thousands of
+                // warps polling at full rate load the L2 the chain's own loads and
+                // stores go through
+                if (COL_BACKOFF)
+                    __nanosleep(np > 16 ? 2048 : (np > 4 ? 512 : (np > 1 ? 128 : 32)));
+                else if (naps >= COL_SPIN)
+                    __nanosleep(naps < COL_SPIN + 8 ? 32 : 128);
                 ++naps;
             }
         }
@@ -133,6 +148,127 @@ __global__ void __launch_bounds__(32 * kColWarps) colour_dataflow_kernel(
         if (lane == 0) st_relaxed_i32(colr + (i - T), first);
         __syncwarp();
     }
+}
+
+// The same greedy colouring inside ONE thread-block cluster (kClusterCtas SMs)
+// when S is small enough for every CTA to hold all of S's colours (u16) in
+// its shared memory: a published colour is written into every CTA's copy
+// through distributed shared memory (st to cluster.map_shared_rank: ~200
+// cycles, not an L2 round trip), and a waiting warp polls its own CTA's copy.
+// A step of the critical chain then costs one DSMEM store plus a shared-memory
+// poll instead of an L2 store plus an L2 poll (rmat22: 2581 steps).  Vertices
+// are taken in order from a counter in CTA 0's shared memory; every warp of
+// the cluster is resident, so a waited-for vertex is always being coloured.
+constexpr int kClusterCtas = 8;        // portable cluster size
+constexpr int kClusterWarps = 32;      // warps per CTA
+#ifndef COL_PEND
+#define COL_PEND 12
+#endif
+constexpr int kClusterPend = COL_PEND;  // pending predecessors a lane keeps (shared memory); measured 4 / 12 / 24 = 4.7 / 2.4 / 2.4 ms on rmat22
+constexpr uint16_t kNoColour = 0xffffu;
+
+__global__ void __launch_bounds__(32 * kClusterWarps) colour_cluster_kernel(
+    int64_t n, int64_t m, int64_t T, const int32_t *__restrict__ order, const int32_t *__restrict__ pid,
+    const int64_t *__restrict__ orp, const int32_t *__restrict__ ocol, int MW, int32_t *colr) {
+    namespace cg = cooperative_groups;
+    cg::cluster_group cluster = cg::this_cluster();
+    extern __shared__ unsigned char csm[];
+    unsigned long long *next = reinterpret_cast<unsigned long long *>(csm);           // (CTA 0's is used)
+    int32_t *pends = reinterpret_cast<int32_t *>(csm + 16);                            // threads x kClusterPend
+    unsigned *masks = reinterpret_cast<unsigned *>(pends + (size_t)32 * kClusterWarps * kClusterPend);
+    uint16_t *scol = reinterpret_cast<uint16_t *>(masks + (size_t)kClusterWarps * MW);  // m colours
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    unsigned *mask = masks + (size_t)wib * MW;
+    int32_t *pend = pends + (size_t)threadIdx.x * kClusterPend;  // this lane's pending predecessors
+    for (int64_t j = threadIdx.x; j < m; j += blockDim.x) scol[j] = kNoColour;
+    if (threadIdx.x == 0) *next = 0ull;
+    cluster.sync();
+    unsigned long long *gnext = cluster.map_shared_rank(next, 0);
+    while (true) {
+        unsigned long long j = 0;
+        if (lane == 0) j = atomicAdd(gnext, 1ull);
+        j = __shfl_sync(0xffffffffu, j, 0);
+        if ((int64_t)j >= m) break;
+        const int32_t i = pid[order[n - 1 - (int64_t)j]];
+        const int64_t rb = orp[i], re = orp[i + 1];
+        for (int w = lane; w < MW; w += 32) mask[w] = 0u;
+        __syncwarp();
+        int np = 0;
+        bool rescan = false;  // more than kClusterPend pending in this lane's elements
+        // the row's ids are loaded 8 per lane at a time, all in flight together (a
+        // dense-core row of ~1000 ids is then a few L2 latencies, not ~30)
+        for (int64_t e0 = rb; e0 < re; e0 += 32 * 8) {
+            int32_t uu[8];
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+                const int64_t e = e0 + 32 * q + lane;
+                uu[q] = e < re ? __ldg(ocol + e) - (int32_t)T : -1;
+            }
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+                if (uu[q] < 0) continue;
+                const uint16_t c = *(volatile uint16_t *)(scol + uu[q]);
+                if (c != kNoColour) {
+                    atomicOr(mask + (c >> 5), 1u << (c & 31));
+                } else if (np < kClusterPend) {
+                    pend[np++] = uu[q];
+                } else {
+                    rescan = true;
+                }
+            }
+        }
+        // wait for the missing colours (predecessors are taken earlier by resident warps)
+        while (__any_sync(0xffffffffu, np > 0 || rescan)) {
+            int left = 0;
+            for (int q = 0; q < np; ++q) {
+                const int32_t u = pend[q];
+                const uint16_t c = *(volatile uint16_t *)(scol + u);
+                if (c != kNoColour)
+                    atomicOr(mask + (c >> 5), 1u << (c & 31));
+                else
+                    pend[left++] = u;
+            }
+            np = left;
+            if (rescan && np == 0) {  // re-read this lane's elements for the overflowed ones
+                rescan = false;
+                for (int64_t e0 = rb; e0 < re; e0 += 32 * 8) {
+                    int32_t uu[8];
+#pragma unroll
+                    for (int q = 0; q < 8; ++q) {
+                        const int64_t e = e0 + 32 * q + lane;
+                        uu[q] = e < re ? __ldg(ocol + e) - (int32_t)T : -1;
+                    }
+#pragma unroll
+                    for (int q = 0; q < 8; ++q) {
+                        if (uu[q] < 0) continue;
+                        const uint16_t c = *(volatile uint16_t *)(scol + uu[q]);
+                        if (c != kNoColour)
+                            atomicOr(mask + (c >> 5), 1u << (c & 31));  // (idempotent)
+                        else if (np < kClusterPend)
+                            pend[np++] = uu[q];
+                        else
+                            rescan = true;
+                    }
+                }
+            }
+            if (np > 0 || rescan) __nanosleep(20);
+        }
+        __syncwarp();
+        int first = INT32_MAX;
+        for (int w = lane; w < MW; w += 32) {
+            const unsigned z = ~mask[w];
+            if (z) {
+                first = w * 32 + __ffs((int)z) - 1;
+                break;
+            }
+        }
+        first = __reduce_min_sync(0xffffffffu, first);
+        if (lane < kClusterCtas)  // every CTA's copy, through distributed shared memory
+            *(volatile uint16_t *)cluster.map_shared_rank(scol + (i - T), lane) = (uint16_t)first;
+        if (lane == 0) colr[i - T] = first;
+        __syncwarp();
+    }
+    cluster.sync();  // no CTA leaves while others may still write into its shared memory
 }
 
 // keep[r - T] = 1 + |colours(N+(r))| >= need (and |N+(r)| >= need - 1), warp per root
@@ -200,6 +336,30 @@ bool root_colour_filter(mce_graph *g, int32_t need, int64_t min_s, uint8_t *keep
         MCE_CUDA(cudaFuncSetAttribute(colour_dataflow_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_df));
     if (smem > 48 * 1024)
         MCE_CUDA(cudaFuncSetAttribute(root_colour_bound_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    const size_t csmem = 16 + (size_t)32 * kClusterWarps * kClusterPend * 4 + (size_t)kClusterWarps * MW * 4 +
+                         (size_t)m * 2;
+    if (COL_CLUSTER && csmem <= 200 * 1024 && MW <= 64) {
+        static size_t attr = 0;
+        if (attr < csmem) {
+            MCE_CUDA(cudaFuncSetAttribute(colour_cluster_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)csmem));
+            attr = csmem;
+        }
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3(kClusterCtas, 1, 1);
+        cfg.blockDim = dim3(32 * kClusterWarps, 1, 1);
+        cfg.dynamicSmemBytes = csmem;
+        cfg.stream = s;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeClusterDimension;
+        at[0].val.clusterDim.x = kClusterCtas;
+        at[0].val.clusterDim.y = 1;
+        at[0].val.clusterDim.z = 1;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
+        const int32_t *ord = g->order.get(), *pd = g->pid.get(), *oc = g->ocol.get();
+        const int64_t *op = g->orp.get();
+        MCE_CUDA(cudaLaunchKernelEx(&cfg, colour_cluster_kernel, n, m, T, ord, pd, op, oc, MW, colr));
+    } else {
     // persistent dataflow: only resident warps may take vertices (a waiting
     // warp's predecessors must be running), so the grid is the resident capacity
     int per_sm = 0;
@@ -209,6 +369,7 @@ bool root_colour_filter(mce_graph *g, int32_t need, int64_t min_s, uint8_t *keep
     colour_dataflow_kernel<<<grid, 32 * kColWarps, smem_df, s>>>(n, m, T, g->order.get(), g->pid.get(), g->orp.get(),
                                                                  g->ocol.get(), MW, PW, colr, ctr);
     MCE_LAUNCH_CHECK();
+    }
     root_colour_bound_kernel<<<grid_for(m * 32, 32 * kColWarps, 8), 32 * kColWarps, smem, s>>>(
         n, T, g->orp.get(), g->ocol.get(), colr, MW, need, keep, ctr + 1);
     MCE_LAUNCH_CHECK();
