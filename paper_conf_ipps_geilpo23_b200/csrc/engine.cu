@@ -464,6 +464,9 @@ bool Engine::run_small(int32_t k, const Level &L) {
         fprintf(stderr, "[mce] fused levels k=%d..%lld entries=%lld -> children=%lld leaves=%lld status=%lld\n", k,
                 (long long)(k + o.levels - 1), (long long)L.count, (long long)o.children, (long long)o.leaves,
                 (long long)o.status);
+    if (o_.verbose > 1)
+        fprintf(stderr, "[mce]   cycles: setup %lld staging %lld entry0 %lld (colouring %lld completions %lld branching %lld, %lld vertices) wait %lld tail %lld\n",
+                o.prof[0], o.prof[1], o.prof[2], o.prof[6], o.prof[7], o.prof[8], o.prof[9], o.prof[3], o.prof[4]);
     if (o.leaves > 0 || o.cliques > 0) {  // leaves of size k_next / completions of size need, last level
         ExpandArgs la = a;
         la.P = o.inP;

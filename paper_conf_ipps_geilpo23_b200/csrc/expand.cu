@@ -435,10 +435,13 @@ __device__ __forceinline__ unsigned long long warp_excl_u64(unsigned long long x
 // adjacency row word: read-only global (LDG) or a copy in shared memory (SROWS)
 template <bool SROWS>
 __device__ __forceinline__ uint64_t ldrow(const uint64_t *p) {
-    if constexpr (SROWS)
-        return *p;
-    else
+    if constexpr (SROWS) {  // an explicit shared-space load (a generic load costs the address-window check)
+        uint64_t v;
+        asm("ld.shared.u64 %0, [%1];" : "=l"(v) : "r"((unsigned)__cvta_generic_to_shared(p)));
+        return v;
+    } else {
         return __ldg(p);
+    }
 }
 
 // SROWS: the root's rows 0 .. 64 W - 1 (first W words each) are staged at
@@ -458,6 +461,9 @@ __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, 
     uint8_t colr[64 * W];  // colour - 1 (a full 4-word set has 256 colours)
     int np = 0;
     int ncol = 0;
+    int maxcls = 0, cls_start = 0;  // largest colour class (a matching complement has classes of at most 2)
+    const bool prof = a.dbg && active && e == a.begin;
+    long long c0 = prof ? clock64() : 0;
     if (a.bound == 1) {
         uint64_t U[W];
 #pragma unroll
@@ -467,6 +473,8 @@ __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, 
 #pragma unroll
             for (int w = 0; w < W; ++w) any |= U[w] != 0;
             if (!any) break;
+            maxcls = max(maxcls, np - cls_start);
+            cls_start = np;
             ++ncol;
             uint64_t Q[W];
 #pragma unroll
@@ -501,6 +509,11 @@ __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, 
         }
         ncol = np;
     }
+    if (prof) {
+        const long long c1 = clock64();
+        a.dbg[0] += c1 - c0;
+        c0 = c1;
+    }
     // P is a clique iff every colour class is a single vertex (reading 10)
     bool done = false;
     if (a.shortcut && a.bound == 1 && np >= 2 && ncol == np && a.k + np == a.need) {
@@ -513,9 +526,11 @@ __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, 
     }
     // P's complement a matching with |C| + #colours == need: 2^m completions
     // (the greedy colouring then makes every colour class a pair or a single
-    // vertex, so #colours = |P| - m)
+    // vertex, so #colours = |P| - m; a class of three or more rules it out
+    // without the pairwise test)
+    maxcls = max(maxcls, np - cls_start);
     if (!done && a.shortcut && a.bound == 1 && ncol < np && np - ncol <= 40 && a.k + ncol == a.need &&
-        a.need <= 4096) {
+        a.need <= 4096 && maxcls <= 2) {
         bool matching = true;
         for (int i = 0; i < np && matching; ++i) {
             const int v = ord[i];
@@ -537,6 +552,11 @@ __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, 
             done = true;
             if (!fused) return 0;
         }
+    }
+    if (prof) {
+        const long long c1 = clock64();
+        a.dbg[1] += c1 - c0;
+        c0 = c1;
     }
     // the branching loop (Algorithm 2 lines 3-9 with the colouring order):
     // MODE 0 count (+ leaves), 1 write at `at` with word stride `ws`
@@ -583,6 +603,12 @@ __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, 
     };
     if (WRITE) return branch(1, out, a.Wc);
     const int32_t cnt = branch(0, 0, 0);
+    if (prof) {
+        const long long c1 = clock64();
+        a.dbg[2] += c1 - c0;
+        a.dbg[3] += np;
+        c0 = c1;
+    }
     if (fused) {
         unsigned long long total;
         const unsigned long long excl = warp_excl_u64((unsigned long long)cnt, total);
@@ -627,7 +653,8 @@ __global__ void __launch_bounds__(256) expand_thread(const ExpandArgs a) {
 // ---------------------------------------------------------------------------
 // small-frontier fused levels (see expand.cuh)
 // ---------------------------------------------------------------------------
-constexpr int kSmallThreads = 1024;
+constexpr int kSmallThreads = 512;  // (1024 capped the colouring loop at 64 registers: Q/U spilled, ~360 cycles a step)
+constexpr int kSmallPer = kSmallMax / kSmallThreads;  // candidates per thread
 constexpr int kSmallRoots = 4;  // roots whose rows expand_small stages in shared memory (8 KB each)
 
 template <bool WRITE>
@@ -645,7 +672,7 @@ __device__ __forceinline__ int32_t expand_entry_w(int W, const ExpandArgs &a, in
     return expand_entry<4, WRITE>(a, e, out, nleaf, nclq, hb, ub, active, fused);
 }
 
-__global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a0, uint8_t *scratch,
+__global__ void __launch_bounds__(kSmallThreads, 1) expand_small(const ExpandArgs a0, uint8_t *scratch,
                                                               int64_t scratch_bytes, SmallOut *out,
                                                               LevelLink *chain) {
     __shared__ ExpandArgs A;
@@ -672,6 +699,19 @@ __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a
         out->slot = const_cast<int32_t *>(a0.slot);
         out->parent = const_cast<int32_t *>(a0.parent);
         out->vloc = const_cast<int32_t *>(a0.vloc);
+    }
+    __syncthreads();
+    long long pt = clock64();
+    auto phase = [&](int i) {  // thread 0: cycles since the previous mark into prof[i]
+        if (t == 0) {
+            const long long now = clock64();
+            out->prof[i] += now - pt;
+            pt = now;
+        }
+    };
+    if (t == 0) {
+        for (int i = 0; i < 10; ++i) out->prof[i] = 0;
+        A.dbg = out->prof + 6;
     }
     __syncthreads();
     for (int lev = 0; lev < kSmallMaxLevels; ++lev) {
@@ -714,17 +754,24 @@ __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a
         // hub roots): the roots' rows are staged in shared memory, so the
         // colouring's dependent row loads are shared-memory hits instead of
         // L2 round trips
+        phase(0);
         if (t < kSmallRoots) s_slots[t] = -1;
         if (t == 0) s_over = 0;
         __syncthreads();
-        int my = -1;
-        if (t < N) {
-            const int32_t sl = A.slot[A.begin + t];
-            for (int j = 0; j < kSmallRoots && my < 0; ++j) {
-                const int old = atomicCAS(&s_slots[j], -1, sl);
-                if (old == -1 || old == sl) my = j;
+        int mys[kSmallPer];
+#pragma unroll
+        for (int r = 0; r < kSmallPer; ++r) {
+            int my = -1;
+            const int idx = t + r * kSmallThreads;
+            if (idx < N) {
+                const int32_t sl = A.slot[A.begin + idx];
+                for (int j = 0; j < kSmallRoots && my < 0; ++j) {
+                    const int old = atomicCAS(&s_slots[j], -1, sl);
+                    if (old == -1 || old == sl) my = j;
+                }
+                if (my < 0) s_over = 1;
             }
-            if (my < 0) s_over = 1;
+            mys[r] = my;
         }
         __syncthreads();
         const bool staged = !s_over;
@@ -740,17 +787,24 @@ __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a
             }
         }
         __syncthreads();
+        phase(1);
         unsigned nleaf = 0;
         unsigned long long nclq = 0;
         int hb = -1, ub = 0;
-        const int32_t cnt = expand_entry_w<false>(W, A, A.begin + t, 0, nleaf, nclq, hb, ub, t < N, true,
-                                                  staged ? s_rows[max(my, 0)] : nullptr);  // block-uniform path
-        (void)cnt;
+#pragma unroll
+        for (int r = 0; r < kSmallPer; ++r) {
+            if (r * kSmallThreads >= N) break;  // (block-uniform)
+            const int idx = t + r * kSmallThreads;
+            expand_entry_w<false>(W, A, A.begin + idx, 0, nleaf, nclq, hb, ub, idx < N, true,
+                                  staged ? s_rows[max(mys[r], 0)] : nullptr);  // block-uniform path
+        }
+        phase(2);  // (thread 0's own entries)
         if (nleaf) atomicAdd(&s_leaf, nleaf);
         if (nclq) atomicAdd(&s_clq, nclq);
         if (hb >= 0) atomicMax(&s_hb, hb);
         if (ub > 0) atomicMax(&s_ub, ub);
         __syncthreads();
+        phase(3);  // (waiting for the block's slowest entry)
         const int64_t total = (int64_t)s_cnt;
         if (t == 0) {
             out->level_n[lev] = N;
@@ -824,6 +878,7 @@ __global__ void __launch_bounds__(kSmallThreads) expand_small(const ExpandArgs a
             A.k = A.k + 1;
         }
         __syncthreads();
+        phase(4);
         if (stop) break;
     }
 }

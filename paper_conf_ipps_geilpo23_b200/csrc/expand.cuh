@@ -98,6 +98,7 @@ struct ExpandArgs {
     // wide count pass (expand_wide, W >= 32): per-tile colouring-order scratch (u16 entries)
     uint16_t *wscratch;
     int64_t wscratch_n;
+    long long *dbg;  // diagnostics (expand_small, verbose >= 2): cycles of the first entry's phases
 };
 
 // Fused root level for W == 1 roots (roots.cu): one warp per root builds the
@@ -146,6 +147,7 @@ struct SmallOut {
     int32_t *inslot, *inparent, *invloc;
     int64_t inN, inW, inPs;
     int64_t level_n[kSmallMaxLevels];  // entries of every processed level
+    long long prof[10];                // clock64 cycles per phase, summed over levels (verbose >= 2 prints them)
 };
 // write the rows of the pair completions recorded by the last count pass over
 // the level described by `a` (its P / slot / chain); n = descriptors recorded
