@@ -53,6 +53,9 @@ def parse():
                    choices=["auto", "none", "single_degree", "single_core", "multi_degree", "multi_core"],
                    help="lower-bound heuristic (PAPER.md IV-A); auto: the per-config choice of HEURISTIC below "
                         "(PAPER.md V line 315 reports each dataset under its fastest heuristic)")
+    p.add_argument("--orientation", default="auto", choices=["auto", "degeneracy", "degree", "degeneracy_det"],
+                   help="edge orientation (PAPER.md IV-C: the paper keeps the edge from the lower-degree vertex; "
+                        "the degeneracy orders bound every out-degree by the core number); auto: ORIENTATION below")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--shard-depth", type=int, default=-1,
@@ -243,6 +246,15 @@ HEURISTIC = {"er2000": "multi_degree", "ba1m": "multi_degree", "rmat22": "multi_
              "dense800": "multi_degree", "rmat26": "multi_degree"}
 
 
+# per-config orientation (same reasoning as HEURISTIC: the answer never depends on it), from the sweep in
+# profiles/r02_orientation_sweep_v1.md: the paper's degree orientation skips the k-core peel and wins on
+# er2000 and dense800; rmat22 needs the degeneracy order (out-degree <= core: the root colour filter and
+# narrow root spaces); ba1m keeps it too -- 1.20 ms with degree vs 1.41, but its sparse root kernel
+# (out-degrees <= 4 only under the degeneracy order) is the north star's >= 50% HBM roofline kernel
+ORIENTATION = {"er2000": "degree", "ba1m": "degeneracy", "rmat22": "degeneracy", "dense800": "degree",
+               "rmat26": "degeneracy"}
+
+
 def bench_defaults(args):
     mode = args.mode or ("find_one" if args.config == "dense800" else "enumerate")
     shard_depth = args.shard_depth if args.shard_depth >= 0 else (3 if args.config == "rmat26" else 0)
@@ -250,6 +262,8 @@ def bench_defaults(args):
     max_cl = args.max_cliques if args.max_cliques >= 0 else (1 << 16 if args.config.startswith("rmat") else 0)
     if args.heuristic == "auto":
         args.heuristic = HEURISTIC[args.config]
+    if args.orientation == "auto":
+        args.orientation = ORIENTATION[args.config]
     return mode, shard_depth, window, max_cl
 
 
@@ -338,6 +352,9 @@ def main():
     rdev = "cpu" if (world > 1 and dist.get_backend() == "gloo") else f"cuda:{local}"
     mode, shard_depth, args.window, max_cl = bench_defaults(args)
     heur = args.heuristic
+    orient = args.orientation
+    if world > 1 and orient == "degeneracy":
+        orient = "degeneracy_det"  # every rank must orient identically (reading 18)
 
     g = build_graph(args.config, f"cuda:{local}")
     edges = g.num_edges
@@ -349,11 +366,12 @@ def main():
         gr.clear_cache()
         if world > 1:
             if mode == "enumerate":
-                return mdist.enumerate_distributed(gr, max_cliques=max_cl, shard_depth=shard_depth, heuristic=heur)
-            return mdist.find_one_distributed(gr, window=args.window, heuristic=heur)
+                return mdist.enumerate_distributed(gr, max_cliques=max_cl, shard_depth=shard_depth, heuristic=heur,
+                                                   orientation=orient)
+            return mdist.find_one_distributed(gr, window=args.window, heuristic=heur, orientation=orient)
         if mode == "enumerate":
-            return gr.enumerate(max_cliques=max_cl, heuristic=heur)
-        return gr.find_one(window=args.window, heuristic=heur)
+            return gr.enumerate(max_cliques=max_cl, heuristic=heur, orientation=orient)
+        return gr.find_one(window=args.window, heuristic=heur, orientation=orient)
 
     for _ in range(args.warmup):
         res = one_step(graph)
@@ -430,9 +448,10 @@ def main():
             torch.cuda.synchronize()
             t0 = time.perf_counter()
             gh = mce.Graph(rp_h, col_h, device=local)
-            r2 = mdist.enumerate_distributed(gh, max_cliques=max_cl, shard_depth=shard_depth, heuristic=heur) if (world > 1 and mode == "enumerate") else (
-                mdist.find_one_distributed(gh, window=args.window, heuristic=heur) if world > 1 else
-                (gh.enumerate(max_cliques=max_cl, heuristic=heur) if mode == "enumerate" else gh.find_one(window=args.window, heuristic=heur)))
+            ok = dict(heuristic=heur, orientation=orient)
+            r2 = mdist.enumerate_distributed(gh, max_cliques=max_cl, shard_depth=shard_depth, **ok) if (world > 1 and mode == "enumerate") else (
+                mdist.find_one_distributed(gh, window=args.window, **ok) if world > 1 else
+                (gh.enumerate(max_cliques=max_cl, **ok) if mode == "enumerate" else gh.find_one(window=args.window, **ok)))
             dt = time.perf_counter() - t0
             gh.close()
             if i >= e2e_warm:
@@ -466,7 +485,7 @@ def main():
             "dtype": "int32",
             "data": "synthetic",
             "config": config_dict(args.config, mode, args.window, g.n, edges, max_cl, world, shard_depth),
-            "details": {"heuristic": heur, "omega": res.omega, "multiplicity": res.count, "stored_cliques": int(res.cliques.shape[0]),
+            "details": {"heuristic": heur, "orientation": orient, "omega": res.omega, "multiplicity": res.count, "stored_cliques": int(res.cliques.shape[0]),
                         "phases_ms": phases, "levels": res.levels, "step_ms": [round(t, 4) for t in times]},
             "verified": verified,
             "paper_context": PAPER_CONTEXT,

@@ -82,13 +82,31 @@ void *dev_alloc(size_t bytes) {
     return p;
 }
 
+// The cache keeps at most a quarter of the device's memory: blocks beyond it
+// go back to the driver at once, so a run that needed a huge frontier does not
+// leave the device full for the rest of the process (other allocators --
+// PyTorch's -- cannot see or reclaim what this cache holds).
+static size_t cache_cap(int dev) {
+    static size_t cap[64] = {0};
+    if (dev >= 0 && dev < 64 && !cap[dev]) {
+        size_t f = 0, t = 0;
+        if (cudaMemGetInfo(&f, &t) == cudaSuccess) cap[dev] = t / 4;
+    }
+    return dev >= 0 && dev < 64 && cap[dev] ? cap[dev] : (size_t)16 << 30;
+}
+
 void dev_free(void *p, size_t bytes) {
     if (!p) return;
     const size_t r = round_size(bytes);
     int dev = 0;
     if (cudaGetDevice(&dev) != cudaSuccess) return;
+    const size_t cap = cache_cap(dev);
     std::lock_guard<std::mutex> lk(g_mu);
     DeviceCache &c = g_cache[dev];
+    if (c.cached + r > cap) {
+        cudaFree(p);
+        return;
+    }
     c.free_blocks.emplace(r, p);
     c.cached += r;
 }

@@ -237,6 +237,7 @@ mce_status mce_preprocess(mce_graph *g, int32_t orientation, int32_t *core_out, 
             fail(MCE_ERR_INVALID, "bad orientation");
         MCE_CUDA(cudaSetDevice(g->device));
         preprocess(g, orientation);
+        if (core_out || degeneracy_out) kcore(g);  // (the degree orientation does not need them)
         auto kind = where == MCE_WHERE_HOST ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice;
         if (core_out && g->n) MCE_CUDA(cudaMemcpy(core_out, g->core.get(), sizeof(int32_t) * g->n, kind));
         if (order_out && g->n) MCE_CUDA(cudaMemcpy(order_out, g->order.get(), sizeof(int32_t) * g->n, kind));

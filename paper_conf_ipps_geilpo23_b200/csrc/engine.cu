@@ -1166,7 +1166,7 @@ mce_result *Engine::run() {
     int heur = o_.heuristic;
     if (find_one_ && heur == 0) heur = 1;  // find-one needs an incumbent clique
     HeuristicResult hr;
-    const bool need_pre = !(g_->have_core && g_->orientation == o_.orientation);
+    const bool need_pre = !preprocessed(g_, o_.orientation);
     if (!o_.no_overlap && need_pre && (heur == MCE_HEUR_SINGLE_DEGREE || heur == MCE_HEUR_MULTI_DEGREE)) {
         // the degree heuristics read only the CSR: run them on a second stream
         // and host thread while the k-core peel and the orientation run here

@@ -61,8 +61,9 @@ namespace mce {
 void kcore(mce_graph *g);
 // rank/order by the requested orientation + oriented CSR with sorted rows
 void orient(mce_graph *g, int orientation);
-// both, cached on the handle
+// both (the k-core only for the degeneracy orientations), cached on the handle
 void preprocess(mce_graph *g, int orientation);
+bool preprocessed(const mce_graph *g, int orientation);
 // device time of the last preprocessing (waits for it if still pending)
 double preprocess_ms(mce_graph *g);
 // orientation from a given order (mce_set_order)

@@ -521,7 +521,7 @@ __global__ void degrees_kernel(int64_t n, const int64_t *__restrict__ rowptr, in
 __global__ void priority_keys_kernel(int64_t n, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ core,
                                      uint64_t span, uint64_t *keys, int32_t *vals) {
     for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
-        keys[v] = (uint64_t)(uint32_t)core[v] * span + (uint64_t)(rowptr[v + 1] - rowptr[v]);
+        keys[v] = (core ? (uint64_t)(uint32_t)core[v] * span : 0ull) + (uint64_t)(rowptr[v + 1] - rowptr[v]);
         vals[v] = (int32_t)v;
     }
 }
@@ -529,19 +529,6 @@ __global__ void priority_keys_kernel(int64_t n, const int64_t *__restrict__ rowp
 __global__ void invert_kernel(int64_t n, const int32_t *__restrict__ order, int32_t *rank) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
         rank[order[i]] = (int32_t)i;
-}
-
-// degree order: counting sort by degree (ties in arbitrary order)
-__global__ void degree_hist(int64_t n, const int64_t *__restrict__ rowptr, int32_t *bins) {
-    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
-        atomicAdd(bins + (rowptr[v + 1] - rowptr[v]), 1);
-}
-__global__ void degree_scatter(int64_t n, const int64_t *__restrict__ rowptr, unsigned long long *cursor,
-                               int32_t *order) {
-    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
-        unsigned long long p = atomicAdd(cursor + (rowptr[v + 1] - rowptr[v]), 1ull);
-        order[p] = (int32_t)v;
-    }
 }
 
 // Tile of G lanes (8 or 32) inside a warp: lane index, first lane, member mask.
@@ -1005,18 +992,14 @@ void orient(mce_graph *g, int orientation) {
         MCE_CUDA(cudaMemcpyAsync(g->order.get(), g->peel.get(), sizeof(int32_t) * n, cudaMemcpyDeviceToDevice, s));
     } else if (orientation == 2) {  // deterministic degeneracy order: (core, shell round, id)
         deterministic_order(g);
-    } else {  // degree order
-        int64_t nb = g->max_deg + 1;
-        int32_t *bins = g->pool.take<int32_t>(nb);
-        int64_t *cursor = g->pool.take<int64_t>(nb + 1), *tmp = g->pool.take<int64_t>(scan_tmp_items(nb));
-        MCE_CUDA(cudaMemsetAsync(bins, 0, sizeof(int32_t) * nb, s));
-        degree_hist<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(), bins);
+    } else {  // degree order, ties by vertex id (a stable radix sort: deterministic, so every rank
+              // of a sharded run orients identically)
+        uint64_t *keys = g->pool.take<uint64_t>(n), *keys_out = g->pool.take<uint64_t>(n);
+        int32_t *vals = g->pool.take<int32_t>(n);
+        priority_keys_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(), nullptr, 0, keys, vals);
         MCE_LAUNCH_CHECK();
-        exclusive_scan_i32(bins, cursor, nb, tmp, s);
-        degree_scatter<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(), (unsigned long long *)cursor,
-                                                         g->order.get());
-        MCE_LAUNCH_CHECK();
-        g->kernels += 5;
+        sort_by_key_stable(keys, keys_out, vals, g->order.get(), n, (uint64_t)g->max_deg + 1, g->pool, s);
+        g->kernels += 4;
     }
     invert_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->order.get(), g->rank.get());
     MCE_LAUNCH_CHECK();
@@ -1108,15 +1091,22 @@ void orient_from(mce_graph *g, int orientation, const int32_t *order, bool on_de
     stream_sync(g->stream);
 }
 
+bool preprocessed(const mce_graph *g, int orientation) {
+    return g->orientation == orientation && (g->have_core || orientation == 1);
+}
+
 void preprocess(mce_graph *g, int orientation) {
-    if (g->have_core && g->orientation == orientation) return;
+    if (preprocessed(g, orientation)) return;
     if (!g->pre_ev[0]) {
         MCE_CUDA(cudaEventCreate(&g->pre_ev[0]));
         MCE_CUDA(cudaEventCreate(&g->pre_ev[1]));
     }
     MCE_CUDA(cudaEventRecord(g->pre_ev[0], g->stream));
     g->kernels = 0;
-    kcore(g);
+    // the degree orientation (PAPER.md IV-C) needs no core numbers: the k-core
+    // peel runs only for the degeneracy orientations (and on demand for the
+    // core-number heuristics, mce_preprocess and the root colour filter)
+    if (orientation != 1) kcore(g);
     orient(g, orientation);
     // no host sync here: the device time is read after the caller's next one
     MCE_CUDA(cudaEventRecord(g->pre_ev[1], g->stream));
