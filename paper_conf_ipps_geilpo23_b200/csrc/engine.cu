@@ -318,6 +318,7 @@ void Engine::leaf_args(ExpandArgs &a) const {
     // (leaves only) does not depend on the bound, and every deeper clique sits
     // under exactly one dealt level-d entry.
     a.shortcut = (o_.no_clique_shortcut || (entry_shard_ && !split_)) ? 0 : 1;
+    a.universal = 1;  // (process() turns it off for levels counted by the lockstep kernel)
     a.clq_total = clq_total_;
     a.clq_slot = clq_slot_;
     a.clq_rows = g_->cstage.get();
@@ -743,6 +744,7 @@ void Engine::process(int32_t k, const Level &L) {
         kernels_ += 5;
         a.perm = perm;
         a.chunk_ctr = chunk_ctr_;
+        a.universal = 0;  // (the lockstep count pass colours every candidate: the write pass must too)
     }
 
     a.chunk_ctr = chunk_ctr_;  // (dynamic work counter of the shared-memory and wide count passes)

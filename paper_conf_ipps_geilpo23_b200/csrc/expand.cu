@@ -446,6 +446,9 @@ __device__ __forceinline__ uint64_t ldrow(const uint64_t *p) {
 
 // SROWS: the root's rows 0 .. 64 W - 1 (first W words each) are staged at
 // srows with stride W (expand_small, every candidate under one root)
+#ifndef UNIVERSAL_RULE
+#define UNIVERSAL_RULE 1  // 0: every candidate coloured and branched as in round 1
+#endif
 #ifndef THREAD_COLOUR_FLAT
 #define THREAD_COLOUR_FLAT 0  // 1: one branch-free loop per class; measured slower (rmat22 chain: 624 vs 348 cycles per coloured vertex)
 #endif
@@ -467,7 +470,71 @@ __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, 
     int maxcls = 0, cls_start = 0;  // largest colour class (a matching complement has classes of at most 2)
     const bool prof = a.dbg && active && e == a.begin;
     long long c0 = prof ? clock64() : 0;
-    if (a.bound == 1) {
+    // Universal vertices (reading 19): u in P adjacent to every other
+    // vertex of P is in every maximal clique below (C, P), so (C + u, P - u) is
+    // the ONLY child needed -- it holds every clique of (C, P), each once -- and
+    // no colouring is needed for it (its bound k + |P| is the trivial one).
+    // When every vertex of P is universal, P is a clique: its colouring is one
+    // class per vertex, written directly (the clique completion then applies).
+    int uni = -1;       // the lowest universal vertex, if P has a non-universal one too
+    bool all_uni = false;
+    if (UNIVERSAL_RULE && a.universal && a.shortcut && a.bound == 1 && active) {
+        int npc = 0, nuni = 0, maxmiss = 0;
+#pragma unroll
+        for (int w = 0; w < W; ++w) npc += __popcll(P[w]);
+        // (only near-cliques -- |P| at most twice what is still needed -- are
+        // scanned: elsewhere universal vertices are rare and the scan is waste)
+        if (npc >= 2 && npc <= 2 * (a.need - a.k)) {
+#pragma unroll
+            for (int w = 0; w < W; ++w) {
+                uint64_t q = P[w];
+                while (q) {
+                    const int b = __ffsll((long long)q) - 1;
+                    q &= q - 1;
+                    const int v = w * 64 + b;
+                    const uint64_t *row = A + (int64_t)v * Wa;
+                    int miss = 0;
+#pragma unroll
+                    for (int x = 0; x < W; ++x)
+                        miss += __popcll(P[x] & ~ldrow<SROWS>(row + x) & ~(x == w ? 1ull << b : 0ull));
+                    maxmiss = max(maxmiss, miss);
+                    if (!miss) {
+                        ++nuni;
+                        if (uni < 0) uni = v;
+                    }
+                }
+            }
+            all_uni = nuni == npc;
+            // P's complement a matching: the colouring path's pair completion
+            // (reading 13) takes every clique at once -- keep that path
+            if (!all_uni && maxmiss <= 1) uni = -1;
+            if (all_uni) {  // P is a clique: one colour class per vertex, ascending
+#pragma unroll
+                for (int w = 0; w < W; ++w) {
+                    uint64_t q = P[w];
+                    while (q) {
+                        const int b = __ffsll((long long)q) - 1;
+                        q &= q - 1;
+                        ord[np] = (uint8_t)(w * 64 + b);
+                        colr[np] = (uint8_t)np;
+                        ++np;
+                    }
+                }
+                ncol = np;
+                maxcls = 1;
+                cls_start = np;
+                uni = -1;
+            } else if (uni >= 0) {  // the single child on u; its bound k + 1 + (|P| - 1)
+                ord[0] = (uint8_t)uni;
+                colr[0] = (uint8_t)(npc - 1);
+                np = 1;
+                ncol = npc;
+                maxcls = 3;  // (no pair completion at this level)
+                cls_start = np;
+            }
+        }
+    }
+    if (a.bound == 1 && !all_uni && uni < 0) {
         uint64_t U[W];
 #pragma unroll
         for (int w = 0; w < W; ++w) U[w] = P[w];
@@ -522,7 +589,7 @@ __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, 
             }
 #endif
         }
-    } else {
+    } else if (a.bound != 1) {
 #pragma unroll
         for (int w = 0; w < W; ++w) {
             uint64_t q = P[w];

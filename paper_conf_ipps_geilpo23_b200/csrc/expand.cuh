@@ -99,6 +99,10 @@ struct ExpandArgs {
     uint16_t *wscratch;
     int64_t wscratch_n;
     long long *dbg;  // diagnostics (expand_small, verbose >= 2): cycles of the first entry's phases
+    // universal-vertex rule (reading 19) in the thread path: the count and
+    // write passes of one level must agree, so it is off when the level's count pass
+    // is the shared-memory lockstep kernel (which does not apply it)
+    int32_t universal;
 };
 
 // Fused root level for W == 1 roots (roots.cu): one warp per root builds the
