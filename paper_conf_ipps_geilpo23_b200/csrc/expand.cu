@@ -446,6 +446,9 @@ __device__ __forceinline__ uint64_t ldrow(const uint64_t *p) {
 
 // SROWS: the root's rows 0 .. 64 W - 1 (first W words each) are staged at
 // srows with stride W (expand_small, every candidate under one root)
+constexpr int kUniCompute = -3;  // expand_entry's universal-vertex hint: compute it
+constexpr int kUniAll = -2;      // P is a clique
+constexpr int kUniNone = -1;     // colour as usual
 #ifndef UNIVERSAL_RULE
 #define UNIVERSAL_RULE 1  // 0: every candidate coloured and branched as in round 1
 #endif
@@ -455,7 +458,8 @@ __device__ __forceinline__ uint64_t ldrow(const uint64_t *p) {
 template <int W, bool WRITE, bool SROWS = false>
 __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, int64_t out, unsigned &nleaf,
                                                 unsigned long long &nclq, int &hb, int &ub, bool active = true,
-                                                bool fused = false, const uint64_t *srows = nullptr) {
+                                                bool fused = false, const uint64_t *srows = nullptr,
+                                                int uhint = kUniCompute) {
     uint64_t P[W];
 #pragma unroll
     for (int w = 0; w < W; ++w) P[w] = active ? a.P[e * a.Ps + w] : 0ull;
@@ -478,7 +482,38 @@ __device__ __forceinline__ int32_t expand_entry(const ExpandArgs &a, int64_t e, 
     // class per vertex, written directly (the clique completion then applies).
     int uni = -1;       // the lowest universal vertex, if P has a non-universal one too
     bool all_uni = false;
-    if (UNIVERSAL_RULE && a.universal && a.shortcut && a.bound == 1 && active) {
+    if (uhint != kUniCompute && active) {  // decided cooperatively by expand_small (same rule)
+        uni = uhint >= 0 ? uhint : -1;
+        all_uni = uhint == kUniAll;
+        if (all_uni || uni >= 0) {
+            int npc = 0;
+#pragma unroll
+            for (int w = 0; w < W; ++w) npc += __popcll(P[w]);
+            if (all_uni) {
+#pragma unroll
+                for (int w = 0; w < W; ++w) {
+                    uint64_t q = P[w];
+                    while (q) {
+                        const int b = __ffsll((long long)q) - 1;
+                        q &= q - 1;
+                        ord[np] = (uint8_t)(w * 64 + b);
+                        colr[np] = (uint8_t)np;
+                        ++np;
+                    }
+                }
+                ncol = np;
+                maxcls = 1;
+                cls_start = np;
+            } else {
+                ord[0] = (uint8_t)uni;
+                colr[0] = (uint8_t)(npc - 1);
+                np = 1;
+                ncol = npc;
+                maxcls = 3;
+                cls_start = np;
+            }
+        }
+    } else if (UNIVERSAL_RULE && a.universal && a.shortcut && a.bound == 1 && active) {
         int npc = 0, nuni = 0, maxmiss = 0;
 #pragma unroll
         for (int w = 0; w < W; ++w) npc += __popcll(P[w]);
@@ -749,17 +784,18 @@ __global__ void __launch_bounds__(256) expand_thread(const ExpandArgs a) {
 // ---------------------------------------------------------------------------
 constexpr int kSmallThreads = 512;  // (1024 capped the colouring loop at 64 registers: Q/U spilled, ~360 cycles a step)
 constexpr int kSmallPer = kSmallMax / kSmallThreads;  // candidates per thread
+constexpr int kSmallCoop = 16;  // levels of at most this many candidates take the block's universal-vertex scan
 constexpr int kSmallRoots = 4;  // roots whose rows expand_small stages in shared memory (8 KB each)
 
 template <bool WRITE>
 __device__ __forceinline__ int32_t expand_entry_w(int W, const ExpandArgs &a, int64_t e, int64_t out,
                                                   unsigned &nleaf, unsigned long long &nclq, int &hb, int &ub,
                                                   bool active = true, bool fused = false,
-                                                  const uint64_t *srows = nullptr) {
+                                                  const uint64_t *srows = nullptr, int uhint = kUniCompute) {
     if (srows) {
-        if (W == 1) return expand_entry<1, WRITE, true>(a, e, out, nleaf, nclq, hb, ub, active, fused, srows);
-        if (W == 2) return expand_entry<2, WRITE, true>(a, e, out, nleaf, nclq, hb, ub, active, fused, srows);
-        return expand_entry<4, WRITE, true>(a, e, out, nleaf, nclq, hb, ub, active, fused, srows);
+        if (W == 1) return expand_entry<1, WRITE, true>(a, e, out, nleaf, nclq, hb, ub, active, fused, srows, uhint);
+        if (W == 2) return expand_entry<2, WRITE, true>(a, e, out, nleaf, nclq, hb, ub, active, fused, srows, uhint);
+        return expand_entry<4, WRITE, true>(a, e, out, nleaf, nclq, hb, ub, active, fused, srows, uhint);
     }
     if (W == 1) return expand_entry<1, WRITE>(a, e, out, nleaf, nclq, hb, ub, active, fused);
     if (W == 2) return expand_entry<2, WRITE>(a, e, out, nleaf, nclq, hb, ub, active, fused);
@@ -776,6 +812,7 @@ __global__ void __launch_bounds__(kSmallThreads, 1) expand_small(const ExpandArg
     __shared__ int s_hb, s_ub;
     __shared__ int64_t s_used;
     __shared__ int s_slots[kSmallRoots], s_over;
+    __shared__ int s_umin, s_unum, s_umiss, s_uhint[kSmallCoop];
     __shared__ uint64_t s_rows[kSmallRoots][256 * 4];  // per root: rows 0 .. 64 W - 1, W words each (W <= 4)
     const int t = threadIdx.x;
     if (t == 0) {
@@ -881,6 +918,59 @@ __global__ void __launch_bounds__(kSmallThreads, 1) expand_small(const ExpandArg
             }
         }
         __syncthreads();
+        // levels of a few candidates (the deep chains): the universal-vertex scan
+        // of each candidate by the whole block, one vertex per thread (a single
+        // thread's scan is a chain of dependent instructions, ~200 cycles per
+        // vertex); the entries then take the decision as a hint (same rule)
+        const bool coop = UNIVERSAL_RULE && staged && N <= kSmallCoop && A.universal && A.shortcut && A.bound == 1;
+        if (coop) {
+            for (int c = 0; c < N; ++c) {
+                const int64_t ec = A.begin + c;
+                int cj = 0;  // the staged root of candidate c
+                const int32_t slc = A.slot[ec];
+                for (int j = 0; j < kSmallRoots; ++j)
+                    if (s_slots[j] == slc) cj = j;
+                if (t == 0) {
+                    s_umin = INT32_MAX;
+                    s_unum = 0;
+                    s_umiss = 0;
+                }
+                __syncthreads();
+                int npc = 0;
+                uint64_t Pc[4] = {0, 0, 0, 0};
+#pragma unroll
+                for (int w = 0; w < 4; ++w)
+                    if (w < W) {
+                        Pc[w] = A.P[ec * A.Ps + w];
+                        npc += __popcll(Pc[w]);
+                    }
+                const bool scan = npc >= 2 && npc <= 2 * (A.need - A.k);
+                if (scan && t < 64 * W && ((Pc[t >> 6] >> (t & 63)) & 1ull)) {
+                    const uint64_t *row = s_rows[cj] + (int64_t)t * W;
+                    int miss = 0;
+#pragma unroll
+                    for (int x = 0; x < 4; ++x)
+                        if (x < W) miss += __popcll(Pc[x] & ~row[x] & ~(x == (t >> 6) ? 1ull << (t & 63) : 0ull));
+                    atomicMax(&s_umiss, miss);
+                    if (!miss) {
+                        atomicAdd(&s_unum, 1);
+                        atomicMin(&s_umin, t);
+                    }
+                }
+                __syncthreads();
+                if (t == 0) {
+                    int h = kUniNone;
+                    if (scan) {
+                        if (s_unum == npc)
+                            h = kUniAll;
+                        else if (s_unum > 0 && s_umiss > 1)
+                            h = s_umin;
+                    }
+                    s_uhint[c] = h;
+                }
+                __syncthreads();
+            }
+        }
         phase(1);
         unsigned nleaf = 0;
         unsigned long long nclq = 0;
@@ -890,7 +980,8 @@ __global__ void __launch_bounds__(kSmallThreads, 1) expand_small(const ExpandArg
             if (r * kSmallThreads >= N) break;  // (block-uniform)
             const int idx = t + r * kSmallThreads;
             expand_entry_w<false>(W, A, A.begin + idx, 0, nleaf, nclq, hb, ub, idx < N, true,
-                                  staged ? s_rows[max(mys[r], 0)] : nullptr);  // block-uniform path
+                                  staged ? s_rows[max(mys[r], 0)] : nullptr,  // block-uniform path
+                                  coop && idx < N ? s_uhint[idx] : kUniCompute);
         }
         phase(2);  // (thread 0's own entries)
         if (nleaf) atomicAdd(&s_leaf, nleaf);
