@@ -32,6 +32,7 @@ struct mce_graph {
     bool pre_pending = false;
     bool pre_overlapped = false;   // set by the engine while the heuristic runs concurrently
     bool order_given = false;      // g->order was set by mce_set_order: orient() keeps it
+    bool pre_started = false;      // pre_ev[0] already recorded (the engine ran kcore before preprocess)
     int64_t kernels = 0;           // kernels launched by the last preprocessing
 
     // ---- reusable memory (no cudaMalloc/cudaFree on the steady-state path) ----

@@ -91,8 +91,9 @@ __device__ __forceinline__ int32_t ld_best(const int32_t *best) {
 #ifndef HEUR_FILTER
 #define HEUR_FILTER 1
 #endif
-__device__ __forceinline__ bool useful(const int32_t *__restrict__ thr, int32_t x, int32_t b) {
-    return !HEUR_FILTER || b <= 1 || __ldg(thr + x) + 1 >= b;
+__device__ __forceinline__ bool useful(const int32_t *__restrict__ thr, int32_t x, int32_t b,
+                                       const int32_t *__restrict__ core = nullptr) {
+    return !HEUR_FILTER || b <= 1 || (__ldg(thr + x) + 1 >= b && (!core || __ldg(core + x) + 1 >= b));
 }
 
 // Hub bit matrix (exact acceleration of the runs on power-law graphs).  H =
@@ -213,7 +214,7 @@ __device__ __forceinline__ bool adjacent_h(const Hub &H, int hw, const int64_t *
 template <int G>
 __device__ int32_t greedy_run(int32_t s, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
                               const int32_t *__restrict__ thr, int32_t *__restrict__ scratch, const int32_t *best,
-                              const Hub &H) {
+                              const Hub &H, const int32_t *__restrict__ fcore = nullptr) {
     const int lane = threadIdx.x & 31;
     const int gl = lane & (G - 1);
     const int gbase = lane & ~(G - 1);
@@ -250,7 +251,7 @@ __device__ int32_t greedy_run(int32_t s, const int64_t *__restrict__ rowptr, con
             int64_t i = i0 + gl;
             int32_t x = i < len ? src[i] : -1;
             bool xh = true;
-            bool keep = i < len && x != w && useful(thr, x, b) && adjacent_h(H, hw, rowptr, col, x, w, wb, we, xh);
+            bool keep = i < len && x != w && useful(thr, x, b, fcore) && adjacent_h(H, hw, rowptr, col, x, w, wb, we, xh);
             const unsigned m = (__ballot_sync(gmask, keep) & gmask) >> gbase;
             if (keep) buf[out + __popc(m & ((1u << gl) - 1u))] = x;
             out += __popc(m);
@@ -276,7 +277,7 @@ constexpr int64_t kBigSeed = 1024;
 template <int NT>
 __device__ int32_t block_run(int32_t s, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
                              const int32_t *__restrict__ thr, int32_t *__restrict__ scratch, int32_t *clique,
-                             const int32_t *best, const Hub &H) {
+                             const int32_t *best, const Hub &H, const int32_t *__restrict__ fcore = nullptr) {
     __shared__ unsigned long long wkey[NT / 32];
     __shared__ int32_t wcnt[NT / 32], wnon[NT / 32];
     __shared__ int32_t sbest, sres;
@@ -321,7 +322,7 @@ __device__ int32_t block_run(int32_t s, const int64_t *__restrict__ rowptr, cons
             const int64_t i = i0 + threadIdx.x;
             const int32_t x = i < len ? src[i] : -1;
             bool xh = true;
-            const bool keep = i < len && x != w && useful(thr, x, b) && adjacent_h(H, hw, rowptr, col, x, w, wb, we, xh);
+            const bool keep = i < len && x != w && useful(thr, x, b, fcore) && adjacent_h(H, hw, rowptr, col, x, w, wb, we, xh);
             const unsigned m = __ballot_sync(0xffffffffu, keep);
             const unsigned nh = H.K ? __ballot_sync(0xffffffffu, keep && !xh) : 0u;
             __syncthreads();  // wkey/wcnt reuse, and every read of this chunk precedes its writes
@@ -380,7 +381,8 @@ __global__ void __launch_bounds__(kBlockRun) greedy_big_kernel(int64_t nbig, con
         const int32_t s = big[i];
         int32_t c = 1;
         if (!abort_runs || seed_cap(s, rowptr, core) >= ld_best(best_size))
-            c = block_run<kBlockRun>(s, rowptr, col, thr, scratch, nullptr, abort_runs ? best_size : nullptr, H);
+            c = block_run<kBlockRun>(s, rowptr, col, thr, scratch, nullptr, abort_runs ? best_size : nullptr, H,
+                                     abort_runs ? core : nullptr);
         if (threadIdx.x == 0) {
             run_size[s] = c;
             atomicMax(best_size, c);
@@ -421,7 +423,7 @@ __global__ void __launch_bounds__(256) greedy_kernel(int64_t nseeds, const int32
         if (!__ballot_sync(0xffffffffu, s_mine >= 0)) continue;
         if (__all_sync(0xffffffffu, d_mine <= 64)) {
             if (s_mine >= 0) {
-                const int32_t c = greedy_run<8>(s_mine, rowptr, col, thr, scratch, best, none);
+                const int32_t c = greedy_run<8>(s_mine, rowptr, col, thr, scratch, best, none, best ? core : nullptr);
                 if ((lane & 7) == 0) run_size[s_mine] = c;
                 mybest = c;
             }
@@ -429,7 +431,7 @@ __global__ void __launch_bounds__(256) greedy_kernel(int64_t nseeds, const int32
             for (int t = 0; t < 4; ++t) {
                 const int32_t s = __shfl_sync(0xffffffffu, s_mine, 8 * t);
                 if (s < 0) continue;
-                const int32_t c = greedy_run<32>(s, rowptr, col, thr, scratch, best, H);
+                const int32_t c = greedy_run<32>(s, rowptr, col, thr, scratch, best, H, best ? core : nullptr);
                 if (lane == 0) run_size[s] = c;
                 mybest = max(mybest, c);
             }
@@ -476,6 +478,7 @@ __global__ void best_seed_kernel(int64_t nseeds, const int32_t *__restrict__ see
 // Replay of the winning run to recover its clique (one block, nothing else running)
 constexpr int kReplay = 1024;
 __global__ void __launch_bounds__(kReplay) replay_kernel(const unsigned long long *best_key, const int32_t *best,
+                                                         const int32_t *__restrict__ core,
                                                          const int64_t *__restrict__ rowptr,
                                                          const int32_t *__restrict__ col,
                                                          const int32_t *__restrict__ thr,
@@ -483,7 +486,7 @@ __global__ void __launch_bounds__(kReplay) replay_kernel(const unsigned long lon
     const int32_t s = (int32_t)(0x7fffffffu - (uint32_t)(*best_key & 0xffffffffull));
     // the winning run reaches *best, so the filter (and the abort) against it
     // leaves its picks unchanged (see useful())
-    block_run<kReplay>(s, rowptr, col, thr, scratch, clique, best, H);
+    block_run<kReplay>(s, rowptr, col, thr, scratch, clique, best, H, core);
 }
 
 __global__ void degree_thr_kernel(int64_t n, const int64_t *__restrict__ rowptr, int32_t *thr) {
@@ -609,7 +612,7 @@ __global__ void __launch_bounds__(256) hub_matrix_kernel(int K, int KW, const in
 }  // namespace
 
 HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_rank, int32_t shard_count,
-                              bool want_runs, bool concurrent) {
+                              bool want_runs, bool concurrent, bool with_core) {
     HeuristicResult res;
     const int64_t n = g->n;
     cudaStream_t s = concurrent ? g->hstream : g->stream;
@@ -702,7 +705,7 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
     MCE_CUDA(cudaMemsetAsync(run_size, 0, sizeof(int32_t) * n, s));
     MCE_CUDA(cudaMemsetAsync(best, 0, sizeof(int32_t), s));
     MCE_CUDA(cudaMemsetAsync(best_key, 0, sizeof(unsigned long long), s));
-    const int32_t *core = (!concurrent && g->have_core) ? g->core.get() : nullptr;
+    const int32_t *core = ((!concurrent || with_core) && g->have_core) ? g->core.get() : nullptr;
     const int abort_runs = want_runs ? 0 : 1;
     Hub H;
     int64_t nbig = 0;
@@ -804,7 +807,10 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
         MCE_LAUNCH_CHECK();
         best_seed_kernel<<<grid_for(nseeds, 256), 256, 0, s>>>(nseeds, seed_ptr, thr, run_size, best, best_key);
         MCE_LAUNCH_CHECK();
-        replay_kernel<<<1, kReplay, 0, s>>>(best_key, best, g->rowptr.get(), g->col.get(), thr, scratch, clique, H);
+        // (the winning run never picks a vertex of core + 1 < best: the same
+        // filter leaves its picks unchanged, reading 15)
+        replay_kernel<<<1, kReplay, 0, s>>>(best_key, best, abort_runs ? core : nullptr, g->rowptr.get(),
+                                            g->col.get(), thr, scratch, clique, H);
         MCE_LAUNCH_CHECK();
         kernels += 3;
     }

@@ -12,8 +12,10 @@ struct HeuristicResult {
     int64_t kernels = 0;
 };
 // kind: MCE_HEUR_*; h <= 0 means |V|; runs sharded cyclically when shard_count > 1
-// concurrent: run on g->hstream / g->hpool / g->hhost without core numbers
-// (overlapped with preprocessing by the engine; degree kinds only)
+// concurrent: run on g->hstream / g->hpool / g->hhost (overlapped with
+// preprocessing by the engine; degree kinds only); with_core: the core numbers
+// are on the device (stream-ordered before the heuristic) and prune seeds and
+// candidates (core + 1 < best)
 HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_rank, int32_t shard_count,
-                              bool want_runs, bool concurrent = false);
+                              bool want_runs, bool concurrent = false, bool with_core = false);
 }  // namespace mce

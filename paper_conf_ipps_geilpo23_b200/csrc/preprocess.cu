@@ -1101,7 +1101,8 @@ void preprocess(mce_graph *g, int orientation) {
         MCE_CUDA(cudaEventCreate(&g->pre_ev[0]));
         MCE_CUDA(cudaEventCreate(&g->pre_ev[1]));
     }
-    MCE_CUDA(cudaEventRecord(g->pre_ev[0], g->stream));
+    if (!g->pre_started) MCE_CUDA(cudaEventRecord(g->pre_ev[0], g->stream));  // (else the caller's, before its kcore)
+    g->pre_started = false;
     g->kernels = 0;
     // the degree orientation (PAPER.md IV-C) needs no core numbers: the k-core
     // peel runs only for the degeneracy orientations (and on demand for the
