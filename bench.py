@@ -44,8 +44,9 @@ def parse():
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
     p.add_argument("--mode", default=None, choices=[None, "enumerate", "find_one"])
     p.add_argument("--window", type=int, default=-1,
-                   help="find-one roots per window (PAPER.md IV-E); -1: 64 for dense800 (the best of the "
-                        "window sweep, profiles/r01_window_sweep_dense800_*.json), else 0 = all roots")
+                   help="find-one roots per window (PAPER.md IV-E); -1: 96 for dense800 (the best of the "
+                        "window sweep under the degree orientation, profiles/r02_window_sweep_dense800_v2.md), "
+                        "else 0 = all roots")
     p.add_argument("--max-cliques", type=int, default=-1,
                    help="stored-clique capacity (multiplicity stays exact); -1: 2^16 for the R-MAT configs "
                         "(~10^8 maximum cliques of size ~223 there), unbounded otherwise")
@@ -258,7 +259,7 @@ ORIENTATION = {"er2000": "degree", "ba1m": "degeneracy", "rmat22": "degeneracy",
 def bench_defaults(args):
     mode = args.mode or ("find_one" if args.config == "dense800" else "enumerate")
     shard_depth = args.shard_depth if args.shard_depth >= 0 else (3 if args.config == "rmat26" else 0)
-    window = args.window if args.window >= 0 else (64 if args.config == "dense800" else 0)
+    window = args.window if args.window >= 0 else (96 if args.config == "dense800" else 0)
     max_cl = args.max_cliques if args.max_cliques >= 0 else (1 << 16 if args.config.startswith("rmat") else 0)
     if args.heuristic == "auto":
         args.heuristic = HEURISTIC[args.config]
