@@ -550,12 +550,20 @@ struct Tile {
 // the start of v's own undirected row in `stage` (rowptr-indexed), their
 // number at odeg[pid[v]]; orient_copy moves them to the oriented CSR once the
 // out-degrees are scanned (one gather pass over rank/pid instead of two)
+// (rank, CSR id) of a vertex in one 8-byte word: the stage pass gathers both
+// with one load per neighbour (one sector instead of two)
+__global__ void pack_rank_pid_kernel(int64_t n, const int32_t *__restrict__ rank, const int32_t *__restrict__ pid,
+                                     int2 *rp) {
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+        rp[v] = make_int2(rank[v], pid[v]);
+}
+
 template <int G, int KL>
 __device__ void stage_one(int64_t v, const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
-                          const int32_t *__restrict__ rank, const int32_t *__restrict__ pid, int32_t *odeg,
-                          int32_t *stage) {
+                          const int2 *__restrict__ rp, int32_t *odeg, int32_t *stage) {
     Tile<G> t;
-    const int32_t r = rank[v];
+    const int2 rv = rp[v];
+    const int32_t r = rv.x;
     const int64_t eb = rowptr[v], ee = rowptr[v + 1];
     int64_t out = eb;
     // whole warps (long rows): KL chunks' ids and ranks gathered before any
@@ -563,30 +571,30 @@ __device__ void stage_one(int64_t v, const int64_t *__restrict__ rowptr, const i
     constexpr int K = G == 32 ? KL : 1;
     for (int64_t e0 = eb; e0 < ee; e0 += G * K) {
         int32_t u[K];
-        bool up[K];
+        int2 x[K];
 #pragma unroll
         for (int k = 0; k < K; ++k) {
             const int64_t e = e0 + G * k + t.gl;
-            u[k] = e < ee ? col[e] : 0;
+            u[k] = e < ee ? col[e] : -1;
         }
 #pragma unroll
-        for (int k = 0; k < K; ++k) up[k] = e0 + G * k + t.gl < ee && rank[u[k]] > r;
+        for (int k = 0; k < K; ++k) x[k] = u[k] >= 0 ? __ldg(rp + u[k]) : make_int2(INT32_MIN, 0);
 #pragma unroll
         for (int k = 0; k < K; ++k) {
-            const unsigned m = t.ballot(up[k]);
-            if (up[k]) stage[out + __popc(m & t.lt())] = pid[u[k]];
+            const bool up = x[k].x > r;
+            const unsigned m = t.ballot(up);
+            if (up) stage[out + __popc(m & t.lt())] = x[k].y;
             out += __popc(m);
         }
     }
-    if (t.gl == 0) odeg[pid[v]] = (int32_t)(out - eb);
+    if (t.gl == 0) odeg[rv.y] = (int32_t)(out - eb);
 }
 
 // Warp w takes vertices [4w, 4w+4): 8-lane tiles when all four have degree <= 64, else a warp each
 template <int KL>
 __global__ void __launch_bounds__(256) orient_stage_kernel(int64_t n, const int64_t *__restrict__ rowptr,
                                                            const int32_t *__restrict__ col,
-                                                           const int32_t *__restrict__ rank,
-                                                           const int32_t *__restrict__ pid, int32_t *odeg,
+                                                           const int2 *__restrict__ rp, int32_t *odeg,
                                                            int32_t *stage) {
     const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -595,9 +603,9 @@ __global__ void __launch_bounds__(256) orient_stage_kernel(int64_t n, const int6
         const int64_t v = v0 + (lane >> 3);
         const int64_t d = v < n ? rowptr[v + 1] - rowptr[v] : 0;
         if (__all_sync(0xffffffffu, d <= 64)) {
-            if (v < n) stage_one<8, 1>(v, rowptr, col, rank, pid, odeg, stage);
+            if (v < n) stage_one<8, 1>(v, rowptr, col, rp, odeg, stage);
         } else {
-            for (int t = 0; t < 4 && v0 + t < n; ++t) stage_one<32, KL>(v0 + t, rowptr, col, rank, pid, odeg, stage);
+            for (int t = 0; t < 4 && v0 + t < n; ++t) stage_one<32, KL>(v0 + t, rowptr, col, rp, odeg, stage);
         }
         __syncwarp();
     }
@@ -714,8 +722,11 @@ __global__ void sort_rows_block(const int64_t *__restrict__ orp, int32_t *ocol, 
 }
 
 // rows longer than a warp (sorted by one block each) and the largest out-degree
-__global__ void long_rows_kernel(int64_t n, const int64_t *__restrict__ orp, int32_t *rows, int32_t *count,
-                                 int32_t *max_out) {
+// rows by length class: (32, 256] -> mid (a warp each, in registers), (256,
+// 8192] -> big (a block each, shared memory), longer -> huge (one block,
+// global scratch); meta = counts [mid, big, huge], then the largest out-degree
+__global__ void long_rows_kernel(int64_t n, const int64_t *__restrict__ orp, int32_t *mid, int32_t *big,
+                                 int32_t *huge, int32_t *meta) {
     const int lane = threadIdx.x & 31;
     int32_t mx = 0;
     for (int64_t r0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) & ~31ll; r0 < n;
@@ -723,14 +734,73 @@ __global__ void long_rows_kernel(int64_t n, const int64_t *__restrict__ orp, int
         const int64_t r = r0 + lane;
         const int32_t len = r < n ? (int32_t)(orp[r + 1] - orp[r]) : 0;
         mx = max(mx, len);
-        const unsigned m = __ballot_sync(0xffffffffu, len > 32);
-        int32_t b = 0;
-        if (lane == 0 && m) b = atomicAdd(count, __popc(m));
-        b = __shfl_sync(0xffffffffu, b, 0);
-        if (len > 32) rows[b + __popc(m & lanemask_lt())] = (int32_t)r;
+        const int cls = len <= 32 ? -1 : (len <= 256 ? 0 : (len <= 8192 ? 1 : 2));
+#pragma unroll
+        for (int c = 0; c < 3; ++c) {
+            const unsigned m = __ballot_sync(0xffffffffu, cls == c);
+            int32_t b = 0;
+            if (lane == 0 && m) b = atomicAdd(meta + c, __popc(m));
+            b = __shfl_sync(0xffffffffu, b, 0);
+            int32_t *dst = c == 0 ? mid : (c == 1 ? big : huge);
+            if (cls == c) dst[b + __popc(m & lanemask_lt())] = (int32_t)r;
+        }
     }
     mx = __reduce_max_sync(0xffffffffu, mx);
-    if (lane == 0 && mx) atomicMax(max_out, mx);
+    if (lane == 0 && mx) atomicMax(meta + 3, mx);
+}
+
+// rows of (32, 32 E] ids by one warp each, E per lane in registers ("blocked":
+// lane l holds positions l E .. l E + E - 1): a bitonic network whose strides
+// below E stay inside a lane and the rest are lane shuffles -- no barrier
+// (a 256-thread block per row with a barrier per stage was 3.3 ms on rmat22)
+template <int E>
+__global__ void __launch_bounds__(256) sort_rows_mid(const int64_t *__restrict__ orp, int32_t *ocol,
+                                                      const int32_t *__restrict__ rows, int32_t nrows) {
+    const int lane = threadIdx.x & 31;
+    const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t ri = warp; ri < nrows; ri += nwarps) {
+        const int32_t r = rows[ri];
+        const int64_t b = orp[r];
+        const int len = (int)(orp[r + 1] - b);
+        int32_t x[E];
+#pragma unroll
+        for (int j = 0; j < E; ++j) {
+            const int i = lane * E + j;
+            x[j] = i < len ? ocol[b + i] : INT32_MAX;
+        }
+#pragma unroll
+        for (int size = 2; size <= 32 * E; size <<= 1) {
+#pragma unroll
+            for (int stride = size >> 1; stride > 0; stride >>= 1) {
+                if (stride >= E) {
+#pragma unroll
+                    for (int j = 0; j < E; ++j) {
+                        const int i = lane * E + j;
+                        const int32_t y = __shfl_xor_sync(0xffffffffu, x[j], stride / E);
+                        const bool up = (i & size) == 0, lower = (i & stride) == 0;
+                        x[j] = (lower == up) ? min(x[j], y) : max(x[j], y);
+                    }
+                } else {
+#pragma unroll
+                    for (int j = 0; j < E; ++j) {
+                        const int p = j ^ stride;
+                        if (p > j) {
+                            const bool up = ((lane * E + j) & size) == 0;
+                            const int32_t a = x[j], c = x[p];
+                            x[j] = up ? min(a, c) : max(a, c);
+                            x[p] = up ? max(a, c) : min(a, c);
+                        }
+                    }
+                }
+            }
+        }
+#pragma unroll
+        for (int j = 0; j < E; ++j) {
+            const int i = lane * E + j;
+            if (i < len) ocol[b + i] = x[j];
+        }
+    }
 }
 
 // ---------------------------------------------------------------------------
@@ -1035,12 +1105,14 @@ void orient(mce_graph *g, int orientation) {
     // are rare (mean degree <= 16: ba1m preprocessing 1.27 -> 1.17 ms); with
     // many (rmat22, mean 31) the wider gathers slow the greedy heuristic that
     // runs beside this pass more than they gain (step 82.6 -> 88-93 ms)
+    int2 *rp2 = g->pool.take<int2>(n);
+    pack_rank_pid_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->rank.get(), g->pid.get(), rp2);
+    MCE_LAUNCH_CHECK();
     if (g->nnz <= 16 * n)
-        orient_stage_kernel<ORIENT_KL><<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), g->rank.get(),
-                                                              g->pid.get(), odeg, stage);
+        orient_stage_kernel<ORIENT_KL><<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), rp2, odeg,
+                                                                           stage);
     else
-        orient_stage_kernel<1><<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), g->rank.get(),
-                                                              g->pid.get(), odeg, stage);
+        orient_stage_kernel<1><<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), rp2, odeg, stage);
     MCE_LAUNCH_CHECK();
     exclusive_scan_i32(odeg, g->orp.get(), n, g->pool.take<int64_t>(scan_tmp_items(n)), s);
     orient_copy_kernel<<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->vid.get(), g->orp.get(), stage,
@@ -1048,30 +1120,36 @@ void orient(mce_graph *g, int orientation) {
     MCE_LAUNCH_CHECK();
     sort_rows_warp<<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->orp.get(), g->ocol.get());
     MCE_LAUNCH_CHECK();
-    int32_t *rows = g->pool.take<int32_t>(n), *meta = g->pool.take<int32_t>(2);
-    MCE_CUDA(cudaMemsetAsync(meta, 0, 2 * sizeof(int32_t), s));
-    long_rows_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->orp.get(), rows, meta, meta + 1);
+    int32_t *rmid = g->pool.take<int32_t>(n), *rbig = g->pool.take<int32_t>(n), *rhuge = g->pool.take<int32_t>(n);
+    int32_t *meta = g->pool.take<int32_t>(4);
+    MCE_CUDA(cudaMemsetAsync(meta, 0, 4 * sizeof(int32_t), s));
+    long_rows_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->orp.get(), rmid, rbig, rhuge, meta);
     MCE_LAUNCH_CHECK();
-    int32_t *hmeta = g->host.get<int32_t>(2);
-    MCE_CUDA(cudaMemcpyAsync(hmeta, meta, 2 * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+    int32_t *hmeta = g->host.get<int32_t>(4);
+    MCE_CUDA(cudaMemcpyAsync(hmeta, meta, 4 * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
     stream_sync(s);
     g->kernels += 8;
-    g->max_out = hmeta[1];
-    const int32_t n_long = hmeta[0];
-    if (n_long > 0) {
-        const int32_t smem_cap = 8192;  // ints (32 KB)
+    g->max_out = hmeta[3];
+    const int32_t n_mid = hmeta[0], n_big = hmeta[1], n_huge = hmeta[2];
+    const int32_t smem_cap = 8192;  // ints (32 KB)
+    if (n_mid > 0) {
+        sort_rows_mid<8><<<grid_for((int64_t)n_mid * 32, 256), 256, 0, s>>>(g->orp.get(), g->ocol.get(), rmid, n_mid);
+        MCE_LAUNCH_CHECK();
+        g->kernels += 1;
+    }
+    if (n_big > 0) {
+        sort_rows_block<<<grid_for(n_big, 1, 16), 256, smem_cap * sizeof(int32_t), s>>>(
+            g->orp.get(), g->ocol.get(), rbig, n_big, nullptr, smem_cap);
+        MCE_LAUNCH_CHECK();
+        g->kernels += 1;
+    }
+    if (n_huge > 0) {  // rows beyond shared memory: one block, global scratch
         int32_t p2 = 1;
         while (p2 < g->max_out) p2 <<= 1;
-        if (p2 <= smem_cap) {
-            sort_rows_block<<<grid_for(n_long, 1, 16), 256, smem_cap * sizeof(int32_t), s>>>(
-                g->orp.get(), g->ocol.get(), rows, n_long, nullptr, smem_cap);
-            MCE_LAUNCH_CHECK();
-        } else {  // some row exceeds shared memory: one block, global scratch
-            int32_t *scratch = g->pool.take<int32_t>(p2);
-            sort_rows_block<<<1, 1024, smem_cap * sizeof(int32_t), s>>>(g->orp.get(), g->ocol.get(), rows, n_long,
-                                                                        scratch, smem_cap);
-            MCE_LAUNCH_CHECK();
-        }
+        int32_t *scratch = g->pool.take<int32_t>(p2);
+        sort_rows_block<<<1, 1024, smem_cap * sizeof(int32_t), s>>>(g->orp.get(), g->ocol.get(), rhuge, n_huge,
+                                                                    scratch, smem_cap);
+        MCE_LAUNCH_CHECK();
         g->kernels += 1;
     }
     g->orientation = orientation;  // (stream-ordered: no sync needed before the consumers)
