@@ -722,11 +722,12 @@ __global__ void sort_rows_block(const int64_t *__restrict__ orp, int32_t *ocol, 
 }
 
 // rows longer than a warp (sorted by one block each) and the largest out-degree
-// rows by length class: (32, 256] -> mid (a warp each, in registers), (256,
-// 8192] -> big (a block each, shared memory), longer -> huge (one block,
-// global scratch); meta = counts [mid, big, huge], then the largest out-degree
+// rows by length class: (32, 256] -> mid and (256, 1024] -> wide (a warp each,
+// in registers), (1024, 8192] -> big (a block each, shared memory), longer ->
+// huge (one block, global scratch); meta = counts [mid, big, huge], the largest
+// out-degree, count [wide]
 __global__ void long_rows_kernel(int64_t n, const int64_t *__restrict__ orp, int32_t *mid, int32_t *big,
-                                 int32_t *huge, int32_t *meta) {
+                                 int32_t *huge, int32_t *wide, int32_t *meta) {
     const int lane = threadIdx.x & 31;
     int32_t mx = 0;
     for (int64_t r0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) & ~31ll; r0 < n;
@@ -734,14 +735,14 @@ __global__ void long_rows_kernel(int64_t n, const int64_t *__restrict__ orp, int
         const int64_t r = r0 + lane;
         const int32_t len = r < n ? (int32_t)(orp[r + 1] - orp[r]) : 0;
         mx = max(mx, len);
-        const int cls = len <= 32 ? -1 : (len <= 256 ? 0 : (len <= 8192 ? 1 : 2));
+        const int cls = len <= 32 ? -1 : (len <= 256 ? 0 : (len <= 1024 ? 3 : (len <= 8192 ? 1 : 2)));
 #pragma unroll
-        for (int c = 0; c < 3; ++c) {
+        for (int c = 0; c < 4; ++c) {
             const unsigned m = __ballot_sync(0xffffffffu, cls == c);
             int32_t b = 0;
-            if (lane == 0 && m) b = atomicAdd(meta + c, __popc(m));
+            if (lane == 0 && m) b = atomicAdd(meta + (c == 3 ? 4 : c), __popc(m));
             b = __shfl_sync(0xffffffffu, b, 0);
-            int32_t *dst = c == 0 ? mid : (c == 1 ? big : huge);
+            int32_t *dst = c == 0 ? mid : (c == 1 ? big : (c == 2 ? huge : wide));
             if (cls == c) dst[b + __popc(m & lanemask_lt())] = (int32_t)r;
         }
     }
@@ -1121,19 +1122,26 @@ void orient(mce_graph *g, int orientation) {
     sort_rows_warp<<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->orp.get(), g->ocol.get());
     MCE_LAUNCH_CHECK();
     int32_t *rmid = g->pool.take<int32_t>(n), *rbig = g->pool.take<int32_t>(n), *rhuge = g->pool.take<int32_t>(n);
-    int32_t *meta = g->pool.take<int32_t>(4);
-    MCE_CUDA(cudaMemsetAsync(meta, 0, 4 * sizeof(int32_t), s));
-    long_rows_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->orp.get(), rmid, rbig, rhuge, meta);
+    int32_t *rwide = g->pool.take<int32_t>(n);
+    int32_t *meta = g->pool.take<int32_t>(5);
+    MCE_CUDA(cudaMemsetAsync(meta, 0, 5 * sizeof(int32_t), s));
+    long_rows_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->orp.get(), rmid, rbig, rhuge, rwide, meta);
     MCE_LAUNCH_CHECK();
-    int32_t *hmeta = g->host.get<int32_t>(4);
-    MCE_CUDA(cudaMemcpyAsync(hmeta, meta, 4 * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+    int32_t *hmeta = g->host.get<int32_t>(5);
+    MCE_CUDA(cudaMemcpyAsync(hmeta, meta, 5 * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
     stream_sync(s);
     g->kernels += 8;
     g->max_out = hmeta[3];
-    const int32_t n_mid = hmeta[0], n_big = hmeta[1], n_huge = hmeta[2];
+    const int32_t n_mid = hmeta[0], n_big = hmeta[1], n_huge = hmeta[2], n_wide = hmeta[4];
     const int32_t smem_cap = 8192;  // ints (32 KB)
     if (n_mid > 0) {
         sort_rows_mid<8><<<grid_for((int64_t)n_mid * 32, 256), 256, 0, s>>>(g->orp.get(), g->ocol.get(), rmid, n_mid);
+        MCE_LAUNCH_CHECK();
+        g->kernels += 1;
+    }
+    if (n_wide > 0) {
+        sort_rows_mid<32><<<grid_for((int64_t)n_wide * 32, 256), 256, 0, s>>>(g->orp.get(), g->ocol.get(), rwide,
+                                                                               n_wide);
         MCE_LAUNCH_CHECK();
         g->kernels += 1;
     }
