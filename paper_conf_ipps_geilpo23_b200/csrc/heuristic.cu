@@ -111,7 +111,10 @@ __device__ __forceinline__ bool useful(const int32_t *__restrict__ thr, int32_t 
 #define HUB_BIG 131072
 #endif
 constexpr int kHubBig = HUB_BIG;          // lookup matrix: at most 2^17 rows of 2^11 words (2 GiB)
-constexpr int kHubTail = 8192;            // bit-set tail: the first kHubTail hubs
+#ifndef HUB_TAIL
+#define HUB_TAIL 2048  // measured 2048 / 4096 / 8192 / 16384 / 32768: rmat22 43.4 / 44.5 / 44.3 / 49.5 / 58.0 ms (one word per lane)
+#endif
+constexpr int kHubTail = HUB_TAIL;        // bit-set tail: the first kHubTail hubs
 constexpr int kHubWords = kHubTail / 64;  // 128
 constexpr int kHubWPL = kHubWords / 32;   // words per lane
 struct Hub {
