@@ -44,8 +44,10 @@ struct mce_graph {
     mce::Pool hpool;
     mce::PinnedBuf hhost{1};
     cudaStream_t hstream = nullptr;
+    cudaStream_t pstream = nullptr;  // greatest-priority stream of the overlapped preprocessing
     ~mce_graph() {
         if (hstream) cudaStreamDestroy(hstream);
+        if (pstream) cudaStreamDestroy(pstream);
         if (pre_ev[0]) cudaEventDestroy(pre_ev[0]);
         if (pre_ev[1]) cudaEventDestroy(pre_ev[1]);
     }
