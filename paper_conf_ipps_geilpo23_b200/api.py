@@ -180,7 +180,7 @@ class Graph:
                                   runs.ctypes.data_as(ctypes.c_void_p)))
         return int(w.value), clique[: ln.value].tolist(), runs[: self.n]
 
-    def _result(self, handle) -> Result:
+    def _result(self, handle, cliques: str = "host") -> Result:
         L = lib()
         try:
             om = ctypes.c_int32()
@@ -188,9 +188,17 @@ class Graph:
             st = ctypes.c_int64()
             tr = ctypes.c_int32()
             check(L.mce_result_info(handle, ctypes.byref(om), ctypes.byref(cnt), ctypes.byref(st), ctypes.byref(tr)))
-            cl = np.empty((st.value, max(om.value, 0)), np.int32)
-            check(L.mce_result_cliques(handle, cl.ctypes.data_as(ctypes.c_void_p) if cl.size else None,
-                                       _lib.WHERE_HOST))
+            if cliques == "device":  # the canonical rows stay in HBM: a torch tensor on the graph's device
+                if torch is None:
+                    raise RuntimeError("cliques='device' needs torch")
+                cl = torch.empty((st.value, max(om.value, 0)), dtype=torch.int32,
+                                 device=torch.device("cuda", self.device))
+                check(L.mce_result_cliques(handle, ctypes.c_void_p(cl.data_ptr()) if cl.numel() else None,
+                                           _lib.WHERE_DEVICE))
+            else:
+                cl = np.empty((st.value, max(om.value, 0)), np.int32)
+                check(L.mce_result_cliques(handle, cl.ctypes.data_as(ctypes.c_void_p) if cl.size else None,
+                                           _lib.WHERE_HOST))
             nl = ctypes.c_int32()
             ent = (ctypes.c_int64 * 512)()
             check(L.mce_result_levels(handle, ent, 512, ctypes.byref(nl)))
@@ -208,14 +216,17 @@ class Graph:
         finally:
             L.mce_result_free(handle)
 
-    def enumerate(self, **opts) -> Result:
+    def enumerate(self, cliques: str = "host", **opts) -> Result:
+        """All maximum cliques (mce_enumerate).  cliques='host': numpy rows;
+        'device': a torch.int32 tensor in the graph's device memory (no copy to
+        the host)."""
         o, keep = make_options(**opts)
         h = ctypes.c_void_p()
         st = lib().mce_enumerate(self._h, ctypes.byref(o), ctypes.byref(h))
         if keep is not None:
             keep.reraise()
         check(st)
-        return self._result(h)
+        return self._result(h, cliques)
 
     def find_one(self, window: int = 0, **opts) -> Result:
         o, keep = make_options(**opts)
