@@ -273,7 +273,7 @@ __device__ int32_t greedy_run(int32_t s, const int64_t *__restrict__ rowptr, con
 // run this way so a long run is not serialised on one warp; the replay of the
 // winning run uses it too, writing the clique (in order added).
 #ifndef BLOCK_RUN
-#define BLOCK_RUN 512  // measured on rmat22: 256 / 512 / 1024 threads = 95.4 / 81.8 / 90.7 ms per step
+#define BLOCK_RUN 256  // rmat22, round 2: 256 / 512 / 1024 threads = 37.5 / 37.8 / 40.6 ms per step (round 1, before the candidate filter: 95.4 / 81.8 / 90.7)
 #endif
 constexpr int kBlockRun = BLOCK_RUN;
 constexpr int64_t kBigSeed = 1024;

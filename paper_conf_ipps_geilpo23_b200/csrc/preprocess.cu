@@ -64,6 +64,9 @@ constexpr int kPeelThreads = 1024;  // launch bound; the launch uses kcore_threa
 #ifndef KCORE_OVL_PCT
 #define KCORE_OVL_PCT 50  // percent of the SMs the peel takes beside the heuristic; measured 35 / 50 / 65 = ba1m 1.51 / 1.43 / 1.49 ms, rmat22 81.5 / 81.7 / 83.9 ms
 #endif
+#ifndef ORIENT_KL_DENSE
+#define ORIENT_KL_DENSE 4  // (mean degree > 16) rmat22, round 2: 1 / 2 / 4 chunks = 37.8 / 36.8 / 36.6 ms per step
+#endif
 #ifndef KCORE_OVL_PCT_DENSE
 #define KCORE_OVL_PCT_DENSE 35
 #endif
@@ -1110,10 +1113,11 @@ void orient(mce_graph *g, int orientation) {
     }
     int32_t *odeg = g->pool.take<int32_t>(n);
     int32_t *stage = g->pool.take<int32_t>(std::max<int64_t>(g->nnz, 1));
-    // Long rows (degree > 64, a warp each) gather 4 chunks per trip when they
-    // are rare (mean degree <= 16: ba1m preprocessing 1.27 -> 1.17 ms); with
-    // many (rmat22, mean 31) the wider gathers slow the greedy heuristic that
-    // runs beside this pass more than they gain (step 82.6 -> 88-93 ms)
+    // Long rows (degree > 64, a warp each) gather ORIENT_KL chunks per trip when
+    // they are rare (mean degree <= 16: ba1m preprocessing 1.27 -> 1.17 ms) and
+    // ORIENT_KL_DENSE otherwise (round 1, beside a 44 ms heuristic, 4 chunks
+    // slowed rmat22's step 82.6 -> 88-93 ms; round 2, beside a 20 ms one, they
+    // gain 37.8 -> 36.6 ms)
     int2 *rp2 = g->pool.take<int2>(n);
     pack_rank_pid_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->rank.get(), g->pid.get(), rp2);
     MCE_LAUNCH_CHECK();
@@ -1121,7 +1125,8 @@ void orient(mce_graph *g, int orientation) {
         orient_stage_kernel<ORIENT_KL><<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), rp2, odeg,
                                                                            stage);
     else
-        orient_stage_kernel<1><<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), rp2, odeg, stage);
+        orient_stage_kernel<ORIENT_KL_DENSE><<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), rp2,
+                                                                                 odeg, stage);
     MCE_LAUNCH_CHECK();
     exclusive_scan_i32(odeg, g->orp.get(), n, g->pool.take<int64_t>(scan_tmp_items(n)), s);
     orient_copy_kernel<<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->vid.get(), g->orp.get(), stage,
