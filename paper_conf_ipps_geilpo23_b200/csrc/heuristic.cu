@@ -115,6 +115,10 @@ constexpr int kHubBig = HUB_BIG;          // lookup matrix: at most 2^17 rows of
 #define HUB_TAIL 2048  // measured 2048 / 4096 / 8192 / 16384 / 32768: rmat22 43.4 / 44.5 / 44.3 / 49.5 / 58.0 ms (one word per lane)
 #endif
 constexpr int kHubTail = HUB_TAIL;        // bit-set tail: the first kHubTail hubs
+#ifndef HUB_ROWS
+#define HUB_ROWS 16384  // rmat22: 4096 / 16384 / 131072 (every hub) rows = 35.5 / 35.4 / 36.3 ms per step
+#endif
+constexpr int kHubRows = HUB_ROWS;        // hubs with a matrix row (the rest: columns only)
 constexpr int kHubWords = kHubTail / 64;  // 128
 constexpr int kHubWPL = kHubWords / 32;   // words per lane
 struct Hub {
@@ -123,6 +127,7 @@ struct Hub {
     const unsigned long long *hkey = nullptr;  // [K] pick keys
     const uint64_t *M = nullptr;               // [K][KW]
     int K = 0, KW = 0, KT = 0;                 // KT: hubs of the tail set (indices < KT), <= kHubTail
+    int KR = 0;                                // hubs with a matrix row (indices < KR, the highest degrees)
 };
 
 // The rest of a run whose candidates are all hubs, by one warp: P = the
@@ -205,7 +210,7 @@ __device__ __forceinline__ bool adjacent_h(const Hub &H, int hw, const int64_t *
     if (H.K) {
         const int hx = __ldg(H.hid + x);
         x_hub = hx >= 0 && hx < H.KT;
-        if (hx >= 0 && hw >= 0) return (__ldg(H.M + (int64_t)hw * H.KW + (hx >> 6)) >> (hx & 63)) & 1ull;
+        if (hx >= 0 && hw >= 0 && hw < H.KR) return (__ldg(H.M + (int64_t)hw * H.KW + (hx >> 6)) >> (hx & 63)) & 1ull;
     } else {
         x_hub = false;
     }
@@ -553,25 +558,28 @@ __global__ void deg_bucket_hist(int64_t n, const int64_t *__restrict__ rowptr, u
 }
 
 // hub index of every vertex (-1: not a hub), by warp-aggregated appends:
-// buckets >= btail take [0, KT) (cnt[0]), buckets in [bstar, btail) take
-// [KT, K) (cnt[1] starts at KT); order inside each range is immaterial (keys
-// carry the tie-break)
-__global__ void hub_index_kernel(int64_t n, const int64_t *__restrict__ rowptr, int bstar, int btail, int32_t *hid,
-                                 int32_t *hv, int32_t *cnt) {
+// buckets >= btail take [0, KT) (cnt[0]), buckets in [brows, btail) take
+// [KT, KR) (cnt[1] starts at KT), buckets in [bstar, brows) take [KR, K)
+// (cnt[2] starts at KR); order inside each range is immaterial (keys carry
+// the tie-break)
+__global__ void hub_index_kernel(int64_t n, const int64_t *__restrict__ rowptr, int bstar, int brows, int btail,
+                                 int32_t *hid, int32_t *hv, int32_t *cnt) {
     const int lane = threadIdx.x & 31;
     for (int64_t v0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) & ~31ll; v0 < n;
          v0 += (int64_t)gridDim.x * blockDim.x) {
         const int64_t v = v0 + lane;
         const int bk = v < n ? deg_bucket(rowptr[v + 1] - rowptr[v]) : -1;
-        const bool t = bk >= btail, h = bk >= bstar && !t;
-        const unsigned mt = __ballot_sync(0xffffffffu, t), mh = __ballot_sync(0xffffffffu, h);
-        int bt = 0, bh = 0;
-        if (lane == 0 && mt) bt = atomicAdd(cnt, __popc(mt));
-        if (lane == 0 && mh) bh = atomicAdd(cnt + 1, __popc(mh));
-        bt = __shfl_sync(0xffffffffu, bt, 0);
-        bh = __shfl_sync(0xffffffffu, bh, 0);
+        const int cls = bk >= btail ? 0 : (bk >= brows ? 1 : (bk >= bstar ? 2 : -1));
+        int idx = -1;
+#pragma unroll
+        for (int c = 0; c < 3; ++c) {
+            const unsigned m = __ballot_sync(0xffffffffu, cls == c);
+            int b = 0;
+            if (lane == 0 && m) b = atomicAdd(cnt + c, __popc(m));
+            b = __shfl_sync(0xffffffffu, b, 0);
+            if (cls == c) idx = b + __popc(m & lanemask_lt());
+        }
         if (v < n) {
-            const int idx = t ? bt + __popc(mt & lanemask_lt()) : (h ? bh + __popc(mh & lanemask_lt()) : -1);
             hid[v] = idx;
             if (idx >= 0) hv[idx] = (int32_t)v;
         }
@@ -742,8 +750,8 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
         const size_t free_b = dev_free_memory();
         unsigned long long kcap = kHubBig;
         while (kcap > kHubTail && (kcap * ((kcap + 63) / 64) * 8ull) > free_b / 4) kcap >>= 1;
-        int bstar = kBuckets, btail = kBuckets;
-        unsigned long long above = 0, tail = 0;
+        int bstar = kBuckets, btail = kBuckets, brows = kBuckets;
+        unsigned long long above = 0, tail = 0, rows = 0;
         for (int b = kBuckets - 1; b >= 0; --b) {
             if (above + hb[b] > kcap) break;
             above += hb[b];
@@ -752,22 +760,30 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
                 tail = above;
                 if (hb[b]) btail = b;
             }
+            if (above <= (unsigned long long)kHubRows) {
+                rows = above;
+                if (hb[b]) brows = b;
+            }
         }
         kernels += 1;
         if (above >= 64) {  // enough hubs to matter
             const int K = (int)above;
             const int KW = (K + 63) / 64;
-            int32_t *hid = pool.take<int32_t>(n), *hv = pool.take<int32_t>(K), *cnt = pool.take<int32_t>(2);
-            const int32_t cnt0[2] = {0, (int32_t)tail};
+            const int KR = std::max<int>((int)rows, (int)tail);
+            int32_t *hid = pool.take<int32_t>(n), *hv = pool.take<int32_t>(K), *cnt = pool.take<int32_t>(3);
+            const int32_t cnt0[3] = {0, (int32_t)tail, KR};
             MCE_CUDA(cudaMemcpyAsync(cnt, cnt0, sizeof(cnt0), cudaMemcpyHostToDevice, s));
-            hub_index_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(), bstar, btail, hid, hv, cnt);
+            hub_index_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->rowptr.get(), bstar, brows, btail, hid, hv, cnt);
             MCE_LAUNCH_CHECK();
-            uint64_t *M = pool.take<uint64_t>((int64_t)K * KW);
+            // rows only for the KR highest-degree hubs (the picks of the runs; a
+            // test against a lower pick falls back to the binary search), columns
+            // for all K of them
+            uint64_t *M = pool.take<uint64_t>((int64_t)KR * KW);
             unsigned long long *hkey = pool.take<unsigned long long>(K);
             const size_t smem = (size_t)8 * KW * sizeof(unsigned long long);
             MCE_CUDA(cudaFuncSetAttribute(hub_matrix_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-            hub_matrix_kernel<<<std::max(1, std::min((K + 7) / 8, num_sms() * 8)), 256, smem, s>>>(
-                K, KW, hv, g->rowptr.get(), g->col.get(), hid, thr, M, hkey);
+            hub_matrix_kernel<<<std::max(1, std::min((KR + 7) / 8, num_sms() * 8)), 256, smem, s>>>(
+                KR, KW, hv, g->rowptr.get(), g->col.get(), hid, thr, M, hkey);
             MCE_LAUNCH_CHECK();
             kernels += 2;
             H.hid = hid;
@@ -777,6 +793,7 @@ HeuristicResult run_heuristic(mce_graph *g, int kind, int64_t h, int32_t shard_r
             H.K = K;
             H.KW = KW;
             H.KT = (int)tail;
+            H.KR = KR;
         }
     }
     if (nseeds > 0) {
