@@ -65,10 +65,10 @@ constexpr int kPeelThreads = 1024;  // launch bound; the launch uses kcore_threa
 #define KCORE_OVL_PCT 50  // percent of the SMs the peel takes beside the heuristic; measured 35 / 50 / 65 = ba1m 1.51 / 1.43 / 1.49 ms, rmat22 81.5 / 81.7 / 83.9 ms
 #endif
 #ifndef ORIENT_KL_DENSE
-#define ORIENT_KL_DENSE 4  // (mean degree > 16) rmat22, round 2: 1 / 2 / 4 chunks = 37.8 / 36.8 / 36.6 ms per step
+#define ORIENT_KL_DENSE 8  // (mean degree > 16) rmat22, round 2: 1 / 2 / 4 / 8 chunks = 37.8 / 36.8 / 36.6 / 36.2 ms per step
 #endif
 #ifndef KCORE_OVL_PCT_DENSE
-#define KCORE_OVL_PCT_DENSE 35
+#define KCORE_OVL_PCT_DENSE 30  // rmat22 after the round-2 heuristic work: 25 / 30 / 35 / 42% = 35.7 / 34.5 / 35.2 / 35.5 ms
 #endif
 #ifndef KCORE_CHUNK
 #define KCORE_CHUNK 32  // measured: 128 / 64 / 32 / 16 / 8 = ba1m 1.49 / 1.46 / 1.43 / 1.44 / 1.50 ms, rmat22 82.5 / 81.8 / 82.1 / 81.4 / - ms
@@ -1011,8 +1011,9 @@ void kcore(mce_graph *g) {
     if (blocks_per_sm < 1) fail(2, "kcore: cooperative kernel does not fit an SM");
     // beside the heuristic: a smaller share on graphs of mean degree > 16, whose
     // heuristic is long and whose peel gains nothing from more blocks (rmat22:
-    // 20 / 27 / 35 / 42 / 50% = 40.4 / 38.3 / 37.7 / 38.1 / 39.0 ms per step;
-    // ba1m keeps 50%: 35% = 1.45 ms, 42% = 1.37, 50% = 1.37)
+    // 20 / 27 / 35 / 42 / 50% = 40.4 / 38.3 / 37.7 / 38.1 / 39.0 ms per step,
+    // re-swept after the later heuristic changes: 30% best; ba1m keeps 50%:
+    // 35% = 1.45 ms, 42% = 1.37, 50% = 1.37)
     const int pct = g->nnz > 16 * n ? KCORE_OVL_PCT_DENSE : KCORE_OVL_PCT;
     const int grid = half ? std::max(1, num_sms() * pct / 100) : num_sms();
     int64_t n_arg = n;
