@@ -837,17 +837,34 @@ __global__ void __launch_bounds__(512)
     const int64_t nthreads = (int64_t)gridDim.x * blockDim.x;
     const int lane = threadIdx.x & 31;
     // d(v) and frontier 0: a warp per 32 vertices, 8-lane tiles over the rows
+    // (rows of more than 64 neighbours by the whole warp: a hub's row is
+    // 4x shorter per lane)
     for (int64_t v0 = (tid >> 5) * 32; v0 < n; v0 += (nthreads >> 5) * 32) {
         for (int q = 0; q < 32; q += 4) {
             const int64_t v = v0 + q + (lane >> 3);
             int32_t cnt = 0, c = 0;
+            int64_t eb = 0, ee = 0;
             if (v < n) {
                 c = core[v];
-                for (int64_t e = rowptr[v] + (lane & 7); e < rowptr[v + 1]; e += 8) cnt += core[col[e]] >= c;
+                eb = rowptr[v];
+                ee = rowptr[v + 1];
             }
+            const bool longrow = ee - eb > 64;
+            if (v < n && !longrow)
+                for (int64_t e = eb + (lane & 7); e < ee; e += 8) cnt += core[col[e]] >= c;
             cnt += __shfl_xor_sync(0xffffffffu, cnt, 1);
             cnt += __shfl_xor_sync(0xffffffffu, cnt, 2);
             cnt += __shfl_xor_sync(0xffffffffu, cnt, 4);
+            const unsigned lm = __ballot_sync(0xffffffffu, longrow && (lane & 7) == 0);
+            for (unsigned mm = lm; mm; mm &= mm - 1) {  // the tiles' long rows, one at a time by the warp
+                const int src = __ffs(mm) - 1;
+                const int64_t lb = __shfl_sync(0xffffffffu, eb, src), le = __shfl_sync(0xffffffffu, ee, src);
+                const int32_t lc = __shfl_sync(0xffffffffu, c, src);
+                int32_t lcnt = 0;
+                for (int64_t e = lb + lane; e < le; e += 32) lcnt += core[col[e]] >= lc;
+                lcnt = __reduce_add_sync(0xffffffffu, lcnt);
+                if (lane == src) cnt = lcnt;
+            }
             const bool take = v < n && (lane & 7) == 0 && cnt <= c;
             if (v < n && (lane & 7) == 0) {
                 d[v] = cnt;
@@ -882,12 +899,16 @@ __global__ void __launch_bounds__(512)
                 eb = rowptr[v];
                 ee = rowptr[v + 1];
             }
-            const int iters = __reduce_max_sync(0xffffffffu, (unsigned)((ee - eb + 7) >> 3));
+            // rows of more than 64 neighbours by the whole warp, the rest by 8-lane tiles
+            const bool longrow = ee - eb > 64;
+            const unsigned lm = __ballot_sync(0xffffffffu, longrow && (lane & 7) == 0);
+            const int64_t seb = longrow ? 0 : eb, see = longrow ? 0 : ee;
+            const int iters = __reduce_max_sync(0xffffffffu, (unsigned)((see - seb + 7) >> 3));
             for (int it = 0; it < iters; ++it) {
-                const int64_t e = eb + it * 8 + (lane & 7);
+                const int64_t e = seb + it * 8 + (lane & 7);
                 bool fell = false;
                 int32_t w = -1;
-                if (e < ee) {
+                if (e < see) {
                     w = col[e];
                     if (core[w] == c && __ldcg(round + w) < 0) fell = atomicSub(d + w, 1) == c + 1;
                 }
@@ -896,6 +917,25 @@ __global__ void __launch_bounds__(512)
                 if (lane == 0 && m) b = atomicAdd(ctrl + 2 + ((t + 1) & 1), (unsigned long long)__popc(m));
                 b = __shfl_sync(0xffffffffu, b, 0);
                 if (fell) nxt[b + __popc(m & lanemask_lt())] = w;
+            }
+            for (unsigned mm = lm; mm; mm &= mm - 1) {
+                const int src = __ffs(mm) - 1;
+                const int64_t lb = __shfl_sync(0xffffffffu, eb, src), le = __shfl_sync(0xffffffffu, ee, src);
+                const int32_t lc = __shfl_sync(0xffffffffu, c, src);
+                for (int64_t e0 = lb; e0 < le; e0 += 32) {
+                    const int64_t e = e0 + lane;
+                    bool fell = false;
+                    int32_t w = -1;
+                    if (e < le) {
+                        w = col[e];
+                        if (core[w] == lc && __ldcg(round + w) < 0) fell = atomicSub(d + w, 1) == lc + 1;
+                    }
+                    const unsigned m = __ballot_sync(0xffffffffu, fell);
+                    unsigned long long b = 0;
+                    if (lane == 0 && m) b = atomicAdd(ctrl + 2 + ((t + 1) & 1), (unsigned long long)__popc(m));
+                    b = __shfl_sync(0xffffffffu, b, 0);
+                    if (fell) nxt[b + __popc(m & lanemask_lt())] = w;
+                }
             }
         }
         grid.sync();
@@ -936,6 +976,8 @@ void deterministic_order(mce_graph *g) {
     int blocks_per_sm = 0;
     MCE_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm, shell_round_peel, 512, 0));
     if (blocks_per_sm < 1) fail(2, "shell_round_peel: cooperative kernel does not fit an SM");
+    // (all SMs even beside the heuristic: the rounds are the longer branch --
+    // rmat22 with the k-core's 30% share 57.9 ms per step, with all SMs 54.4)
     const int grid = num_sms() * std::min(blocks_per_sm, 2);
     int64_t n_arg = n;
     const int64_t *rp = g->rowptr.get();
