@@ -354,8 +354,8 @@ def main():
     mode, shard_depth, args.window, max_cl = bench_defaults(args)
     heur = args.heuristic
     orient = args.orientation
-    if world > 1 and orient == "degeneracy":
-        orient = "degeneracy_det"  # every rank must orient identically (reading 18)
+    # world > 1 with "degeneracy": rank 0 peels and broadcasts its cores and
+    # order, every rank orients from them (distributed.agree_core)
 
     g = build_graph(args.config, f"cuda:{local}")
     edges = g.num_edges

@@ -187,6 +187,20 @@ mce_status mce_preprocess(mce_graph *g, int32_t orientation, int32_t *core_out, 
  * mce_preprocess output; MCE_ERR_INVALID for a NULL order. */
 mce_status mce_set_order(mce_graph *g, int32_t orientation, const int32_t *order, int32_t where);
 
+/* Install k-core numbers and a degeneracy (peel) order computed elsewhere
+ * instead of peeling on this handle (PAPER.md IV-C: the degeneracy ordering
+ * and core numbers of the preprocessing step).  core: int32[n], core number of
+ * each vertex; peel: int32[n], vertex of rank i in a degeneracy order (each
+ * vertex has at most core(v) later neighbours) -- both host or device per
+ * `where`, copied, caller keeps ownership.  Not validated: they must be exact
+ * (e.g. another handle's mce_preprocess(MCE_ORIENT_DEGENERACY) output on the
+ * same graph).  The handle's orientation is dropped and rebuilt from them on
+ * the next call; the degeneracy is recomputed as max core.  Multi-GPU: rank 0
+ * peels, broadcasts both arrays and the other ranks set them here, so every
+ * rank orients the edges the same way without a second (or a deterministic,
+ * slower) peel (distributed.py).  MCE_ERR_INVALID for NULL arrays (n > 0). */
+mce_status mce_set_core(mce_graph *g, const int32_t *core, const int32_t *peel, int32_t where);
+
 /* Greedy heuristic (PAPER.md IV-A, Algorithm 1).  kind = MCE_HEUR_*; h = runs
  * (<=0: |V|; single-run kinds ignore h and use 1).  *omega_bar_out = size of the
  * best clique found; clique_out (host, capacity >= max degree + 1, may be NULL)

@@ -71,7 +71,7 @@ def build(force: bool = False, jobs: int = 8) -> str:
 
 
 EXPORTS = [
-    "mce_default_options", "mce_load_csr", "mce_graph_free", "mce_graph_clear_cache", "mce_preprocess", "mce_set_order", "mce_heuristic", "mce_enumerate",
+    "mce_default_options", "mce_load_csr", "mce_graph_free", "mce_graph_clear_cache", "mce_preprocess", "mce_set_order", "mce_set_core", "mce_heuristic", "mce_enumerate",
     "mce_find_one", "mce_result_info", "mce_result_cliques", "mce_result_levels", "mce_result_timing",
     "mce_result_free", "mce_empty_cache", "mce_last_error", "mce_version",
 ]
@@ -102,6 +102,8 @@ def lib():
     L.mce_preprocess.argtypes = [vp, i32, vp, vp, i32, p32]
     L.mce_set_order.restype = i32
     L.mce_set_order.argtypes = [vp, i32, vp, i32]
+    L.mce_set_core.restype = i32
+    L.mce_set_core.argtypes = [vp, vp, vp, i32]
     L.mce_heuristic.restype = i32
     L.mce_heuristic.argtypes = [vp, i32, i64, p32, vp, p32, vp]
     L.mce_enumerate.restype = i32

@@ -164,6 +164,27 @@ class Graph:
         check(lib().mce_preprocess(self._h, ORIENT[orientation], None, ptr, where, ctypes.byref(d)))
         return out
 
+    def core_into(self, core, peel):
+        """Preprocess with the degeneracy orientation (cached) and copy its core
+        numbers and peel order into `core` / `peel` (int32[n], both torch tensors
+        on this graph's device or both host arrays)."""
+        cptr, where, _k1 = _ptr_and_where(core, np.int32)
+        pptr, where2, _k2 = _ptr_and_where(peel, np.int32)
+        if where != where2:
+            raise ValueError("core and peel must both be on the host or both on the device")
+        d = ctypes.c_int32()
+        check(lib().mce_preprocess(self._h, ORIENT["degeneracy"], cptr, pptr, where, ctypes.byref(d)))
+        return core, peel
+
+    def set_core(self, core, peel):
+        """mce_set_core: take core numbers and a degeneracy (peel) order computed
+        elsewhere (another rank's core_into) instead of peeling here."""
+        cptr, where, _k1 = _ptr_and_where(core, np.int32)
+        pptr, where2, _k2 = _ptr_and_where(peel, np.int32)
+        if where != where2:
+            raise ValueError("core and peel must both be on the host or both on the device")
+        check(lib().mce_set_core(self._h, cptr, pptr, where))
+
     def set_order(self, order, orientation: str = "degeneracy"):
         """mce_set_order: orient the edges along `order` (vertex of rank i)."""
         ptr, where, _keep = _ptr_and_where(order, np.int32)

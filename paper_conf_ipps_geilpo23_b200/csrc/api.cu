@@ -229,6 +229,15 @@ mce_status mce_set_order(mce_graph *g, int32_t orientation, const int32_t *order
     });
 }
 
+mce_status mce_set_core(mce_graph *g, const int32_t *core, const int32_t *peel, int32_t where) {
+    return run_guarded([&] {
+        if (!g) fail(MCE_ERR_INVALID, "graph is NULL");
+        if ((!core || !peel) && g->n) fail(MCE_ERR_INVALID, "core or peel is NULL");
+        MCE_CUDA(cudaSetDevice(g->device));
+        set_core(g, core, peel, where == MCE_WHERE_DEVICE);
+    });
+}
+
 mce_status mce_preprocess(mce_graph *g, int32_t orientation, int32_t *core_out, int32_t *order_out, int32_t where,
                           int32_t *degeneracy_out) {
     return run_guarded([&] {

@@ -71,4 +71,6 @@ bool preprocessed(const mce_graph *g, int orientation);
 double preprocess_ms(mce_graph *g);
 // orientation from a given order (mce_set_order)
 void orient_from(mce_graph *g, int orientation, const int32_t *order, bool on_device);
+// core numbers + peel order from another handle (mce_set_core): no peel here
+void set_core(mce_graph *g, const int32_t *core, const int32_t *peel, bool on_device);
 }  // namespace mce

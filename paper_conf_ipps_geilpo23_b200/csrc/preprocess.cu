@@ -1233,6 +1233,44 @@ void orient_from(mce_graph *g, int orientation, const int32_t *order, bool on_de
     stream_sync(g->stream);
 }
 
+__global__ void max_core_kernel(int64_t n, const int32_t *__restrict__ core, int32_t *out) {
+    int m = 0;
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+        m = max(m, core[v]);
+    for (int o = 16; o; o >>= 1) m = max(m, __shfl_xor_sync(0xffffffffu, m, o));
+    if ((threadIdx.x & 31) == 0) atomicMax(out, m);
+}
+
+// Multi-GPU: rank 0 peels once, the others take its
+// core numbers and peel order instead of re-peeling -- the asynchronous peel's
+// order depends on timing, and root / candidate ownership needs every rank to
+// orient the edges the same way.  The degeneracy is max core (recomputed, so a
+// degree-ordered `peel` would still give the right value).
+void set_core(mce_graph *g, const int32_t *core, const int32_t *peel, bool on_device) {
+    const int64_t n = g->n;
+    cudaStream_t s = g->stream;
+    g->core.ensure(std::max<int64_t>(n, 1));
+    g->peel.ensure(std::max<int64_t>(n, 1));
+    g->have_core = false;
+    g->orientation = -1;  // the oriented CSR (and its CSR-id priorities) follow the new cores
+    g->degeneracy = 0;
+    if (n) {
+        const auto kind = on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice;
+        MCE_CUDA(cudaMemcpyAsync(g->core.get(), core, sizeof(int32_t) * n, kind, s));
+        MCE_CUDA(cudaMemcpyAsync(g->peel.get(), peel, sizeof(int32_t) * n, kind, s));
+        g->pool.reset();
+        int32_t *mx = g->pool.take<int32_t>(1);
+        MCE_CUDA(cudaMemsetAsync(mx, 0, sizeof(int32_t), s));
+        max_core_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->core.get(), mx);
+        MCE_LAUNCH_CHECK();
+        int32_t *h = g->host.get<int32_t>(1);
+        MCE_CUDA(cudaMemcpyAsync(h, mx, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+        stream_sync(s);
+        g->degeneracy = h[0];
+    }
+    g->have_core = true;
+}
+
 bool preprocessed(const mce_graph *g, int orientation) {
     return g->orientation == orientation && (g->have_core || orientation == 1);
 }

@@ -4,11 +4,15 @@ North star: "Work is partitioned ... by sharding first-level root vertices,
 whose subtrees are independent, with a small NCCL max-allreduce of the omega
 lower bound each level and a final gather of the cliques over NVLink."
 
- * every rank loads the whole graph and runs the whole preprocessing itself,
-   concurrently, with the DETERMINISTIC degeneracy orientation
-   (MCE_ORIENT_DEGENERACY_DET: order (core, shell round, id), a function of
-   the graph alone), so every rank orients the edges identically with no
-   broadcast and no second k-core -- clique ownership depends on it;
+ * every rank loads the whole graph; rank 0 runs the k-core peel and
+   broadcasts its core numbers and peel order (one int32[2n] broadcast over
+   NVLink), the other ranks install them with mce_set_core instead of peeling,
+   and every rank orients its edges from them -- identically, which clique
+   ownership depends on (the asynchronous peel's order depends on timing).
+   orientation="degeneracy_det" instead has every rank compute the
+   deterministic order (core, shell round, id) itself, with no broadcast but
+   a slower peel (reading 18); the degree orientation is a function
+   of the graph and needs neither;
  * heuristic seeds are dealt cyclically (seed position % world == rank) and
    root vertices by CSR id (id % world == rank) inside the library
    (mce_options.shard_rank / shard_count), or level-d candidates by path hash
@@ -100,17 +104,33 @@ def gather_result(res: Result, group=None, find_one: bool = False, max_cliques: 
     return Result(omega, total, allrows, bool(trunc), res.levels, res.timing)
 
 
-def sharded_orientation(orientation: str, world: int) -> str:
-    """The orientation every rank uses: the asynchronous peel's order depends
-    on timing, so a multi-rank degeneracy run takes the deterministic one."""
-    return "degeneracy_det" if world > 1 and orientation == "degeneracy" else orientation
+def agree_core(graph: Graph, group=None):
+    """Rank 0 peels (or reuses its cached peel) and broadcasts its core numbers
+    and degeneracy order; the others set them (mce_set_core) so every rank
+    orients the edges identically with one peel in the whole job."""
+    if dist.get_world_size(group) == 1 or graph.n == 0:
+        return
+    n = graph.n
+    dev = torch.device("cuda", graph.device) if _device(group).type == "cuda" else torch.device("cpu")
+    buf = torch.empty(2 * n, dtype=torch.int32, device=dev)
+    src = dist.get_global_rank(group, 0) if group is not None else 0
+    if dist.get_rank(group) == 0:
+        graph.core_into(buf[:n], buf[n:])
+    dist.broadcast(buf, src=src, group=group)
+    if dist.get_rank(group) != 0:
+        graph.set_core(buf[:n], buf[n:])
+
+
+def _agree(graph: Graph, group, world: int, opts: dict):
+    if world > 1 and opts.setdefault("orientation", "degeneracy") == "degeneracy":
+        agree_core(graph, group)
 
 
 def agree_orientation(graph: Graph, group=None, orientation: str = "degeneracy"):
     """Fallback for callers that need rank 0's own (asynchronous-peel) order on
-    every rank: broadcast it and set it on the others.  enumerate_distributed /
-    find_one_distributed do not use it (each rank computes the deterministic
-    order itself)."""
+    every rank: broadcast it and set it on the others (each rank re-peels for
+    its core numbers; enumerate_distributed / find_one_distributed use
+    agree_core, which broadcasts those too)."""
     if dist.get_world_size(group) == 1 or graph.n == 0:
         return
     dev = _device(group)
@@ -129,7 +149,7 @@ def agree_orientation(graph: Graph, group=None, orientation: str = "degeneracy")
 def enumerate_distributed(graph: Graph, group=None, **opts) -> Result:
     rank = dist.get_rank(group)
     world = dist.get_world_size(group)
-    opts["orientation"] = sharded_orientation(opts.get("orientation", "degeneracy"), world)
+    _agree(graph, group, world, opts)
     res = graph.enumerate(shard_rank=rank, shard_count=world, bound_sync=make_bound_sync(group), **opts)
     return gather_result(res, group, max_cliques=int(opts.get("max_cliques", 0) or 0))
 
@@ -137,7 +157,7 @@ def enumerate_distributed(graph: Graph, group=None, **opts) -> Result:
 def find_one_distributed(graph: Graph, window: int = 0, group=None, **opts) -> Result:
     rank = dist.get_rank(group)
     world = dist.get_world_size(group)
-    opts["orientation"] = sharded_orientation(opts.get("orientation", "degeneracy"), world)
+    _agree(graph, group, world, opts)
     res = graph.find_one(window=window, shard_rank=rank, shard_count=world, bound_sync=make_bound_sync(group),
                          **opts)
     return gather_result(res, group, find_one=True)

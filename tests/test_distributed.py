@@ -253,6 +253,49 @@ def test_shards_on_separate_handles_agree_after_set_order(key, depth):
 
 
 @pytest.mark.gpu
+@pytest.mark.parametrize("where", ["device", "host"])
+@pytest.mark.parametrize("depth", [0, 3])
+@pytest.mark.parametrize("key", ["RMAT13", "planted", "BA5k", "T(30,6)"])
+def test_shards_on_separate_handles_agree_after_set_core(key, depth, where):
+    """Handle 0 peels; the others take its core numbers and peel order with
+    mce_set_core (no peel of their own, distributed.agree_core): they orient
+    identically, report the same cores and degeneracy, and their shards
+    partition the maximum cliques exactly."""
+    import torch
+
+    import oracle
+    from tests.test_gpu_parity import GRAPHS
+
+    import paper_conf_ipps_geilpo23_b200 as m
+    from paper_conf_ipps_geilpo23_b200 import _lib
+
+    g = GRAPHS[key]()
+    om, cl = oracle.max_cliques(*g.numpy())
+    shards = 3
+    hs = [m.Graph(g.rowptr, g.col) for _ in range(shards)]
+    dev = "cuda" if where == "device" else "cpu"
+    core = torch.empty(g.n, dtype=torch.int32, device=dev)
+    peel = torch.empty(g.n, dtype=torch.int32, device=dev)
+    hs[0].core_into(core, peel)
+    for h in hs[1:]:
+        h.set_core(core, peel)
+    c0, o0, d0 = hs[0].preprocess()
+    for h in hs[1:]:
+        c1, o1, d1 = h.preprocess()
+        assert np.array_equal(c0, c1) and np.array_equal(o0, o1) and d0 == d1
+    assert d0 == int(c0.max())
+    assert _lib.lib().mce_set_core(hs[1]._h, None, None, _lib.WHERE_HOST) == 1  # MCE_ERR_INVALID
+    parts = [h.enumerate(shard_rank=r, shard_count=shards, shard_depth=depth) for r, h in enumerate(hs)]
+    for h in hs:
+        h.close()
+    omega = max(p.omega for p in parts)
+    count = sum(p.count for p in parts if p.omega == omega)
+    rows = np.concatenate([p.cliques for p in parts if p.omega == omega], 0)
+    rows = rows[np.lexsort(rows.T[::-1])]
+    assert omega == om and count == len(cl) and np.array_equal(rows, cl)
+
+
+@pytest.mark.gpu
 @pytest.mark.parametrize("depth", [0, 2, 3])
 @pytest.mark.parametrize("key", ["planted", "RMAT13", "BA5k", "T(30,6)", "ER400d", "RMAT11"])
 def test_shards_with_different_bounds(key, depth, monkeypatch):
@@ -333,6 +376,10 @@ def _enumerate_mp_body(rank, world):
             f = mdist.find_one_distributed(gg, window=8, shard_depth=depth)
             okf = f.omega == om and oracle.is_clique(*g.numpy(), f.cliques[0])
             out.append((key, depth, bool(ok), bool(okf), r.omega, r.count))
+        gg.clear_cache()
+        r = mdist.enumerate_distributed(gg, orientation="degeneracy_det")
+        ok = r.omega == om and r.count == len(cl) and np.array_equal(r.cliques, cl)
+        out.append((key, "det", bool(ok), True, r.omega, r.count))
         gg.close()
     return out
 
@@ -340,7 +387,9 @@ def _enumerate_mp_body(rank, world):
 @pytest.mark.gpu
 def test_enumerate_distributed_end_to_end():
     """Two processes (gloo process group, both on cuda:0) run the whole
-    sharded path -- deterministic orientation computed by each rank, cyclic
+    sharded path -- rank 0's cores and peel order broadcast and set on the
+    other rank (agree_core; and the deterministic orientation computed by
+    each rank, orientation="degeneracy_det"), cyclic
     root deal or level-3 hash deal, per-step bound all-reduce, final gather --
     and get the oracle's answer (PAPER.md IV-E line 146: root subsets are
     independent)."""
