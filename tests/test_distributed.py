@@ -396,3 +396,35 @@ def test_enumerate_distributed_end_to_end():
     for rank_out in spawn(_enumerate_mp_body, timeout=900):
         for key, depth, ok, okf, om, cnt in rank_out:
             assert ok and okf, (key, depth, om, cnt)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("config", ["er2000", "ba1m"])
+def test_bench_two_ranks(config):
+    """bench.py's N > 1 path (torchrun, two ranks; on this one-GPU box both on
+    cuda:0 with gloo, the test hooks MCE_BENCH_SAME_DEVICE / MCE_BENCH_BACKEND):
+    rank 0 prints one JSON line whose omega and multiplicity equal a one-GPU
+    run of the library on the same seeded graph."""
+    import json
+    import subprocess
+    import sys
+
+    import paper_conf_ipps_geilpo23_b200 as m
+    from synth import graphs as G
+
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, MCE_BENCH_SAME_DEVICE="1", MCE_BENCH_BACKEND="gloo")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+           "--master-addr", "127.0.0.1", "--master-port", str(_free_port()), "bench.py", "--gpus", "2",
+           "--steps", "3", "--warmup", "3", "--config", config, "--no-cpu-baseline"]
+    out = subprocess.run(cmd, cwd=root, env=env, capture_output=True, text=True, timeout=900)
+    assert out.returncode == 0, out.stderr[-3000:]
+    lines = [ln for ln in out.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, out.stdout[-2000:]
+    rec = json.loads(lines[0])
+    assert rec["n_gpus"] == 2 and rec["value"] > 0
+    g = G.make_config(config)
+    gg = m.Graph(g.rowptr.cuda(), g.col.cuda())
+    r = gg.enumerate()
+    gg.close()
+    assert rec["details"]["omega"] == r.omega and rec["details"]["multiplicity"] == r.count
