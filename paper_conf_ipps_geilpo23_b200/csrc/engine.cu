@@ -990,6 +990,7 @@ void Engine::do_class_w1(const int32_t *list, int64_t count) {
         ra.stride = 1;
         ra.orp = g_->orp.get();
         ra.ocol = g_->ocol.get();
+        ra.ocol4 = g_->have_ocol4 ? g_->ocol4.get() : nullptr;
         ra.order = g_->vid.get();
         ra.need = need();
         ra.bound = o_.bound;

@@ -113,6 +113,7 @@ struct RootArgs {
     int64_t count, stride;
     const int64_t *orp;
     const int32_t *ocol;
+    const int4 *ocol4;  // rows padded to 16-byte slots (mce_graph::ocol4) or nullptr
     const int32_t *order;
     int32_t need, bound;
     // outputs (appended; ctr = {roots, adjacency rows, level-2 entries, leaves})

@@ -26,6 +26,8 @@ struct mce_graph {
     mce::DevBuf<int32_t> pid;      // [n] vertex -> CSR id
     mce::DevBuf<int64_t> orp;      // [n+1] oriented CSR (edges to higher rank), indexed by CSR id
     mce::DevBuf<int32_t> ocol;     // [nnz/2] out-neighbour CSR ids, rows ascending
+    mce::DevBuf<int4> ocol4;       // [n] the same rows padded to 16-byte slots (-1 fill), only when max_out <= 4
+    bool have_ocol4 = false;       // ocol4 matches the current orientation
     int32_t max_out = 0;           // largest out-degree
     double t_pre_ms = 0.0;         // device time of the last preprocessing (see preprocess_ms)
     cudaEvent_t pre_ev[2] = {nullptr, nullptr};

@@ -1095,8 +1095,30 @@ void kcore(mce_graph *g) {
     g->have_core = true;
 }
 
+// Out-rows of <= 4 ids padded to one aligned 16-byte slot per vertex (-1
+// fill): the sparse root level (roots.cu root_expand_l4) then fetches a row
+// with one LDG.128 and no row bounds -- two dependent loads per root instead
+// of four.
+__global__ void pad_rows4_kernel(int64_t n, const int64_t *__restrict__ orp, const int32_t *__restrict__ ocol,
+                                 int4 *__restrict__ out) {
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t b = orp[v];
+        const int d = (int)(orp[v + 1] - b);
+        int4 x;
+        x.x = d > 0 ? ocol[b] : -1;
+        x.y = d > 1 ? ocol[b + 1] : -1;
+        x.z = d > 2 ? ocol[b + 2] : -1;
+        x.w = d > 3 ? ocol[b + 3] : -1;
+        out[v] = x;
+    }
+}
+
+#ifndef PAD_ROWS4
+#define PAD_ROWS4 1
+#endif
 void orient(mce_graph *g, int orientation) {
     if (g->orientation == orientation) return;
+    g->have_ocol4 = false;
     const int64_t n = g->n;
     cudaStream_t s = g->stream;
     g->order.ensure(std::max<int64_t>(n, 1));
@@ -1188,6 +1210,14 @@ void orient(mce_graph *g, int orientation) {
     stream_sync(s);
     g->kernels += 8;
     g->max_out = hmeta[3];
+    g->have_ocol4 = false;
+    if (g->max_out <= 4 && PAD_ROWS4) {  // (rows this short need no further sort)
+        g->ocol4.ensure(n);
+        pad_rows4_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->orp.get(), g->ocol.get(), g->ocol4.get());
+        MCE_LAUNCH_CHECK();
+        g->kernels += 1;
+        g->have_ocol4 = true;
+    }
     const int32_t n_mid = hmeta[0], n_big = hmeta[1], n_huge = hmeta[2], n_wide = hmeta[4];
     const int32_t smem_cap = 8192;  // ints (32 KB)
     if (n_mid > 0) {

@@ -295,16 +295,46 @@ __device__ __forceinline__ void load4(const int32_t *__restrict__ col, int64_t s
 
 // kShort: every out-row of the launch has <= 4 ids (the orientation's largest
 // out-degree is <= 4), so the tail and binary-search paths are compiled out
-template <int LM, bool kShort = false>
+// kPad: the rows come from the 16-byte padded copy (a.ocol4; kShort only):
+// a root's row and each neighbour's row are one aligned load each, with no
+// row bounds (vb and L are derived here; vb is read only for survivors)
+template <int LM, bool kShort = false, bool kPad = false>
 __device__ void root_thread(const RootArgs &a, int32_t r, int64_t vb, int L, unsigned long long &bytes) {
+    static_assert(!kPad || (kShort && LM == 4), "padded rows: sparse launches only");
     uint64_t adj = 0;
     typename std::conditional<kShort, unsigned, unsigned long long>::type T = 0;
+    int32_t V[LM];
     if (r < 0) {
         vb = 0;
         L = 0;
     }
-    if (r >= 0) {
-        int32_t V[LM];
+    if (kPad && r >= 0) {
+        const int4 x = __ldg(a.ocol4 + r);
+        V[0] = x.x;
+        V[1] = x.y;
+        V[2] = x.z;
+        V[3] = x.w;
+        L = (x.x >= 0) + (x.y >= 0) + (x.z >= 0) + (x.w >= 0);
+        int4 y[4];
+#pragma unroll
+        for (int p = 0; p < 4; ++p) y[p] = p < L ? __ldg(a.ocol4 + V[p]) : make_int4(-2, -2, -2, -2);
+#pragma unroll
+        for (int p = 0; p < 4; ++p) {
+            if (p >= L) break;
+            const int32_t u0 = y[p].x, u1 = y[p].y, u2 = y[p].z, u3 = y[p].w;
+            T += (u0 >= 0) + (u1 >= 0) + (u2 >= 0) + (u3 >= 0);
+            unsigned m = 0;
+#pragma unroll
+            for (int c = 0; c < 4; ++c)
+                m |= (unsigned)((V[c] == u0) | (V[c] == u1) | (V[c] == u2) | (V[c] == u3)) << c;
+            const unsigned lm = (__brev(m) >> (32 - L)) & 0xffu;
+            adj |= (uint64_t)lm << (8 * (L - 1 - p));
+        }
+        adj |= transpose8(adj);
+        // the method's bytes over the CSR, as for the unpadded path
+        bytes += 16ull + 20ull * (unsigned long long)L + 4ull * T;
+    }
+    if (!kPad && r >= 0) {
         if constexpr (LM == 4) {
             load4(a.ocol, vb, L, -1, V);
         } else {
@@ -421,7 +451,14 @@ __device__ void root_thread(const RootArgs &a, int32_t r, int64_t vb, int L, uns
                     const unsigned long long idx = atomicAdd(a.ctr + 3, 1ull);
                     if ((int64_t)idx < a.leaf_cap) {
                         a.leaf_rows[idx * 2] = __ldg(a.order + r);
-                        a.leaf_rows[idx * 2 + 1] = __ldg(a.order + __ldg(a.ocol + vb + (L - 1 - v)));
+                        int32_t w;
+                        if constexpr (kPad) {
+                            const int q = L - 1 - v;
+                            w = q == 0 ? V[0] : q == 1 ? V[1] : q == 2 ? V[2] : V[3];
+                        } else {
+                            w = __ldg(a.ocol + vb + (L - 1 - v));
+                        }
+                        a.leaf_rows[idx * 2 + 1] = __ldg(a.order + w);
                     }
                 }
             } else if (2 + pc >= a.need) {
@@ -448,6 +485,7 @@ __device__ void root_thread(const RootArgs &a, int32_t r, int64_t vb, int L, uns
         bl = __shfl_sync(0xffffffffu, bl, 0) + ol;
         bc = __shfl_sync(0xffffffffu, bc, 0) + oc;
         if (surv) {
+            if constexpr (kPad) vb = __ldg(a.orp + r);
             RootInfo ri;
             ri.r = r;
             ri.L = L;
@@ -547,6 +585,10 @@ __global__ void __launch_bounds__(kRootWarps * 32, ROOT_SPARSE_BLOCKS) root_expa
         const int64_t i = base + threadIdx.x;
         const int32_t r = i < a.count ? __ldg(a.list + i * a.stride) : -1;
 #endif
+        if (a.ocol4) {
+            root_thread<4, true, true>(a, r, 0, 0, bytes);
+            continue;
+        }
         int64_t vb = 0, ve = 0;
         if (r >= 0) row_bounds(a.orp, r, vb, ve);
         root_thread<4, true>(a, r, vb, (int)(ve - vb), bytes);

@@ -10,7 +10,7 @@ for ex in "$@"; do
   for c in $CFGS; do
     timeout 600 python bench.py --config $c --steps 5 --warmup 3 --no-cpu-baseline --no-e2e > gpurun_out/${TAG}_bench_${k}_$c.log 2>&1
     python -c "
-import json;l=[x for x in open('gpurun_out/${TAG}_bench_${k}_$c.log') if x.startswith('{')][-1];d=json.loads(l);p=d['details']['phases_ms'];print('[$ex] $c', d['details'].get('heuristic'), round(d['ms_per_step'],3), 'pre', round(p['preprocess_ms'],3), 'heur', round(p['heuristic_ms'],3), 'enum', round(p['host_enum_ms'],3), d['details']['omega'], d['details']['multiplicity'], d.get('verified',{}).get('ok'))" || tail -5 gpurun_out/${TAG}_bench_${k}_$c.log
+import json;l=[x for x in open('gpurun_out/${TAG}_bench_${k}_$c.log') if x.startswith('{')][-1];d=json.loads(l);p=d['details']['phases_ms'];print('[$ex] $c', d['details'].get('heuristic'), round(d['ms_per_step'],3), 'pre', round(p['preprocess_ms'],3), 'heur', round(p['heuristic_ms'],3), 'enum', round(p['host_enum_ms'],3), 'rootk', round(d['roofline'].get('kernel_ms_per_step') or 0,4), 'frac', round(d['roofline']['frac'],3), d['details']['omega'], d['details']['multiplicity'], d.get('verified',{}).get('ok'))" || tail -5 gpurun_out/${TAG}_bench_${k}_$c.log
   done
 done
 make -s -C paper_conf_ipps_geilpo23_b200/csrc clean > /dev/null
