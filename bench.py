@@ -394,6 +394,9 @@ def main():
     timings = []
     py_ms = []
     start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    start.record(stream)  # (the CUDA events are created at their first record: not inside a timed step)
+    end.record(stream)
+    torch.cuda.synchronize()
     with clocks:
         for _ in range(args.steps):
             flush.fill_(1)  # L2 flush (256 MiB > 126 MB L2) before every timed step
