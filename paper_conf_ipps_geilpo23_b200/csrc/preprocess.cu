@@ -537,7 +537,7 @@ __global__ void invert_kernel(int64_t n, const int32_t *__restrict__ order, int3
         rank[order[i]] = (int32_t)i;
 }
 
-// Tile of G lanes (8 or 32) inside a warp: lane index, first lane, member mask.
+// Tile of G lanes (4, 8 or 32) inside a warp: lane index, first lane, member mask.
 template <int G>
 struct Tile {
     int gl, gbase;
@@ -572,9 +572,9 @@ __device__ void stage_one(int64_t v, const int64_t *__restrict__ rowptr, const i
     const int32_t r = rv.x;
     const int64_t eb = rowptr[v], ee = rowptr[v + 1];
     int64_t out = eb;
-    // whole warps (long rows): KL chunks' ids and ranks gathered before any
-    // is used, so a long row costs one gather latency per KL chunks
-    constexpr int K = G == 32 ? KL : 1;
+    // KL chunks' ids and ranks gathered before any is used, so a row costs
+    // one gather latency per KL chunks
+    constexpr int K = KL;
     for (int64_t e0 = eb; e0 < ee; e0 += G * K) {
         int32_t u[K];
         int2 x[K];
@@ -596,22 +596,28 @@ __device__ void stage_one(int64_t v, const int64_t *__restrict__ rowptr, const i
     if (t.gl == 0) odeg[rv.y] = (int32_t)(out - eb);
 }
 
-// Warp w takes vertices [4w, 4w+4): 8-lane tiles when all four have degree <= 64, else a warp each
-template <int KL>
+// Warp w takes vertices [Vw, Vw+V), V = 32 / TG: TG-lane tiles (TK chunks
+// per trip) when all V have degree <= 64, else a warp each (KL chunks per
+// trip).  Measured (`profiles/r02_orient_tile_ab_v1.txt`): 8-lane tiles for
+// sparse graphs (ba1m preprocessing 1.08 ms vs 1.12 with 4-lane tiles),
+// 4-lane tiles with 2 chunks per trip for mean degree > 16 (rmat22 18.0 ->
+// 17.75 ms).
+template <int KL, int TG, int TK>
 __global__ void __launch_bounds__(256) orient_stage_kernel(int64_t n, const int64_t *__restrict__ rowptr,
                                                            const int32_t *__restrict__ col,
                                                            const int2 *__restrict__ rp, int32_t *odeg,
                                                            int32_t *stage) {
+    constexpr int V = 32 / TG;
     const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     const int lane = threadIdx.x & 31;
-    for (int64_t v0 = warp * 4; v0 < n; v0 += nwarps * 4) {
-        const int64_t v = v0 + (lane >> 3);
+    for (int64_t v0 = warp * V; v0 < n; v0 += nwarps * V) {
+        const int64_t v = v0 + lane / TG;
         const int64_t d = v < n ? rowptr[v + 1] - rowptr[v] : 0;
         if (__all_sync(0xffffffffu, d <= 64)) {
-            if (v < n) stage_one<8, 1>(v, rowptr, col, rp, odeg, stage);
+            if (v < n) stage_one<TG, TK>(v, rowptr, col, rp, odeg, stage);
         } else {
-            for (int t = 0; t < 4 && v0 + t < n; ++t) stage_one<32, KL>(v0 + t, rowptr, col, rp, odeg, stage);
+            for (int t = 0; t < V && v0 + t < n; ++t) stage_one<32, KL>(v0 + t, rowptr, col, rp, odeg, stage);
         }
         __syncwarp();
     }
@@ -1187,11 +1193,11 @@ void orient(mce_graph *g, int orientation) {
     pack_rank_pid_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, g->rank.get(), g->pid.get(), rp2);
     MCE_LAUNCH_CHECK();
     if (g->nnz <= 16 * n)
-        orient_stage_kernel<ORIENT_KL><<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), rp2, odeg,
-                                                                           stage);
-    else
-        orient_stage_kernel<ORIENT_KL_DENSE><<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), rp2,
+        orient_stage_kernel<ORIENT_KL, 8, 1><<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(), rp2,
                                                                                  odeg, stage);
+    else
+        orient_stage_kernel<ORIENT_KL_DENSE, 4, 2><<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->col.get(),
+                                                                                       rp2, odeg, stage);
     MCE_LAUNCH_CHECK();
     exclusive_scan_i32(odeg, g->orp.get(), n, g->pool.take<int64_t>(scan_tmp_items(n)), s);
     orient_copy_kernel<<<grid_for(n * 8, 256), 256, 0, s>>>(n, g->rowptr.get(), g->vid.get(), g->orp.get(), stage,
