@@ -159,6 +159,50 @@ def test_find_one_gather_takes_a_holder_of_omega():
         assert omega == 3 and count == 1 and cliques == [[9, 10, 11]]
 
 
+class _FakeGraph:
+    """Stands in for a graph handle in agree_core's host logic (CPU, gloo):
+    rank 0 "peels" (fills known cores and a peel order), the others record
+    what they are given."""
+
+    def __init__(self, n, rank):
+        self.n, self.rank, self.device = n, rank, 0
+        self.calls = []
+
+    def core_into(self, core, peel):
+        self.calls.append("core_into")
+        core.copy_(torch.arange(self.n, dtype=torch.int32) % 5)
+        peel.copy_(torch.arange(self.n - 1, -1, -1, dtype=torch.int32))
+
+    def set_core(self, core, peel):
+        self.calls.append(("set_core", core.tolist(), peel.tolist()))
+
+
+def _agree_core_body(rank, world):
+    g = _FakeGraph(7, rank)
+    mdist.agree_core(g)
+    opts = {}
+    mdist._agree(g, None, world, opts)  # default orientation: agree again
+    det = {"orientation": "degeneracy_det"}
+    mdist._agree(g, None, world, det)   # the deterministic order: no broadcast
+    deg = {"orientation": "degree"}
+    mdist._agree(g, None, world, deg)   # the degree order: no broadcast
+    return g.calls, opts
+
+
+def test_agree_core_broadcasts_rank0_cores_and_order():
+    """Multi-GPU orientation (distributed.agree_core): rank 0 peels once; every
+    other rank receives exactly its core numbers and peel order through one
+    broadcast and installs them (mce_set_core), for the degeneracy orientation
+    only."""
+    out = spawn(_agree_core_body)
+    want = ("set_core", [i % 5 for i in range(7)], list(range(6, -1, -1)))
+    calls0, opts0 = out[0]
+    calls1, opts1 = out[1]
+    assert calls0 == ["core_into", "core_into"]
+    assert calls1 == [want, want]
+    assert opts0 == opts1 == {"orientation": "degeneracy"}
+
+
 def test_cyclic_deal_partitions_every_root():
     for world in (1, 2, 3, 8):
         for count in (0, 1, 7, 100):
